@@ -1,0 +1,208 @@
+/*
+ * wg.h -- C ABI of the B200-native gTask graph-convolution layer
+ * (WiseGraph, Huang et al., EuroSys '24; this build's hot path is named by
+ * BASELINE.json north_star and SURVEY.md §8).
+ *
+ * Every entry point returns a wg_status; nothing throws, aborts or exits, and
+ * no CUDA or torch type appears in a signature (streams are passed as the
+ * opaque value of a cudaStream_t).  There is no CPU fallback: a call that
+ * cannot run on the GPU returns WG_ERR_UNSUPPORTED / WG_ERR_CUDA.
+ *
+ * Citations: "P:L<a>-<b>" = line range of the paper text and the
+ * section / figure / equation it falls in; "Q<n>" = a reading listed in
+ * DESIGN.md for a point the paper leaves open.
+ *
+ * Layout conventions (all calls):
+ *   - Vertex tensors are row-major [rows x ld] in the conv dtype (fp32 or
+ *     bf16); ld >= F and ld * sizeof(dtype) is a multiple of 16 bytes.
+ *     Input columns >= F are never read into a result; output columns in
+ *     [F, round_up(F, 16 B)) are written as 0, later pad columns untouched.
+ *   - Weights and biases are fp32 (master copies), row-major, exact shapes;
+ *     the library casts them to the conv dtype internally (RNE for bf16, Q23).
+ *   - Weight gradients are fp32, exact shapes, OVERWRITTEN (not accumulated).
+ *   - bf16 results are rounded to nearest even; accumulation is fp32.
+ * Ownership: the caller owns every tensor passed in (x, y, params, grads,
+ * saved, workspace, exchange).  The library owns graph / plan internals
+ * (device memory allocated on the creation stream, freed by *_destroy).
+ * Graphs and plans are immutable after creation; a plan must not outlive
+ * its graph.
+ * Errors: argument / range errors are detected synchronously in *_create
+ * (WG_ERR_INVALID / WG_ERR_RANGE); kernel faults surface as WG_ERR_CUDA on a
+ * later call.  wg_last_error() returns a thread-local message.
+ */
+#ifndef WG_H_
+#define WG_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  WG_OK = 0,
+  WG_ERR_INVALID = 1,      /* bad argument / descriptor                     */
+  WG_ERR_RANGE = 2,        /* vertex id or type out of range                */
+  WG_ERR_NOMEM = 3,        /* device allocation failed                      */
+  WG_ERR_CUDA = 4,         /* CUDA runtime / kernel error                   */
+  WG_ERR_UNSUPPORTED = 6,  /* valid but not implemented combination         */
+  WG_ERR_STATE = 7         /* misuse of handles                             */
+} wg_status;
+
+typedef enum { WG_GCN = 0, WG_GIN = 1, WG_SAGE = 2, WG_GAT = 3, WG_RGCN = 4 } wg_model;
+typedef enum { WG_F32 = 0, WG_BF16 = 1 } wg_dtype;
+/* GCN [24] / RGCN [34] edge coefficient c_e (Q2, Q3):
+ * NONE: 1; RIGHT: 1/deg_in(dst) (RGCN: 1/|in(dst) of type r|);
+ * BOTH: deg_out(src)^-1/2 * deg_in(dst)^-1/2.  Degrees clamp to >= 1.    */
+typedef enum { WG_NORM_NONE = 0, WG_NORM_RIGHT = 1, WG_NORM_BOTH = 2 } wg_norm;
+/* Per-gTask operation plan (a4): EDGE = gather-then-transform, VERTEX =
+ * transform-before-gather (T2 "indexing swapping").          */
+typedef enum { WG_PLAN_AUTO = 0, WG_PLAN_ALL_EDGE = 1, WG_PLAN_ALL_VERTEX = 2,
+               WG_PLAN_RANDOM = 3 } wg_plan_policy;
+
+typedef void* wg_stream;                 /* a cudaStream_t value (0 = legacy) */
+typedef struct wg_graph_s* wg_graph;
+typedef struct wg_plan_s* wg_plan;
+
+/* ------------------------------------------------------------------------ */
+/* Graph ingest + gTask partition (a1-a3).                                  */
+/* Edge attributes src-id / dst-id / edge-type (Fig 5a).      */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+  int64_t num_vertices;     /* V (global), 1 <= V < 2^31                          */
+  int64_t num_edges;        /* E, 0 <= E < 2^31                                   */
+  const int64_t* indptr;    /* CSR over dst, length V+1; NULL => COO (dst given)  */
+  const int32_t* src;       /* length E                                           */
+  const int32_t* dst;       /* length E (COO); ignored when indptr != NULL        */
+  const int32_t* etype;     /* length E, in [0, num_types); NULL => one relation  */
+  int32_t num_types;        /* R >= 1; gTasks are split by type iff R > 1 && etype */
+  int32_t tile_rows;        /* T (dst-range restriction, Q11); 0 => 128           */
+  int64_t max_task_edges;   /* E_max (uniq(edge-id) <= E_max, Q13); 0 => default  */
+  int64_t v_begin, v_end;   /* owned vertex range for a 1-D partition (multiple of */
+                            /* T, except v_end == V); both 0 => [0, V)            */
+} wg_graph_desc;
+/* Pointers may be host or device memory (detected with
+ * cudaPointerGetAttributes); the call copies what it needs and returns after
+ * the partition is complete (synchronous on `stream`).                      */
+
+/* gTask record (D5).  Forward graph: key vertex = dst; transposed graph
+ * (backward): key vertex = src.  e_begin/e_end are positions in this
+ * graph's perm order; tile / d_lo / d_hi are GLOBAL vertex-derived ids.     */
+typedef struct {
+  int32_t tile, type;
+  int64_t e_begin, e_end;
+  int32_t d_lo, d_hi;       /* first / last key vertex                            */
+  int32_t flags;            /* WG_TASK_SPLIT: chunk of a key segment > E_max      */
+  int32_t n_uniq_src;       /* distinct other-endpoint ids in the task            */
+} wg_task;
+#define WG_TASK_SPLIT 1
+
+wg_status wg_graph_create(const wg_graph_desc* desc, int device, wg_stream stream, wg_graph* out);
+/* info[0..9]: V, owned rows, E_fwd (local in-edges), E_T (local out-edges),
+ * n_tasks, n_tasks_T, T, E_max, by_type, max in-degree                      */
+wg_status wg_graph_info(wg_graph g, int64_t info[10]);
+/* Copies the partition to HOST memory.  transposed = 0: forward tables
+ * (perm = GLOBAL edge ids in sorted order); 1: transposed tables.  fwdpos
+ * (transposed only, may be NULL): fwdpos_of_T[j] = inv(perm)[perm_T[j]],
+ * valid when the graph owns all rows.                                      */
+wg_status wg_graph_export(wg_graph g, int transposed, int64_t* perm, wg_task* tasks, int64_t* fwdpos);
+wg_status wg_graph_destroy(wg_graph g);
+
+/* ------------------------------------------------------------------------ */
+/* Plan (a4): per-gTask EDGE / VERTEX choice by an integer cost model of     */
+/* FLOP + memory volume.             */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+  wg_model model;
+  wg_dtype dtype;
+  int32_t f_in, f_out;      /* GAT: f_out is per head                            */
+  int32_t heads;            /* GAT only (>= 1)                                   */
+  int32_t concat_heads;     /* GAT: 1 = concat heads, 0 = mean (last layer, Q6)  */
+  wg_norm norm;             /* GCN / RGCN                                        */
+  int32_t self_loop;        /* RGCN: add x[v] W_0                                */
+  int32_t bias;             /* add a bias                                        */
+  int32_t fuse_relu;        /* ReLU applied to the conv output (Q7)              */
+  float gin_eps;            /* GIN epsilon (Q5: 0)                               */
+  float neg_slope;          /* GAT LeakyReLU slope (Q6: 0.2)                     */
+  wg_plan_policy policy;
+  uint64_t policy_seed;     /* WG_PLAN_RANDOM                                    */
+  int32_t need_dx;          /* backward produces dx (0 for the input layer)      */
+} wg_conv_desc;
+
+wg_status wg_plan_create(wg_graph g, const wg_conv_desc* desc, wg_plan* out);
+/* Bytes of the caller-owned `saved` (forward -> backward) and `workspace`
+ * buffers; both 256-byte aligned device memory.                            */
+wg_status wg_plan_sizes(wg_plan p, size_t* saved_bytes, size_t* workspace_bytes);
+/* per_task_plan (host, n_tasks bytes, may be NULL): 0 = EDGE, 1 = VERTEX.
+ * stats (host, may be NULL) [0..7]: n EDGE tasks, n VERTEX tasks, backward
+ * path (0 = dAgg, 1 = G), exchange width fwd, exchange width bwd (elements,
+ * 0 = the exchanged table is x itself), n work items fwd, n work items T,
+ * n split rows fwd.                                                        */
+wg_status wg_plan_export(wg_plan p, uint8_t* per_task_plan, int64_t stats[8]);
+wg_status wg_plan_destroy(wg_plan p);
+
+/* ------------------------------------------------------------------------ */
+/* Forward / backward (a5-a11).  Parameters (fp32, device):                  */
+/*   GCN : W [f_in x f_out], bias [f_out]                                   */
+/*   SAGE: W = W_neigh, W_self [f_in x f_out], bias [f_out]                 */
+/*   GIN : W = W1 [f_in x f_out], bias = b1, W2 [f_out x f_out], b2         */
+/*   GAT : W [f_in x heads*f_out], attn_l / attn_r [heads x f_out],         */
+/*         bias [heads*f_out] (concat) or [f_out] (mean)                    */
+/*   RGCN: W [R x f_in x f_out], W_self = W_0 (self_loop), bias             */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+  const float *W, *W_self, *bias, *attn_l, *attn_r, *W2, *b2;
+} wg_params;
+typedef struct {
+  float *W, *W_self, *bias, *attn_l, *attn_r, *W2, *b2;   /* NULL => skip */
+} wg_grads;
+
+/* Phases for the 1-D multi-GPU layer (§8(e)).  Single GPU: WG_PHASE_ALL.
+ * PRE computes this rank's rows of the exchange table into
+ * `xchg + row_offset * ld_xchg`; the caller all-gathers `xchg` (in place);
+ * POST consumes the gathered table.                                        */
+typedef enum { WG_PHASE_ALL = 0, WG_PHASE_PRE = 1, WG_PHASE_POST = 2 } wg_phase;
+
+typedef struct {
+  int32_t phase;
+  const void* x;            /* [V_global x ldx]: all rows (gathered when distributed) */
+  int64_t ldx;
+  void* y;                  /* [owned rows x ldy] output                          */
+  int64_t ldy;
+  void* saved;              /* wg_plan_sizes().saved bytes                        */
+  void* workspace;          /* wg_plan_sizes().workspace bytes                    */
+  void* xchg;               /* exchange table [V_global x ld_xchg] (or NULL)      */
+  int64_t ld_xchg;
+} wg_fwd_args;
+
+typedef struct {
+  int32_t phase;
+  const void* dy;           /* [owned rows x lddy] gradient of the conv output    */
+  int64_t lddy;
+  const void* x;            /* forward input, as in wg_fwd_args                   */
+  int64_t ldx;
+  const void* y;            /* forward output (needed when fuse_relu)             */
+  int64_t ldy;
+  const void* saved;
+  void* dx;                 /* [owned rows x lddx], written when need_dx          */
+  int64_t lddx;
+  void* workspace;
+  void* xchg;
+  int64_t ld_xchg;
+} wg_bwd_args;
+
+wg_status wg_conv_forward(wg_plan p, const wg_params* params, const wg_fwd_args* a, wg_stream stream);
+wg_status wg_conv_backward(wg_plan p, const wg_params* params, const wg_bwd_args* a,
+                           const wg_grads* grads, wg_stream stream);
+
+/* ------------------------------------------------------------------------ */
+const char* wg_status_string(wg_status s);
+const char* wg_last_error(void);
+/* Number of kernels this library has launched on the calling thread. */
+int64_t wg_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* WG_H_ */

@@ -1,0 +1,294 @@
+"""B200-native gTask graph-convolution layer (WiseGraph, EuroSys '24 hot path).
+
+Python binding over the C ABI of ``include/wg.h`` (``libwg.so``).  PyTorch is
+used for device memory, streams and process groups only; every step of the
+layer runs in the library's CUDA kernels.  There is no CPU fallback.
+
+    g = Graph(src, dst, num_vertices=V)                  # a1-a3 (GPU partition)
+    conv = Conv(g, "sage", f_in, f_out, dtype=torch.bfloat16, fuse_relu=True)
+    y = conv(x, params)                                  # autograd-aware
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+import torch
+
+from . import _capi as C
+from ._capi import WGError, TASK_DTYPE
+
+__all__ = ["Graph", "Conv", "WGError", "TASK_DTYPE", "padded", "pad_to", "ld_of", "launch_count", "init_params"]
+
+
+def _ptr(t):
+    if t is None:
+        return None
+    if isinstance(t, torch.Tensor):
+        return ctypes.c_void_p(t.data_ptr())
+    if isinstance(t, np.ndarray):
+        return t.ctypes.data_as(ctypes.c_void_p)
+    return t
+
+
+def _stream(stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _dt(dtype):
+    if dtype == torch.float32:
+        return C.WG_F32
+    if dtype == torch.bfloat16:
+        return C.WG_BF16
+    raise WGError(f"unsupported dtype {dtype}")
+
+
+def pitch(F: int, dtype) -> int:
+    """Row pitch (elements): rows padded to 32 bytes (one DRAM sector)."""
+    s = torch.empty((), dtype=dtype).element_size()
+    return -(-F * s // 32) * 32 // s
+
+
+def padded(rows: int, F: int, dtype, device="cuda", zero=True):
+    """[rows x F] view of a [rows x pitch(F)] buffer."""
+    ld = pitch(F, dtype)
+    buf = (torch.zeros if zero else torch.empty)((rows, ld), dtype=dtype, device=device)
+    return buf[:, :F]
+
+
+def ld_of(t: torch.Tensor) -> int:
+    if t.dim() != 2 or t.stride(1) != 1:
+        raise WGError("vertex tensors must be 2-D row-major views")
+    if (t.stride(0) * t.element_size()) % 16:
+        raise WGError("row pitch must be a multiple of 16 bytes (use padded())")
+    return t.stride(0)
+
+
+def pad_to(t: torch.Tensor) -> torch.Tensor:
+    """Return a view of ``t`` whose row pitch satisfies the ABI (copies if needed)."""
+    if t.dim() == 2 and t.stride(1) == 1 and (t.stride(0) * t.element_size()) % 16 == 0 and t.stride(0) >= t.shape[1]:
+        return t
+    out = padded(t.shape[0], t.shape[1], t.dtype, t.device, zero=True)
+    out.copy_(t)
+    return out
+
+
+def launch_count() -> int:
+    return int(C.lib().wg_launch_count())
+
+
+class Graph:
+    """Device graph + forward / transposed gTask partitions (wg_graph_create)."""
+
+    def __init__(self, src, dst=None, *, num_vertices: int, indptr=None, etype=None, num_types: int = 1,
+                 tile_rows: int = 128, max_task_edges: int = 0, v_begin: int = 0, v_end: int = 0,
+                 device: int | None = None, stream=None):
+        L = C.lib()
+        self._keep = []
+
+        def arr(a, dt):
+            if a is None:
+                return None
+            if isinstance(a, torch.Tensor):
+                a = a.to(dt).contiguous()
+            else:
+                a = np.ascontiguousarray(a, dtype={torch.int32: np.int32, torch.int64: np.int64}[dt])
+            self._keep.append(a)
+            return a
+
+        s = arr(src, torch.int32)
+        d = arr(dst, torch.int32)
+        ip = arr(indptr, torch.int64)
+        et = arr(etype, torch.int32)
+        E = (s.shape[0] if s is not None else 0)
+        desc = C.GraphDesc(num_vertices, E, _ptr(ip), _ptr(s), _ptr(d), _ptr(et), num_types, tile_rows,
+                           max_task_edges, v_begin, v_end)
+        self.device = torch.cuda.current_device() if device is None else device
+        h = ctypes.c_void_p()
+        with torch.cuda.device(self.device):
+            C.check(L.wg_graph_create(ctypes.byref(desc), self.device, _stream(stream), ctypes.byref(h)),
+                    "wg_graph_create")
+        self._h = h
+        self._keep = []
+        info = (ctypes.c_int64 * 10)()
+        C.check(L.wg_graph_info(self._h, info), "wg_graph_info")
+        (self.V, self.n_rows, self.E_fwd, self.E_T, self.n_tasks, self.n_tasks_T, self.T, self.E_max,
+         self.by_type, self.max_in_degree) = list(info)
+        self.v_begin = v_begin
+        self.num_types = num_types
+        self._plans = 0
+
+    @property
+    def handle(self):
+        return self._h
+
+    def export(self, transposed: bool = False):
+        """(perm int64[E], tasks TASK_DTYPE[n], fwdpos or None) as numpy (host) arrays."""
+        E = self.E_T if transposed else self.E_fwd
+        n = self.n_tasks_T if transposed else self.n_tasks
+        perm = np.empty(max(E, 1), np.int64)
+        tasks = np.empty(max(n, 1), TASK_DTYPE)
+        fwdpos = np.empty(max(E, 1), np.int64) if (transposed and self.n_rows == self.V) else None
+        C.check(C.lib().wg_graph_export(self._h, int(transposed), _ptr(perm), _ptr(tasks), _ptr(fwdpos)),
+                "wg_graph_export")
+        return perm[:E], tasks[:n], (fwdpos[:E] if fwdpos is not None else None)
+
+    def close(self):
+        if getattr(self, "_h", None):
+            C.check(C.lib().wg_graph_destroy(self._h), "wg_graph_destroy")
+            self._h = None
+
+    def __del__(self):
+        try:
+            if getattr(self, "_h", None) and self._plans == 0:
+                C.lib().wg_graph_destroy(self._h)
+                self._h = None
+        except Exception:
+            pass
+
+
+PARAM_NAMES = ("W", "W_self", "bias", "attn_l", "attn_r", "W2", "b2")
+
+
+class Conv:
+    """One gTask graph-convolution layer bound to a graph (wg_plan_create)."""
+
+    def __init__(self, graph: Graph, model: str, f_in: int, f_out: int, *, dtype=torch.float32, heads: int = 1,
+                 concat: bool = True, norm: str = "both", self_loop: bool = False, bias: bool = True,
+                 fuse_relu: bool = False, gin_eps: float = 0.0, neg_slope: float = 0.2, policy: str = "auto",
+                 seed: int = 0, need_dx: bool = True):
+        self.graph = graph
+        self.model = model
+        self.f_in, self.f_out, self.heads, self.concat = f_in, f_out, heads, concat
+        self.dtype = dtype
+        self.fuse_relu = fuse_relu
+        self.bias = bias
+        self.need_dx = need_dx
+        self.desc = C.ConvDesc(C.MODELS[model], _dt(dtype), f_in, f_out, heads, int(concat), C.NORMS[norm],
+                               int(self_loop), int(bias), int(fuse_relu), gin_eps, neg_slope, C.POLICIES[policy],
+                               seed, int(need_dx))
+        h = ctypes.c_void_p()
+        C.check(C.lib().wg_plan_create(graph.handle, ctypes.byref(self.desc), ctypes.byref(h)), "wg_plan_create")
+        self._h = h
+        graph._plans += 1
+        sb, wb = ctypes.c_size_t(), ctypes.c_size_t()
+        C.check(C.lib().wg_plan_sizes(self._h, ctypes.byref(sb), ctypes.byref(wb)), "wg_plan_sizes")
+        self.saved_bytes, self.ws_bytes = sb.value, wb.value
+        dev = torch.device("cuda", graph.device)
+        self.workspace = torch.empty(max(self.ws_bytes, 256), dtype=torch.uint8, device=dev)
+        stats = (ctypes.c_int64 * 8)()
+        C.check(C.lib().wg_plan_export(self._h, None, stats), "wg_plan_export")
+        (self.n_edge_tasks, self.n_vertex_tasks, self.bwd_path, self.xchg_fwd, self.xchg_bwd, self.n_items,
+         self.n_items_T, self.n_split_rows) = list(stats)
+        self.out_dim = heads * f_out if (model == "gat" and concat) else f_out
+
+    def plan_bits(self) -> np.ndarray:
+        out = np.empty(max(self.graph.n_tasks, 1), np.uint8)
+        C.check(C.lib().wg_plan_export(self._h, _ptr(out), None), "wg_plan_export")
+        return out[: self.graph.n_tasks]
+
+    def new_saved(self):
+        return torch.empty(max(self.saved_bytes, 256), dtype=torch.uint8, device=self.workspace.device)
+
+    # ------------------------------------------------------------------ raw calls
+    def forward_raw(self, x, params: dict, y=None, saved=None, phase=C.PHASE_ALL, xchg=None, stream=None):
+        rows = self.graph.n_rows
+        if y is None:
+            y = padded(rows, self.out_dim, self.dtype, x.device, zero=False)
+        if saved is None:
+            saved = self.new_saved()
+        pr = C.Params(*[_ptr(params.get(n)) for n in PARAM_NAMES])
+        a = C.FwdArgs(phase, _ptr(x), ld_of(x), _ptr(y), ld_of(y), _ptr(saved), _ptr(self.workspace),
+                      _ptr(xchg), ld_of(xchg) if xchg is not None else 0)
+        C.check(C.lib().wg_conv_forward(self._h, ctypes.byref(pr), ctypes.byref(a), _stream(stream)),
+                "wg_conv_forward")
+        return y, saved
+
+    def backward_raw(self, dy, x, y, saved, params: dict, dx=None, phase=C.PHASE_ALL, xchg=None, stream=None,
+                     grads: dict | None = None):
+        dev = dy.device
+        if grads is None:
+            grads = {n: torch.empty_like(params[n], dtype=torch.float32) for n in PARAM_NAMES
+                     if params.get(n) is not None}
+        if self.need_dx and dx is None:
+            dx = padded(self.graph.n_rows, self.f_in, self.dtype, dev, zero=False)
+        pr = C.Params(*[_ptr(params.get(n)) for n in PARAM_NAMES])
+        gr = C.Grads(*[_ptr(grads.get(n)) for n in PARAM_NAMES])
+        a = C.BwdArgs(phase, _ptr(dy), ld_of(dy), _ptr(x), ld_of(x), _ptr(y), ld_of(y) if y is not None else 0,
+                      _ptr(saved), _ptr(dx), ld_of(dx) if dx is not None else 0, _ptr(self.workspace),
+                      _ptr(xchg), ld_of(xchg) if xchg is not None else 0)
+        C.check(C.lib().wg_conv_backward(self._h, ctypes.byref(pr), ctypes.byref(a), ctypes.byref(gr),
+                                         _stream(stream)), "wg_conv_backward")
+        return dx, grads
+
+    # ------------------------------------------------------------------ autograd
+    def __call__(self, x, params: dict):
+        names = [n for n in PARAM_NAMES if params.get(n) is not None]
+        return _ConvFn.apply(self, names, pad_to(x), *[params[n] for n in names])
+
+    def close(self):
+        if getattr(self, "_h", None):
+            C.check(C.lib().wg_plan_destroy(self._h), "wg_plan_destroy")
+            self._h = None
+            self.graph._plans -= 1
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class _ConvFn(torch.autograd.Function):
+    @staticmethod
+    def forward(ctx, conv: Conv, names, x, *tensors):
+        params = dict(zip(names, tensors))
+        y, saved = conv.forward_raw(x, params)
+        ctx.conv, ctx.names = conv, names
+        ctx.save_for_backward(x, y, *tensors)
+        ctx.saved_buf = saved
+        return y
+
+    @staticmethod
+    def backward(ctx, dy):
+        conv = ctx.conv
+        x, y, *tensors = ctx.saved_tensors
+        params = dict(zip(ctx.names, tensors))
+        dx, grads = conv.backward_raw(pad_to(dy.contiguous() if dy.stride(1) != 1 else dy), x, y, ctx.saved_buf,
+                                      params)
+        return (None, None, dx if conv.need_dx else None, *[grads.get(n) for n in ctx.names])
+
+
+def init_params(model: str, f_in: int, f_out: int, *, heads: int = 1, concat: bool = True, R: int = 1,
+                self_loop: bool = False, bias: bool = True, device="cuda", seed: int = 0) -> dict:
+    """Glorot-initialised fp32 master parameters for one layer (random init, no checkpoint)."""
+    g = torch.Generator(device="cpu").manual_seed(seed)
+
+    def glorot(*shape, fan_in, fan_out):
+        lim = (6.0 / (fan_in + fan_out)) ** 0.5
+        return ((torch.rand(*shape, generator=g) * 2 - 1) * lim).to(device)
+
+    p = {}
+    if model == "gat":
+        p["W"] = glorot(f_in, heads * f_out, fan_in=f_in, fan_out=heads * f_out)
+        p["attn_l"] = glorot(heads, f_out, fan_in=f_out, fan_out=1)
+        p["attn_r"] = glorot(heads, f_out, fan_in=f_out, fan_out=1)
+        if bias:
+            p["bias"] = torch.zeros(heads * f_out if concat else f_out, device=device)
+    elif model == "rgcn":
+        p["W"] = glorot(R, f_in, f_out, fan_in=f_in, fan_out=f_out)
+        if self_loop:
+            p["W_self"] = glorot(f_in, f_out, fan_in=f_in, fan_out=f_out)
+        if bias:
+            p["bias"] = torch.zeros(f_out, device=device)
+    else:
+        p["W"] = glorot(f_in, f_out, fan_in=f_in, fan_out=f_out)
+        if model == "sage":
+            p["W_self"] = glorot(f_in, f_out, fan_in=f_in, fan_out=f_out)
+        if model == "gin":
+            p["W2"] = glorot(f_out, f_out, fan_in=f_out, fan_out=f_out)
+            p["b2"] = torch.zeros(f_out, device=device)
+        if bias or model == "gin":
+            p["bias"] = torch.zeros(f_out, device=device)
+    return p

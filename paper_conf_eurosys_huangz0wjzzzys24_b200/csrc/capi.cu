@@ -1,0 +1,60 @@
+// C-ABI glue: status strings, thread-local error text, launch counter and
+// the forward / backward dispatch by model.
+#include "plan.h"
+
+namespace wg {
+namespace {
+thread_local std::string g_err;
+thread_local int64_t g_launches = 0;
+}  // namespace
+void set_error(const std::string& msg) { g_err = msg; }
+int64_t& launch_counter() { return g_launches; }
+}  // namespace wg
+
+extern "C" {
+
+const char* wg_status_string(wg_status s) {
+  switch (s) {
+    case WG_OK: return "ok";
+    case WG_ERR_INVALID: return "invalid argument";
+    case WG_ERR_RANGE: return "out of range";
+    case WG_ERR_NOMEM: return "out of device memory";
+    case WG_ERR_CUDA: return "CUDA error";
+    case WG_ERR_UNSUPPORTED: return "unsupported";
+    case WG_ERR_STATE: return "invalid state";
+  }
+  return "unknown status";
+}
+
+const char* wg_last_error(void) { return wg::g_err.c_str(); }
+
+int64_t wg_launch_count(void) { return wg::launch_counter(); }
+
+wg_status wg_conv_forward(wg_plan p, const wg_params* params, const wg_fwd_args* a, wg_stream stream) {
+  WG_REQ(p && params && a, WG_ERR_INVALID, "wg_conv_forward: null argument");
+  WG_CK(cudaSetDevice(p->g->device));
+  WG_CK(cudaGetLastError());
+  cudaStream_t s = (cudaStream_t)stream;
+  switch (p->d.model) {
+    case WG_GCN: case WG_SAGE: case WG_GIN: return wg::lin_forward(p, params, a, s);
+    case WG_GAT: return wg::gat_forward(p, params, a, s);
+    case WG_RGCN: return wg::rgcn_forward(p, params, a, s);
+  }
+  return WG_ERR_INVALID;
+}
+
+wg_status wg_conv_backward(wg_plan p, const wg_params* params, const wg_bwd_args* a, const wg_grads* grads,
+                           wg_stream stream) {
+  WG_REQ(p && params && a, WG_ERR_INVALID, "wg_conv_backward: null argument");
+  WG_CK(cudaSetDevice(p->g->device));
+  WG_CK(cudaGetLastError());
+  cudaStream_t s = (cudaStream_t)stream;
+  switch (p->d.model) {
+    case WG_GCN: case WG_SAGE: case WG_GIN: return wg::lin_backward(p, params, a, grads, s);
+    case WG_GAT: return wg::gat_backward(p, params, a, grads, s);
+    case WG_RGCN: return wg::rgcn_backward(p, params, a, grads, s);
+  }
+  return WG_ERR_INVALID;
+}
+
+}  // extern "C"

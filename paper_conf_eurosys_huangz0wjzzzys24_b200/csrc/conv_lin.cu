@@ -1,0 +1,387 @@
+// GCN / GraphSAGE-mean / GIN layers: forward (a5-a8) and backward (a9-a11).
+//
+// All three are "aggregate + linear transform" layers, so the two operation
+// plans of the paper apply (T2 indexing swapping):
+//   EDGE   (gather-then-transform): Agg = A_hat x   ->  y = Agg W
+//   VERTEX (transform-before-gather): Y = x W      ->  y = A_hat Y
+// chosen per gTask by the plan (plan.cu).  A mixed plan writes Agg rows for
+// EDGE gTasks and Z rows for VERTEX gTasks (each row belongs to exactly one
+// gTask or SPLIT row) and the final GEMM computes y = Agg W + Z + b.
+//
+// Backward (the paper is silent, Q8; exact gradients of the definitions in
+// DESIGN.md "Backward") runs the same gather pattern over the transposed gTask
+// partition, in one of two orders:
+//   dAgg path (all-EDGE forward, Agg saved):  dAgg = dT W^T, dx = A_hat^T dAgg,
+//                                             dW = Agg^T dT
+//   G path (otherwise):                       G = A_hat^T dT, dx = G W^T,
+//                                             dW = x^T G
+// where dT is dy masked by the fused ReLU.
+#include "plan.h"
+
+namespace wg {
+
+namespace {
+
+struct Ctx {
+  wg_plan_s* p;
+  wg_graph_s* g;
+  wg_dtype dt;
+  int s;        // dtype bytes
+  int fi, fo;
+  int64_t pi, po, nr, Vg, vb;
+  int64_t wrows_o, wrows_i;   // padded weight row counts
+};
+
+Ctx mk(wg_plan_s* p) {
+  Ctx c;
+  c.p = p; c.g = p->g; c.dt = p->d.dtype; c.s = dsize(c.dt);
+  c.fi = p->d.f_in; c.fo = p->d.f_out;
+  c.pi = p->pi; c.po = p->po;
+  c.nr = c.g->ve - c.g->vb; c.Vg = c.g->V; c.vb = c.g->vb;
+  c.wrows_o = rup(c.fo, 16); c.wrows_i = rup(c.fi, 16);
+  return c;
+}
+
+int64_t part_ld(const Ctx& c) { return rup(std::max(c.fi, c.fo), 8); }
+
+char* off(const void* base, int64_t rows, int64_t ld, int s) {
+  return (char*)base + rows * ld * s;
+}
+
+}  // namespace
+
+void lin_layout(wg_plan_s* p) {
+  const wg_conv_desc& d = p->d;
+  p->pi = pitch(d.f_in, d.dtype);
+  p->po = pitch(d.f_out, d.dtype);
+  Ctx c = mk(p);
+  const int s = c.s;
+  Layout& S = p->saved;
+  Layout& W = p->ws;
+  S = Layout();
+  W = Layout();
+  const bool sage = d.model == WG_SAGE, gin = d.model == WG_GIN;
+  if (p->n_edge_tasks > 0) S.add("agg", (size_t)c.nr * c.pi * s);
+  if (gin) S.add("h", (size_t)c.nr * c.po * s);
+  // prepped weights (forward: transposed [rows_o x pi]; backward: [rows_i x po])
+  W.add("wt", (size_t)c.wrows_o * c.pi * s);          // W^T (GCN W, SAGE W_n, GIN W1)
+  W.add("w", (size_t)c.wrows_i * c.po * s);           // W
+  if (sage) {
+    W.add("wst", (size_t)c.wrows_o * c.pi * s);
+    W.add("ws", (size_t)c.wrows_i * c.po * s);
+    W.add("wys", (size_t)2 * c.po * c.pi * s);       // [W_n^T ; W_s^T] stacked along N
+    W.add("wbs", (size_t)2 * c.pi * c.po * s);       // [W_n ; W_s] stacked along N
+    W.add("s", (size_t)c.nr * c.po * s);             // x W_s (all-VERTEX forward)
+    W.add("dxs", (size_t)c.nr * c.pi * s);           // dy W_s^T (dAgg path)
+  }
+  if (gin) {
+    W.add("w2t", (size_t)c.wrows_o * c.po * s);
+    W.add("w2", (size_t)c.wrows_o * c.po * s);
+    W.add("da", (size_t)c.Vg * c.po * s);
+  }
+  if (p->n_vert_tasks > 0) W.add("y", (size_t)c.Vg * c.po * s);
+  if (p->mixed) W.add("z", (size_t)c.nr * c.po * s);
+  const int64_t pl = part_ld(c);
+  W.add("part", sizeof(float) * (size_t)std::max(1, p->n_slots_f) * pl);
+  W.add("partT", sizeof(float) * (size_t)std::max(1, p->n_slots_t) * pl);
+  // backward
+  W.add("dt", (size_t)c.Vg * c.po * s);
+  W.add("colsum", bias_grad_scratch(c.nr, (int)std::max(c.po, c.pi)));
+  W.add("tn", gemm_tn_scratch(c.nr, (int)c.fi, (int)c.fo) + gemm_tn_scratch(c.nr, (int)c.fo, (int)c.fo));
+  W.add("dagg", (size_t)c.Vg * c.pi * s);
+  W.add("g", (size_t)c.nr * c.po * s);
+}
+
+namespace {
+
+AggArgs agg_base(const Ctx& c, const ItemList& L, const Side& S) {
+  AggArgs a{};
+  a.items = L.d;
+  a.n_items = L.n;
+  a.row_ptr = S.row_ptr;
+  a.idx = S.idx;
+  a.row_base = c.vb;
+  a.self_coef = 1.f;
+  a.E_max = c.g->E_max;
+  return a;
+}
+
+CombineArgs comb_from(const AggArgs& a, const ItemList& L, int plan_filter) {
+  CombineArgs b{};
+  b.rows = L.split; b.n_rows = L.n_split;
+  b.partial = a.partial; b.ld_part = a.ld_part;
+  b.rscale = a.rscale; b.row_base = a.row_base;
+  b.self_tab = a.self_tab; b.ld_self = a.ld_self; b.self_coef = a.self_coef;
+  b.bias = a.bias; b.relu = a.relu; b.mask_ref = a.mask_ref; b.ld_mask = a.ld_mask;
+  b.out = a.out; b.ld_out = a.ld_out;
+  b.zero_out = a.zero_out; b.ld_zero = a.ld_zero; b.zero_cols = a.zero_cols;
+  b.F = a.F; b.plan_filter = plan_filter;
+  return b;
+}
+
+wg_status run_agg(const Ctx& c, AggArgs a, const ItemList& L, cudaStream_t st) {
+  WG_TRY(launch_agg(c.dt, a, st));
+  WG_TRY(launch_combine(c.dt, comb_from(a, L, -1), st));
+  return WG_OK;
+}
+
+// GCN edge coefficient c_e = gs[src] * rs[dst] (Q3)
+void gcn_scales(const Ctx& c, const float** gs_src, const float** rs_dst) {
+  *gs_src = nullptr; *rs_dst = nullptr;
+  if (c.p->d.model == WG_SAGE) { *rs_dst = c.g->inv_in; return; }
+  if (c.p->d.model != WG_GCN) return;
+  if (c.p->d.norm == WG_NORM_BOTH) { *gs_src = c.g->rs_out; *rs_dst = c.g->rs_in; }
+  else if (c.p->d.norm == WG_NORM_RIGHT) { *rs_dst = c.g->inv_in; }
+}
+
+}  // namespace
+
+wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cudaStream_t st) {
+  Ctx c = mk(p);
+  const wg_conv_desc& d = p->d;
+  const bool sage = d.model == WG_SAGE, gin = d.model == WG_GIN;
+  const bool pre = A->phase != WG_PHASE_POST, post = A->phase != WG_PHASE_PRE;
+  WG_REQ(P && P->W, WG_ERR_INVALID, "params->W is NULL");
+  WG_REQ(!sage || P->W_self, WG_ERR_INVALID, "SAGE needs W_self");
+  WG_REQ(!gin || P->W2, WG_ERR_INVALID, "GIN needs W2");
+  WG_REQ(A->x && A->y && A->workspace, WG_ERR_INVALID, "x / y / workspace is NULL");
+  WG_REQ(p->n_edge_tasks == 0 || A->saved, WG_ERR_INVALID, "saved is NULL");
+  WG_REQ((A->ldx * c.s) % 16 == 0 && A->ldx >= c.fi && (A->ldy * c.s) % 16 == 0 && A->ldy >= c.fo, WG_ERR_INVALID,
+         "ldx / ldy must be >= F and 16-byte multiples");
+  const bool dist = c.nr != c.Vg;
+  WG_REQ(!dist || !p->mixed, WG_ERR_UNSUPPORTED, "mixed EDGE/VERTEX plans are not supported with a 1-D partition");
+  void* ws = A->workspace;
+  const Layout& L = p->ws;
+  const char* x_own = off(A->x, c.vb, A->ldx, c.s);
+  const float *gs, *rs;
+  gcn_scales(c, &gs, &rs);
+  const bool all_vertex = p->n_edge_tasks == 0;
+  const bool has_bias = d.bias && P->bias;
+  // prepped weights
+  void* wt = L.at<void>(ws, "wt");
+  WG_TRY(prep_weight(c.dt, P->W, c.fi, c.fo, 1, wt, c.pi, (int)c.wrows_o, st));
+  void* wst = nullptr;
+  if (sage) {
+    wst = L.at<void>(ws, "wst");
+    WG_TRY(prep_weight(c.dt, P->W_self, c.fi, c.fo, 1, wst, c.pi, (int)c.wrows_o, st));
+  }
+  // ---- VERTEX table: Y = x W (own rows), exchanged in the distributed case
+  void* ytab = nullptr;
+  int64_t ldY = c.po;
+  if (p->n_vert_tasks > 0) {
+    ytab = A->xchg ? A->xchg : L.at<void>(ws, "y");
+    ldY = A->xchg ? A->ld_xchg : c.po;
+    if (pre) {
+      GemmPart part{x_own, A->ldx, wt, c.pi, c.fi};
+      GemmEpi e;
+      e.D = off(ytab, c.vb, ldY, c.s);
+      e.ldd = ldY;
+      WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), &part, 1, e, nullptr, 0, st));
+      if (sage && all_vertex) {  // S = x W_s (self term of the VERTEX plan)
+        GemmPart ps{x_own, A->ldx, wst, c.pi, c.fi};
+        GemmEpi es;
+        es.D = L.at<void>(ws, "s");
+        es.ldd = c.po;
+        WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), &ps, 1, es, nullptr, 0, st));
+      }
+    }
+  }
+  if (!post) return WG_OK;
+  void* agg = p->n_edge_tasks > 0 ? L.at<void>(A->saved, "agg") : nullptr;
+  void* z = p->mixed ? L.at<void>(ws, "z") : nullptr;
+  void* h = gin ? L.at<void>(A->saved, "h") : nullptr;
+  const int64_t pl = part_ld(c);
+  // ---- EDGE gTasks: Agg = A_hat x  (GIN: z = (1+eps) x + A x)
+  if (p->n_edge_tasks > 0) {
+    AggArgs a = agg_base(c, p->fe, c.g->fwd);
+    a.table = A->x; a.ld_tab = A->ldx;
+    a.gscale = gs; a.rscale = rs;
+    if (gin) { a.self_tab = x_own; a.ld_self = A->ldx; a.self_coef = 1.f + d.gin_eps; }
+    a.out = agg; a.ld_out = c.pi;
+    a.zero_out = z; a.ld_zero = c.po; a.zero_cols = (int)c.po;
+    a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
+    a.F = c.fi;
+    WG_TRY(run_agg(c, a, p->fe, st));
+  }
+  // ---- VERTEX gTasks: out = A_hat Y (+ self, bias, relu when all-VERTEX)
+  if (p->n_vert_tasks > 0) {
+    AggArgs a = agg_base(c, p->fv, c.g->fwd);
+    a.table = ytab; a.ld_tab = ldY;
+    a.gscale = gs; a.rscale = rs;
+    a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
+    a.F = c.fo;
+    if (gin) { a.self_tab = off(ytab, c.vb, ldY, c.s); a.ld_self = ldY; a.self_coef = 1.f + d.gin_eps; }
+    if (all_vertex) {
+      if (sage) { a.self_tab = L.at<void>(ws, "s"); a.ld_self = c.po; a.self_coef = 1.f; }
+      if (gin) {  // a = A_hat-stage output + b1 -> h = relu(a)
+        a.bias = P->bias; a.relu = 1; a.out = h; a.ld_out = c.po;
+      } else {
+        a.bias = has_bias ? P->bias : nullptr; a.relu = d.fuse_relu; a.out = A->y; a.ld_out = A->ldy;
+      }
+    } else {
+      a.out = z; a.ld_out = c.po;
+      a.zero_out = agg; a.ld_zero = c.pi; a.zero_cols = (int)c.pi;
+    }
+    WG_TRY(run_agg(c, a, p->fv, st));
+  }
+  // ---- EDGE transform: y = Agg W (+ x W_s) + Z + b
+  if (p->n_edge_tasks > 0) {
+    GemmPart parts[2];
+    int np = 0;
+    if (sage) parts[np++] = GemmPart{x_own, A->ldx, wst, c.pi, c.fi};
+    parts[np++] = GemmPart{agg, c.pi, wt, c.pi, c.fi};
+    GemmEpi e;
+    e.addend = z; e.ld_add = c.po;
+    if (gin) {
+      e.bias = P->bias; e.relu = 1; e.D = h; e.ldd = c.po;
+    } else {
+      e.bias = has_bias ? P->bias : nullptr; e.relu = d.fuse_relu; e.D = A->y; e.ldd = A->ldy;
+    }
+    WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), parts, np, e, nullptr, 0, st));
+  }
+  // ---- GIN second linear: y = h W2 + b2
+  if (gin) {
+    void* w2t = L.at<void>(ws, "w2t");
+    WG_TRY(prep_weight(c.dt, P->W2, c.fo, c.fo, 1, w2t, c.po, (int)c.wrows_o, st));
+    GemmPart part{h, c.po, w2t, c.po, c.fo};
+    GemmEpi e;
+    e.bias = P->b2; e.relu = d.fuse_relu; e.D = A->y; e.ldd = A->ldy;
+    WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), &part, 1, e, nullptr, 0, st));
+  }
+  return WG_OK;
+}
+
+wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, const wg_grads* G, cudaStream_t st) {
+  Ctx c = mk(p);
+  const wg_conv_desc& d = p->d;
+  const bool sage = d.model == WG_SAGE, gin = d.model == WG_GIN;
+  const bool pre = A->phase != WG_PHASE_POST, post = A->phase != WG_PHASE_PRE;
+  WG_REQ(P && P->W && A->dy && A->x && A->workspace, WG_ERR_INVALID, "backward: null argument");
+  WG_REQ(!d.fuse_relu || A->y, WG_ERR_INVALID, "fuse_relu backward needs y");
+  WG_REQ(!d.need_dx || A->dx, WG_ERR_INVALID, "need_dx but dx is NULL");
+  WG_REQ(p->n_edge_tasks == 0 || A->saved, WG_ERR_INVALID, "saved is NULL");
+  const bool dist = c.nr != c.Vg;
+  void* ws = A->workspace;
+  const Layout& L = p->ws;
+  const char* x_own = off(A->x, c.vb, A->ldx, c.s);
+  const float *gs, *rs;
+  gcn_scales(c, &gs, &rs);
+  const int path = p->bwd_path;
+  void* xchg = A->xchg;
+  const int64_t pl = part_ld(c);
+  float* colsum = L.at<float>(ws, "colsum");
+  void* tn = L.at<void>(ws, "tn");
+  // prepped weights for backward
+  void* w = L.at<void>(ws, "w");
+  WG_TRY(prep_weight(c.dt, P->W, c.fi, c.fo, 0, w, c.po, (int)c.wrows_i, st));
+  void* wsb = nullptr;
+  if (sage) {
+    wsb = L.at<void>(ws, "ws");
+    WG_TRY(prep_weight(c.dt, P->W_self, c.fi, c.fo, 0, wsb, c.po, (int)c.wrows_i, st));
+  }
+  // ---- dT = dy (masked by the fused ReLU); db
+  // The table the transposed gather reads (dT in the G path, dAgg in the
+  // dAgg path) lives in the exchange buffer when distributed.
+  // (single GPU: vb == 0 and every table is indexed by global == local rows)
+  const bool gpath_lin = (path == 1 && !gin);
+  void* dt_buf = nullptr;
+  int64_t ld_dtb = c.po;
+  if (gpath_lin && xchg) { dt_buf = off(xchg, c.vb, A->ld_xchg, c.s); ld_dtb = A->ld_xchg; }
+  else if (d.fuse_relu) { dt_buf = off(L.at<void>(ws, "dt"), c.vb, c.po, c.s); ld_dtb = c.po; }
+  if (pre) {
+    float* db = gin ? (G ? G->b2 : nullptr) : (G ? G->bias : nullptr);
+    if (dt_buf || db)
+      WG_TRY(bias_grad_mask(c.dt, c.nr, c.fo, A->dy, A->lddy, d.fuse_relu ? A->y : nullptr, A->ldy, dt_buf, ld_dtb,
+                            db, colsum, st));
+  }
+  const void* dT = dt_buf ? dt_buf : A->dy;
+  const int64_t lddT = dt_buf ? ld_dtb : A->lddy;
+  const void* dTT;        // gradient w.r.t. the swappable transform's output
+  int64_t lddTT;
+  const void* gtab = nullptr;   // G-path gathered table (global rows)
+  int64_t ldg = lddT;
+  if (gpath_lin) { gtab = xchg ? xchg : dT; ldg = xchg ? A->ld_xchg : lddT; }
+  dTT = dT; lddTT = lddT;
+  // ---- GIN MLP tail: dW2 = h^T dT, da = (dT W2^T) * [h > 0], db1 = sum da
+  void* gin_tab = nullptr;
+  int64_t ld_gin = c.po;
+  if (gin) {
+    void* h = L.at<void>(A->saved, "h");
+    gin_tab = (path == 1 && xchg) ? xchg : L.at<void>(ws, "da");
+    ld_gin = (path == 1 && xchg) ? A->ld_xchg : c.po;
+    void* da = off(gin_tab, c.vb, ld_gin, c.s);
+    if (pre) {
+      if (G && G->W2) WG_TRY(gemm_tn(c.dt, c.nr, c.fo, c.fo, h, c.po, dT, lddT, G->W2, tn, st));
+      void* w2 = L.at<void>(ws, "w2");
+      WG_TRY(prep_weight(c.dt, P->W2, c.fo, c.fo, 0, w2, c.po, (int)c.wrows_o, st));
+      GemmPart part{dT, lddT, w2, c.po, c.fo};
+      GemmEpi e;
+      e.mask_ref = h; e.ld_mask = c.po; e.D = da; e.ldd = ld_gin;
+      WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), &part, 1, e, nullptr, 0, st));
+      if (G && G->bias) WG_TRY(bias_grad_mask(c.dt, c.nr, c.fo, da, ld_gin, nullptr, 0, nullptr, 0, G->bias, colsum, st));
+    }
+    dTT = da; lddTT = ld_gin;
+    if (path == 1) { gtab = gin_tab; ldg = ld_gin; }
+  }
+  // ---- dAgg path
+  if (path == 0) {
+    void* agg = L.at<void>(A->saved, "agg");
+    void* dtab = xchg ? xchg : L.at<void>(ws, "dagg");
+    const int64_t ldd = xchg ? A->ld_xchg : c.pi;
+    if (pre) {
+      if (G && G->W) WG_TRY(gemm_tn(c.dt, c.nr, c.fi, c.fo, agg, c.pi, dTT, lddTT, G->W, tn, st));
+      if (sage && G && G->W_self) WG_TRY(gemm_tn(c.dt, c.nr, c.fi, c.fo, x_own, A->ldx, dT, lddT, G->W_self, tn, st));
+      if (d.need_dx) {
+        GemmPart part{dTT, lddTT, w, c.po, c.fo};
+        GemmEpi e;
+        e.D = off(dtab, c.vb, ldd, c.s); e.ldd = ldd;
+        WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), &part, 1, e, nullptr, 0, st));
+        if (sage) {  // dXs = dT W_s^T (self term)
+          GemmPart ps{dT, lddT, wsb, c.po, c.fo};
+          GemmEpi es;
+          es.D = L.at<void>(ws, "dxs"); es.ldd = c.pi;
+          WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), &ps, 1, es, nullptr, 0, st));
+        }
+      }
+    }
+    if (post && d.need_dx) {
+      AggArgs a = agg_base(c, p->bt, c.g->bwd);
+      a.table = dtab; a.ld_tab = ldd;
+      a.gscale = rs; a.rscale = gs;       // transposed: c_e = gs[u] * rs[d]
+      if (sage) { a.self_tab = L.at<void>(ws, "dxs"); a.ld_self = c.pi; a.self_coef = 1.f; }
+      if (gin) { a.self_tab = off(dtab, c.vb, ldd, c.s); a.ld_self = ldd; a.self_coef = 1.f + d.gin_eps; }
+      a.out = A->dx; a.ld_out = A->lddx;
+      a.partial = L.at<float>(ws, "partT"); a.ld_part = pl;
+      a.F = c.fi;
+      WG_TRY(run_agg(c, a, p->bt, st));
+    }
+    return WG_OK;
+  }
+  // ---- G path
+  if (pre && sage && G && G->W_self) WG_TRY(gemm_tn(c.dt, c.nr, c.fi, c.fo, x_own, A->ldx, dT, lddT, G->W_self, tn, st));
+  if (!post) return WG_OK;
+  void* gbuf = L.at<void>(ws, "g");
+  {
+    AggArgs a = agg_base(c, p->bt, c.g->bwd);
+    a.table = gtab; a.ld_tab = ldg;
+    a.gscale = rs; a.rscale = gs;
+    if (gin) { a.self_tab = off(gtab, c.vb, ldg, c.s); a.ld_self = ldg; a.self_coef = 1.f + d.gin_eps; }
+    a.out = gbuf; a.ld_out = c.po;
+    a.partial = L.at<float>(ws, "partT"); a.ld_part = pl;
+    a.F = c.fo;
+    WG_TRY(run_agg(c, a, p->bt, st));
+  }
+  if (G && G->W) WG_TRY(gemm_tn(c.dt, c.nr, c.fi, c.fo, x_own, A->ldx, gbuf, c.po, G->W, tn, st));
+  if (d.need_dx) {
+    GemmPart parts[2];
+    int np = 0;
+    parts[np++] = GemmPart{gbuf, c.po, w, c.po, c.fo};
+    if (sage) parts[np++] = GemmPart{dT, lddT, wsb, c.po, c.fo};
+    GemmEpi e;
+    e.D = A->dx; e.ldd = A->lddx;
+    WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), parts, np, e, nullptr, 0, st));
+  }
+  return WG_OK;
+}
+
+}  // namespace wg

@@ -1,0 +1,187 @@
+// CUDA-core (FFMA) GEMMs.  Used for the fp32 path (tf32 tensor cores alone
+// cannot meet the 1e-4 fp32 tolerance) and as the bf16
+// fallback for shapes the tcgen05 kernel does not take.
+#include <algorithm>
+
+#include "wg_internal.cuh"
+
+namespace wg {
+
+bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi,
+                cudaStream_t s, wg_status* st);
+bool tc_gemm_tn(int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb, float* D,
+                float* part, cudaStream_t s, wg_status* st);
+
+namespace {
+
+template <typename T> __device__ __forceinline__ float tof(T v) { return (float)v; }
+template <> __device__ __forceinline__ float tof<__nv_bfloat16>(__nv_bfloat16 v) { return __bfloat162float(v); }
+
+constexpr int BM = 64, BN = 64, BK = 16;
+
+struct NTArgs {
+  int64_t M;
+  int N;
+  GemmPart parts[3];
+  int n_parts;
+  GemmEpi epi;
+};
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_gemm_nt(NTArgs a) {
+  __shared__ float As[BK][BM + 4];
+  __shared__ float Bs[BK][BN + 4];
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  const int64_t m0 = (int64_t)blockIdx.x * BM;
+  const int n0 = blockIdx.y * BN;
+  float acc[4][4] = {};
+  for (int p = 0; p < a.n_parts; ++p) {
+    const GemmPart P = a.parts[p];
+    const T* A = static_cast<const T*>(P.A);
+    const T* B = static_cast<const T*>(P.B);
+    for (int k0 = 0; k0 < P.K; k0 += BK) {
+      for (int t = threadIdx.x; t < BM * BK; t += 256) {
+        int mm = t / BK, kk = t % BK;
+        int64_t m = m0 + mm;
+        int k = k0 + kk;
+        As[kk][mm] = (m < a.M && k < P.K) ? tof<T>(A[m * P.lda + k]) : 0.f;
+        int n = n0 + mm;
+        Bs[kk][mm] = (n < a.N && k < P.K) ? tof<T>(B[(int64_t)n * P.ldb + k]) : 0.f;
+      }
+      __syncthreads();
+#pragma unroll
+      for (int kk = 0; kk < BK; ++kk) {
+        float av[4], bv[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) { av[i] = As[kk][ty * 4 + i]; bv[i] = Bs[kk][tx * 4 + i]; }
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+      }
+      __syncthreads();
+    }
+  }
+  const GemmEpi& e = a.epi;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int64_t m = m0 + ty * 4 + i;
+    if (m >= a.M) continue;
+    const float rs = e.rscale ? e.rscale[m] : 1.f;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int n = n0 + tx * 4 + j;
+      if (n >= a.N) continue;
+      float v = rs * acc[i][j];
+      if (e.addend) v += tof<T>(static_cast<const T*>(e.addend)[m * e.ld_add + n]);
+      if (e.bias) v += e.bias[n];
+      if (e.relu) v = fmaxf(v, 0.f);
+      if (e.mask_ref && !(tof<T>(static_cast<const T*>(e.mask_ref)[m * e.ld_mask + n]) > 0.f)) v = 0.f;
+      if (e.d_f32) static_cast<float*>(e.D)[m * e.ldd + n] = v;
+      else static_cast<T*>(e.D)[m * e.ldd + n] = (T)v;
+    }
+  }
+}
+
+// D[M x N] partials: part[z][m][n] = sum_{k in split z} A[k][m] * B[k][n]
+template <typename T>
+__global__ void __launch_bounds__(256) k_gemm_tn(int64_t K, int M, int N, const T* A, int64_t lda, const T* B,
+                                                 int64_t ldb, float* part, int64_t kchunk) {
+  __shared__ float As[BK][BM + 4];
+  __shared__ float Bs[BK][BN + 4];
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  const int m0 = blockIdx.x * BM, n0 = blockIdx.y * BN;
+  const int64_t kb = (int64_t)blockIdx.z * kchunk, ke = min(K, kb + kchunk);
+  float acc[4][4] = {};
+  for (int64_t k0 = kb; k0 < ke; k0 += BK) {
+    for (int t = threadIdx.x; t < BM * BK; t += 256) {
+      int kk = t / BM, mm = t % BM;
+      int64_t k = k0 + kk;
+      As[kk][mm] = (k < ke && m0 + mm < M) ? tof<T>(A[k * lda + m0 + mm]) : 0.f;
+      Bs[kk][mm] = (k < ke && n0 + mm < N) ? tof<T>(B[k * ldb + n0 + mm]) : 0.f;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int kk = 0; kk < BK; ++kk) {
+      float av[4], bv[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) { av[i] = As[kk][ty * 4 + i]; bv[i] = Bs[kk][tx * 4 + i]; }
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+  float* P = part + (int64_t)blockIdx.z * M * N;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    int m = m0 + ty * 4 + i;
+    if (m >= M) continue;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      int n = n0 + tx * 4 + j;
+      if (n < N) P[(int64_t)m * N + n] = acc[i][j];
+    }
+  }
+}
+
+__global__ void k_split_reduce(const float* part, int splits, int64_t MN, float* D) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= MN) return;
+  float s = 0.f;
+  for (int z = 0; z < splits; ++z) s += part[z * MN + i];
+  D[i] = s;
+}
+
+int tn_splits(int64_t K, int M, int N) {
+  const int64_t tiles = cdiv(M, BM) * cdiv(N, BN);
+  int64_t want = std::max<int64_t>(1, (148 * 4) / std::max<int64_t>(1, tiles));
+  want = std::min<int64_t>(want, std::max<int64_t>(1, cdiv(K, 512)));
+  return (int)std::min<int64_t>(want, 1024);
+}
+
+}  // namespace
+
+wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi,
+                  void* scratch, size_t scratch_bytes, cudaStream_t s) {
+  (void)scratch; (void)scratch_bytes;
+  if (M == 0 || N == 0) return WG_OK;
+  WG_REQ(n_parts >= 1 && n_parts <= 3, WG_ERR_INVALID, "gemm_nt: 1..3 parts");
+  wg_status st = WG_OK;
+  if (dt == WG_BF16 && tc_gemm_nt(dt, M, N, parts, n_parts, epi, s, &st)) return st;
+  NTArgs a{};
+  a.M = M; a.N = N; a.n_parts = n_parts; a.epi = epi;
+  for (int i = 0; i < n_parts; ++i) a.parts[i] = parts[i];
+  dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN));
+  if (dt == WG_BF16) WG_LAUNCH(k_gemm_nt<__nv_bfloat16>, grid, 256, 0, s, a);
+  else WG_LAUNCH(k_gemm_nt<float>, grid, 256, 0, s, a);
+  return WG_OK;
+}
+
+size_t gemm_tn_scratch(int64_t K, int M, int N) {
+  return sizeof(float) * (size_t)std::max(tn_splits(K, M, N), 160) * M * N;
+}
+
+wg_status gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb,
+                  float* D, void* scratch, cudaStream_t s) {
+  if (M == 0 || N == 0) return WG_OK;
+  if (K == 0) { WG_CK(cudaMemsetAsync(D, 0, sizeof(float) * M * N, s)); return WG_OK; }
+  float* part = static_cast<float*>(scratch);
+  int splits = tn_splits(K, M, N);
+  wg_status st = WG_OK;
+  if (dt == WG_BF16 && tc_gemm_tn(K, M, N, A, lda, B, ldb, D, part, s, &st)) return st;
+  const int64_t kchunk = rup(cdiv(K, splits), BK);
+  splits = (int)cdiv(K, kchunk);
+  dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN), (unsigned)splits);
+  if (dt == WG_BF16)
+    WG_LAUNCH(k_gemm_tn<__nv_bfloat16>, grid, 256, 0, s, K, M, N, (const __nv_bfloat16*)A, lda,
+              (const __nv_bfloat16*)B, ldb, part, kchunk);
+  else
+    WG_LAUNCH(k_gemm_tn<float>, grid, 256, 0, s, K, M, N, (const float*)A, lda, (const float*)B, ldb, part, kchunk);
+  const int64_t MN = (int64_t)M * N;
+  WG_LAUNCH(k_split_reduce, (unsigned)cdiv(MN, 256), 256, 0, s, part, splits, MN, D);
+  return WG_OK;
+}
+
+}  // namespace wg

@@ -1,0 +1,241 @@
+// Plan selection (a4) and execution structures.
+//
+// Cost model ("computation workload, memory access volume, and
+// parallelism"; the paper gives no formula): integer
+// milli-femtoseconds per gTask,
+//   t_edge = max(n_e (A+4) k_mem + n_rows 2A k_mem, 2 n_rows F_in F_out k_mma)
+// (n_rows = d_hi - d_lo + 1: the unfused EDGE path writes and re-reads Agg)
+//   t_vert = n_e (B+4) k_mem + floor(n_uniq U / S) (A+B) k_mem
+// with A / B the padded row bytes of f_in / f_out wide rows, U the number of
+// vertices with out-edges, S = sum over gTasks of n_uniq_src (each Y row is
+// shared by the gTasks that read it: T1 unique extraction, and
+// T2 indexing swapping).  VERTEX iff t_vert < t_edge.
+#include <algorithm>
+#include <random>
+
+#include "plan.h"
+
+namespace wg {
+
+namespace {
+
+// Build work items from one side's gTask table (untyped graphs).
+// plan: per task bit (nullptr => all EDGE).  out[0] EDGE items, out[1] VERTEX.
+void build_items(const wg_graph_s* g, const Side& S, const std::vector<uint8_t>* plan, ItemList* out0,
+                 ItemList* out1, int* n_slots) {
+  const int64_t T = g->T, vb = g->vb, ve = g->ve;
+  const int64_t t0 = vb / T, t1 = cdiv(ve, T);
+  size_t ti = 0;
+  int slot = 0;
+  std::vector<std::pair<int64_t, WorkItem>> lists[2];
+  for (int64_t tile = t0; tile < t1; ++tile) {
+    const int32_t lo = (int32_t)(tile * T - vb), hi = (int32_t)(std::min<int64_t>((tile + 1) * T, ve) - vb);
+    // tasks of this tile
+    size_t tj = ti;
+    while (tj < S.h_tasks.size() && S.h_tasks[tj].tile == tile) ++tj;
+    int32_t cur_lo = lo;
+    int64_t cur_task = -1;
+    auto flush = [&](int32_t end) {
+      if (end <= cur_lo) return;
+      WorkItem w{};
+      w.row_lo = cur_lo; w.row_hi = end;
+      w.e_lo = S.h_row_ptr[cur_lo]; w.e_hi = S.h_row_ptr[end];
+      w.split_slot = -1;
+      w.task = (int32_t)cur_task;
+      int b = (cur_task >= 0 && plan) ? (*plan)[cur_task] : 0;
+      int64_t weight = cur_task >= 0 ? S.h_tasks[cur_task].e_end - S.h_tasks[cur_task].e_begin : 0;
+      lists[b].push_back({weight, w});
+    };
+    bool first = true;
+    int32_t split_row = -1;
+    for (size_t k = ti; k < tj; ++k) {
+      const wg_task& t = S.h_tasks[k];
+      if (t.flags & WG_TASK_SPLIT) {
+        int b = plan ? (*plan)[k] : 0;
+        int32_t row = (int32_t)(t.d_lo - vb);
+        ItemList* L = b ? out1 : out0;
+        if (row != split_row) {
+          L->hs.push_back(SplitRow{row, slot, 0, b});
+          split_row = row;
+        }
+        L->hs.back().n_slots++;
+        WorkItem w{};
+        w.row_lo = row; w.row_hi = row + 1; w.e_lo = t.e_begin; w.e_hi = t.e_end;
+        w.split_slot = slot++;
+        w.task = (int32_t)k;
+        // SPLIT chunks first (heaviest: overfill / frequent-value)
+        lists[b].push_back({INT64_MAX / 2 + (t.e_end - t.e_begin), w});
+        continue;
+      }
+      if (first) {
+        cur_task = (int64_t)k;
+        first = false;
+      } else {
+        flush((int32_t)(t.d_lo - vb));
+        cur_lo = (int32_t)(t.d_lo - vb);
+        cur_task = (int64_t)k;
+      }
+    }
+    flush(hi);
+    ti = tj;
+  }
+  ItemList* outs[2] = {out0, out1};
+  for (int b = 0; b < 2; ++b) {
+    auto& L = lists[b];
+    std::stable_sort(L.begin(), L.end(), [](const auto& x, const auto& y) { return x.first > y.first; });
+    outs[b]->h.clear();
+    for (auto& e : L) outs[b]->h.push_back(e.second);
+  }
+  *n_slots = slot;
+}
+
+// per-task plan bits for the untyped models (GCN / SAGE / GIN)
+void choose_plans(wg_plan_s* p) {
+  const wg_graph_s* g = p->g;
+  const auto& tasks = g->fwd.h_tasks;
+  const int64_t n = (int64_t)tasks.size();
+  p->plan_bits.assign(n, 0);
+  const wg_conv_desc& d = p->d;
+  if (d.model == WG_GAT) {  // GAT: transform-before-gather only
+    std::fill(p->plan_bits.begin(), p->plan_bits.end(), 1);
+  } else if (d.policy == WG_PLAN_ALL_VERTEX) {
+    std::fill(p->plan_bits.begin(), p->plan_bits.end(), 1);
+  } else if (d.policy == WG_PLAN_RANDOM) {
+    std::mt19937_64 rng(d.policy_seed);
+    for (int64_t i = 0; i < n; ++i) p->plan_bits[i] = (uint8_t)(rng() & 1);
+  } else if (d.policy == WG_PLAN_AUTO) {
+    const int s = dsize(d.dtype);
+    const int64_t A = rup((int64_t)d.f_in * s, 32), B = rup((int64_t)d.f_out * s, 32);
+    const int64_t k_mma = d.dtype == WG_BF16 ? K_MMA_BF16 : K_MMA_F32;
+    int64_t S = 0;
+    for (auto& t : tasks) S += t.n_uniq_src;
+    // U: vertices with out-edges (each needs one Y row)
+    int64_t U = 0;
+    {
+      std::vector<int32_t> dout(g->V);
+      cudaMemcpy(dout.data(), g->deg_out, 4 * g->V, cudaMemcpyDeviceToHost);
+      for (auto x : dout) U += x > 0;
+    }
+    for (int64_t i = 0; i < n; ++i) {
+      const wg_task& t = tasks[i];
+      const int64_t ne = t.e_end - t.e_begin;
+      const int64_t nrows = (int64_t)t.d_hi - t.d_lo + 1;
+      const int64_t t_edge = std::max<int64_t>(ne * (A + 4) * K_MEM + nrows * 2 * A * K_MEM,
+                                      2LL * nrows * d.f_in * d.f_out * k_mma);
+      const int64_t share = S > 0 ? (int64_t)t.n_uniq_src * U / S : 0;
+      const int64_t t_vert = ne * (B + 4) * K_MEM + share * (A + B) * K_MEM;
+      p->plan_bits[i] = t_vert < t_edge ? 1 : 0;
+    }
+  }
+  // all SPLIT chunks of one row take the plan of the row's first chunk
+  for (int64_t i = 1; i < n; ++i)
+    if ((tasks[i].flags & WG_TASK_SPLIT) && (tasks[i - 1].flags & WG_TASK_SPLIT) && tasks[i].d_lo == tasks[i - 1].d_lo &&
+        tasks[i].type == tasks[i - 1].type)
+      p->plan_bits[i] = p->plan_bits[i - 1];
+  p->n_vert_tasks = std::count(p->plan_bits.begin(), p->plan_bits.end(), 1);
+  p->n_edge_tasks = n - p->n_vert_tasks;
+}
+
+template <typename T>
+wg_status upload(wg_plan_s* p, const std::vector<T>& h, T** d) {
+  *d = nullptr;
+  if (h.empty()) return WG_OK;
+  void* q = nullptr;
+  WG_CK(cudaMalloc(&q, sizeof(T) * h.size()));
+  p->allocs.push_back(q);
+  WG_CK(cudaMemcpy(q, h.data(), sizeof(T) * h.size(), cudaMemcpyHostToDevice));
+  *d = static_cast<T*>(q);
+  return WG_OK;
+}
+
+wg_status upload_list(wg_plan_s* p, ItemList& L) {
+  L.n = (int)L.h.size();
+  L.n_split = (int)L.hs.size();
+  WG_TRY(upload(p, L.h, &L.d));
+  WG_TRY(upload(p, L.hs, &L.split));
+  return WG_OK;
+}
+
+}  // namespace
+
+wg_status plan_create(wg_graph g, const wg_conv_desc* d, wg_plan* out) {
+  WG_REQ(g && d && out, WG_ERR_INVALID, "wg_plan_create: null argument");
+  WG_REQ(d->f_in >= 1 && d->f_out >= 1, WG_ERR_INVALID, "f_in / f_out must be >= 1");
+  WG_REQ(d->dtype == WG_F32 || d->dtype == WG_BF16, WG_ERR_INVALID, "dtype");
+  WG_REQ(d->model >= WG_GCN && d->model <= WG_RGCN, WG_ERR_INVALID, "model");
+  if (d->model != WG_RGCN)
+    WG_REQ(!g->by_type, WG_ERR_UNSUPPORTED, "typed graph (num_types > 1) is only supported by RGCN");
+  if (d->model == WG_GAT) WG_REQ(d->heads >= 1, WG_ERR_INVALID, "GAT needs heads >= 1");
+  WG_CK(cudaSetDevice(g->device));
+  auto* p = new wg_plan_s();
+  p->g = g;
+  p->d = *d;
+  if (p->d.heads < 1) p->d.heads = 1;
+  if (d->model == WG_RGCN) {
+    wg_status s = rgcn_plan(p, 0);
+    if (s != WG_OK) { delete p; return s; }
+  } else {
+    choose_plans(p);
+    build_items(g, g->fwd, &p->plan_bits, &p->fe, &p->fv, &p->n_slots_f);
+    ItemList dummy;
+    build_items(g, g->bwd, nullptr, &p->bt, &dummy, &p->n_slots_t);
+    wg_status s;
+    if ((s = upload_list(p, p->fe)) != WG_OK || (s = upload_list(p, p->fv)) != WG_OK ||
+        (s = upload_list(p, p->bt)) != WG_OK) {
+      for (void* q : p->allocs) cudaFree(q);
+      delete p;
+      return s;
+    }
+    p->mixed = (p->n_edge_tasks > 0 && p->n_vert_tasks > 0) ? 1 : 0;
+    // backward path: dAgg (needs Agg of every row, i.e. no VERTEX task) else G
+    p->bwd_path = p->n_vert_tasks > 0 ? 1 : 0;
+    if (d->model == WG_GAT) gat_layout(p); else lin_layout(p);
+  }
+  g->live_plans++;
+  *out = p;
+  return WG_OK;
+}
+
+}  // namespace wg
+
+extern "C" {
+
+wg_status wg_plan_create(wg_graph g, const wg_conv_desc* desc, wg_plan* out) {
+  return wg::plan_create(g, desc, out);
+}
+
+wg_status wg_plan_sizes(wg_plan p, size_t* saved_bytes, size_t* workspace_bytes) {
+  WG_REQ(p, WG_ERR_INVALID, "wg_plan_sizes: null plan");
+  if (saved_bytes) *saved_bytes = p->saved.total;
+  if (workspace_bytes) *workspace_bytes = p->ws.total;
+  return WG_OK;
+}
+
+wg_status wg_plan_export(wg_plan p, uint8_t* per_task_plan, int64_t stats[8]) {
+  WG_REQ(p, WG_ERR_INVALID, "wg_plan_export: null plan");
+  if (per_task_plan) std::copy(p->plan_bits.begin(), p->plan_bits.end(), per_task_plan);
+  if (stats) {
+    stats[0] = p->n_edge_tasks;
+    stats[1] = p->n_vert_tasks;
+    stats[2] = p->bwd_path;
+    stats[3] = 0;
+    stats[4] = 0;
+    stats[5] = p->fe.n + p->fv.n;
+    stats[6] = p->bt.n;
+    stats[7] = p->fe.n_split + p->fv.n_split;
+  }
+  return WG_OK;
+}
+
+wg_status wg_plan_destroy(wg_plan p) {
+  if (!p) return WG_OK;
+  cudaSetDevice(p->g->device);
+  cudaDeviceSynchronize();
+  if (p->rg) wg::rgcn_plan_free(p);
+  for (void* q : p->allocs) cudaFree(q);
+  p->g->live_plans--;
+  delete p;
+  return WG_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,64 @@
+// Plan object: per-gTask operation plan (a4) plus the execution structures
+// derived from the gTask tables (work items, split rows, buffer layout).
+#pragma once
+#include <map>
+#include <string>
+
+#include "wg_internal.cuh"
+
+namespace wg {
+
+// Named, 256-byte aligned sub-buffers of one caller-owned allocation.
+struct Layout {
+  std::map<std::string, size_t> off;
+  size_t total = 0;
+  void add(const std::string& name, size_t bytes) {
+    off[name] = total;
+    total += rup(std::max<size_t>(bytes, 1), 256);
+  }
+  bool has(const std::string& n) const { return off.count(n) != 0; }
+  template <typename T> T* at(const void* base, const std::string& n) const {
+    auto it = off.find(n);
+    return it == off.end() ? nullptr : reinterpret_cast<T*>(const_cast<char*>(static_cast<const char*>(base)) + it->second);
+  }
+};
+
+struct ItemList {
+  WorkItem* d = nullptr;
+  int n = 0;
+  SplitRow* split = nullptr;
+  int n_split = 0;
+  std::vector<WorkItem> h;
+  std::vector<SplitRow> hs;
+};
+
+}  // namespace wg
+
+struct wg_plan_s {
+  wg_graph g = nullptr;
+  wg_conv_desc d{};
+  std::vector<uint8_t> plan_bits;    // per forward gTask: 0 EDGE, 1 VERTEX
+  int64_t n_edge_tasks = 0, n_vert_tasks = 0;
+  wg::ItemList fe, fv, bt;           // forward EDGE items, forward VERTEX items, transposed items
+  int n_slots_f = 0, n_slots_t = 0;  // SPLIT partial slots
+  int bwd_path = 0;                  // 0: dAgg path (Agg saved), 1: G path
+  int mixed = 0;
+  int64_t pi = 0, po = 0;            // row pitches (elements) of f_in / f_out wide tensors
+  wg::Layout saved, ws;
+  std::vector<void*> allocs;
+  // RGCN structures (rgcn.cu)
+  void* rg = nullptr;
+};
+
+namespace wg {
+wg_status rgcn_plan(wg_plan_s* p, cudaStream_t s);
+void rgcn_plan_free(wg_plan_s* p);
+wg_status rgcn_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* a, cudaStream_t s);
+wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, const wg_grads* G, cudaStream_t s);
+wg_status gat_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* a, cudaStream_t s);
+wg_status gat_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, const wg_grads* G, cudaStream_t s);
+wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* a, cudaStream_t s);
+wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, const wg_grads* G, cudaStream_t s);
+void gat_layout(wg_plan_s* p);
+void lin_layout(wg_plan_s* p);
+}  // namespace wg

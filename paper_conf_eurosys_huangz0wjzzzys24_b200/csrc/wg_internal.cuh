@@ -1,0 +1,207 @@
+// Internal declarations of the B200 gTask graph-convolution library (libwg.so).
+// Product code: never includes or links anything under oracle/.
+#pragma once
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+#include <string>
+#include <vector>
+
+#include "../../include/wg.h"
+
+namespace wg {
+
+// ----------------------------------------------------------------- errors
+void set_error(const std::string& msg);
+int64_t& launch_counter();
+
+#define WG_CK(call)                                                                    \
+  do {                                                                                 \
+    cudaError_t e_ = (call);                                                           \
+    if (e_ != cudaSuccess) {                                                           \
+      ::wg::set_error(std::string(#call) + ": " + cudaGetErrorString(e_) + " @" +      \
+                      __FILE__ + ":" + std::to_string(__LINE__));                      \
+      return WG_ERR_CUDA;                                                              \
+    }                                                                                  \
+  } while (0)
+
+#define WG_REQ(cond, code, msg)                                                        \
+  do {                                                                                 \
+    if (!(cond)) {                                                                     \
+      ::wg::set_error(msg);                                                            \
+      return code;                                                                     \
+    }                                                                                  \
+  } while (0)
+
+#define WG_TRY(expr)                                                                   \
+  do {                                                                                 \
+    wg_status s_ = (expr);                                                             \
+    if (s_ != WG_OK) return s_;                                                        \
+  } while (0)
+
+// every kernel launch goes through this so wg_launch_count() is exact
+#define WG_LAUNCH(kernel, grid, block, smem, stream, ...)                              \
+  do {                                                                                 \
+    kernel<<<(grid), (block), (smem), (stream)>>>(__VA_ARGS__);                        \
+    ++::wg::launch_counter();                                                          \
+    cudaError_t e_ = cudaGetLastError();                                               \
+    if (e_ != cudaSuccess) {                                                           \
+      ::wg::set_error(std::string("launch ") + #kernel + ": " + cudaGetErrorString(e_)); \
+      return WG_ERR_CUDA;                                                              \
+    }                                                                                  \
+  } while (0)
+
+static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+static inline int64_t rup(int64_t a, int64_t b) { return cdiv(a, b) * b; }
+static inline int dsize(wg_dtype t) { return t == WG_BF16 ? 2 : 4; }
+// row pitch in elements: rows padded to 32 bytes (sector size)
+static inline int64_t pitch(int64_t F, wg_dtype t) { return rup(F * dsize(t), 32) / dsize(t); }
+
+// ------------------------------------------------------------ work items
+// A work item is the unit a CTA executes: the rows of one gTask (plus the
+// empty rows next to it in the same tile), or one SPLIT chunk of a row.
+struct WorkItem {
+  int32_t row_lo, row_hi;   // local rows [row_lo, row_hi)
+  int64_t e_lo, e_hi;       // SPLIT: edge positions of the chunk; regular: row_ptr range
+  int32_t split_slot;       // >= 0: SPLIT chunk -> partial slot; -1: regular
+  int32_t task;             // gTask index (for plans / debugging)
+};
+static_assert(sizeof(WorkItem) == 32, "WorkItem layout");
+
+struct SplitRow {
+  int32_t row;              // local row
+  int32_t first_slot, n_slots;
+  int32_t plan;
+};
+
+// --------------------------------------------------- one partition side
+struct Side {
+  int64_t E = 0;            // local edges (in-edges of owned rows, or out-edges)
+  int64_t n_rows = 0;       // owned rows
+  int32_t* perm = nullptr;  // [E] global edge ids in sorted order
+  int32_t* idx = nullptr;   // [E] other endpoint (global vertex id) in sorted order
+  int32_t* key = nullptr;   // [E] key vertex (global) in sorted order
+  int32_t* type = nullptr;  // [E] edge type in sorted order (typed graphs)
+  int64_t* row_ptr = nullptr;  // [n_rows+1] local CSR over key rows (untyped graphs)
+  wg_task* tasks = nullptr; // device task table
+  int64_t n_tasks = 0;
+  std::vector<wg_task> h_tasks;  // host copy (plan building)
+  std::vector<int64_t> h_row_ptr;
+};
+
+}  // namespace wg
+
+struct wg_graph_s {
+  int device = 0;
+  int64_t V = 0, vb = 0, ve = 0, E_total = 0;
+  int32_t T = 128, R = 1, by_type = 0;
+  int64_t E_max = 0;
+  int64_t max_in_deg = 0;
+  int32_t* deg_in = nullptr;   // [V] global
+  int32_t* deg_out = nullptr;  // [V]
+  float* rs_in = nullptr;      // [V] 1/sqrt(max(1,deg_in))
+  float* rs_out = nullptr;     // [V] 1/sqrt(max(1,deg_out))
+  float* inv_in = nullptr;     // [V] 1/max(1,deg_in)
+  wg::Side fwd, bwd;
+  int64_t* fwdpos = nullptr;   // [E_T] (owning all rows)
+  int32_t* etype_all = nullptr; // [E_total] types by global edge id (typed graphs)
+  std::vector<void*> allocs;
+  int live_plans = 0;
+};
+
+namespace wg {
+
+// ------------------------------------------------------------- kernels
+struct AggArgs {
+  const WorkItem* items;
+  int n_items;
+  const int64_t* row_ptr;     // [n_rows+1]
+  const int32_t* idx;         // gathered row id per position
+  const void* table;          // gathered table [.. x ld_tab]
+  int64_t ld_tab;
+  const float* gscale;        // per gathered row (nullable)
+  const float* rscale;        // per output row, indexed by GLOBAL row (local + row_base) (nullable)
+  int64_t row_base;           // local row -> global row offset (for rscale / self rows)
+  const void* self_tab;       // self term rows (local row indexing) (nullable)
+  int64_t ld_self;
+  float self_coef;
+  const float* bias;          // [F] (nullable)
+  int relu;
+  const void* mask_ref;       // relu mask reference (output row r kept where ref[r] > 0) (nullable)
+  int64_t ld_mask;
+  void* out;                  // [n_rows x ld_out]
+  int64_t ld_out;
+  void* zero_out;             // optional second output zeroed for the same rows
+  int64_t ld_zero;
+  int zero_cols;              // columns (elements) of zero_out to clear
+  float* partial;             // SPLIT partials [slots x ld_part] fp32
+  int64_t ld_part;
+  int F;                      // real columns
+  int64_t E_max;              // rows with deg > E_max belong to SPLIT items
+};
+
+struct CombineArgs {
+  const SplitRow* rows;
+  int n_rows;
+  const float* partial;
+  int64_t ld_part;
+  const float* rscale;
+  int64_t row_base;
+  const void* self_tab;
+  int64_t ld_self;
+  float self_coef;
+  const float* bias;
+  int relu;
+  const void* mask_ref;
+  int64_t ld_mask;
+  void* out;
+  int64_t ld_out;
+  void* zero_out;
+  int64_t ld_zero;
+  int zero_cols;
+  int F;
+  int plan_filter;            // -1 all, else only rows with this plan
+};
+
+wg_status launch_agg(wg_dtype dt, const AggArgs& a, cudaStream_t s);
+wg_status launch_combine(wg_dtype dt, const CombineArgs& a, cudaStream_t s);
+
+// GEMM: D[M x N] = sum_p A_p[M x K_p] * B_p[N x K_p]^T  (+ epilogue)
+struct GemmPart {
+  const void* A; int64_t lda;   // row-major [M x K]
+  const void* B; int64_t ldb;   // row-major [N x K]
+  int K;
+};
+struct GemmEpi {
+  const float* rscale = nullptr;      // per row
+  const float* bias = nullptr;        // per column [N]
+  const void* addend = nullptr;       // add [M x N] (conv dtype), ld_add
+  int64_t ld_add = 0;
+  int relu = 0;
+  const void* mask_ref = nullptr;     // keep where ref > 0 (conv dtype), ld_mask
+  int64_t ld_mask = 0;
+  void* D = nullptr; int64_t ldd = 0; // output (conv dtype unless d_f32)
+  int d_f32 = 0;
+};
+wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts,
+                  const GemmEpi& epi, void* scratch, size_t scratch_bytes, cudaStream_t s);
+// dW[M x N] (fp32, exact shape, ld = N) = A[K x M]^T * B[K x N] (split-K, deterministic)
+size_t gemm_tn_scratch(int64_t K, int M, int N);
+wg_status gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda,
+                  const void* B, int64_t ldb, float* D, void* scratch, cudaStream_t s);
+
+// weight prep: fp32 [rows x cols] -> dtype, optionally transposed, into [out_rows x ldo]
+wg_status prep_weight(wg_dtype dt, const float* W, int rows, int cols, int transpose,
+                      void* out, int64_t ldo, int out_rows, cudaStream_t s);
+// column sums (deterministic) of dy (optionally relu-masked by ref, written to dt_out)
+wg_status bias_grad_mask(wg_dtype dt, int64_t M, int N, const void* dy, int64_t lddy,
+                         const void* ref, int64_t ldref, void* dt_out, int64_t ldt,
+                         float* db, float* scratch, cudaStream_t s);
+size_t bias_grad_scratch(int64_t M, int N);
+
+// cost-model constants (milli-femtoseconds per byte / per flop), from MEASURED_PEAKS
+constexpr int64_t K_MEM = 152952;   // 1e6 / 6.538 GB/s-per-fs
+constexpr int64_t K_MMA_BF16 = 720; // 1e6 / 1389.2
+constexpr int64_t K_MMA_F32 = 16000;
+
+}  // namespace wg
