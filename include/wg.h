@@ -140,6 +140,12 @@ wg_status wg_plan_sizes(wg_plan p, size_t* saved_bytes, size_t* workspace_bytes)
  * 0 = the exchanged table is x itself), n work items fwd, n work items T,
  * n split rows fwd.                                                        */
 wg_status wg_plan_export(wg_plan p, uint8_t* per_task_plan, int64_t stats[8]);
+/* Introspection (tests / tools): byte offset of a named sub-buffer of the
+ * saved (which = 0) or workspace (which = 1) buffer, e.g. "agg" (the saved
+ * aggregation, [owned rows x pitch(f_in)]) or "h" (GIN hidden activation,
+ * [owned rows x pitch(f_out)]).  WG_ERR_INVALID if the plan has no such
+ * buffer.  Pitches are 32-byte padded rows in the conv dtype.              */
+wg_status wg_plan_buffer(wg_plan p, int which, const char* name, size_t* offset);
 wg_status wg_plan_destroy(wg_plan p);
 
 /* ------------------------------------------------------------------------ */
@@ -201,6 +207,18 @@ const char* wg_status_string(wg_status s);
 const char* wg_last_error(void);
 /* Number of kernels this library has launched on the calling thread. */
 int64_t wg_launch_count(void);
+
+/* Live per-kernel-class timing (CUDA events recorded on the launching stream
+ * around every launch of the class).  cmd 0: disable; 1: enable and reset;
+ * 2: synchronize the recorded events and write, for each class k in
+ * [0, WG_PROF_KINDS), out[4k+0] = total ms, out[4k+1] = launches,
+ * out[4k+2] = algorithmic bytes, out[4k+3] = algorithmic flops.
+ * Classes: 0 gather/segment-reduce (a6/a10), 1 split combine (a8),
+ * 2 tcgen05 GEMM NT (a5/a7/a9), 3 tcgen05 GEMM TN + reduce (a11),
+ * 4 CUDA-core GEMM, 5 small kernels (weight prep, bias grad),
+ * 6 GAT edge kernels, 7 RGCN kernels.                                      */
+#define WG_PROF_KINDS 8
+wg_status wg_profile(int cmd, double* out);
 
 #ifdef __cplusplus
 }

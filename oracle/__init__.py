@@ -60,7 +60,7 @@ def _L():
         _lib.wgo_sage_forward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P]
         _lib.wgo_sage_backward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P, P, P, P]
         _lib.wgo_gin_forward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, f64, P, P, P, P, P, P]
-        _lib.wgo_gin_backward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, f64, P, P, P, P, P, P, P, P, P, P]
+        _lib.wgo_gin_backward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, f64, P, P, P, P, P, P, P, P, P, P, P]
         _lib.wgo_rgcn_forward.argtypes = [i64, i64, P, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P]
         _lib.wgo_rgcn_backward.argtypes = [i64, i64, P, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P, P, P, P]
         _lib.wgo_gat_forward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, f64, P, P, P, P, P, P, P]
@@ -179,13 +179,15 @@ def gin_forward(src, dst, V, x, W1, b1, W2, b2, eps=0.0):
     return y
 
 
-def gin_backward(src, dst, V, x, W1, b1, W2, dy, eps=0.0):
+def gin_backward(src, dst, V, x, W1, b1, W2, dy, eps=0.0, amask=None):
+    """amask: optional [V x fo] ReLU decisions taken by the implementation under test."""
     x, W1, b1, W2, dy = map(_f64, (x, W1, b1, W2, dy))
+    am = None if amask is None else np.ascontiguousarray(amask, dtype=np.uint8)
     fi, fo = W1.shape
     dx, dW1, db1, dW2, db2 = np.zeros((V, fi)), np.zeros((fi, fo)), np.zeros(fo), np.zeros((fo, fo)), np.zeros(fo)
     s, d = _i32(src), _i32(dst)
     _L().wgo_gin_backward(V, s.shape[0], _p(s), _p(d), fi, fo, float(eps), _p(x), _p(W1), _p(b1), _p(W2), _p(dy),
-                          _p(dx), _p(dW1), _p(db1), _p(dW2), _p(db2))
+                          _p(am), _p(dx), _p(dW1), _p(db1), _p(dW2), _p(db2))
     return dx, dW1, db1, dW2, db2
 
 

@@ -312,10 +312,13 @@ void wgo_gin_forward(int64_t V, int64_t E, const int32_t* src, const int32_t* ds
 
 /* dW2 = h^T dy ; da = (dy W2^T) * [a > 0] ; dW1 = z^T da ; dz = da W1^T ;
  * dx[u] = (1+eps) dz[u] + sum_{e in out(u)} dz[d_e] ; db1 = sum da ; db2 = sum dy */
+/* amask (nullable, [V x fo] bytes): the ReLU decision [a > 0] taken by the
+ * implementation under test in its own precision (a float deciding an integer
+ * is decided by one side only); NULL = use a > 0. */
 void wgo_gin_backward(int64_t V, int64_t E, const int32_t* src, const int32_t* dst, int fi, int fo,
                       double eps, const double* x, const double* W1, const double* b1,
-                      const double* W2, const double* dy, double* dx, double* dW1, double* db1,
-                      double* dW2, double* db2) {
+                      const double* W2, const double* dy, const uint8_t* amask, double* dx, double* dW1,
+                      double* db1, double* dW2, double* db2) {
     double* z = malloc(sizeof(double) * V * fi);
     double* dz = malloc(sizeof(double) * V * fi);
     double* a = malloc(sizeof(double) * fo);
@@ -331,10 +334,14 @@ void wgo_gin_backward(int64_t V, int64_t E, const int32_t* src, const int32_t* d
     for (int64_t v = 0; v < V; ++v) {
         for (int j = 0; j < fo; ++j) a[j] = b1 ? b1[j] : 0.0;
         add_msg(fi, fo, 1.0, z + v * fi, W1, a);
-        for (int j = 0; j < fo; ++j) { h[j] = a[j] > 0.0 ? a[j] : 0.0; dh[j] = 0.0; }
+        for (int j = 0; j < fo; ++j) {
+            int on = amask ? amask[v * fo + j] != 0 : a[j] > 0.0;
+            h[j] = on ? a[j] : 0.0;
+            dh[j] = 0.0;
+        }
         if (db2) for (int j = 0; j < fo; ++j) db2[j] += dy[v * fo + j];
         add_msg_grad(fo, fo, 1.0, h, W2, dy + v * fo, dh, dW2);
-        for (int j = 0; j < fo; ++j) da[j] = a[j] > 0.0 ? dh[j] : 0.0;
+        for (int j = 0; j < fo; ++j) da[j] = (amask ? amask[v * fo + j] != 0 : a[j] > 0.0) ? dh[j] : 0.0;
         if (db1) for (int j = 0; j < fo; ++j) db1[j] += da[j];
         add_msg_grad(fi, fo, 1.0, z + v * fi, W1, da, dz + v * fi, dW1);
     }

@@ -78,6 +78,18 @@ def launch_count() -> int:
     return int(C.lib().wg_launch_count())
 
 
+def profile(cmd: str):
+    """'start' | 'stop' | 'collect' -> {kind: {ms, launches, bytes, flops}} (wg_profile)."""
+    L = C.lib()
+    if cmd in ("start", "stop"):
+        C.check(L.wg_profile(1 if cmd == "start" else 0, None), "wg_profile")
+        return None
+    out = (ctypes.c_double * (4 * len(C.PROF_KINDS)))()
+    C.check(L.wg_profile(2, out), "wg_profile")
+    return {k: {"ms": out[4 * i], "launches": int(out[4 * i + 1]), "bytes": out[4 * i + 2], "flops": out[4 * i + 3]}
+            for i, k in enumerate(C.PROF_KINDS)}
+
+
 class Graph:
     """Device graph + forward / transposed gTask partitions (wg_graph_create)."""
 
@@ -187,6 +199,15 @@ class Conv:
         out = np.empty(max(self.graph.n_tasks, 1), np.uint8)
         C.check(C.lib().wg_plan_export(self._h, _ptr(out), None), "wg_plan_export")
         return out[: self.graph.n_tasks]
+
+    def buffer_view(self, buf: torch.Tensor, name: str, rows: int, F: int, which: int = 0) -> torch.Tensor:
+        """[rows x F] view of the named sub-buffer of `saved` (which=0) or the workspace (1)."""
+        off = ctypes.c_size_t()
+        C.check(C.lib().wg_plan_buffer(self._h, which, name.encode(), ctypes.byref(off)), "wg_plan_buffer")
+        es = torch.empty((), dtype=self.dtype).element_size()
+        ld = pitch(F, self.dtype)
+        raw = buf[off.value: off.value + rows * ld * es]
+        return raw.view(self.dtype).view(rows, ld)[:, :F]
 
     def new_saved(self):
         return torch.empty(max(self.saved_bytes, 256), dtype=torch.uint8, device=self.workspace.device)

@@ -23,10 +23,11 @@ PHASE_ALL, PHASE_PRE, PHASE_POST = 0, 1, 2
 # every symbol include/wg.h declares (checked by tests/test_abi.py)
 EXPORTS = [
     "wg_graph_create", "wg_graph_info", "wg_graph_export", "wg_graph_destroy",
-    "wg_plan_create", "wg_plan_sizes", "wg_plan_export", "wg_plan_destroy",
+    "wg_plan_create", "wg_plan_sizes", "wg_plan_export", "wg_plan_buffer", "wg_plan_destroy",
     "wg_conv_forward", "wg_conv_backward",
-    "wg_status_string", "wg_last_error", "wg_launch_count",
+    "wg_status_string", "wg_last_error", "wg_launch_count", "wg_profile",
 ]
+PROF_KINDS = ["gather_reduce", "split_combine", "tc_gemm_nt", "tc_gemm_tn", "simt_gemm", "misc", "gat", "rgcn"]
 
 P = ctypes.c_void_p
 i32, i64, u64, f32 = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64, ctypes.c_float
@@ -99,6 +100,8 @@ def lib():
     L.wg_plan_sizes.argtypes = [P, ctypes.POINTER(ctypes.c_size_t), ctypes.POINTER(ctypes.c_size_t)]
     L.wg_plan_export.restype = st
     L.wg_plan_export.argtypes = [P, P, P]
+    L.wg_plan_buffer.restype = st
+    L.wg_plan_buffer.argtypes = [P, ctypes.c_int, ctypes.c_char_p, ctypes.POINTER(ctypes.c_size_t)]
     L.wg_plan_destroy.restype = st
     L.wg_plan_destroy.argtypes = [P]
     L.wg_conv_forward.restype = st
@@ -111,6 +114,8 @@ def lib():
     L.wg_last_error.argtypes = []
     L.wg_launch_count.restype = i64
     L.wg_launch_count.argtypes = []
+    L.wg_profile.restype = st
+    L.wg_profile.argtypes = [ctypes.c_int, P]
     _lib = L
     return L
 

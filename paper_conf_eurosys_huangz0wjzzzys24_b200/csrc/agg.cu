@@ -324,6 +324,14 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
 
 wg_status launch_agg(wg_dtype dt, const AggArgs& a, cudaStream_t s) {
   if (a.n_items == 0) return WG_OK;
+  // algorithmic bytes: per edge the index (4 B), the gathered row (F elements)
+  // and the source scale if any; per row the output, row_ptr and optional
+  // self / mask rows
+  const double es = dt == WG_BF16 ? 2.0 : 4.0, rb = a.F * es;
+  const double bytes = a.n_edges * (4.0 + rb + (a.gscale ? 4.0 : 0.0)) +
+                       a.n_rows * (rb + 8.0 + (a.self_tab ? rb : 0.0) + (a.mask_ref ? rb : 0.0) +
+                                   (a.zero_out ? a.zero_cols * es : 0.0));
+  ProfScope ps(PK_AGG, s, bytes, 2.0 * a.n_edges * a.F);
   return dt == WG_BF16 ? launch_t<__nv_bfloat16>(a, s) : launch_t<float>(a, s);
 }
 
@@ -331,6 +339,7 @@ wg_status launch_combine(wg_dtype dt, const CombineArgs& a, cudaStream_t s) {
   if (a.n_rows == 0) return WG_OK;
   const int EPV = dt == WG_BF16 ? 8 : 4;
   const int VPR = (int)cdiv(a.F, EPV);
+  ProfScope ps(PK_COMBINE, s, (double)a.n_rows * a.F * (EPV == 8 ? 2 : 4), 0.0);
   if (dt == WG_BF16) WG_LAUNCH(k_combine<__nv_bfloat16>, a.n_rows, 128, 0, s, a, VPR);
   else WG_LAUNCH(k_combine<float>, a.n_rows, 128, 0, s, a, VPR);
   return WG_OK;
@@ -385,6 +394,7 @@ wg_status prep_weight(wg_dtype dt, const float* W, int rows, int cols, int trans
                       int out_rows, cudaStream_t s) {
   int64_t n = (int64_t)out_rows * ldo;
   unsigned grid = (unsigned)std::min<int64_t>(cdiv(n, 256), 1184);
+  ProfScope ps(PK_MISC, s, (double)rows * cols * 4.0 + (double)n * (dt == WG_BF16 ? 2.0 : 4.0), 0.0);
   if (grid == 0) return WG_OK;
   if (dt == WG_BF16)
     WG_LAUNCH(k_prep_weight<__nv_bfloat16>, grid, 256, 0, s, W, rows, cols, transpose, (__nv_bfloat16*)out, ldo, out_rows);
@@ -399,6 +409,8 @@ wg_status bias_grad_mask(wg_dtype dt, int64_t M, int N, const void* dy, int64_t 
                          int64_t ldref, void* dt_out, int64_t ldt, float* db, float* scratch, cudaStream_t s) {
   const int64_t rpb = std::max<int64_t>(1, cdiv(M, COLSUM_BLKS));
   const int nblk = (int)std::max<int64_t>(1, cdiv(M, rpb));
+  const double es = dt == WG_BF16 ? 2.0 : 4.0;
+  ProfScope ps(PK_MISC, s, (double)M * N * es * (1 + (ref ? 1 : 0) + (dt_out ? 1 : 0)), (double)M * N);
   const int threads = N >= 256 ? 256 : (int)rup(N, 32);
   if (dt == WG_BF16)
     WG_LAUNCH(k_colsum<__nv_bfloat16>, nblk, threads, 0, s, M, N, (const __nv_bfloat16*)dy, lddy,

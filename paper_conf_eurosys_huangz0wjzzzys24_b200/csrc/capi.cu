@@ -9,6 +9,38 @@ thread_local int64_t g_launches = 0;
 }  // namespace
 void set_error(const std::string& msg) { g_err = msg; }
 int64_t& launch_counter() { return g_launches; }
+
+namespace {
+struct ProfRec {
+  int kind;
+  cudaEvent_t a, b;
+  double bytes, flops;
+};
+struct Profiler {
+  bool on = false;
+  std::vector<cudaEvent_t> pool;
+  std::vector<ProfRec> recs;
+  cudaEvent_t get() {
+    if (!pool.empty()) { cudaEvent_t e = pool.back(); pool.pop_back(); return e; }
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    return e;
+  }
+};
+Profiler g_prof;
+}  // namespace
+
+ProfScope::ProfScope(int kind, cudaStream_t s, double bytes, double flops) : s_(s) {
+  if (!g_prof.on) return;
+  ProfRec r{kind, g_prof.get(), g_prof.get(), bytes, flops};
+  cudaEventRecord(r.a, s);
+  rec_ = (int)g_prof.recs.size();
+  g_prof.recs.push_back(r);
+}
+
+ProfScope::~ProfScope() {
+  if (rec_ >= 0 && rec_ < (int)g_prof.recs.size()) cudaEventRecord(g_prof.recs[rec_].b, s_);
+}
 }  // namespace wg
 
 extern "C" {
@@ -29,6 +61,31 @@ const char* wg_status_string(wg_status s) {
 const char* wg_last_error(void) { return wg::g_err.c_str(); }
 
 int64_t wg_launch_count(void) { return wg::launch_counter(); }
+
+wg_status wg_profile(int cmd, double* out) {
+  using namespace wg;
+  if (cmd == 0 || cmd == 1) {
+    for (auto& r : g_prof.recs) { cudaEventSynchronize(r.b); g_prof.pool.push_back(r.a); g_prof.pool.push_back(r.b); }
+    g_prof.recs.clear();
+    g_prof.on = cmd == 1;
+    return WG_OK;
+  }
+  WG_REQ(cmd == 2 && out, WG_ERR_INVALID, "wg_profile: cmd must be 0, 1 or 2 (with out)");
+  for (int i = 0; i < 4 * PK_KINDS; ++i) out[i] = 0.0;
+  for (auto& r : g_prof.recs) {
+    WG_CK(cudaEventSynchronize(r.b));
+    float ms = 0.f;
+    WG_CK(cudaEventElapsedTime(&ms, r.a, r.b));
+    out[4 * r.kind + 0] += ms;
+    out[4 * r.kind + 1] += 1;
+    out[4 * r.kind + 2] += r.bytes;
+    out[4 * r.kind + 3] += r.flops;
+    g_prof.pool.push_back(r.a);
+    g_prof.pool.push_back(r.b);
+  }
+  g_prof.recs.clear();
+  return WG_OK;
+}
 
 wg_status wg_conv_forward(wg_plan p, const wg_params* params, const wg_fwd_args* a, wg_stream stream) {
   WG_REQ(p && params && a, WG_ERR_INVALID, "wg_conv_forward: null argument");

@@ -103,6 +103,8 @@ AggArgs agg_base(const Ctx& c, const ItemList& L, const Side& S) {
   a.row_base = c.vb;
   a.self_coef = 1.f;
   a.E_max = c.g->E_max;
+  a.n_edges = L.n_edges;
+  a.n_rows = L.n_rows;
   return a;
 }
 
@@ -172,13 +174,13 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
     ytab = A->xchg ? A->xchg : L.at<void>(ws, "y");
     ldY = A->xchg ? A->ld_xchg : c.po;
     if (pre) {
-      GemmPart part{x_own, A->ldx, wt, c.pi, c.fi};
+      GemmPart part{x_own, A->ldx, wt, c.pi, c.fi, (int)c.wrows_o};
       GemmEpi e;
       e.D = off(ytab, c.vb, ldY, c.s);
       e.ldd = ldY;
       WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), &part, 1, e, nullptr, 0, st));
       if (sage && all_vertex) {  // S = x W_s (self term of the VERTEX plan)
-        GemmPart ps{x_own, A->ldx, wst, c.pi, c.fi};
+        GemmPart ps{x_own, A->ldx, wst, c.pi, c.fi, (int)c.wrows_o};
         GemmEpi es;
         es.D = L.at<void>(ws, "s");
         es.ldd = c.po;
@@ -187,9 +189,9 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
     }
   }
   if (!post) return WG_OK;
-  void* agg = p->n_edge_tasks > 0 ? L.at<void>(A->saved, "agg") : nullptr;
+  void* agg = p->n_edge_tasks > 0 ? p->saved.at<void>(A->saved, "agg") : nullptr;
   void* z = p->mixed ? L.at<void>(ws, "z") : nullptr;
-  void* h = gin ? L.at<void>(A->saved, "h") : nullptr;
+  void* h = gin ? p->saved.at<void>(A->saved, "h") : nullptr;
   const int64_t pl = part_ld(c);
   // ---- EDGE gTasks: Agg = A_hat x  (GIN: z = (1+eps) x + A x)
   if (p->n_edge_tasks > 0) {
@@ -228,8 +230,8 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
   if (p->n_edge_tasks > 0) {
     GemmPart parts[2];
     int np = 0;
-    if (sage) parts[np++] = GemmPart{x_own, A->ldx, wst, c.pi, c.fi};
-    parts[np++] = GemmPart{agg, c.pi, wt, c.pi, c.fi};
+    if (sage) parts[np++] = GemmPart{x_own, A->ldx, wst, c.pi, c.fi, (int)c.wrows_o};
+    parts[np++] = GemmPart{agg, c.pi, wt, c.pi, c.fi, (int)c.wrows_o};
     GemmEpi e;
     e.addend = z; e.ld_add = c.po;
     if (gin) {
@@ -243,7 +245,7 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
   if (gin) {
     void* w2t = L.at<void>(ws, "w2t");
     WG_TRY(prep_weight(c.dt, P->W2, c.fo, c.fo, 1, w2t, c.po, (int)c.wrows_o, st));
-    GemmPart part{h, c.po, w2t, c.po, c.fo};
+    GemmPart part{h, c.po, w2t, c.po, c.fo, (int)c.wrows_o};
     GemmEpi e;
     e.bias = P->b2; e.relu = d.fuse_relu; e.D = A->y; e.ldd = A->ldy;
     WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), &part, 1, e, nullptr, 0, st));
@@ -306,7 +308,7 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   void* gin_tab = nullptr;
   int64_t ld_gin = c.po;
   if (gin) {
-    void* h = L.at<void>(A->saved, "h");
+    void* h = p->saved.at<void>(A->saved, "h");
     gin_tab = (path == 1 && xchg) ? xchg : L.at<void>(ws, "da");
     ld_gin = (path == 1 && xchg) ? A->ld_xchg : c.po;
     void* da = off(gin_tab, c.vb, ld_gin, c.s);
@@ -314,7 +316,7 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
       if (G && G->W2) WG_TRY(gemm_tn(c.dt, c.nr, c.fo, c.fo, h, c.po, dT, lddT, G->W2, tn, st));
       void* w2 = L.at<void>(ws, "w2");
       WG_TRY(prep_weight(c.dt, P->W2, c.fo, c.fo, 0, w2, c.po, (int)c.wrows_o, st));
-      GemmPart part{dT, lddT, w2, c.po, c.fo};
+      GemmPart part{dT, lddT, w2, c.po, c.fo, (int)c.wrows_o};
       GemmEpi e;
       e.mask_ref = h; e.ld_mask = c.po; e.D = da; e.ldd = ld_gin;
       WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), &part, 1, e, nullptr, 0, st));
@@ -325,19 +327,19 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   }
   // ---- dAgg path
   if (path == 0) {
-    void* agg = L.at<void>(A->saved, "agg");
+    void* agg = p->saved.at<void>(A->saved, "agg");
     void* dtab = xchg ? xchg : L.at<void>(ws, "dagg");
     const int64_t ldd = xchg ? A->ld_xchg : c.pi;
     if (pre) {
       if (G && G->W) WG_TRY(gemm_tn(c.dt, c.nr, c.fi, c.fo, agg, c.pi, dTT, lddTT, G->W, tn, st));
       if (sage && G && G->W_self) WG_TRY(gemm_tn(c.dt, c.nr, c.fi, c.fo, x_own, A->ldx, dT, lddT, G->W_self, tn, st));
       if (d.need_dx) {
-        GemmPart part{dTT, lddTT, w, c.po, c.fo};
+        GemmPart part{dTT, lddTT, w, c.po, c.fo, (int)c.wrows_i};
         GemmEpi e;
         e.D = off(dtab, c.vb, ldd, c.s); e.ldd = ldd;
         WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), &part, 1, e, nullptr, 0, st));
         if (sage) {  // dXs = dT W_s^T (self term)
-          GemmPart ps{dT, lddT, wsb, c.po, c.fo};
+          GemmPart ps{dT, lddT, wsb, c.po, c.fo, (int)c.wrows_i};
           GemmEpi es;
           es.D = L.at<void>(ws, "dxs"); es.ldd = c.pi;
           WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), &ps, 1, es, nullptr, 0, st));
@@ -375,8 +377,8 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   if (d.need_dx) {
     GemmPart parts[2];
     int np = 0;
-    parts[np++] = GemmPart{gbuf, c.po, w, c.po, c.fo};
-    if (sage) parts[np++] = GemmPart{dT, lddT, wsb, c.po, c.fo};
+    parts[np++] = GemmPart{gbuf, c.po, w, c.po, c.fo, (int)c.wrows_i};
+    if (sage) parts[np++] = GemmPart{dT, lddT, wsb, c.po, c.fo, (int)c.wrows_i};
     GemmEpi e;
     e.D = A->dx; e.ldd = A->lddx;
     WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), parts, np, e, nullptr, 0, st));

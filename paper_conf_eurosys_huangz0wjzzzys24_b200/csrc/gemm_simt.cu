@@ -46,7 +46,7 @@ __global__ void __launch_bounds__(256) k_gemm_nt(NTArgs a) {
         int k = k0 + kk;
         As[kk][mm] = (m < a.M && k < P.K) ? tof<T>(A[m * P.lda + k]) : 0.f;
         int n = n0 + mm;
-        Bs[kk][mm] = (n < a.N && k < P.K) ? tof<T>(B[(int64_t)n * P.ldb + k]) : 0.f;
+        Bs[kk][mm] = (n < a.N && n < P.nb && k < P.K) ? tof<T>(B[(int64_t)n * P.ldb + k]) : 0.f;
       }
       __syncthreads();
 #pragma unroll
@@ -152,7 +152,10 @@ wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_pa
   if (dt == WG_BF16 && tc_gemm_nt(dt, M, N, parts, n_parts, epi, s, &st)) return st;
   NTArgs a{};
   a.M = M; a.N = N; a.n_parts = n_parts; a.epi = epi;
-  for (int i = 0; i < n_parts; ++i) a.parts[i] = parts[i];
+  double kt = 0;
+  for (int i = 0; i < n_parts; ++i) { a.parts[i] = parts[i]; kt += parts[i].K; }
+  const double es = dt == WG_BF16 ? 2.0 : 4.0;
+  ProfScope ps(PK_SIMT, s, (double)M * (kt + N) * es, 2.0 * M * N * kt);
   dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN));
   if (dt == WG_BF16) WG_LAUNCH(k_gemm_nt<__nv_bfloat16>, grid, 256, 0, s, a);
   else WG_LAUNCH(k_gemm_nt<float>, grid, 256, 0, s, a);
@@ -173,6 +176,7 @@ wg_status gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t l
   if (dt == WG_BF16 && tc_gemm_tn(K, M, N, A, lda, B, ldb, D, part, s, &st)) return st;
   const int64_t kchunk = rup(cdiv(K, splits), BK);
   splits = (int)cdiv(K, kchunk);
+  ProfScope ps(PK_SIMT, s, (double)K * (M + N) * (dt == WG_BF16 ? 2.0 : 4.0), 2.0 * K * M * N);
   dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN), (unsigned)splits);
   if (dt == WG_BF16)
     WG_LAUNCH(k_gemm_tn<__nv_bfloat16>, grid, 256, 0, s, K, M, N, (const __nv_bfloat16*)A, lda,

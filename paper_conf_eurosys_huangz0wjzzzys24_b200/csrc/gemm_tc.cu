@@ -1,13 +1,423 @@
-// tcgen05 / TMEM / TMA GEMMs for sm_100a (placeholder until the tensor-core
-// kernels land; returning false routes to the CUDA-core kernels).
+// tcgen05 / TMEM / TMA GEMMs for sm_100a (bf16 in, fp32 accumulate).
+//
+// The dense per-gTask / per-vertex transforms of the layer (a5, a7, a9, a11):
+// "a batch of K src rows becomes a matrix-matrix product on tensor cores"
+// (Fig 10c).  Two variants share one pipeline:
+//   NT  D[M x N] = sum_p A_p[M x K_p] B_p[N x K_p]^T   (A, B K-major)
+//       + epilogue (row scale, bias, addend, ReLU, ReLU-mask, RNE cast)
+//   TN  D[M x N] = A[K x M]^T B[K x N]                   (A, B MN-major)
+//       split-K over K (= vertices) with fp32 partials reduced in a fixed
+//       order (deterministic weight gradients, a11).
+// Structure: one CTA = 128 threads computes a 128 x BN tile.  Thread 0
+// issues TMA loads (128-byte swizzle) into a STAGES-deep smem ring guarded by
+// full/empty mbarriers; thread 32 issues tcgen05.mma (M=128, N=BN, K=16)
+// into a TMEM accumulator and releases ring slots with tcgen05.commit; all
+// four warps then drain TMEM with tcgen05.ld (warp w owns lanes 32w..32w+31)
+// and run the epilogue.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <mutex>
+
 #include "wg_internal.cuh"
 
 namespace wg {
-bool tc_gemm_nt(wg_dtype, int64_t, int, const GemmPart*, int, const GemmEpi&, cudaStream_t, wg_status*) {
-  return false;
+
+namespace {
+
+constexpr int BM = 128, BK = 64;
+constexpr int A_STAGE = BM * BK * 2;   // 16 KB
+
+struct TcParams {
+  int64_t M;
+  int N;          // columns written (NT) / real N (TN)
+  int BN;         // MMA N (multiple of 16, <= 256)
+  int stages;
+  int nparts;
+  int kblocks[3];
+  int64_t k_base; // TN: first K row of split z = blockIdx.z * k_span
+  int64_t k_span;
+  int64_t K;      // TN total K
+  GemmEpi epi;
+  float* part;    // TN partial output [splits x M x N]
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
-bool tc_gemm_tn(int64_t, int, int, const void*, int64_t, const void*, int64_t, float*, float*, cudaStream_t,
-                wg_status*) {
-  return false;
+
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
 }
+
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map, int c0, int c1, uint32_t bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(bar)
+      : "memory");
+}
+
+// UMMA shared-memory descriptor (sm100): start>>4 [0,14), LBO>>4 [16,30),
+// SBO>>4 [32,46), version 1 [46,48), layout SWIZZLE_128B = 2 [61,64)
+__device__ __forceinline__ uint64_t umma_desc(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((addr >> 4) & 0x3FFF);
+  d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
+  d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)2 << 61;
+  return d;
+}
+
+__device__ __forceinline__ void umma_bf16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                          uint32_t accumulate) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n"
+      "}\n" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
+}
+
+__device__ __forceinline__ void umma_commit(uint32_t bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+}
+
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float* v) {
+  uint32_t r[16];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+__device__ __forceinline__ void bf16x8_unpack(const int4& q, float* f) {
+  const uint32_t w[4] = {(uint32_t)q.x, (uint32_t)q.y, (uint32_t)q.z, (uint32_t)q.w};
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    f[2 * i] = __uint_as_float(w[i] << 16);
+    f[2 * i + 1] = __uint_as_float(w[i] & 0xffff0000u);
+  }
+}
+
+__device__ __forceinline__ int4 bf16x8_pack(const float* f) {
+  uint32_t w[4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(f[2 * i], f[2 * i + 1]);
+    w[i] = *reinterpret_cast<uint32_t*>(&h);
+  }
+  return make_int4((int)w[0], (int)w[1], (int)w[2], (int)w[3]);
+}
+
+template <bool MN>
+__global__ void __launch_bounds__(128, 1)
+    k_tc_gemm(const __grid_constant__ CUtensorMap tA0, const __grid_constant__ CUtensorMap tB0,
+              const __grid_constant__ CUtensorMap tA1, const __grid_constant__ CUtensorMap tB1,
+              const __grid_constant__ CUtensorMap tA2, const __grid_constant__ CUtensorMap tB2, TcParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int BN = p.BN, S = p.stages;
+  const int b_stage = MN ? ((BN + 63) / 64) * BK * 128 : BN * 128;
+  uint8_t* a_smem = smem;
+  uint8_t* b_smem = smem + S * A_STAGE;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(b_smem + S * b_stage);
+  uint64_t* full = bars;
+  uint64_t* empty = bars + 4;
+  uint64_t* accf = bars + 8;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 9);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint32_t tcols = 32;
+  while ((int)tcols < BN) tcols <<= 1;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(smem_u32(&full[s]), 1);
+      mbar_init(smem_u32(&empty[s]), 1);
+    }
+    mbar_init(smem_u32(accf), 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(tcols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tmem_slot;
+
+  const int64_t m0 = (int64_t)blockIdx.x * BM;
+  const int n0 = blockIdx.y * BN;
+  int total_kb = 0;
+  for (int i = 0; i < p.nparts; ++i) total_kb += p.kblocks[i];
+  const int64_t kz = MN ? p.k_base + (int64_t)blockIdx.z * p.k_span : 0;
+
+  if (threadIdx.x == 0) {
+    // ---------------- TMA producer
+    const uint32_t tx = A_STAGE + b_stage;
+    int part = 0, kk = 0;
+    for (int kb = 0; kb < total_kb; ++kb) {
+      const int s = kb % S;
+      const uint32_t ph = (kb / S) & 1;
+      mbar_wait(smem_u32(&empty[s]), ph ^ 1);
+      mbar_expect_tx(smem_u32(&full[s]), tx);
+      const uint32_t fb = smem_u32(&full[s]);
+      const uint32_t ad = smem_u32(a_smem + s * A_STAGE), bd = smem_u32(b_smem + s * b_stage);
+      if (MN) {
+        const int krow = (int)(kz + (int64_t)kb * BK);
+        tma_load_2d(ad, &tA0, (int)m0, krow, fb);
+        tma_load_2d(ad + BK * 128, &tA0, (int)m0 + 64, krow, fb);
+        for (int j = 0; j * 64 < BN; ++j) tma_load_2d(bd + j * BK * 128, &tB0, n0 + 64 * j, krow, fb);
+      } else {
+        const CUtensorMap* ta = part == 0 ? &tA0 : (part == 1 ? &tA1 : &tA2);
+        const CUtensorMap* tb = part == 0 ? &tB0 : (part == 1 ? &tB1 : &tB2);
+        tma_load_2d(ad, ta, kk * BK, (int)m0, fb);
+        tma_load_2d(bd, tb, kk * BK, n0, fb);
+        if (++kk == p.kblocks[part]) { kk = 0; ++part; }
+      }
+    }
+  } else if (threadIdx.x == 32) {
+    // ---------------- MMA issuer
+    // instruction descriptor: D f32 [4,6)=1, A bf16 [7,10)=1, B bf16 [10,13)=1,
+    // A/B major [15],[16], N>>3 [17,23), M>>4 [24,29)
+    const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((MN ? 1u : 0u) << 15) | ((MN ? 1u : 0u) << 16) |
+                           ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+    for (int kb = 0; kb < total_kb; ++kb) {
+      const int s = kb % S;
+      const uint32_t ph = (kb / S) & 1;
+      mbar_wait(smem_u32(&full[s]), ph);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      const uint32_t ad = smem_u32(a_smem + s * A_STAGE), bd = smem_u32(b_smem + s * b_stage);
+#pragma unroll
+      for (int k = 0; k < BK / 16; ++k) {
+        uint64_t adesc, bdesc;
+        if (MN) {  // MN-major SW128: LBO = next 64-wide MN chunk, SBO = next 8 K rows
+          adesc = umma_desc(ad + k * 16 * 128, BK * 128, 1024);
+          bdesc = umma_desc(bd + k * 16 * 128, BK * 128, 1024);
+        } else {   // K-major SW128: K step of 16 elements = +32 bytes inside the atom
+          adesc = umma_desc(ad + k * 32, 16, 1024);
+          bdesc = umma_desc(bd + k * 32, 16, 1024);
+        }
+        umma_bf16(tmem, adesc, bdesc, idesc, (kb | k) != 0 ? 1u : 0u);
+      }
+      umma_commit(smem_u32(&empty[s]));
+    }
+    umma_commit(smem_u32(accf));
+  }
+  __syncwarp();
+  // ---------------- epilogue: warp w owns TMEM lanes / tile rows 32w..32w+31
+  mbar_wait(smem_u32(accf), 0);
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const int r = warp * 32 + lane;
+  const int64_t m = m0 + r;
+  const GemmEpi& e = p.epi;
+  const float rs = (!MN && e.rscale && m < p.M) ? e.rscale[m] : 1.f;
+  for (int c0 = 0; c0 < BN; c0 += 16) {
+    float v[16];
+    tmem_ld16(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0, v);
+    if (m >= p.M) continue;
+    if (MN) {
+      float* out = p.part + (int64_t)blockIdx.z * p.M * p.N + m * p.N;
+#pragma unroll
+      for (int i = 0; i < 16; ++i) {
+        const int n = n0 + c0 + i;
+        if (n < p.N) out[n] = v[i];
+      }
+      continue;
+    }
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int n = n0 + c0 + 8 * h;
+      if (n >= p.N) continue;
+      float* f = v + 8 * h;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) f[i] *= rs;
+      if (e.addend) {
+        float t[8];
+        bf16x8_unpack(*reinterpret_cast<const int4*>(static_cast<const __nv_bfloat16*>(e.addend) + m * e.ld_add + n), t);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) f[i] += t[i];
+      }
+      if (e.bias) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) f[i] += (n + i < p.N) ? e.bias[n + i] : 0.f;
+      }
+      if (e.relu) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) f[i] = fmaxf(f[i], 0.f);
+      }
+      if (e.mask_ref) {
+        float t[8];
+        bf16x8_unpack(*reinterpret_cast<const int4*>(static_cast<const __nv_bfloat16*>(e.mask_ref) + m * e.ld_mask + n), t);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) f[i] = t[i] > 0.f ? f[i] : 0.f;
+      }
+      if (e.d_f32) {
+        float* o = static_cast<float*>(e.D) + m * e.ldd + n;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) o[i] = f[i];
+      } else {
+        *reinterpret_cast<int4*>(static_cast<__nv_bfloat16*>(e.D) + m * e.ldd + n) = bf16x8_pack(f);
+      }
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(tcols));
+}
+
+__global__ void k_split_reduce_tc(const float* part, int splits, int64_t MN, float* D) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= MN) return;
+  float s = 0.f;
+  for (int z = 0; z < splits; ++z) s += part[z * MN + i];
+  D[i] = s;
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  return fn;
+}
+
+// 2-D bf16 tensor map, 128-byte swizzle; dims {inner, outer}, row pitch ld_bytes
+bool make_map(CUtensorMap* m, const void* ptr, uint64_t inner, uint64_t outer, uint64_t ld_bytes, uint32_t box_in,
+              uint32_t box_out) {
+  auto fn = encode_fn();
+  if (!fn) return false;
+  if ((reinterpret_cast<uintptr_t>(ptr) & 15) || (ld_bytes & 15)) return false;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {ld_bytes};
+  cuuint32_t box[2] = {box_in, box_out};
+  cuuint32_t estr[2] = {1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+int g_tc_disabled = -1;
+bool tc_enabled() {
+  if (g_tc_disabled < 0) {
+    const char* e = getenv("WG_DISABLE_TC");
+    g_tc_disabled = (e && e[0] == '1') ? 1 : 0;
+  }
+  return !g_tc_disabled;
+}
+
+size_t smem_bytes(bool mn, int BN, int stages) {
+  const int b_stage = mn ? ((BN + 63) / 64) * BK * 128 : BN * 128;
+  return 1024 + (size_t)stages * (A_STAGE + b_stage) + 128;
+}
+
+template <bool MN>
+wg_status launch(dim3 grid, size_t smem, const CUtensorMap* maps, const TcParams& p, cudaStream_t s) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_tc_gemm<MN>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    attr = true;
+  }
+  WG_LAUNCH(k_tc_gemm<MN>, grid, 128, smem, s, maps[0], maps[1], maps[2], maps[3], maps[4], maps[5], p);
+  return WG_OK;
+}
+
+}  // namespace
+
+bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi,
+                cudaStream_t s, wg_status* st) {
+  if (dt != WG_BF16 || !tc_enabled() || n_parts > 3 || M <= 0) return false;
+  const int n_tiles = (int)cdiv(N, 256);
+  const int BN = (int)rup(cdiv(N, n_tiles), 16);
+  if (BN > 256) return false;
+  CUtensorMap maps[6];
+  memset(maps, 0, sizeof(maps));
+  TcParams p{};
+  p.M = M; p.N = N; p.BN = BN; p.nparts = n_parts; p.epi = epi;
+  for (int i = 0; i < n_parts; ++i) {
+    const GemmPart& q = parts[i];
+    if (!make_map(&maps[2 * i], q.A, (uint64_t)q.K, (uint64_t)M, (uint64_t)q.lda * 2, BK, BM)) return false;
+    if (!make_map(&maps[2 * i + 1], q.B, (uint64_t)q.K, (uint64_t)q.nb, (uint64_t)q.ldb * 2, BK, BN))
+      return false;
+    p.kblocks[i] = (int)cdiv(q.K, BK);
+  }
+  for (int i = n_parts; i < 3; ++i) { maps[2 * i] = maps[0]; maps[2 * i + 1] = maps[1]; }
+  if ((epi.addend && ((uintptr_t)epi.addend & 15)) || ((uintptr_t)epi.D & 15)) return false;
+  int stages = 4;
+  while (stages > 2 && smem_bytes(false, BN, stages) > 110 * 1024) --stages;
+  p.stages = stages;
+  dim3 grid((unsigned)cdiv(M, BM), (unsigned)n_tiles, 1);
+  double kt = 0;
+  for (int i = 0; i < n_parts; ++i) kt += parts[i].K;
+  ProfScope ps(PK_TC_NT, s, (double)M * (kt + N + (epi.addend ? N : 0) + (epi.mask_ref ? N : 0)) * 2.0,
+               2.0 * M * N * kt);
+  *st = launch<false>(grid, smem_bytes(false, BN, stages), maps, p, s);
+  return true;
+}
+
+bool tc_gemm_tn(int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb, float* D,
+                float* part, cudaStream_t s, wg_status* st) {
+  if (!tc_enabled() || K <= 0) return false;
+  const int n_tiles = (int)cdiv(N, 256);
+  const int BN = (int)rup(cdiv(N, n_tiles), 16);
+  const int m_tiles = (int)cdiv(M, BM);
+  CUtensorMap maps[6];
+  memset(maps, 0, sizeof(maps));
+  if (!make_map(&maps[0], A, (uint64_t)M, (uint64_t)K, (uint64_t)lda * 2, 64, BK)) return false;
+  if (!make_map(&maps[1], B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb * 2, 64, BK)) return false;
+  for (int i = 2; i < 6; ++i) maps[i] = maps[i & 1];
+  // split K so that the grid covers the SMs twice
+  const int tiles = m_tiles * n_tiles;
+  int64_t splits = std::max<int64_t>(1, (148 * 2) / tiles);
+  splits = std::min<int64_t>(splits, cdiv(K, BK));
+  splits = std::min<int64_t>(splits, 160);
+  const int64_t span = rup(cdiv(K, splits), BK);
+  splits = cdiv(K, span);
+  TcParams p{};
+  p.M = M; p.N = N; p.BN = BN; p.nparts = 1; p.kblocks[0] = (int)(span / BK);
+  p.k_base = 0; p.k_span = span; p.K = K; p.part = part;
+  int stages = 4;
+  while (stages > 2 && smem_bytes(true, BN, stages) > 200 * 1024) --stages;
+  p.stages = stages;
+  dim3 grid((unsigned)m_tiles, (unsigned)n_tiles, (unsigned)splits);
+  ProfScope ps(PK_TC_TN, s, (double)K * (M + N) * 2.0 + (double)M * N * 4.0, 2.0 * K * M * N);
+  *st = launch<true>(grid, smem_bytes(true, BN, stages), maps, p, s);
+  if (*st != WG_OK) return true;
+  const int64_t MN = (int64_t)M * N;
+  cudaStream_t ss = s;
+  k_split_reduce_tc<<<(unsigned)cdiv(MN, 256), 256, 0, ss>>>(part, (int)splits, MN, D);
+  ++launch_counter();
+  if (cudaGetLastError() != cudaSuccess) *st = WG_ERR_CUDA;
+  return true;
+}
+
 }  // namespace wg

@@ -45,6 +45,8 @@ void build_items(const wg_graph_s* g, const Side& S, const std::vector<uint8_t>*
       int b = (cur_task >= 0 && plan) ? (*plan)[cur_task] : 0;
       int64_t weight = cur_task >= 0 ? S.h_tasks[cur_task].e_end - S.h_tasks[cur_task].e_begin : 0;
       lists[b].push_back({weight, w});
+      (b ? out1 : out0)->n_edges += weight;
+      (b ? out1 : out0)->n_rows += end - cur_lo;
     };
     bool first = true;
     int32_t split_row = -1;
@@ -59,6 +61,7 @@ void build_items(const wg_graph_s* g, const Side& S, const std::vector<uint8_t>*
           split_row = row;
         }
         L->hs.back().n_slots++;
+        L->n_edges += t.e_end - t.e_begin;
         WorkItem w{};
         w.row_lo = row; w.row_hi = row + 1; w.e_lo = t.e_begin; w.e_hi = t.e_end;
         w.split_slot = slot++;
@@ -224,6 +227,15 @@ wg_status wg_plan_export(wg_plan p, uint8_t* per_task_plan, int64_t stats[8]) {
     stats[6] = p->bt.n;
     stats[7] = p->fe.n_split + p->fv.n_split;
   }
+  return WG_OK;
+}
+
+wg_status wg_plan_buffer(wg_plan p, int which, const char* name, size_t* offset) {
+  WG_REQ(p && name && offset, WG_ERR_INVALID, "wg_plan_buffer: null argument");
+  const wg::Layout& L = which ? p->ws : p->saved;
+  auto it = L.off.find(name);
+  WG_REQ(it != L.off.end(), WG_ERR_INVALID, std::string("no buffer named ") + name);
+  *offset = it->second;
   return WG_OK;
 }
 

@@ -30,6 +30,7 @@ struct ItemList {
   int n_split = 0;
   std::vector<WorkItem> h;
   std::vector<SplitRow> hs;
+  int64_t n_edges = 0, n_rows = 0;   // totals (algorithmic-byte accounting)
 };
 
 }  // namespace wg

@@ -51,6 +51,16 @@ int64_t& launch_counter();
     }                                                                                  \
   } while (0)
 
+// live per-kernel-class timing (wg_profile): events around each launch
+enum ProfKind { PK_AGG = 0, PK_COMBINE = 1, PK_TC_NT = 2, PK_TC_TN = 3, PK_SIMT = 4, PK_MISC = 5, PK_GAT = 6,
+                PK_RGCN = 7, PK_KINDS = 8 };
+struct ProfScope {
+  ProfScope(int kind, cudaStream_t s, double bytes, double flops);
+  ~ProfScope();
+  int rec_ = -1;
+  cudaStream_t s_;
+};
+
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 static inline int64_t rup(int64_t a, int64_t b) { return cdiv(a, b) * b; }
 static inline int dsize(wg_dtype t) { return t == WG_BF16 ? 2 : 4; }
@@ -138,6 +148,7 @@ struct AggArgs {
   int64_t ld_part;
   int F;                      // real columns
   int64_t E_max;              // rows with deg > E_max belong to SPLIT items
+  int64_t n_edges, n_rows;    // totals over the items (profiling: algorithmic bytes)
 };
 
 struct CombineArgs {
@@ -169,8 +180,9 @@ wg_status launch_combine(wg_dtype dt, const CombineArgs& a, cudaStream_t s);
 // GEMM: D[M x N] = sum_p A_p[M x K_p] * B_p[N x K_p]^T  (+ epilogue)
 struct GemmPart {
   const void* A; int64_t lda;   // row-major [M x K]
-  const void* B; int64_t ldb;   // row-major [N x K]
+  const void* B; int64_t ldb;   // row-major [nb x K]; rows >= nb read as 0
   int K;
+  int nb;
 };
 struct GemmEpi {
   const float* rscale = nullptr;      // per row

@@ -1,0 +1,148 @@
+"""Multi-layer full-graph training step over the gTask layer (single GPU and
+the 1-D multi-GPU partition of SURVEY §8(e)).
+
+Forward: layer i reads the previous activation table and writes its own rows
+straight into the next layer's table.  Distributed (one process per GPU,
+torch.distributed / NCCL): rank p owns the T-aligned vertex block
+[p*B, (p+1)*B) of every activation and gradient table; before a layer the
+table its gathers read is all-gathered in place -- the activation itself for
+EDGE (gather-then-transform) layers, or Y = h W for VERTEX layers when the
+transformed rows are narrower (transform-before-communicate, P:L2279-2289,
+Fig 11c).  Backward mirrors it: the per-layer PRE phase writes this rank's
+rows of dAgg (or dT) into the exchange table, the table is all-gathered, and
+the POST phase runs the transposed gather over the rank's out-edges.  Weight
+gradients are all-reduced (sum).  Rows >= V in the last block are padding.
+"""
+from __future__ import annotations
+
+import torch
+import torch.nn.functional as F
+
+from . import Conv, Graph, init_params, padded, pitch
+from . import _capi as C
+
+
+class GNNStack:
+    """L gTask layers (hidden ReLU fused into the layer epilogue) + CE loss + Adam."""
+
+    def __init__(self, graph: Graph, model: str, dims, *, dtype=torch.bfloat16, heads: int = 1, policy="auto",
+                 seed: int = 0, lr: float = 1e-3, group=None, block: int | None = None, R: int = 1):
+        self.g, self.model, self.dims, self.dtype = graph, model, list(dims), dtype
+        self.L = len(dims) - 1
+        self.dev = torch.device("cuda", graph.device)
+        self.group = group
+        self.dist = group is not None and torch.distributed.get_world_size(group) > 1
+        self.world = torch.distributed.get_world_size(group) if group is not None else 1
+        self.rank = torch.distributed.get_rank(group) if group is not None else 0
+        self.rows = graph.n_rows
+        self.vb = graph.v_begin
+        self.block = block if block is not None else self.rows
+        self.Vtab = self.block * self.world if self.dist else graph.V
+        self.convs, self.params = [], []
+        for i in range(self.L):
+            last = i == self.L - 1
+            kw = dict(dtype=dtype, fuse_relu=not last, need_dx=i > 0, seed=seed + i)
+            if model == "gat":
+                kw.update(heads=heads, concat=not last)
+            pol = policy
+            conv = Conv(graph, model, dims[i], dims[i + 1], policy=pol, **kw)
+            if self.dist and conv.n_edge_tasks and conv.n_vertex_tasks:   # uniform plan per layer when distributed
+                pol = "vertex" if conv.n_vertex_tasks > conv.n_edge_tasks else "edge"
+                conv.close()
+                conv = Conv(graph, model, dims[i], dims[i + 1], policy=pol, **kw)
+            self.convs.append(conv)
+            fo = dims[i + 1] if model != "gat" else (heads * dims[i + 1] if not last else dims[i + 1])
+            self.params.append(init_params(model, dims[i], dims[i + 1], heads=heads, concat=not last, R=R,
+                                           device=self.dev, seed=seed + 100 + i))
+        # activation tables: h[0] = input, h[i+1] = output of layer i (global rows when distributed)
+        self.h = [None] + [padded(self.Vtab, c.out_dim, dtype, self.dev) for c in self.convs]
+        self.saved = [c.new_saved() for c in self.convs]
+        self.dx = [None] + [padded(self.Vtab if self.dist else self.rows, dims[i], dtype, self.dev)
+                            for i in range(1, self.L)]
+        self.grads = [{k: torch.zeros_like(v) for k, v in p.items()} for p in self.params]
+        self.xchg_f, self.xchg_b = [], []
+        for c in self.convs:
+            self.xchg_f.append(padded(self.Vtab, pitch(c.f_out, dtype), dtype, self.dev)
+                               if (self.dist and c.n_vertex_tasks) else None)
+            wb = (c.f_out if c.bwd_path == 1 else c.f_in)
+            self.xchg_b.append(padded(self.Vtab, pitch(wb, dtype), dtype, self.dev) if self.dist else None)
+        for p in self.params:
+            for v in p.values():
+                v.requires_grad_(True)
+        self.opt = torch.optim.Adam([v for p in self.params for v in p.values()], lr=lr)
+
+    # -------------------------------------------------------------- helpers
+    def _own(self, t):
+        return t[self.vb:self.vb + self.rows] if self.dist else t
+
+    def _allgather(self, t):
+        if not self.dist:
+            return
+        full = t.as_strided((self.Vtab, t.stride(0)), (t.stride(0), 1))
+        mine = full[self.rank * self.block:(self.rank + 1) * self.block]
+        torch.distributed.all_gather_into_tensor(full, mine, group=self.group)
+
+    def forward(self, x):
+        """x: [V_tab x f0] (replicated input features); returns this rank's logits rows."""
+        h = x
+        for i, c in enumerate(self.convs):
+            y = self._own(self.h[i + 1])
+            if self.dist and c.n_vertex_tasks:
+                xg = self.xchg_f[i]
+                c.forward_raw(h, self.params[i], y=y, saved=self.saved[i], phase=C.PHASE_PRE, xchg=xg)
+                self._allgather(xg)
+                c.forward_raw(h, self.params[i], y=y, saved=self.saved[i], phase=C.PHASE_POST, xchg=xg)
+            else:
+                c.forward_raw(h, self.params[i], y=y, saved=self.saved[i])
+            if self.dist and i + 1 < self.L and not self.convs[i + 1].n_vertex_tasks:
+                self._allgather(self.h[i + 1])       # next EDGE layer gathers raw rows
+            h = self.h[i + 1]
+        self.x = x
+        return self._own(self.h[self.L])
+
+    def backward(self, dlogits):
+        g = dlogits
+        for i in reversed(range(self.L)):
+            c = self.convs[i]
+            xin = self.x if i == 0 else self.h[i]
+            dx = self._own(self.dx[i]) if i > 0 else None
+            y = self._own(self.h[i + 1])
+            if self.dist:
+                xb = self.xchg_b[i]
+                c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, phase=C.PHASE_PRE, xchg=xb,
+                               grads=self.grads[i])
+                self._allgather(xb)
+                c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, phase=C.PHASE_POST, xchg=xb,
+                               grads=self.grads[i])
+            else:
+                c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, grads=self.grads[i])
+            g = dx
+        if self.dist:
+            flat = torch.cat([v.reshape(-1) for gr in self.grads for v in gr.values()])
+            torch.distributed.all_reduce(flat, group=self.group)
+            o = 0
+            for gr in self.grads:
+                for v in gr.values():
+                    v.copy_(flat[o:o + v.numel()].view_as(v))
+                    o += v.numel()
+
+    def step(self, x, labels, n_global: int):
+        """One epoch step: forward, CE loss (mean over all vertices), backward, Adam."""
+        logits = self.forward(x)
+        lf = logits.float().detach().requires_grad_(True)
+        loss = F.cross_entropy(lf, labels, reduction="sum") / n_global
+        loss.backward()
+        dl = padded(self.rows, logits.shape[1], self.dtype, self.dev, zero=False)
+        dl.copy_(lf.grad)
+        self.backward(dl)
+        for p, gr in zip(self.params, self.grads):
+            for k, v in p.items():
+                v.grad = gr[k]
+        self.opt.step()
+        return loss.detach()
+
+
+def partition_1d(V: int, world: int, T: int = 128):
+    """Equal T-aligned vertex blocks: returns (block_rows, [(v_begin, v_end)] per rank)."""
+    block = -(-(-(-V // world)) // T) * T
+    return block, [(min(V, p * block), min(V, (p + 1) * block)) for p in range(world)]

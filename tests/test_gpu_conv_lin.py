@@ -32,7 +32,7 @@ def make_inputs(V, E, fi, fo, dtype, seed, alpha=0.6, ints=False):
     return src, dst, x.to(dtype), dy.to(dtype)
 
 
-def oracle_layer(model, src, dst, V, x, params, dy, dtype, norm, eps=0.0):
+def oracle_layer(model, src, dst, V, x, params, dy, dtype, norm, eps=0.0, amask=None):
     Wq = {k: q(v, dtype) for k, v in params.items()}
     xo = f64(x)
     if model == "gcn":
@@ -45,7 +45,8 @@ def oracle_layer(model, src, dst, V, x, params, dy, dtype, norm, eps=0.0):
         return y, dx, {"W": dWn, "W_self": dWs, "bias": db}
     if model == "gin":
         y = oracle.gin_forward(src, dst, V, xo, Wq["W"], Wq["bias"], Wq["W2"], Wq["b2"], eps)
-        dx, dW1, db1, dW2, db2 = oracle.gin_backward(src, dst, V, xo, Wq["W"], Wq["bias"], Wq["W2"], dy, eps)
+        dx, dW1, db1, dW2, db2 = oracle.gin_backward(src, dst, V, xo, Wq["W"], Wq["bias"], Wq["W2"], dy, eps,
+                                                     amask=amask)
         return y, dx, {"W": dW1, "bias": db1, "W2": dW2, "b2": db2}
     raise ValueError(model)
 
@@ -63,7 +64,8 @@ def run(model, dtype=torch.float32, policy="auto", V=900, E=12000, fi=37, fo=20,
         params = {k: torch.from_numpy(synth.small_ints(tuple(v.shape), seed=seed + 7 + i)).cuda()
                   for i, (k, v) in enumerate(params.items())}
     else:
-        params = {k: (v + 0.1 * torch.randn_like(v)) for k, v in params.items()}  # non-zero biases
+        gen = torch.Generator(device="cuda").manual_seed(seed)   # non-zero biases, seeded
+        params = {k: (v + 0.1 * torch.randn(v.shape, generator=gen, device=v.device)) for k, v in params.items()}
     xd = m.pad_to(x.cuda())
     y, saved = conv.forward_raw(xd, params)
     dyd = m.pad_to(dy.cuda())
@@ -73,7 +75,10 @@ def run(model, dtype=torch.float32, policy="auto", V=900, E=12000, fi=37, fo=20,
     dyo = f64(dy)
     if fuse_relu:
         dyo = dyo * (yg > 0)       # the mask decision is the kernel's (its own output)
-    yo, dxo, go = oracle_layer(model, src, dst, V, x, params, dyo, dtype, norm)
+    amask = None
+    if model == "gin":   # GIN's inner ReLU decision is the kernel's (taken on its fp32 accumulator)
+        amask = (f64(conv.buffer_view(saved, "h", V, fo)) > 0).astype(np.uint8)
+    yo, dxo, go = oracle_layer(model, src, dst, V, x, params, dyo, dtype, norm, amask=amask)
     if fuse_relu:
         yo = np.maximum(yo, 0)
     return dict(conv=conv, y=(yg, yo), dx=(f64(dx) if need_dx else None, dxo),
