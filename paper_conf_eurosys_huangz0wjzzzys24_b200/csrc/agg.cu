@@ -3,22 +3,24 @@
 //
 // Indexing ops of the paper: Index (h[src-id]) then Index-add (h[dst-id] +=)
 // (Fig 2b); "indexing dominates" tensor-centric execution
-// (P:L821-831).  Here one CTA executes one work item (the rows of one gTask);
-// the destination ordering inside a gTask is sorted, so every output row is
-// reduced in registers and stored ONCE with 16-byte vector stores -- no global
-// atomics.  Per-edge coefficients are factored into a per-source scale
-// (gathered with the row) and a per-destination scale.
+// (P:L821-831).  One CTA executes one work item (the rows of one gTask, or one
+// SPLIT chunk of an over-long row).  Inside a gTask the edges are sorted by
+// destination, so the reduction is a warp-segmented scan over a flat edge
+// range -- no global atomics:
+//   * the item's edge range is cut into 8*G equal chunks, one per "worker"
+//     (a group of LPE lanes; G = 32/LPE workers per warp), so every worker
+//     streams the same number of rows of the table regardless of the degree
+//     mix (overfill rows are shared by all workers);
+//   * a worker keeps U row loads (16 B per lane) in flight across row
+//     boundaries and flushes a destination row (epilogue + one 16-byte store
+//     per lane) as soon as it is complete;
+//   * a row cut by a chunk boundary leaves fp32 partials in shared memory; the
+//     worker where the row starts sums them in worker order and stores it.
+// Every reduction has a fixed order, so results are run-to-run deterministic.
 //
 //   out[r] = epi( rscale[r] * sum_{j in seg(r)} gscale[idx_j] * table[idx_j]
 //                 + self_coef * self[r] )
 //   epi(v) = mask( relu( v + bias ) )
-//
-// Differentiated execution: SPLIT chunks (frequent-value /
-// overfill rows) run first and write fp32 partials that a combine kernel sums
-// in chunk order; rows heavier than HEAVY_DEG inside a regular gTask are
-// processed by all 8 warps of the CTA (edge-parallel, smem reduction); the
-// other rows get one warp each.  All reductions use a fixed order, so results
-// are run-to-run deterministic.
 #include "wg_internal.cuh"
 
 namespace wg {
@@ -26,7 +28,6 @@ namespace wg {
 namespace {
 
 constexpr int WARPS = 8;
-constexpr int HEAVY_DEG = 256;
 
 template <typename T> struct VT;
 template <> struct VT<float> {
@@ -73,12 +74,12 @@ template <> struct VT<__nv_bfloat16> {
 
 __device__ __forceinline__ int4 ldg16(const void* p) { return __ldg(reinterpret_cast<const int4*>(p)); }
 
-// epilogue on one 16-byte output vector (EPV columns starting at column c0)
+// epilogue on one 16-byte output vector (EPV columns starting at column c0) of local row r
 template <typename T>
-__device__ __forceinline__ void epilogue_store(const float* acc_in, int64_t grow, int r, int cv, int c0,
-                                               float rs, const void* self_tab, int64_t ld_self, float self_coef,
-                                               const float* bias, int relu, const void* mask_ref, int64_t ld_mask,
-                                               void* out, int64_t ld_out, int F) {
+__device__ __forceinline__ void epilogue_store(const float* acc_in, int r, int c0, float rs, const void* self_tab,
+                                               int64_t ld_self, float self_coef, const float* bias, int relu,
+                                               const void* mask_ref, int64_t ld_mask, void* out, int64_t ld_out,
+                                               int F) {
   constexpr int EPV = VT<T>::EPV;
   float v[EPV];
 #pragma unroll
@@ -106,166 +107,177 @@ __device__ __forceinline__ void epilogue_store(const float* acc_in, int64_t grow
 #pragma unroll
   for (int i = 0; i < EPV; ++i) if (c0 + i >= F) v[i] = 0.f;
   *reinterpret_cast<int4*>(static_cast<T*>(out) + (int64_t)r * ld_out + c0) = VT<T>::pack(v);
-  (void)grow; (void)cv;
 }
 
+// write a finished row: epilogue store, or (SPLIT chunk) raw fp32 partial
 template <typename T>
-__device__ __forceinline__ void zero_row(void* z, int64_t ldz, int cols, int r, int lane, int nl) {
-  if (!z) return;
+__device__ __forceinline__ void finish_vec(const AggArgs& a, const float* acc, int r, int c0, int slot) {
   constexpr int EPV = VT<T>::EPV;
-  T* p = static_cast<T*>(z) + (int64_t)r * ldz;
-  for (int c = lane * EPV; c < cols; c += nl * EPV) *reinterpret_cast<int4*>(p + c) = make_int4(0, 0, 0, 0);
+  if (slot >= 0) {
+    float* pp = a.partial + (int64_t)slot * a.ld_part + c0;
+#pragma unroll
+    for (int i = 0; i < EPV; ++i) pp[i] = acc[i];
+    return;
+  }
+  const float rs = a.rscale ? a.rscale[a.row_base + r] : 1.f;
+  epilogue_store<T>(acc, r, c0, rs, a.self_tab, a.ld_self, a.self_coef, a.bias, a.relu, a.mask_ref, a.ld_mask, a.out,
+                    a.ld_out, a.F);
 }
 
-// Warp accumulation of the vectors [cv0, cv0 + nvec) of rows table[idx[j]],
-// j in [b, e).  LPE lanes cover one edge's row chunk (NV vectors per lane);
-// G = 32 / LPE edges are processed in parallel, U batches in flight.
+// Warp-segmented gather-reduce.  Template: LPE lanes per edge row chunk, NV
+// 16-byte vectors per lane (chunk width CW = LPE*NV vectors), U edges in flight.
 template <typename T, int LPE, int NV, int U>
-__device__ __forceinline__ void warp_accumulate(const AggArgs& a, int64_t b, int64_t e, int cv0, int nvec,
-                                                float (&acc)[NV][VT<T>::EPV]) {
+__global__ void __launch_bounds__(WARPS * 32, 3) k_agg(AggArgs a, int VPR) {
   constexpr int EPV = VT<T>::EPV;
   constexpr int G = 32 / LPE;
-  const int lane = threadIdx.x & 31, grp = lane / LPE, l = lane % LPE;
-#pragma unroll
-  for (int q = 0; q < NV; ++q)
-#pragma unroll
-    for (int i = 0; i < EPV; ++i) acc[q][i] = 0.f;
+  constexpr int W = WARPS * G;                 // workers per CTA
+  constexpr int CW = LPE * NV;                 // vectors per column chunk
+  constexpr int SLOTF = CW * EPV;              // floats per partial slot
+  extern __shared__ float part_smem[];         // [W][2][SLOTF]
+  __shared__ int slot_row[W][2];               // local row of slot 0 (continuation) / slot 1 (owner), -1 none
+
+  const WorkItem it = a.items[blockIdx.x];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int grp = lane / LPE, l = lane % LPE, worker = warp * G + grp;
+  const unsigned gmask = LPE == 32 ? 0xffffffffu : (((1u << LPE) - 1u) << (grp * LPE));
+  const bool split = it.split_slot >= 0;
+  const int64_t eb = split ? it.e_lo : a.row_ptr[it.row_lo];
+  const int64_t ee = split ? it.e_hi : a.row_ptr[it.row_hi];
+  const int64_t len = ee - eb;
+  const int64_t cb = eb + len * worker / W, ce = eb + len * (worker + 1) / W;
   const T* tab = static_cast<const T*>(a.table);
-  for (int64_t base = b; base < e; base += 32) {
-    const int n = (int)(e - base < 32 ? e - base : 32);
-    const int my_idx = lane < n ? a.idx[base + lane] : 0;
-    const float my_sc = (a.gscale && lane < n) ? a.gscale[my_idx] : 1.f;
-    for (int j = 0; j < n; j += G * U) {
-      int4 v[U][NV];
-      float sc[U];
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int k = j + u * G + grp;
-        const bool ok = k < n;
-        const int s = __shfl_sync(0xffffffffu, my_idx, ok ? k : 0);
-        sc[u] = __shfl_sync(0xffffffffu, my_sc, ok ? k : 0);
-        const T* row = tab + (int64_t)s * a.ld_tab + (int64_t)cv0 * EPV;
-#pragma unroll
-        for (int q = 0; q < NV; ++q) {
-          const int vi = l + q * LPE;
-          v[u][q] = (ok && vi < nvec) ? ldg16(row + vi * EPV) : make_int4(0, 0, 0, 0);
-        }
-        if (!ok) sc[u] = 0.f;
-      }
-#pragma unroll
-      for (int u = 0; u < U; ++u)
-#pragma unroll
-        for (int q = 0; q < NV; ++q) VT<T>::add(acc[q], v[u][q], sc[u]);
-    }
-  }
-#pragma unroll
-  for (int off = LPE; off < 32; off <<= 1)
-#pragma unroll
-    for (int q = 0; q < NV; ++q)
-#pragma unroll
-      for (int i = 0; i < EPV; ++i) acc[q][i] += __shfl_xor_sync(0xffffffffu, acc[q][i], off);
-}
+  const int64_t rb = a.row_base;
+  const int* key = a.key;
 
-template <typename T, int LPE, int NV, int U>
-__device__ void do_row_warp(const AggArgs& a, int r, int64_t b, int64_t e, int VPR) {
-  constexpr int EPV = VT<T>::EPV;
-  constexpr int CW = LPE * NV;
-  const int lane = threadIdx.x & 31, l = lane % LPE;
-  const float rs = a.rscale ? a.rscale[a.row_base + r] : 1.f;
   for (int cv0 = 0; cv0 < VPR; cv0 += CW) {
     const int nvec = min(CW, VPR - cv0);
-    float acc[NV][EPV];
-    warp_accumulate<T, LPE, NV, U>(a, b, e, cv0, nvec, acc);
-    if (lane < LPE) {
-#pragma unroll
-      for (int q = 0; q < NV; ++q) {
-        const int vi = l + q * LPE;
-        if (vi < nvec)
-          epilogue_store<T>(acc[q], a.row_base + r, r, cv0 + vi, (cv0 + vi) * EPV, rs, a.self_tab, a.ld_self,
-                            a.self_coef, a.bias, a.relu, a.mask_ref, a.ld_mask, a.out, a.ld_out, a.F);
-      }
-    }
-  }
-  zero_row<T>(a.zero_out, a.ld_zero, a.zero_cols, r, lane, 32);
-}
-
-// whole CTA on one row (heavy row or SPLIT chunk).  partial_slot >= 0: write
-// the raw fp32 sum to the partial buffer instead of the epilogue.
-template <typename T, int LPE, int NV, int U>
-__device__ void do_row_cta(const AggArgs& a, int r, int64_t b, int64_t e, int VPR, int partial_slot, float* red) {
-  constexpr int EPV = VT<T>::EPV;
-  constexpr int CW = LPE * NV;
-  const int lane = threadIdx.x & 31, l = lane % LPE, w = threadIdx.x >> 5;
-  const int64_t len = e - b;
-  const int64_t wb = b + len * w / WARPS, we = b + len * (w + 1) / WARPS;
-  const float rs = a.rscale ? a.rscale[a.row_base + r] : 1.f;
-  for (int cv0 = 0; cv0 < VPR; cv0 += CW) {
-    const int nvec = min(CW, VPR - cv0);
-    float acc[NV][EPV];
-    warp_accumulate<T, LPE, NV, U>(a, wb, we, cv0, nvec, acc);
-    __syncthreads();  // red[] reuse across chunks
-    if (lane < LPE) {
+    if (l == 0) { slot_row[worker][0] = -1; slot_row[worker][1] = -1; }
+    if (cb < ce) {
+      float acc[NV][EPV];
 #pragma unroll
       for (int q = 0; q < NV; ++q)
 #pragma unroll
-        for (int i = 0; i < EPV; ++i) red[(w * CW + l + q * LPE) * EPV + i] = acc[q][i];
+        for (int i = 0; i < EPV; ++i) acc[q][i] = 0.f;
+      int cur = split ? it.row_lo : (int)(key[cb] - rb);
+      bool first = true;
+      // first row starts before this chunk -> its partial is a continuation
+      const bool first_cont = split ? (cb > eb) : (a.row_ptr[cur] < cb);
+      int64_t pos = cb;
+      int my_idx = 0, my_key = 0;
+      float my_sc = 1.f;
+      if (pos + l < ce) {
+        my_idx = a.idx[pos + l];
+        my_key = split ? it.row_lo : (int)(key[pos + l] - rb);
+        if (a.gscale) my_sc = a.gscale[my_idx];
+      }
+      auto flush = [&](int row, bool as_cont, bool as_owner) {
+        // as_cont: continuation partial (slot 0); as_owner: owner partial (slot 1); else final
+        if (as_cont || as_owner) {
+          const int s = as_cont ? 0 : 1;
+          float* sp = part_smem + ((size_t)worker * 2 + s) * SLOTF;
+#pragma unroll
+          for (int q = 0; q < NV; ++q)
+#pragma unroll
+            for (int i = 0; i < EPV; ++i) sp[(l + q * LPE) * EPV + i] = acc[q][i];
+          if (l == 0) slot_row[worker][s] = row;
+        } else {
+#pragma unroll
+          for (int q = 0; q < NV; ++q) {
+            const int vi = l + q * LPE;
+            if (vi < nvec) finish_vec<T>(a, acc[q], row, (cv0 + vi) * EPV, split ? it.split_slot : -1);
+          }
+        }
+      };
+      while (pos < ce) {
+        const int n = (int)min((int64_t)LPE, ce - pos);
+        // prefetch the next round of indices
+        int nx_idx = 0, nx_key = 0;
+        float nx_sc = 1.f;
+        const int64_t np = pos + LPE + l;
+        if (np < ce) {
+          nx_idx = a.idx[np];
+          nx_key = split ? it.row_lo : (int)(key[np] - rb);
+          if (a.gscale) nx_sc = a.gscale[nx_idx];
+        }
+        for (int j = 0; j < n; j += U) {
+          int4 v[U][NV];
+          float sc[U];
+          int rk[U];
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const int k = j + u;
+            const bool ok = k < n;
+            const int s = __shfl_sync(gmask, my_idx, ok ? k : 0, LPE);
+            sc[u] = __shfl_sync(gmask, my_sc, ok ? k : 0, LPE);
+            rk[u] = __shfl_sync(gmask, my_key, ok ? k : 0, LPE);
+            if (!ok) rk[u] = -1;
+            const T* row = tab + (int64_t)s * a.ld_tab + (int64_t)cv0 * EPV;
+#pragma unroll
+            for (int q = 0; q < NV; ++q) {
+              const int vi = l + q * LPE;
+              v[u][q] = (ok && vi < nvec) ? ldg16(row + vi * EPV) : make_int4(0, 0, 0, 0);
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            if (rk[u] < 0) break;
+            if (rk[u] != cur) {
+              flush(cur, first && first_cont, false);
+              first = false;
+              cur = rk[u];
+#pragma unroll
+              for (int q = 0; q < NV; ++q)
+#pragma unroll
+                for (int i = 0; i < EPV; ++i) acc[q][i] = 0.f;
+            }
+#pragma unroll
+            for (int q = 0; q < NV; ++q) VT<T>::add(acc[q], v[u][q], sc[u]);
+          }
+        }
+        my_idx = nx_idx;
+        my_key = nx_key;
+        my_sc = nx_sc;
+        pos += LPE;
+      }
+      // last row of the chunk: does it continue past the chunk end?
+      const bool last_open = split ? (ce < ee) : (a.row_ptr[cur + 1] > ce);
+      if (first && first_cont) flush(cur, true, false);       // whole chunk inside one cut row
+      else flush(cur, false, last_open);
     }
     __syncthreads();
-    for (int vi = threadIdx.x; vi < nvec; vi += blockDim.x) {
-      float s[EPV];
+    // owners merge the continuation partials of the following workers, in order
+    if (cb < ce && slot_row[worker][1] >= 0) {
+      const int r = slot_row[worker][1];
+      for (int q = 0; q < NV; ++q) {
+        const int vi = l + q * LPE;
+        if (vi >= nvec) continue;
+        float s[EPV];
+        const float* sp = part_smem + ((size_t)worker * 2 + 1) * SLOTF + vi * EPV;
 #pragma unroll
-      for (int i = 0; i < EPV; ++i) s[i] = 0.f;
-      for (int ww = 0; ww < WARPS; ++ww)
+        for (int i = 0; i < EPV; ++i) s[i] = sp[i];
+        for (int w2 = worker + 1; w2 < W; ++w2) {
+          if (len * w2 / W == len * (w2 + 1) / W) continue;   // empty chunk (items shorter than W edges)
+          if (slot_row[w2][0] != r) break;
+          const float* sq = part_smem + ((size_t)w2 * 2 + 0) * SLOTF + vi * EPV;
 #pragma unroll
-        for (int i = 0; i < EPV; ++i) s[i] += red[(ww * CW + vi) * EPV + i];
-      const int c0 = (cv0 + vi) * EPV;
-      if (partial_slot >= 0) {
-        float* pp = a.partial + (int64_t)partial_slot * a.ld_part + c0;
-#pragma unroll
-        for (int i = 0; i < EPV; ++i) pp[i] = s[i];
-      } else {
-        epilogue_store<T>(s, a.row_base + r, r, cv0 + vi, c0, rs, a.self_tab, a.ld_self, a.self_coef, a.bias,
-                          a.relu, a.mask_ref, a.ld_mask, a.out, a.ld_out, a.F);
+          for (int i = 0; i < EPV; ++i) s[i] += sq[i];
+        }
+        finish_vec<T>(a, s, r, (cv0 + vi) * EPV, split ? it.split_slot : -1);
       }
     }
-  }
-  if (partial_slot < 0) zero_row<T>(a.zero_out, a.ld_zero, a.zero_cols, r, threadIdx.x, blockDim.x);
-}
-
-template <typename T, int LPE, int NV, int U>
-__global__ void __launch_bounds__(WARPS * 32) k_agg(AggArgs a, int VPR) {
-  extern __shared__ float red[];
-  __shared__ int heavy[1024];
-  __shared__ int n_heavy;
-  const WorkItem it = a.items[blockIdx.x];
-  if (it.split_slot >= 0) {
-    do_row_cta<T, LPE, NV, U>(a, it.row_lo, it.e_lo, it.e_hi, VPR, it.split_slot, red);
-    return;
-  }
-  if (threadIdx.x == 0) n_heavy = 0;
-  __syncthreads();
-  const int nrows = it.row_hi - it.row_lo;
-  // rows: heavy ones are collected (in row order, one pass of up to 1024 rows)
-  for (int i = threadIdx.x; i < nrows && i < 1024; i += blockDim.x) {
-    const int r = it.row_lo + i;
-    const int64_t deg = a.row_ptr[r + 1] - a.row_ptr[r];
-    if (deg >= HEAVY_DEG && deg <= a.E_max) heavy[atomicAdd(&n_heavy, 1)] = r;
-  }
-  __syncthreads();
-  const int nh = n_heavy;
-  for (int h = 0; h < nh; ++h) {
-    const int r = heavy[h];
-    do_row_cta<T, LPE, NV, U>(a, r, a.row_ptr[r], a.row_ptr[r + 1], VPR, -1, red);
     __syncthreads();
   }
-  const int w = threadIdx.x >> 5;
-  for (int i = w; i < nrows; i += WARPS) {
-    const int r = it.row_lo + i;
-    const int64_t b = a.row_ptr[r], e = a.row_ptr[r + 1];
-    const int64_t deg = e - b;
-    if (deg > a.E_max) continue;                       // SPLIT row: combine kernel
-    if (deg >= HEAVY_DEG && i < 1024) continue;        // done cooperatively
-    do_row_warp<T, LPE, NV, U>(a, r, b, e, VPR);
+  if (split) return;
+  // rows without in-edges (and the optional zeroed second output)
+  for (int r = it.row_lo + warp; r < it.row_hi; r += WARPS) {
+    if (a.row_ptr[r + 1] == a.row_ptr[r]) {
+      const float zero[EPV] = {};
+      for (int vi = lane; vi < VPR; vi += 32) finish_vec<T>(a, zero, r, vi * EPV, -1);
+    }
+    if (a.zero_out) {
+      T* p = static_cast<T*>(a.zero_out) + (int64_t)r * a.ld_zero;
+      for (int c = lane * EPV; c < a.zero_cols; c += 32 * EPV) *reinterpret_cast<int4*>(p + c) = make_int4(0, 0, 0, 0);
+    }
   }
 }
 
@@ -285,16 +297,20 @@ __global__ void k_combine(CombineArgs a, int VPR) {
 #pragma unroll
       for (int i = 0; i < EPV; ++i) s[i] += pp[i];
     }
-    epilogue_store<T>(s, a.row_base + sr.row, sr.row, vi, c0, rs, a.self_tab, a.ld_self, a.self_coef, a.bias, a.relu,
-                      a.mask_ref, a.ld_mask, a.out, a.ld_out, a.F);
+    epilogue_store<T>(s, sr.row, c0, rs, a.self_tab, a.ld_self, a.self_coef, a.bias, a.relu, a.mask_ref, a.ld_mask,
+                      a.out, a.ld_out, a.F);
   }
-  zero_row<T>(a.zero_out, a.ld_zero, a.zero_cols, sr.row, threadIdx.x, blockDim.x);
+  if (a.zero_out) {
+    T* p = static_cast<T*>(a.zero_out) + (int64_t)sr.row * a.ld_zero;
+    for (int c = threadIdx.x * EPV; c < a.zero_cols; c += blockDim.x * EPV)
+      *reinterpret_cast<int4*>(p + c) = make_int4(0, 0, 0, 0);
+  }
 }
 
 template <typename T, int LPE, int NV, int U>
 wg_status launch_cfg(const AggArgs& a, int VPR, cudaStream_t s) {
   constexpr int EPV = VT<T>::EPV;
-  const size_t smem = (size_t)WARPS * LPE * NV * EPV * sizeof(float);
+  const size_t smem = (size_t)WARPS * (32 / LPE) * 2 * LPE * NV * EPV * sizeof(float);
   if (smem > 48 * 1024) {
     static bool done = false;
     if (!done) {
@@ -313,7 +329,7 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
   if (VPR <= 1) return launch_cfg<T, 1, 1, 1>(a, VPR, s);
   if (VPR <= 2) return launch_cfg<T, 2, 1, 2>(a, VPR, s);
   if (VPR <= 4) return launch_cfg<T, 4, 1, 4>(a, VPR, s);
-  if (VPR <= 8) return launch_cfg<T, 8, 1, 4>(a, VPR, s);
+  if (VPR <= 8) return launch_cfg<T, 8, 1, 8>(a, VPR, s);
   if (VPR <= 16) return launch_cfg<T, 16, 1, 8>(a, VPR, s);
   if (VPR <= 32) return launch_cfg<T, 32, 1, 8>(a, VPR, s);
   if (VPR <= 64) return launch_cfg<T, 32, 2, 4>(a, VPR, s);
@@ -324,6 +340,7 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
 
 wg_status launch_agg(wg_dtype dt, const AggArgs& a, cudaStream_t s) {
   if (a.n_items == 0) return WG_OK;
+  WG_REQ(a.key != nullptr, WG_ERR_STATE, "launch_agg: key array missing");
   // algorithmic bytes: per edge the index (4 B), the gathered row (F elements)
   // and the source scale if any; per row the output, row_ptr and optional
   // self / mask rows
@@ -361,19 +378,41 @@ __global__ void k_prep_weight(const float* W, int rows, int cols, int transpose,
   }
 }
 
-// column partial sums of (optionally relu-masked) dy over row blocks
+// Column partial sums of (optionally ReLU-masked) dy over blocks of rows,
+// 16-byte vectors per thread; block partials reduced in a fixed order.
 template <typename T>
-__global__ void k_colsum(int64_t M, int N, const T* dy, int64_t lddy, const T* ref, int64_t ldref, T* dt,
-                         int64_t ldt, float* part, int64_t rows_per_blk) {
+__global__ void __launch_bounds__(256) k_colsum(int64_t M, int N, const T* dy, int64_t lddy, const T* ref,
+                                                int64_t ldref, T* dt, int64_t ldt, float* part, int64_t rows_per_blk) {
+  constexpr int EPV = VT<T>::EPV;
+  extern __shared__ float red[];                       // [nsub][nv*EPV]
+  const int nv = (N + EPV - 1) / EPV;                  // vectors per row (<= 256)
+  const int nsub = blockDim.x / nv;
+  const int vec = threadIdx.x % nv, sub = threadIdx.x / nv;
   const int64_t r0 = blockIdx.x * rows_per_blk, r1 = min(M, r0 + rows_per_blk);
+  float acc[EPV] = {};
+  if (sub < nsub) {
+    for (int64_t r = r0 + sub; r < r1; r += nsub) {
+      float v[EPV];
+      VT<T>::unpack(ldg16(dy + r * lddy + vec * EPV), v);
+      if (ref) {
+        float m[EPV];
+        VT<T>::unpack(ldg16(ref + r * ldref + vec * EPV), m);
+#pragma unroll
+        for (int i = 0; i < EPV; ++i) v[i] = m[i] > 0.f ? v[i] : 0.f;
+      }
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) if (vec * EPV + i >= N) v[i] = 0.f;
+      if (dt) *reinterpret_cast<int4*>(dt + r * ldt + vec * EPV) = VT<T>::pack(v);
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) acc[i] += v[i];
+    }
+#pragma unroll
+    for (int i = 0; i < EPV; ++i) red[sub * nv * EPV + vec * EPV + i] = acc[i];
+  }
+  __syncthreads();
   for (int c = threadIdx.x; c < N; c += blockDim.x) {
     float s = 0.f;
-    for (int64_t r = r0; r < r1; ++r) {
-      float v = (float)dy[r * lddy + c];
-      if (ref && !((float)ref[r * ldref + c] > 0.f)) v = 0.f;
-      if (dt) dt[r * ldt + c] = (T)v;
-      s += v;
-    }
+    for (int k = 0; k < nsub; ++k) s += red[k * nv * EPV + c];
     part[(int64_t)blockIdx.x * N + c] = s;
   }
 }
@@ -407,16 +446,20 @@ size_t bias_grad_scratch(int64_t M, int N) { return sizeof(float) * (size_t)COLS
 
 wg_status bias_grad_mask(wg_dtype dt, int64_t M, int N, const void* dy, int64_t lddy, const void* ref,
                          int64_t ldref, void* dt_out, int64_t ldt, float* db, float* scratch, cudaStream_t s) {
+  const int EPV = dt == WG_BF16 ? 8 : 4;
+  const int nv = (int)cdiv(N, EPV);
+  WG_REQ(nv <= 256, WG_ERR_UNSUPPORTED, "bias gradient: more than 256 vectors per row");
   const int64_t rpb = std::max<int64_t>(1, cdiv(M, COLSUM_BLKS));
   const int nblk = (int)std::max<int64_t>(1, cdiv(M, rpb));
   const double es = dt == WG_BF16 ? 2.0 : 4.0;
   ProfScope ps(PK_MISC, s, (double)M * N * es * (1 + (ref ? 1 : 0) + (dt_out ? 1 : 0)), (double)M * N);
-  const int threads = N >= 256 ? 256 : (int)rup(N, 32);
+  const int threads = 256;
+  const size_t smem = (size_t)(threads / nv) * nv * EPV * sizeof(float);
   if (dt == WG_BF16)
-    WG_LAUNCH(k_colsum<__nv_bfloat16>, nblk, threads, 0, s, M, N, (const __nv_bfloat16*)dy, lddy,
+    WG_LAUNCH(k_colsum<__nv_bfloat16>, nblk, threads, smem, s, M, N, (const __nv_bfloat16*)dy, lddy,
               (const __nv_bfloat16*)ref, ldref, (__nv_bfloat16*)dt_out, ldt, scratch, rpb);
   else
-    WG_LAUNCH(k_colsum<float>, nblk, threads, 0, s, M, N, (const float*)dy, lddy, (const float*)ref, ldref,
+    WG_LAUNCH(k_colsum<float>, nblk, threads, smem, s, M, N, (const float*)dy, lddy, (const float*)ref, ldref,
               (float*)dt_out, ldt, scratch, rpb);
   if (db) WG_LAUNCH(k_colsum_reduce, (unsigned)cdiv(N, 128), 128, 0, s, scratch, nblk, N, db);
   return WG_OK;

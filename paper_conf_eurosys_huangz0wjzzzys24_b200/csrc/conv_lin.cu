@@ -100,6 +100,7 @@ AggArgs agg_base(const Ctx& c, const ItemList& L, const Side& S) {
   a.n_items = L.n;
   a.row_ptr = S.row_ptr;
   a.idx = S.idx;
+  a.key = S.key;
   a.row_base = c.vb;
   a.self_coef = 1.f;
   a.E_max = c.g->E_max;

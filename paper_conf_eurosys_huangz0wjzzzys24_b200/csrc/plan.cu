@@ -2,14 +2,11 @@
 //
 // Cost model ("computation workload, memory access volume, and
 // parallelism"; the paper gives no formula): integer
-// milli-femtoseconds per gTask,
-//   t_edge = max(n_e (A+4) k_mem + n_rows 2A k_mem, 2 n_rows F_in F_out k_mma)
-// (n_rows = d_hi - d_lo + 1: the unfused EDGE path writes and re-reads Agg)
-//   t_vert = n_e (B+4) k_mem + floor(n_uniq U / S) (A+B) k_mem
-// with A / B the padded row bytes of f_in / f_out wide rows, U the number of
-// vertices with out-edges, S = sum over gTasks of n_uniq_src (each Y row is
-// shared by the gTasks that read it: T1 unique extraction, and
-// T2 indexing swapping).  VERTEX iff t_vert < t_edge.
+// HBM bytes per gTask and per layer, see choose_plans().  Both plans do the
+// same GEMM FLOPs (one row transform per vertex: T1 unique extraction
+// P:L1823-1843 + T2 indexing swapping P:L1845-1876 make the VERTEX plan
+// transform each source row once), so on these HBM-bound shapes the bytes
+// decide.  A / B are the 32-byte padded row bytes of f_in / f_out rows.
 #include <algorithm>
 #include <random>
 
@@ -35,18 +32,26 @@ void build_items(const wg_graph_s* g, const Side& S, const std::vector<uint8_t>*
     while (tj < S.h_tasks.size() && S.h_tasks[tj].tile == tile) ++tj;
     int32_t cur_lo = lo;
     int64_t cur_task = -1;
+    // emit the rows [cur_lo, end) as work items, cut around SPLIT rows
+    // (deg > E_max: those rows are produced by their SPLIT chunks + combine)
     auto flush = [&](int32_t end) {
-      if (end <= cur_lo) return;
-      WorkItem w{};
-      w.row_lo = cur_lo; w.row_hi = end;
-      w.e_lo = S.h_row_ptr[cur_lo]; w.e_hi = S.h_row_ptr[end];
-      w.split_slot = -1;
-      w.task = (int32_t)cur_task;
-      int b = (cur_task >= 0 && plan) ? (*plan)[cur_task] : 0;
-      int64_t weight = cur_task >= 0 ? S.h_tasks[cur_task].e_end - S.h_tasks[cur_task].e_begin : 0;
-      lists[b].push_back({weight, w});
-      (b ? out1 : out0)->n_edges += weight;
-      (b ? out1 : out0)->n_rows += end - cur_lo;
+      const int b = (cur_task >= 0 && plan) ? (*plan)[cur_task] : 0;
+      int32_t lo = cur_lo;
+      for (int32_t r = cur_lo; r <= end; ++r) {
+        const bool cut = (r == end) || (S.h_row_ptr[r + 1] - S.h_row_ptr[r] > g->E_max);
+        if (!cut) continue;
+        if (r > lo) {
+          WorkItem w{};
+          w.row_lo = lo; w.row_hi = r;
+          w.e_lo = S.h_row_ptr[lo]; w.e_hi = S.h_row_ptr[r];
+          w.split_slot = -1;
+          w.task = (int32_t)cur_task;
+          lists[b].push_back({w.e_hi - w.e_lo, w});
+          (b ? out1 : out0)->n_edges += w.e_hi - w.e_lo;
+          (b ? out1 : out0)->n_rows += r - lo;
+        }
+        lo = r + 1;
+      }
     };
     bool first = true;
     int32_t split_row = -1;
@@ -107,28 +112,31 @@ void choose_plans(wg_plan_s* p) {
     std::mt19937_64 rng(d.policy_seed);
     for (int64_t i = 0; i < n; ++i) p->plan_bits[i] = (uint8_t)(rng() & 1);
   } else if (d.policy == WG_PLAN_AUTO) {
+    // Per gTask (HBM bytes, both plans' common terms dropped):
+    //   EDGE   t_e = n_e (A + 4) + n_rows 2A      (gather f_in rows, Agg round trip)
+    //   VERTEX t_v = n_e (B + 4)                  (gather f_out rows)
+    // plus per-layer terms: any VERTEX gTask needs Y = x W for every row,
+    // V (A + B); a mixed layer also writes / reads / zeroes Z, 3 B per row.
+    // The layer takes the cheapest of all-EDGE, all-VERTEX and per-gTask
+    // minimum (ties -> EDGE), i.e. the least-workload DFG.
     const int s = dsize(d.dtype);
     const int64_t A = rup((int64_t)d.f_in * s, 32), B = rup((int64_t)d.f_out * s, 32);
-    const int64_t k_mma = d.dtype == WG_BF16 ? K_MMA_BF16 : K_MMA_F32;
-    int64_t S = 0;
-    for (auto& t : tasks) S += t.n_uniq_src;
-    // U: vertices with out-edges (each needs one Y row)
-    int64_t U = 0;
-    {
-      std::vector<int32_t> dout(g->V);
-      cudaMemcpy(dout.data(), g->deg_out, 4 * g->V, cudaMemcpyDeviceToHost);
-      for (auto x : dout) U += x > 0;
-    }
+    const int64_t rows = g->ve - g->vb;
+    int64_t sum_e = 0, sum_v = rows * (A + B), sum_m = rows * (A + B) + rows * 3 * B;
+    std::vector<uint8_t> best(n, 0);
     for (int64_t i = 0; i < n; ++i) {
       const wg_task& t = tasks[i];
       const int64_t ne = t.e_end - t.e_begin;
       const int64_t nrows = (int64_t)t.d_hi - t.d_lo + 1;
-      const int64_t t_edge = std::max<int64_t>(ne * (A + 4) * K_MEM + nrows * 2 * A * K_MEM,
-                                      2LL * nrows * d.f_in * d.f_out * k_mma);
-      const int64_t share = S > 0 ? (int64_t)t.n_uniq_src * U / S : 0;
-      const int64_t t_vert = ne * (B + 4) * K_MEM + share * (A + B) * K_MEM;
-      p->plan_bits[i] = t_vert < t_edge ? 1 : 0;
+      const int64_t te = ne * (A + 4) + nrows * 2 * A, tv = ne * (B + 4);
+      sum_e += te;
+      sum_v += tv;
+      sum_m += std::min(te, tv);
+      best[i] = tv < te ? 1 : 0;
     }
+    if (sum_e <= sum_v && sum_e <= sum_m) std::fill(p->plan_bits.begin(), p->plan_bits.end(), 0);
+    else if (sum_v <= sum_m) std::fill(p->plan_bits.begin(), p->plan_bits.end(), 1);
+    else p->plan_bits = best;
   }
   // all SPLIT chunks of one row take the plan of the row's first chunk
   for (int64_t i = 1; i < n; ++i)

@@ -127,6 +127,7 @@ struct AggArgs {
   int n_items;
   const int64_t* row_ptr;     // [n_rows+1]
   const int32_t* idx;         // gathered row id per position
+  const int32_t* key;         // key (output) vertex per position, GLOBAL id
   const void* table;          // gathered table [.. x ld_tab]
   int64_t ld_tab;
   const float* gscale;        // per gathered row (nullable)
