@@ -203,6 +203,17 @@ wg_status wg_conv_backward(wg_plan p, const wg_params* params, const wg_bwd_args
                            const wg_grads* grads, wg_stream stream);
 
 /* ------------------------------------------------------------------------ */
+/* Training-step utility: fused softmax cross-entropy over the last layer's
+ * logits [M x ld] (C classes): loss_out[0] = scale * sum_r -log softmax(x_r)[label_r],
+ * dlogits = scale * (softmax(x_r) - onehot(label_r)) in the conv dtype
+ * (columns [C, round_up(C, 16 B)) written 0).  Deterministic (fixed-order
+ * block partials).  scratch: WG_XENT_SCRATCH_BYTES of device memory.      */
+#define WG_XENT_SCRATCH_BYTES 8192
+wg_status wg_softmax_xent(wg_dtype dtype, int64_t M, int32_t C, const void* logits, int64_t ld,
+                          const int64_t* labels, float scale, void* dlogits, int64_t ldd, float* loss_out,
+                          void* scratch, wg_stream stream);
+
+/* ------------------------------------------------------------------------ */
 const char* wg_status_string(wg_status s);
 const char* wg_last_error(void);
 /* Number of kernels this library has launched on the calling thread. */

@@ -78,6 +78,20 @@ def launch_count() -> int:
     return int(C.lib().wg_launch_count())
 
 
+_xent_scratch = {}
+
+
+def softmax_xent(logits: torch.Tensor, labels: torch.Tensor, scale: float, dlogits: torch.Tensor,
+                 loss: torch.Tensor, stream=None):
+    """Fused softmax cross-entropy: loss[0] = scale * sum(-log p[label]); dlogits = scale * (p - onehot)."""
+    dev = logits.device
+    if dev not in _xent_scratch:
+        _xent_scratch[dev] = torch.empty(C.XENT_SCRATCH_BYTES, dtype=torch.uint8, device=dev)
+    C.check(C.lib().wg_softmax_xent(_dt(logits.dtype), logits.shape[0], logits.shape[1], _ptr(logits), ld_of(logits),
+                                    _ptr(labels), scale, _ptr(dlogits), ld_of(dlogits), _ptr(loss),
+                                    _ptr(_xent_scratch[dev]), _stream(stream)), "wg_softmax_xent")
+
+
 def profile(cmd: str):
     """'start' | 'stop' | 'collect' -> {kind: {ms, launches, bytes, flops}} (wg_profile)."""
     L = C.lib()

@@ -25,8 +25,9 @@ EXPORTS = [
     "wg_graph_create", "wg_graph_info", "wg_graph_export", "wg_graph_destroy",
     "wg_plan_create", "wg_plan_sizes", "wg_plan_export", "wg_plan_buffer", "wg_plan_destroy",
     "wg_conv_forward", "wg_conv_backward",
-    "wg_status_string", "wg_last_error", "wg_launch_count", "wg_profile",
+    "wg_status_string", "wg_last_error", "wg_launch_count", "wg_profile", "wg_softmax_xent",
 ]
+XENT_SCRATCH_BYTES = 8192
 PROF_KINDS = ["gather_reduce", "split_combine", "tc_gemm_nt", "tc_gemm_tn", "simt_gemm", "misc", "gat", "rgcn"]
 
 P = ctypes.c_void_p
@@ -116,6 +117,8 @@ def lib():
     L.wg_launch_count.argtypes = []
     L.wg_profile.restype = st
     L.wg_profile.argtypes = [ctypes.c_int, P]
+    L.wg_softmax_xent.restype = st
+    L.wg_softmax_xent.argtypes = [ctypes.c_int, i64, i32, P, i64, P, f32, P, i64, P, P, P]
     _lib = L
     return L
 

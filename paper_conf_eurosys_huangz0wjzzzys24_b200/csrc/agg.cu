@@ -281,6 +281,196 @@ __global__ void __launch_bounds__(WARPS * 32, 3) k_agg(AggArgs a, int VPR) {
   }
 }
 
+// ---------------------------------------------------------------------------
+// k_agg_cp: the same warp-segmented reduction, with the gathered rows staged
+// through a per-lane shared-memory ring filled by cp.async (LDGSTS): lane l of
+// a worker copies and later reads only its own 16-byte slices, so no barrier
+// is needed between copy and use, and no register is held per in-flight row.
+// D = NR*RS edges per worker are in flight (NR rounds of RS edges); per SM
+// that is 2 CTAs x 256 lanes x D x 16 B ~ 190 KB, enough to cover HBM latency
+// at full bandwidth (Little's law: 6.5 TB/s x ~2 us / 148 SMs ~ 90 KB).
+// Edge metadata (destination row, source scale) rides in a per-worker ring.
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool pred) {
+  const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
+  const int n = pred ? 16 : 0;
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "r"(n) : "memory");
+}
+__device__ __forceinline__ void cp_async4(void* smem, const void* gmem, bool pred) {
+  const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
+  const int n = pred ? 4 : 0;
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(s), "l"(gmem), "r"(n) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+template <typename T, int LPE, int NV, int RS, int NR>
+__global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
+  constexpr int EPV = VT<T>::EPV;
+  constexpr int G = 32 / LPE;
+  constexpr int W = WARPS * G;
+  constexpr int CW = LPE * NV;
+  constexpr int SLOTF = CW * EPV;
+  constexpr int D = NR * RS;                   // ring depth (edges) per worker
+  static_assert(RS <= LPE, "a round is issued by RS lanes of the worker");
+  extern __shared__ __align__(16) uint8_t smem_cp[];
+  int4* ring = reinterpret_cast<int4*>(smem_cp);                                   // [D][NV][256]
+  float* part_smem = reinterpret_cast<float*>(ring + (size_t)D * NV * WARPS * 32);  // [W][2][SLOTF]
+  int* key_ring = reinterpret_cast<int*>(part_smem + (size_t)W * 2 * SLOTF);       // [W][D]
+  float* sc_ring = reinterpret_cast<float*>(key_ring + W * D);                      // [W][D]
+  __shared__ int slot_row[W][2];
+
+  const WorkItem it = a.items[blockIdx.x];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int grp = lane / LPE, l = lane % LPE, worker = warp * G + grp;
+  const unsigned gmask = LPE == 32 ? 0xffffffffu : (((1u << LPE) - 1u) << (grp * LPE));
+  const bool split = it.split_slot >= 0;
+  const int64_t eb = split ? it.e_lo : a.row_ptr[it.row_lo];
+  const int64_t ee = split ? it.e_hi : a.row_ptr[it.row_hi];
+  const int64_t len = ee - eb;
+  const int64_t cb = eb + len * worker / W, ce = eb + len * (worker + 1) / W;
+  const T* tab = static_cast<const T*>(a.table);
+  const int64_t rb = a.row_base;
+  int* kr = key_ring + worker * D;
+  float* sr = sc_ring + worker * D;
+
+  for (int cv0 = 0; cv0 < VPR; cv0 += CW) {
+    const int nvec = min(CW, VPR - cv0);
+    if (l == 0) { slot_row[worker][0] = -1; slot_row[worker][1] = -1; }
+    if (cb < ce) {
+      // ---- producer state: next round to issue starts at `prod`
+      int64_t prod = cb;
+      int pidx = (prod + l < ce && l < RS) ? a.idx[prod + l] : 0;
+      int round_issued = 0;
+      auto issue = [&]() {
+        const int n = (int)min((int64_t)RS, ce - prod);
+        const int slot0 = (round_issued % NR) * RS;
+#pragma unroll
+        for (int u = 0; u < RS; ++u) {
+          const int s = __shfl_sync(gmask, pidx, u, LPE);
+          const T* row = tab + (int64_t)s * a.ld_tab + (int64_t)cv0 * EPV;
+#pragma unroll
+          for (int q = 0; q < NV; ++q) {
+            const int vi = l + q * LPE;
+            cp_async16(ring + ((size_t)(slot0 + u) * NV + q) * (WARPS * 32) + threadIdx.x, row + vi * EPV,
+                       u < n && vi < nvec);
+          }
+        }
+        if (l < RS) {
+          const bool ok = l < n;
+          if (split) { if (ok) kr[slot0 + l] = (int)(it.row_lo + rb); }
+          else cp_async4(kr + slot0 + l, a.key + (ok ? prod + l : eb), ok);
+          if (a.gscale) cp_async4(sr + slot0 + l, a.gscale + pidx, ok);
+        }
+        cp_async_commit();
+        prod += n;
+        ++round_issued;
+        pidx = (prod + l < ce && l < RS) ? a.idx[prod + l] : 0;
+      };
+#pragma unroll 1
+      for (int r = 0; r < NR; ++r) {
+        if (prod < ce) issue();
+        else { cp_async_commit(); ++round_issued; }
+      }
+      float acc[NV][EPV];
+#pragma unroll
+      for (int q = 0; q < NV; ++q)
+#pragma unroll
+        for (int i = 0; i < EPV; ++i) acc[q][i] = 0.f;
+      int cur = split ? it.row_lo : (int)(a.key[cb] - rb);
+      bool first = true;
+      const bool first_cont = split ? (cb > eb) : (a.row_ptr[cur] < cb);
+      auto flush = [&](int row, bool as_cont, bool as_owner) {
+        if (as_cont || as_owner) {
+          const int s = as_cont ? 0 : 1;
+          float* sp = part_smem + ((size_t)worker * 2 + s) * SLOTF;
+#pragma unroll
+          for (int q = 0; q < NV; ++q)
+#pragma unroll
+            for (int i = 0; i < EPV; ++i) sp[(l + q * LPE) * EPV + i] = acc[q][i];
+          if (l == 0) slot_row[worker][s] = row;
+        } else {
+#pragma unroll
+          for (int q = 0; q < NV; ++q) {
+            const int vi = l + q * LPE;
+            if (vi < nvec) finish_vec<T>(a, acc[q], row, (cv0 + vi) * EPV, split ? it.split_slot : -1);
+          }
+        }
+      };
+      int64_t cons = cb;
+      int round = 0;
+#pragma unroll 1
+      while (cons < ce) {
+        cp_async_wait<NR - 1>();
+        __syncwarp(gmask);
+        const int n = (int)min((int64_t)RS, ce - cons);
+        const int slot0 = (round % NR) * RS;
+#pragma unroll
+        for (int u = 0; u < RS; ++u) {
+          if (u >= n) break;
+          const int rk = split ? it.row_lo : kr[slot0 + u] - (int)rb;
+          const float sc = a.gscale ? sr[slot0 + u] : 1.f;
+          if (rk != cur) {
+            flush(cur, first && first_cont, false);
+            first = false;
+            cur = rk;
+#pragma unroll
+            for (int q = 0; q < NV; ++q)
+#pragma unroll
+              for (int i = 0; i < EPV; ++i) acc[q][i] = 0.f;
+          }
+#pragma unroll
+          for (int q = 0; q < NV; ++q) {
+            const int4 v = ring[((size_t)(slot0 + u) * NV + q) * (WARPS * 32) + threadIdx.x];
+            VT<T>::add(acc[q], v, sc);
+          }
+        }
+        cons += n;
+        ++round;
+        __syncwarp(gmask);
+        if (prod < ce) issue();
+        else { cp_async_commit(); ++round_issued; }
+      }
+      cp_async_wait<0>();
+      const bool last_open = split ? (ce < ee) : (a.row_ptr[cur + 1] > ce);
+      if (first && first_cont) flush(cur, true, false);
+      else flush(cur, false, last_open);
+    }
+    __syncthreads();
+    if (cb < ce && slot_row[worker][1] >= 0) {
+      const int r = slot_row[worker][1];
+      for (int q = 0; q < NV; ++q) {
+        const int vi = l + q * LPE;
+        if (vi >= nvec) continue;
+        float s[EPV];
+        const float* sp = part_smem + ((size_t)worker * 2 + 1) * SLOTF + vi * EPV;
+#pragma unroll
+        for (int i = 0; i < EPV; ++i) s[i] = sp[i];
+        for (int w2 = worker + 1; w2 < W; ++w2) {
+          if (len * w2 / W == len * (w2 + 1) / W) continue;
+          if (slot_row[w2][0] != r) break;
+          const float* sq = part_smem + ((size_t)w2 * 2 + 0) * SLOTF + vi * EPV;
+#pragma unroll
+          for (int i = 0; i < EPV; ++i) s[i] += sq[i];
+        }
+        finish_vec<T>(a, s, r, (cv0 + vi) * EPV, split ? it.split_slot : -1);
+      }
+    }
+    __syncthreads();
+  }
+  if (split) return;
+  for (int r = it.row_lo + warp; r < it.row_hi; r += WARPS) {
+    if (a.row_ptr[r + 1] == a.row_ptr[r]) {
+      const float zero[EPV] = {};
+      for (int vi = lane; vi < VPR; vi += 32) finish_vec<T>(a, zero, r, vi * EPV, -1);
+    }
+    if (a.zero_out) {
+      T* p = static_cast<T*>(a.zero_out) + (int64_t)r * a.ld_zero;
+      for (int c = lane * EPV; c < a.zero_cols; c += 32 * EPV) *reinterpret_cast<int4*>(p + c) = make_int4(0, 0, 0, 0);
+    }
+  }
+}
+
 template <typename T>
 __global__ void k_combine(CombineArgs a, int VPR) {
   constexpr int EPV = VT<T>::EPV;
@@ -322,6 +512,30 @@ wg_status launch_cfg(const AggArgs& a, int VPR, cudaStream_t s) {
   return WG_OK;
 }
 
+template <typename T, int LPE, int NV, int RS, int NR>
+wg_status launch_cp(const AggArgs& a, int VPR, cudaStream_t s) {
+  constexpr int EPV = VT<T>::EPV;
+  constexpr int W = WARPS * (32 / LPE), D = NR * RS;
+  const size_t smem = (size_t)D * NV * WARPS * 32 * 16 + (size_t)W * 2 * LPE * NV * EPV * sizeof(float) +
+                      (size_t)W * D * 8;
+  static bool done = false;
+  if (!done) {
+    cudaFuncSetAttribute(k_agg_cp<T, LPE, NV, RS, NR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    done = true;
+  }
+  WG_LAUNCH((k_agg_cp<T, LPE, NV, RS, NR>), a.n_items, WARPS * 32, smem, s, a, VPR);
+  return WG_OK;
+}
+
+bool use_v2() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("WG_AGG_V2");
+    v = (e && e[0] == '1') ? 1 : 0;
+  }
+  return v == 1;
+}
+
 template <typename T>
 wg_status launch_t(const AggArgs& a, cudaStream_t s) {
   constexpr int EPV = VT<T>::EPV;
@@ -329,11 +543,17 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
   if (VPR <= 1) return launch_cfg<T, 1, 1, 1>(a, VPR, s);
   if (VPR <= 2) return launch_cfg<T, 2, 1, 2>(a, VPR, s);
   if (VPR <= 4) return launch_cfg<T, 4, 1, 4>(a, VPR, s);
-  if (VPR <= 8) return launch_cfg<T, 8, 1, 8>(a, VPR, s);
-  if (VPR <= 16) return launch_cfg<T, 16, 1, 8>(a, VPR, s);
-  if (VPR <= 32) return launch_cfg<T, 32, 1, 8>(a, VPR, s);
-  if (VPR <= 64) return launch_cfg<T, 32, 2, 4>(a, VPR, s);
-  return launch_cfg<T, 32, 4, 2>(a, VPR, s);
+  if (!use_v2()) {
+    if (VPR <= 8) return launch_cp<T, 8, 1, 7, 3>(a, VPR, s);
+    if (VPR <= 16) return launch_cp<T, 16, 1, 7, 3>(a, VPR, s);
+    if (VPR <= 32) return launch_cp<T, 32, 1, 7, 3>(a, VPR, s);
+  } else {
+    if (VPR <= 8) return launch_cfg<T, 8, 1, 4>(a, VPR, s);
+    if (VPR <= 16) return launch_cfg<T, 16, 1, 4>(a, VPR, s);
+    if (VPR <= 32) return launch_cfg<T, 32, 1, 4>(a, VPR, s);
+  }
+  if (VPR <= 64) return launch_cfg<T, 32, 2, 2>(a, VPR, s);
+  return launch_cfg<T, 32, 4, 1>(a, VPR, s);
 }
 
 }  // namespace

@@ -1,0 +1,105 @@
+// Fused softmax cross-entropy (loss + gradient) for the training step: one
+// warp per row, fixed-order block partials for the loss (deterministic).
+#include "wg_internal.cuh"
+
+namespace wg {
+namespace {
+
+constexpr int XENT_BLKS = 1184;   // 8 x 148 SMs; partials fit WG_XENT_SCRATCH_BYTES
+
+template <typename T> __device__ __forceinline__ float ld_f(const T* p) { return (float)*p; }
+template <> __device__ __forceinline__ float ld_f<__nv_bfloat16>(const __nv_bfloat16* p) { return __bfloat162float(*p); }
+
+template <typename T, int PER>
+__global__ void __launch_bounds__(256) k_xent(int64_t M, int C, const T* x, int64_t ld, const int64_t* labels,
+                                              float scale, T* dx, int64_t ldd, float* part, int64_t rows_per_blk) {
+  __shared__ float wsum[8];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t r0 = blockIdx.x * rows_per_blk, r1 = min(M, r0 + rows_per_blk);
+  const int Cpad = (C + 7) / 8 * 8;
+  float lsum = 0.f;
+  for (int64_t r = r0 + warp; r < r1; r += 8) {
+    float v[PER];
+    float m = -INFINITY;
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int j = lane + 32 * k;
+      v[k] = j < C ? ld_f<T>(x + r * ld + j) : -INFINITY;
+      m = fmaxf(m, v[k]);
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    float s = 0.f, t_lab = 0.f;
+    const int64_t lab = labels[r];
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int j = lane + 32 * k;
+      const float t = j < C ? v[k] - m : 0.f;
+      if (j == lab) t_lab = t;
+      v[k] = j < C ? __expf(t) : 0.f;
+      s += v[k];
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const float inv = 1.f / s;
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int j = lane + 32 * k;
+      if (j < Cpad) {
+        const float p = j < C ? v[k] * inv : 0.f;
+        dx[r * ldd + j] = (T)(j < C ? scale * (p - (j == lab ? 1.f : 0.f)) : 0.f);
+        if (j == lab) lsum += scale * (logf(s) - t_lab);
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) lsum += __shfl_xor_sync(0xffffffffu, lsum, o);
+  if (lane == 0) wsum[warp] = lsum;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float t = 0.f;
+    for (int w = 0; w < 8; ++w) t += wsum[w];
+    part[blockIdx.x] = t;
+  }
+}
+
+__global__ void k_sum(const float* part, int n, float* out) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    float t = 0.f;
+    for (int i = 0; i < n; ++i) t += part[i];
+    *out = t;
+  }
+}
+
+template <typename T, int PER>
+wg_status run(int64_t M, int C, const void* x, int64_t ld, const int64_t* labels, float scale, void* dx, int64_t ldd,
+              float* loss, float* part, cudaStream_t s) {
+  const int64_t rpb = std::max<int64_t>(1, cdiv(M, XENT_BLKS));
+  const int nblk = (int)std::max<int64_t>(1, cdiv(M, rpb));
+  WG_LAUNCH((k_xent<T, PER>), nblk, 256, 0, s, M, C, (const T*)x, ld, labels, scale, (T*)dx, ldd, part, rpb);
+  WG_LAUNCH(k_sum, 1, 32, 0, s, part, nblk, loss);
+  return WG_OK;
+}
+
+}  // namespace
+}  // namespace wg
+
+extern "C" wg_status wg_softmax_xent(wg_dtype dtype, int64_t M, int32_t C, const void* logits, int64_t ld,
+                                     const int64_t* labels, float scale, void* dlogits, int64_t ldd, float* loss_out,
+                                     void* scratch, wg_stream stream) {
+  using namespace wg;
+  WG_REQ(logits && labels && dlogits && loss_out && scratch, WG_ERR_INVALID, "wg_softmax_xent: null argument");
+  WG_REQ(C >= 1 && C <= 1024 && ld >= C && ldd >= C, WG_ERR_INVALID, "wg_softmax_xent: C / ld");
+  cudaStream_t s = (cudaStream_t)stream;
+  ProfScope ps(PK_MISC, s, (double)M * C * (dtype == WG_BF16 ? 4.0 : 8.0) + M * 8.0, 0.0);
+  float* part = static_cast<float*>(scratch);
+  const int per = (C + 31) / 32;
+  if (dtype == WG_BF16) {
+    if (per <= 2) return run<__nv_bfloat16, 2>(M, C, logits, ld, labels, scale, dlogits, ldd, loss_out, part, s);
+    if (per <= 8) return run<__nv_bfloat16, 8>(M, C, logits, ld, labels, scale, dlogits, ldd, loss_out, part, s);
+    return run<__nv_bfloat16, 32>(M, C, logits, ld, labels, scale, dlogits, ldd, loss_out, part, s);
+  }
+  if (per <= 2) return run<float, 2>(M, C, logits, ld, labels, scale, dlogits, ldd, loss_out, part, s);
+  if (per <= 8) return run<float, 8>(M, C, logits, ld, labels, scale, dlogits, ldd, loss_out, part, s);
+  return run<float, 32>(M, C, logits, ld, labels, scale, dlogits, ldd, loss_out, part, s);
+}

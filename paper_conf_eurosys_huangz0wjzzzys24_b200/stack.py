@@ -16,9 +16,8 @@ gradients are all-reduced (sum).  Rows >= V in the last block are padding.
 from __future__ import annotations
 
 import torch
-import torch.nn.functional as F
 
-from . import Conv, Graph, init_params, padded, pitch
+from . import Conv, Graph, init_params, padded, pitch, softmax_xent
 from . import _capi as C
 
 
@@ -129,17 +128,16 @@ class GNNStack:
     def step(self, x, labels, n_global: int):
         """One epoch step: forward, CE loss (mean over all vertices), backward, Adam."""
         logits = self.forward(x)
-        lf = logits.float().detach().requires_grad_(True)
-        loss = F.cross_entropy(lf, labels, reduction="sum") / n_global
-        loss.backward()
-        dl = padded(self.rows, logits.shape[1], self.dtype, self.dev, zero=False)
-        dl.copy_(lf.grad)
-        self.backward(dl)
+        if not hasattr(self, "_dl"):
+            self._dl = padded(self.rows, logits.shape[1], self.dtype, self.dev, zero=True)
+            self._loss = torch.zeros(1, dtype=torch.float32, device=self.dev)
+        softmax_xent(logits, labels, 1.0 / n_global, self._dl, self._loss)
+        self.backward(self._dl)
         for p, gr in zip(self.params, self.grads):
             for k, v in p.items():
                 v.grad = gr[k]
         self.opt.step()
-        return loss.detach()
+        return self._loss
 
 
 def partition_1d(V: int, world: int, T: int = 128):

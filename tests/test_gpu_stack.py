@@ -1,0 +1,118 @@
+"""Multi-layer / multi-partition paths on one GPU.
+
+* the fused softmax cross-entropy against its definition (numpy, fp64);
+* the 1-D partition simulated on one GPU: P rank-partitions
+  share one exchange table (each PRE phase writes its own rows, so the
+  all-gather is implicit), then every POST phase runs; the concatenated rank
+  outputs and the summed weight gradients must equal the single-partition
+  layer (and hence the oracle, tested elsewhere);
+* a short training run of GNNStack decreases the loss.
+"""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from tests.util import f64, rel_err
+
+pytestmark = pytest.mark.gpu
+
+
+def wg():
+    import paper_conf_eurosys_huangz0wjzzzys24_b200 as m
+    return m
+
+
+@pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
+@pytest.mark.parametrize("C", [7, 47, 172])
+def test_softmax_xent(dtype, C):
+    m = wg()
+    M = 5000
+    x = torch.from_numpy(synth.normal((M, C), seed=C, std=3.0)).to(dtype)
+    lab = torch.from_numpy(np.random.default_rng(C).integers(0, C, M)).cuda()
+    xd = m.pad_to(x.cuda())
+    dl = m.padded(M, C, dtype)
+    loss = torch.zeros(1, device="cuda")
+    m.softmax_xent(xd, lab, 1.0 / M, dl, loss)
+    xo = f64(x)
+    p = np.exp(xo - xo.max(1, keepdims=True))
+    p /= p.sum(1, keepdims=True)
+    onehot = np.zeros_like(p)
+    onehot[np.arange(M), lab.cpu().numpy()] = 1
+    ref_loss = -np.log(p[np.arange(M), lab.cpu().numpy()]).sum() / M
+    tol = 1e-4 if dtype == torch.float32 else 2e-2
+    assert abs(loss.item() - ref_loss) / abs(ref_loss) < 1e-4
+    assert rel_err(f64(dl), (p - onehot) / M) < tol
+
+
+@pytest.mark.parametrize("model,policy", [("sage", "edge"), ("sage", "vertex"), ("gcn", "edge"), ("gin", "vertex")])
+@pytest.mark.parametrize("P", [2, 3])
+def test_1d_partition_phases_match_single(model, policy, P):
+    m = wg()
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import partition_1d
+    V, E, fi, fo = 3000, 40000, 48, 40
+    dtype = torch.float32
+    src, dst, _ = synth.make_graph(V, E, seed=31, alpha=0.6)
+    x = torch.from_numpy(synth.make_features(V, fi, seed=32)).cuda()
+    dy = torch.from_numpy(synth.normal((V, fo), seed=33, std=0.2)).cuda()
+    params = m.init_params(model, fi, fo, seed=3)
+    ts, td = torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda()
+    # single partition reference (through the same library)
+    g1 = m.Graph(ts, td, num_vertices=V)
+    c1 = m.Conv(g1, model, fi, fo, dtype=dtype, policy=policy, fuse_relu=True)
+    xd = m.pad_to(x)
+    y1, s1 = c1.forward_raw(xd, params)
+    dx1, gr1 = c1.backward_raw(m.pad_to(dy), xd, y1, s1, params)
+    # P rank-partitions sharing one exchange table
+    block, bounds = partition_1d(V, P)
+    Vt = block * P
+    xt = m.padded(Vt, fi, dtype)
+    xt[:V] = x
+    ranks = []
+    for p in range(P):
+        vb, ve = bounds[p]
+        g = m.Graph(ts, td, num_vertices=V, v_begin=vb, v_end=ve)
+        c = m.Conv(g, model, fi, fo, dtype=dtype, policy=policy, fuse_relu=True)
+        ranks.append((g, c, vb, ve))
+    wf = m.pitch(fo, dtype)
+    xf = m.padded(Vt, wf, dtype) if ranks[0][1].n_vertex_tasks else None
+    yt = m.padded(Vt, fo, dtype)
+    saved = [c.new_saved() for _, c, _, _ in ranks]
+    for ph in (1, 2):
+        for (g, c, vb, ve), sv in zip(ranks, saved):
+            if xf is None and ph == 1:
+                continue
+            c.forward_raw(xt, params, y=yt[vb:ve], saved=sv, phase=ph if xf is not None else 0, xchg=xf)
+    np.testing.assert_allclose(f64(yt[:V]), f64(y1), rtol=0, atol=1e-5 * max(1.0, f64(y1).max()))
+    # backward: dy rows per rank, exchange table of dAgg (dAgg path) or dT (G path)
+    bw = ranks[0][1]
+    wb = m.pitch(fi if bw.bwd_path == 0 else fo, dtype)
+    xb = m.padded(Vt, wb, dtype)
+    dyt = m.padded(Vt, fo, dtype)
+    dyt[:V] = dy
+    dxt = m.padded(Vt, fi, dtype)
+    grads = []
+    for ph in (1, 2):
+        for i, ((g, c, vb, ve), sv) in enumerate(zip(ranks, saved)):
+            if ph == 1:
+                grads.append({k: torch.zeros_like(v) for k, v in params.items()})
+            c.backward_raw(dyt[vb:ve], xt, yt[vb:ve], sv, params, dx=dxt[vb:ve], phase=ph, xchg=xb, grads=grads[i])
+    assert rel_err(f64(dxt[:V]), f64(dx1)) < 1e-5
+    for k in gr1:
+        tot = sum(gr[k] for gr in grads)
+        assert rel_err(f64(tot), f64(gr1[k])) < 1e-5, k
+
+
+def test_stack_training_decreases_loss():
+    m = wg()
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack
+    V, E = 4000, 60000
+    src, dst, _ = synth.make_graph(V, E, seed=41, alpha=0.5, symmetric=True)
+    g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V)
+    dims = [32, 64, 64, 8]
+    st = GNNStack(g, "sage", dims, dtype=torch.bfloat16, lr=1e-2)
+    x = m.padded(V, 32, torch.bfloat16)
+    x.copy_(torch.from_numpy(synth.make_features(V, 32, seed=42)))
+    labels = torch.from_numpy(np.random.default_rng(1).integers(0, 8, V)).cuda()
+    losses = [float(st.step(x, labels, V).item()) for _ in range(30)]
+    assert losses[-1] < losses[0] * 0.9, losses
