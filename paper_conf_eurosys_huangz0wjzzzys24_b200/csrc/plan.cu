@@ -252,6 +252,7 @@ wg_status wg_plan_destroy(wg_plan p) {
   cudaSetDevice(p->g->device);
   cudaDeviceSynchronize();
   if (p->rg) wg::rgcn_plan_free(p);
+  if (p->gat) wg::gat_plan_free(p);
   for (void* q : p->allocs) cudaFree(q);
   p->g->live_plans--;
   delete p;

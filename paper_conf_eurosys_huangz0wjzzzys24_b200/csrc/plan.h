@@ -47,8 +47,9 @@ struct wg_plan_s {
   int64_t pi = 0, po = 0;            // row pitches (elements) of f_in / f_out wide tensors
   wg::Layout saved, ws;
   std::vector<void*> allocs;
-  // RGCN structures (rgcn.cu)
+  // model-specific structures (conv_rgcn.cu / conv_gat.cu)
   void* rg = nullptr;
+  void* gat = nullptr;
 };
 
 namespace wg {
@@ -61,5 +62,6 @@ wg_status gat_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, c
 wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* a, cudaStream_t s);
 wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, const wg_grads* G, cudaStream_t s);
 void gat_layout(wg_plan_s* p);
+void gat_plan_free(wg_plan_s* p);
 void lin_layout(wg_plan_s* p);
 }  // namespace wg
