@@ -415,9 +415,12 @@ __global__ void k_gat_der(int64_t rows, int64_t row_base, const int64_t* row_ptr
 }
 
 // dG = dg + del a_l + der a_r (conv dtype, GEMM operand); da_l / da_r block partials
+// dG is written as hi (+ lo residual for bf16: dG = hi + lo to ~16 mantissa
+// bits) so the GEMMs that consume it keep the cancellation in dg + del a_l +
+// der a_r accurate.
 template <typename T>
 __global__ void k_gat_dG(int64_t rows, int64_t row_base, GatArgs a, const float* al, const float* ar,
-                         const float* der, T* dG, int64_t ld_dG, float* part, int64_t rows_per_blk) {
+                         const float* der, T* dG, T* dGlo, int64_t ld_dG, float* part, int64_t rows_per_blk) {
   // thread per column c (HF <= 1024), rows of this block
   const int64_t r0 = blockIdx.x * rows_per_blk, r1 = min(rows, r0 + rows_per_blk);
   const T* G = static_cast<const T*>(a.G);
@@ -427,7 +430,10 @@ __global__ void k_gat_dG(int64_t rows, int64_t row_base, GatArgs a, const float*
     for (int64_t r = r0; r < r1; ++r) {
       const int64_t v = row_base + r;
       const float dlv = a.del[v * a.H + h], drv = der[v * a.H + h];
-      dG[r * ld_dG + c] = (T)(a.dg[v * a.ld_dg + c] + dlv * al[c] + drv * ar[c]);
+      const float val = a.dg[v * a.ld_dg + c] + dlv * al[c] + drv * ar[c];
+      const T hi = (T)val;
+      dG[r * ld_dG + c] = hi;
+      if (dGlo) dGlo[r * ld_dG + c] = (T)(val - (float)hi);
       const float g = (float)G[v * a.ldg + c];
       sl += dlv * g;
       sr += drv * g;
@@ -501,6 +507,7 @@ void gat_layout(wg_plan_s* p) {
   W.add("der", sizeof(float) * V * H);
   W.add("dg", sizeof(float) * V * HF);
   W.add("dG", (size_t)nr * p->po * s);
+  W.add("dGlo", (size_t)nr * p->po * s);
   W.add("dyt", (size_t)nr * p->po * s);
   W.add("colsum", bias_grad_scratch(nr, (int)HF));
   W.add("dgp", sizeof(float) * DG_BLKS * 2 * HF);
@@ -617,22 +624,27 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
   float* der = L.at<float>(ws, "der");
   WG_LAUNCH(k_gat_der, (unsigned)cdiv(nr * 32, 256), 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, H, der);
   void* dG = L.at<void>(ws, "dG");
+  void* dGlo = d.dtype == WG_BF16 ? L.at<void>(ws, "dGlo") : nullptr;
   const int64_t rpb = std::max<int64_t>(1, cdiv(nr, DG_BLKS));
   const int nblk = (int)cdiv(nr, rpb);
   float* dgp = L.at<float>(ws, "dgp");
-  WG_LAUNCH(k_gat_dG<T>, nblk, 256, 0, st, nr, vb, a, P->attn_l, P->attn_r, der, (T*)dG, p->po, dgp, rpb);
+  WG_LAUNCH(k_gat_dG<T>, nblk, 256, 0, st, nr, vb, a, P->attn_l, P->attn_r, der, (T*)dG, (T*)dGlo, p->po, dgp,
+            rpb);
   WG_LAUNCH(k_pair_reduce, (unsigned)cdiv(2 * HF, 128), 128, 0, st, dgp, nblk, HF, Gr ? Gr->attn_l : nullptr,
             Gr ? Gr->attn_r : nullptr);
-  // dW = x^T dG ; dx = dG W^T
-  if (Gr && Gr->W)
+  // dW = x^T dG ; dx = dG W^T   (dG = hi + lo for bf16)
+  if (Gr && Gr->W) {
     WG_TRY(gemm_tn(d.dtype, nr, d.f_in, HF, A->x, A->ldx, dG, p->po, Gr->W, L.at<void>(ws, "tn"), st));
+    if (dGlo) WG_TRY(gemm_tn(d.dtype, nr, d.f_in, HF, A->x, A->ldx, dGlo, p->po, Gr->W, L.at<void>(ws, "tn"), st, 1));
+  }
   if (d.need_dx) {
     void* w = L.at<void>(ws, "w");
     WG_TRY(prep_weight(d.dtype, P->W, d.f_in, HF, 0, w, p->po, (int)rup(d.f_in, 16), st));
-    GemmPart part{dG, p->po, w, p->po, HF, (int)rup(d.f_in, 16)};
+    GemmPart parts[2] = {GemmPart{dG, p->po, w, p->po, HF, (int)rup(d.f_in, 16)},
+                         GemmPart{dGlo, p->po, w, p->po, HF, (int)rup(d.f_in, 16)}};
     GemmEpi e;
     e.D = A->dx; e.ldd = A->lddx;
-    WG_TRY(gemm_nt(d.dtype, nr, (int)rup(d.f_in, 16 / s), &part, 1, e, nullptr, 0, st));
+    WG_TRY(gemm_nt(d.dtype, nr, (int)rup(d.f_in, 16 / s), parts, dGlo ? 2 : 1, e, nullptr, 0, st));
   }
   return WG_OK;
 }

@@ -10,7 +10,7 @@ namespace wg {
 bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi,
                 cudaStream_t s, wg_status* st);
 bool tc_gemm_tn(int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb, float* D,
-                float* part, cudaStream_t s, wg_status* st);
+                float* part, cudaStream_t s, wg_status* st, int acc);
 
 namespace {
 
@@ -126,12 +126,12 @@ __global__ void __launch_bounds__(256) k_gemm_tn(int64_t K, int M, int N, const 
   }
 }
 
-__global__ void k_split_reduce(const float* part, int splits, int64_t MN, float* D) {
+__global__ void k_split_reduce(const float* part, int splits, int64_t MN, float* D, int acc) {
   int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= MN) return;
   float s = 0.f;
   for (int z = 0; z < splits; ++z) s += part[z * MN + i];
-  D[i] = s;
+  D[i] = acc ? D[i] + s : s;
 }
 
 int tn_splits(int64_t K, int M, int N) {
@@ -167,13 +167,16 @@ size_t gemm_tn_scratch(int64_t K, int M, int N) {
 }
 
 wg_status gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb,
-                  float* D, void* scratch, cudaStream_t s) {
+                  float* D, void* scratch, cudaStream_t s, int acc) {
   if (M == 0 || N == 0) return WG_OK;
-  if (K == 0) { WG_CK(cudaMemsetAsync(D, 0, sizeof(float) * M * N, s)); return WG_OK; }
+  if (K == 0) {
+    if (!acc) WG_CK(cudaMemsetAsync(D, 0, sizeof(float) * M * N, s));
+    return WG_OK;
+  }
   float* part = static_cast<float*>(scratch);
   int splits = tn_splits(K, M, N);
   wg_status st = WG_OK;
-  if (dt == WG_BF16 && tc_gemm_tn(K, M, N, A, lda, B, ldb, D, part, s, &st)) return st;
+  if (dt == WG_BF16 && tc_gemm_tn(K, M, N, A, lda, B, ldb, D, part, s, &st, acc)) return st;
   const int64_t kchunk = rup(cdiv(K, splits), BK);
   splits = (int)cdiv(K, kchunk);
   ProfScope ps(PK_SIMT, s, (double)K * (M + N) * (dt == WG_BF16 ? 2.0 : 4.0), 2.0 * K * M * N);
@@ -184,7 +187,7 @@ wg_status gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t l
   else
     WG_LAUNCH(k_gemm_tn<float>, grid, 256, 0, s, K, M, N, (const float*)A, lda, (const float*)B, ldb, part, kchunk);
   const int64_t MN = (int64_t)M * N;
-  WG_LAUNCH(k_split_reduce, (unsigned)cdiv(MN, 256), 256, 0, s, part, splits, MN, D);
+  WG_LAUNCH(k_split_reduce, (unsigned)cdiv(MN, 256), 256, 0, s, part, splits, MN, D, acc);
   return WG_OK;
 }
 

@@ -290,12 +290,12 @@ __global__ void __launch_bounds__(128, 1)
   if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(tcols));
 }
 
-__global__ void k_split_reduce_tc(const float* part, int splits, int64_t MN, float* D) {
+__global__ void k_split_reduce_tc(const float* part, int splits, int64_t MN, float* D, int acc) {
   int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= MN) return;
   float s = 0.f;
   for (int z = 0; z < splits; ++z) s += part[z * MN + i];
-  D[i] = s;
+  D[i] = acc ? D[i] + s : s;
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
@@ -385,7 +385,7 @@ bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_part
 }
 
 bool tc_gemm_tn(int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb, float* D,
-                float* part, cudaStream_t s, wg_status* st) {
+                float* part, cudaStream_t s, wg_status* st, int acc) {
   if (!tc_enabled() || K <= 0) return false;
   const int n_tiles = (int)cdiv(N, 256);
   const int BN = (int)rup(cdiv(N, n_tiles), 16);
@@ -414,7 +414,7 @@ bool tc_gemm_tn(int64_t K, int M, int N, const void* A, int64_t lda, const void*
   if (*st != WG_OK) return true;
   const int64_t MN = (int64_t)M * N;
   cudaStream_t ss = s;
-  k_split_reduce_tc<<<(unsigned)cdiv(MN, 256), 256, 0, ss>>>(part, (int)splits, MN, D);
+  k_split_reduce_tc<<<(unsigned)cdiv(MN, 256), 256, 0, ss>>>(part, (int)splits, MN, D, acc);
   ++launch_counter();
   if (cudaGetLastError() != cudaSuccess) *st = WG_ERR_CUDA;
   return true;

@@ -200,8 +200,9 @@ wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_pa
                   const GemmEpi& epi, void* scratch, size_t scratch_bytes, cudaStream_t s);
 // dW[M x N] (fp32, exact shape, ld = N) = A[K x M]^T * B[K x N] (split-K, deterministic)
 size_t gemm_tn_scratch(int64_t K, int M, int N);
+// acc != 0: D += A^T B (fixed order: the previous D is added after the split sums)
 wg_status gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda,
-                  const void* B, int64_t ldb, float* D, void* scratch, cudaStream_t s);
+                  const void* B, int64_t ldb, float* D, void* scratch, cudaStream_t s, int acc = 0);
 
 // weight prep: fp32 [rows x cols] -> dtype, optionally transposed, into [out_rows x ldo]
 wg_status prep_weight(wg_dtype dt, const float* W, int rows, int cols, int transpose,
