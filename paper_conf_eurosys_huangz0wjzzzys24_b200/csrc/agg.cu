@@ -169,6 +169,7 @@ __global__ void __launch_bounds__(WARPS * 32, 3) k_agg(AggArgs a, int VPR) {
         my_idx = a.idx[pos + l];
         my_key = split ? it.row_lo : (int)(key[pos + l] - rb);
         if (a.gscale) my_sc = a.gscale[my_idx];
+        else if (a.escale) my_sc = a.escale[pos + l];
       }
       auto flush = [&](int row, bool as_cont, bool as_owner) {
         // as_cont: continuation partial (slot 0); as_owner: owner partial (slot 1); else final
@@ -198,6 +199,7 @@ __global__ void __launch_bounds__(WARPS * 32, 3) k_agg(AggArgs a, int VPR) {
           nx_idx = a.idx[np];
           nx_key = split ? it.row_lo : (int)(key[np] - rb);
           if (a.gscale) nx_sc = a.gscale[nx_idx];
+          else if (a.escale) nx_sc = a.escale[np];
         }
         for (int j = 0; j < n; j += U) {
           int4 v[U][NV];
@@ -361,6 +363,7 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
           if (split) { if (ok) kr[slot0 + l] = (int)(it.row_lo + rb); }
           else cp_async4(kr + slot0 + l, a.key + (ok ? prod + l : eb), ok);
           if (a.gscale) cp_async4(sr + slot0 + l, a.gscale + pidx, ok);
+          else if (a.escale) cp_async4(sr + slot0 + l, a.escale + (ok ? prod + l : eb), ok);
         }
         cp_async_commit();
         prod += n;
@@ -409,7 +412,7 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
         for (int u = 0; u < RS; ++u) {
           if (u >= n) break;
           const int rk = split ? it.row_lo : kr[slot0 + u] - (int)rb;
-          const float sc = a.gscale ? sr[slot0 + u] : 1.f;
+          const float sc = (a.gscale || a.escale) ? sr[slot0 + u] : 1.f;
           if (rk != cur) {
             flush(cur, first && first_cont, false);
             first = false;
@@ -565,7 +568,7 @@ wg_status launch_agg(wg_dtype dt, const AggArgs& a, cudaStream_t s) {
   // and the source scale if any; per row the output, row_ptr and optional
   // self / mask rows
   const double es = dt == WG_BF16 ? 2.0 : 4.0, rb = a.F * es;
-  const double bytes = a.n_edges * (4.0 + rb + (a.gscale ? 4.0 : 0.0)) +
+  const double bytes = a.n_edges * (4.0 + rb + (a.gscale || a.escale ? 4.0 : 0.0)) +
                        a.n_rows * (rb + 8.0 + (a.self_tab ? rb : 0.0) + (a.mask_ref ? rb : 0.0) +
                                    (a.zero_out ? a.zero_cols * es : 0.0));
   ProfScope ps(PK_AGG, s, bytes, 2.0 * a.n_edges * a.F);
@@ -659,6 +662,15 @@ wg_status prep_weight(wg_dtype dt, const float* W, int rows, int cols, int trans
     WG_LAUNCH(k_prep_weight<__nv_bfloat16>, grid, 256, 0, s, W, rows, cols, transpose, (__nv_bfloat16*)out, ldo, out_rows);
   else
     WG_LAUNCH(k_prep_weight<float>, grid, 256, 0, s, W, rows, cols, transpose, (float*)out, ldo, out_rows);
+  return WG_OK;
+}
+
+wg_status prep_weight_batched(wg_dtype dt, const float* W, int batch, int rows, int cols, int transpose, void* out,
+                              int64_t ldo, int out_rows, cudaStream_t s) {
+  const int es = dt == WG_BF16 ? 2 : 4;
+  for (int b = 0; b < batch; ++b)
+    WG_TRY(prep_weight(dt, W + (int64_t)b * rows * cols, rows, cols, transpose,
+                       static_cast<char*>(out) + (int64_t)b * out_rows * ldo * es, ldo, out_rows, s));
   return WG_OK;
 }
 

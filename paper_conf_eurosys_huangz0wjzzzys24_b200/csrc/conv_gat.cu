@@ -222,7 +222,9 @@ __global__ void __launch_bounds__(256) k_gat_fwd(GatArgs a, int64_t row_base) {
       const float inv = l[q] > 0.f ? 1.f / l[q] : 0.f;
 #pragma unroll
       for (int i = 0; i < EPV; ++i) o[i] = (c0 + i < a.HF) ? acc[q][i] * inv : 0.f;
-      *reinterpret_cast<int4*>(static_cast<T*>(a.agg) + (int64_t)ch.row * a.ld_agg + c0) = GV<T>::pack(o);
+      float* ag = static_cast<float*>(a.agg) + (int64_t)ch.row * a.ld_agg + c0;
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) ag[i] = o[i];
       if (head_lead) { a.m[d * a.H + hd[q]] = m[q]; a.l[d * a.H + hd[q]] = l[q]; }
     }
   }
@@ -248,7 +250,7 @@ __global__ void k_gat_fwd_combine(GatArgs a, const SplitRow* rows, int64_t row_b
       m = mn;
     }
     const float val = (c < a.HF && l > 0.f) ? o / l : 0.f;
-    static_cast<T*>(a.agg)[(int64_t)sr.row * a.ld_agg + c] = (T)val;
+    static_cast<float*>(a.agg)[(int64_t)sr.row * a.ld_agg + c] = val;
     if (c < a.HF && c % a.Fo == 0) { a.m[d * a.H + h] = m; a.l[d * a.H + h] = l; }
   }
 }
@@ -262,8 +264,8 @@ __global__ void k_gat_out(int64_t rows, GatArgs a, const float* bias, int relu, 
     const int c = (int)(t % ldy);
     float v = 0.f;
     if (c < FO) {
-      const T* ag = static_cast<const T*>(a.agg) + r * a.ld_agg;
-      if (a.concat) v = (float)ag[c];
+      const float* ag = static_cast<const float*>(a.agg) + r * a.ld_agg;
+      if (a.concat) v = ag[c];
       else {
         for (int h = 0; h < a.H; ++h) v += (float)ag[h * a.Fo + c];
         v /= (float)a.H;
@@ -281,7 +283,7 @@ __global__ void k_gat_s(int64_t rows, int64_t row_base, GatArgs a, float* s) {
   const int lane = threadIdx.x & 31;
   const int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (r >= rows) return;
-  const T* ag = static_cast<const T*>(a.agg) + r * a.ld_agg;
+  const float* ag = static_cast<const float*>(a.agg) + r * a.ld_agg;
   const T* dy = static_cast<const T*>(a.dy) + r * a.lddy;
   for (int h = 0; h < a.H; ++h) {
     float acc = 0.f;
@@ -493,7 +495,7 @@ void gat_layout(wg_plan_s* p) {
   S = Layout();
   W = Layout();
   S.add("G", (size_t)V * p->po * s);
-  S.add("agg", (size_t)nr * p->po * s);
+  S.add("agg", sizeof(float) * (size_t)nr * rup(HF, 4));   // fp32: s = dy.agg feeds a cancellation (dt)
   S.add("el", sizeof(float) * V * H);
   S.add("er", sizeof(float) * V * H);
   S.add("m", sizeof(float) * V * H);
@@ -538,7 +540,7 @@ static wg_status gat_fwd_t(wg_plan_s* p, const wg_params* P, const wg_fwd_args* 
   a.G = S.at<void>(A->saved, "G"); a.ldg = p->po;
   a.el = S.at<float>(A->saved, "el"); a.er = S.at<float>(A->saved, "er");
   a.m = S.at<float>(A->saved, "m"); a.l = S.at<float>(A->saved, "l");
-  a.agg = S.at<void>(A->saved, "agg"); a.ld_agg = p->po;
+  a.agg = S.at<void>(A->saved, "agg"); a.ld_agg = rup(HF, 4);
   a.part = L.at<float>(ws, "part"); a.part_ld = HF + 2 * H + 8;
   a.concat = d.concat_heads;
   // G = x W  (vertex-level transform, tcgen05 for bf16)
@@ -590,7 +592,7 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
   a.G = S.at<void>(A->saved, "G"); a.ldg = p->po;
   a.el = S.at<float>(A->saved, "el"); a.er = S.at<float>(A->saved, "er");
   a.m = S.at<float>(A->saved, "m"); a.l = S.at<float>(A->saved, "l");
-  a.agg = S.at<void>(A->saved, "agg"); a.ld_agg = p->po;
+  a.agg = S.at<void>(A->saved, "agg"); a.ld_agg = rup(HF, 4);
   a.part = L.at<float>(ws, "part"); a.part_ld = HF + 2 * H + 8;
   a.concat = d.concat_heads;
   // dT = dy (masked by the fused ReLU) ; db

@@ -1,10 +1,554 @@
-// RGCN layer (placeholder: implemented in a later milestone).
+// RGCN layer, Eq. (1): h^{l+1}[e.dst] += MLP(h^l[e.src], W^l[e.type]),
+// Schlichtkrull et al. [34] (readings Q2): optional c_e = 1/|in_r(v)|,
+// self-loop W_0 and bias.
+//
+// gTasks are (destination tile x relation) blocks (Fig 7(c)(d)).
+// Per gTask the plan (a4) chooses:
+//   EDGE   (gather-then-transform): one stage-1 row per (dst, relation)
+//          segment, S = sum_e c_e x[src_e]; the row is transformed by W_r and
+//          contributes once to y[dst];
+//   VERTEX (transform-before-gather): one stage-1 row per unique source of the
+//          gTask (T1 unique extraction: src-id_unique / src-id_map),
+//          transformed once by W_r (T2 indexing swapping, Index-2D A[B] x C[D] =
+//          (A x C)[B, D]); every edge contributes c_e Y[map(e)].
+// Stage-1 rows of all gTasks are laid out grouped by relation (each group padded
+// to 128 rows), so one grouped GEMM applies W_r to every row of group r
+// ("a batch of K src rows becomes a matrix-matrix product");
+// stage 3 is the contribution-list gather-reduce into destination rows.
+// Backward mirrors this on the transposed partition (source tile x relation):
+// G = sum over (src, relation) segments of c_e dy[dst], dX = G W_r^T (grouped),
+// dx = sum over a source's segments; dW_r = X_g^T G over group r.
+// Round-1 scope: unfused (stage buffers round-trip HBM); DESIGN.md "RGCN".
+#include <algorithm>
+#include <numeric>
+#include <random>
+
 #include "plan.h"
+
 namespace wg {
-wg_status rgcn_plan(wg_plan_s*, cudaStream_t) { set_error("RGCN not implemented yet"); return WG_ERR_UNSUPPORTED; }
-void rgcn_plan_free(wg_plan_s*) {}
-wg_status rgcn_forward(wg_plan_s*, const wg_params*, const wg_fwd_args*, cudaStream_t) { return WG_ERR_UNSUPPORTED; }
-wg_status rgcn_backward(wg_plan_s*, const wg_params*, const wg_bwd_args*, const wg_grads*, cudaStream_t) {
-  return WG_ERR_UNSUPPORTED;
+
+namespace {
+
+constexpr int TILE_M = 128;
+
+struct CsrExec {
+  int64_t rows = 0, nnz = 0;
+  int64_t* row_ptr = nullptr;
+  int32_t* idx = nullptr;
+  int32_t* key = nullptr;
+  float* escale = nullptr;
+  float* rscale = nullptr;
+  ItemList items;
+  int n_slots = 0;
+};
+
+struct RgcnPlan {
+  int R = 1;
+  int64_t n1 = 0, n1T = 0;           // stage-1 typed rows (padded), forward / transposed
+  CsrExec f1, f3, b1, b3, bg;
+  int32_t* tile_type = nullptr;      // [n1 / 128]
+  int32_t* tile_typeT = nullptr;     // [n1T / 128]
+  int64_t* group_offT = nullptr;     // device [R+1] transposed group row offsets
+  std::vector<int64_t> h_group_offT;
+};
+
+template <typename T>
+wg_status up(wg_plan_s* p, const std::vector<T>& h, T** d) {
+  *d = nullptr;
+  if (h.empty()) return WG_OK;
+  void* q = nullptr;
+  WG_CK(cudaMalloc(&q, sizeof(T) * h.size()));
+  p->allocs.push_back(q);
+  WG_CK(cudaMemcpy(q, h.data(), sizeof(T) * h.size(), cudaMemcpyHostToDevice));
+  *d = static_cast<T*>(q);
+  return WG_OK;
 }
+
+// Work items over a generic CSR: consecutive rows grouped until E_max entries
+// or 128 rows; rows with more than E_max entries become SPLIT chunks.
+wg_status build_exec(wg_plan_s* p, const std::vector<int64_t>& rp, const std::vector<int32_t>& idx,
+                     const std::vector<float>* es, const std::vector<float>* rs, int64_t E_max, CsrExec* X) {
+  X->rows = (int64_t)rp.size() - 1;
+  X->nnz = rp.back();
+  std::vector<int32_t> key(X->nnz);
+  for (int64_t r = 0; r < X->rows; ++r)
+    for (int64_t e = rp[r]; e < rp[r + 1]; ++e) key[e] = (int32_t)r;
+  WG_TRY(up(p, rp, &X->row_ptr));
+  WG_TRY(up(p, idx, &X->idx));
+  WG_TRY(up(p, key, &X->key));
+  if (es) WG_TRY(up(p, *es, &X->escale));
+  if (rs) WG_TRY(up(p, *rs, &X->rscale));
+  std::vector<std::pair<int64_t, WorkItem>> L;
+  int slot = 0;
+  ItemList& IL = X->items;
+  int64_t lo = 0;
+  auto close = [&](int64_t hi) {
+    if (hi <= lo) return;
+    WorkItem w{};
+    w.row_lo = (int32_t)lo; w.row_hi = (int32_t)hi; w.e_lo = rp[lo]; w.e_hi = rp[hi];
+    w.split_slot = -1; w.task = -1;
+    L.push_back({w.e_hi - w.e_lo, w});
+    IL.n_edges += w.e_hi - w.e_lo;
+    IL.n_rows += hi - lo;
+  };
+  for (int64_t r = 0; r < X->rows; ++r) {
+    const int64_t deg = rp[r + 1] - rp[r];
+    if (deg > E_max) {
+      close(r);
+      IL.hs.push_back(SplitRow{(int32_t)r, slot, 0, 0});
+      for (int64_t c = rp[r]; c < rp[r + 1]; c += E_max) {
+        WorkItem w{};
+        w.row_lo = (int32_t)r; w.row_hi = (int32_t)r + 1; w.e_lo = c; w.e_hi = std::min(c + E_max, rp[r + 1]);
+        w.split_slot = slot++; w.task = -1;
+        L.push_back({INT64_MAX / 2 + (w.e_hi - w.e_lo), w});
+        IL.hs.back().n_slots++;
+        IL.n_edges += w.e_hi - w.e_lo;
+      }
+      lo = r + 1;
+      continue;
+    }
+    if (rp[r + 1] - rp[lo] > E_max || r - lo >= 128) {
+      close(r);
+      lo = r;
+    }
+  }
+  close(X->rows);
+  std::stable_sort(L.begin(), L.end(), [](const auto& a, const auto& b) { return a.first > b.first; });
+  for (auto& e : L) IL.h.push_back(e.second);
+  IL.n = (int)IL.h.size();
+  IL.n_split = (int)IL.hs.size();
+  WG_TRY(up(p, IL.h, &IL.d));
+  WG_TRY(up(p, IL.hs, &IL.split));
+  X->n_slots = slot;
+  return WG_OK;
+}
+
+template <typename T>
+wg_status down(const T* d, int64_t n, std::vector<T>& h) {
+  h.resize(n);
+  if (n) WG_CK(cudaMemcpy(h.data(), d, sizeof(T) * n, cudaMemcpyDeviceToHost));
+  return WG_OK;
+}
+
+AggArgs exec_args(const CsrExec& X, int64_t E_max) {
+  AggArgs a{};
+  a.items = X.items.d;
+  a.n_items = X.items.n;
+  a.row_ptr = X.row_ptr;
+  a.idx = X.idx;
+  a.key = X.key;
+  a.escale = X.escale;
+  a.rscale = X.rscale;
+  a.row_base = 0;
+  a.self_coef = 1.f;
+  a.E_max = E_max;
+  a.n_edges = X.items.n_edges;
+  a.n_rows = X.items.n_rows;
+  return a;
+}
+
+CombineArgs comb(const AggArgs& a, const CsrExec& X) {
+  CombineArgs b{};
+  b.rows = X.items.split; b.n_rows = X.items.n_split;
+  b.partial = a.partial; b.ld_part = a.ld_part;
+  b.rscale = a.rscale; b.row_base = a.row_base;
+  b.self_tab = a.self_tab; b.ld_self = a.ld_self; b.self_coef = a.self_coef;
+  b.bias = a.bias; b.relu = a.relu; b.mask_ref = a.mask_ref; b.ld_mask = a.ld_mask;
+  b.out = a.out; b.ld_out = a.ld_out;
+  b.F = a.F; b.plan_filter = -1;
+  return b;
+}
+
+wg_status run(wg_dtype dt, const AggArgs& a, const CsrExec& X, cudaStream_t s) {
+  WG_TRY(launch_agg(dt, a, s));
+  WG_TRY(launch_combine(dt, comb(a, X), s));
+  return WG_OK;
+}
+
+}  // namespace
+
+// -------------------------------------------------------------------- plan
+wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
+  wg_graph_s* g = p->g;
+  const wg_conv_desc& d = p->d;
+  WG_REQ(g->vb == 0 && g->ve == g->V, WG_ERR_UNSUPPORTED, "RGCN with a 1-D partition is not implemented");
+  const int R = g->by_type ? g->R : 1;
+  const int64_t E = g->fwd.E, V = g->V;
+  auto* rp = new RgcnPlan();
+  rp->R = R;
+  p->rg = rp;
+  p->pi = pitch(d.f_in, d.dtype);
+  p->po = pitch(d.f_out, d.dtype);
+  // ---- host copies of the forward / transposed sorted edge arrays
+  std::vector<int32_t> fk, fi_, ft, fperm, bk, bi, bt, bperm;
+  WG_TRY(down(g->fwd.key, E, fk));
+  WG_TRY(down(g->fwd.idx, E, fi_));
+  WG_TRY(down(g->fwd.perm, E, fperm));
+  WG_TRY(down(g->bwd.key, E, bk));
+  WG_TRY(down(g->bwd.idx, E, bi));
+  WG_TRY(down(g->bwd.perm, E, bperm));
+  if (g->by_type) {
+    WG_TRY(down(g->fwd.type, E, ft));
+    WG_TRY(down(g->bwd.type, E, bt));
+  } else {
+    ft.assign(E, 0);
+    bt.assign(E, 0);
+  }
+  const auto& tasks = g->fwd.h_tasks;
+  const int64_t nt = (int64_t)tasks.size();
+  // per-edge coefficient c_e (by global edge id): 1 or 1/|in_r(dst)|
+  std::vector<float> coef_eid(E, 1.f);
+  // segment runs in the forward order: (dst, type) constant
+  std::vector<int64_t> seg_len_at(E, 0);   // length of the segment each position belongs to
+  for (int64_t i = 0; i < E;) {
+    int64_t j = i;
+    while (j < E && fk[j] == fk[i] && ft[j] == ft[i]) ++j;
+    for (int64_t k = i; k < j; ++k) seg_len_at[k] = j - i;
+    i = j;
+  }
+  if (d.norm == WG_NORM_RIGHT)
+    for (int64_t i = 0; i < E; ++i) coef_eid[fperm[i]] = 1.f / (float)seg_len_at[i];
+  // ---- plan bits (a4)
+  p->plan_bits.assign(nt, 0);
+  {
+    const int s = dsize(d.dtype);
+    const int64_t A = rup((int64_t)d.f_in * s, 32), B = rup((int64_t)d.f_out * s, 32);
+    std::mt19937_64 rng(d.policy_seed);
+    for (int64_t t = 0; t < nt; ++t) {
+      const wg_task& k = tasks[t];
+      int64_t nseg = 0;
+      for (int64_t i = k.e_begin; i < k.e_end; ++i) nseg += (i == k.e_begin || fk[i] != fk[i - 1]);
+      const int64_t ne = k.e_end - k.e_begin, nu = k.n_uniq_src;
+      const int64_t te = ne * (A + 4) + nseg * (2 * A + 2 * B + 4);
+      const int64_t tv = nu * (2 * A + 2 * B) + ne * (B + 8);
+      uint8_t b = 0;
+      if (d.policy == WG_PLAN_ALL_VERTEX) b = 1;
+      else if (d.policy == WG_PLAN_RANDOM) b = (uint8_t)(rng() & 1);
+      else if (d.policy == WG_PLAN_AUTO) b = tv < te ? 1 : 0;
+      p->plan_bits[t] = b;
+    }
+    for (int64_t t = 1; t < nt; ++t)
+      if ((tasks[t].flags & WG_TASK_SPLIT) && (tasks[t - 1].flags & WG_TASK_SPLIT) && tasks[t].d_lo == tasks[t - 1].d_lo &&
+          tasks[t].type == tasks[t - 1].type)
+        p->plan_bits[t] = p->plan_bits[t - 1];
+    p->n_vert_tasks = std::count(p->plan_bits.begin(), p->plan_bits.end(), 1);
+    p->n_edge_tasks = nt - p->n_vert_tasks;
+  }
+  // ---- forward stage-1 rows, grouped by relation
+  struct Row1 { int64_t ent_b, ent_e; float rs; };
+  std::vector<std::vector<Row1>> rows1(R);
+  std::vector<std::vector<int32_t>> ents(R);                 // per-type stage-1 entries (source ids)
+  struct Contrib { int32_t dst; int32_t type; int64_t row; float c; };
+  std::vector<Contrib> contrib;
+  contrib.reserve(E);
+  int64_t open_seg_dst = -1, open_seg_type = -1;           // EDGE segment continuing across SPLIT tasks
+  for (int64_t t = 0; t < nt; ++t) {
+    const wg_task& k = tasks[t];
+    const int r = k.type;
+    if (p->plan_bits[t] == 0) {
+      for (int64_t i = k.e_begin; i < k.e_end;) {
+        int64_t j = i;
+        while (j < k.e_end && fk[j] == fk[i]) ++j;
+        const bool cont = (i == k.e_begin) && open_seg_dst == fk[i] && open_seg_type == r && (k.flags & WG_TASK_SPLIT);
+        if (!cont) {
+          const float rs = d.norm == WG_NORM_RIGHT ? 1.f / (float)seg_len_at[i] : 1.f;
+          rows1[r].push_back(Row1{(int64_t)ents[r].size(), (int64_t)ents[r].size(), rs});
+          contrib.push_back(Contrib{fk[i], r, (int64_t)rows1[r].size() - 1, 1.f});
+        }
+        for (int64_t q = i; q < j; ++q) ents[r].push_back(fi_[q]);
+        rows1[r].back().ent_e = (int64_t)ents[r].size();
+        open_seg_dst = fk[i];
+        open_seg_type = r;
+        i = j;
+      }
+    } else {
+      open_seg_dst = -1;
+      std::vector<int32_t> us(fi_.begin() + k.e_begin, fi_.begin() + k.e_end);
+      std::sort(us.begin(), us.end());
+      us.erase(std::unique(us.begin(), us.end()), us.end());
+      const int64_t base = (int64_t)rows1[r].size();
+      for (int32_t u : us) {
+        rows1[r].push_back(Row1{(int64_t)ents[r].size(), (int64_t)ents[r].size() + 1, 1.f});
+        ents[r].push_back(u);
+      }
+      for (int64_t i = k.e_begin; i < k.e_end; ++i) {
+        const int64_t m = std::lower_bound(us.begin(), us.end(), fi_[i]) - us.begin();
+        contrib.push_back(Contrib{fk[i], r, base + m, coef_eid[fperm[i]]});
+      }
+    }
+  }
+  // typed layout: group r at base1[r], padded to 128 rows
+  std::vector<int64_t> base1(R + 1, 0);
+  for (int r = 0; r < R; ++r) base1[r + 1] = base1[r] + rup((int64_t)rows1[r].size(), TILE_M);
+  rp->n1 = base1[R];
+  {
+    std::vector<int64_t> rpv(rp->n1 + 1, 0);
+    std::vector<int32_t> idx;
+    std::vector<float> rs(rp->n1, 1.f);
+    bool any_rs = false;
+    idx.reserve(E);
+    int64_t row = 0;
+    for (int r = 0; r < R; ++r) {
+      for (const Row1& w : rows1[r]) {
+        for (int64_t q = w.ent_b; q < w.ent_e; ++q) idx.push_back(ents[r][q]);
+        rs[row] = w.rs;
+        any_rs |= w.rs != 1.f;
+        rpv[++row] = (int64_t)idx.size();
+      }
+      while (row < base1[r + 1]) rpv[++row] = (int64_t)idx.size();
+    }
+    WG_TRY(build_exec(p, rpv, idx, nullptr, any_rs ? &rs : nullptr, g->E_max, &rp->f1));
+    std::vector<int32_t> tt(rp->n1 / TILE_M);
+    for (int r = 0; r < R; ++r)
+      for (int64_t t = base1[r] / TILE_M; t < base1[r + 1] / TILE_M; ++t) tt[t] = r;
+    WG_TRY(up(p, tt, &rp->tile_type));
+  }
+  // stage 3: contributions per destination row (sorted by dst, then typed row)
+  {
+    for (auto& c : contrib) c.row += base1[c.type];
+    std::stable_sort(contrib.begin(), contrib.end(), [](const Contrib& a, const Contrib& b) {
+      return a.dst != b.dst ? a.dst < b.dst : a.row < b.row;
+    });
+    std::vector<int64_t> rpv(V + 1, 0);
+    std::vector<int32_t> idx(contrib.size());
+    std::vector<float> es(contrib.size());
+    bool any = false;
+    for (size_t i = 0; i < contrib.size(); ++i) {
+      rpv[contrib[i].dst + 1]++;
+      idx[i] = (int32_t)contrib[i].row;
+      es[i] = contrib[i].c;
+      any |= es[i] != 1.f;
+    }
+    for (int64_t v = 0; v < V; ++v) rpv[v + 1] += rpv[v];
+    WG_TRY(build_exec(p, rpv, idx, any ? &es : nullptr, nullptr, g->E_max, &rp->f3));
+  }
+  // ---- transposed: (src, relation) segments grouped by relation
+  {
+    std::vector<std::vector<std::pair<int64_t, int64_t>>> segs(R);   // [b, e) in transposed order
+    std::vector<std::vector<int32_t>> seg_src(R);
+    for (int64_t i = 0; i < E;) {
+      int64_t j = i;
+      while (j < E && bk[j] == bk[i] && bt[j] == bt[i]) ++j;
+      segs[bt[i]].push_back({i, j});
+      seg_src[bt[i]].push_back(bk[i]);
+      i = j;
+    }
+    std::vector<int64_t> baseT(R + 1, 0);
+    for (int r = 0; r < R; ++r) baseT[r + 1] = baseT[r] + rup((int64_t)segs[r].size(), TILE_M);
+    rp->n1T = baseT[R];
+    std::vector<int64_t> rpv(rp->n1T + 1, 0), rpg(rp->n1T + 1, 0);
+    std::vector<int32_t> idx, gidx;
+    std::vector<float> es;
+    idx.reserve(E);
+    es.reserve(E);
+    bool any = false;
+    struct SC { int32_t src; int64_t row; };
+    std::vector<SC> sc;
+    int64_t row = 0;
+    for (int r = 0; r < R; ++r) {
+      for (size_t s = 0; s < segs[r].size(); ++s) {
+        for (int64_t q = segs[r][s].first; q < segs[r][s].second; ++q) {
+          idx.push_back(bi[q]);
+          const float c = coef_eid[bperm[q]];
+          es.push_back(c);
+          any |= c != 1.f;
+        }
+        gidx.push_back(seg_src[r][s]);
+        sc.push_back(SC{seg_src[r][s], row});
+        rpg[row + 1] = (int64_t)gidx.size();
+        rpv[++row] = (int64_t)idx.size();
+      }
+      while (row < baseT[r + 1]) { rpg[row + 1] = (int64_t)gidx.size(); rpv[++row] = (int64_t)idx.size(); }
+    }
+    WG_TRY(build_exec(p, rpv, idx, any ? &es : nullptr, nullptr, g->E_max, &rp->b1));
+    WG_TRY(build_exec(p, rpg, gidx, nullptr, nullptr, g->E_max, &rp->bg));
+    std::vector<int32_t> tt(rp->n1T / TILE_M);
+    for (int r = 0; r < R; ++r)
+      for (int64_t t = baseT[r] / TILE_M; t < baseT[r + 1] / TILE_M; ++t) tt[t] = r;
+    WG_TRY(up(p, tt, &rp->tile_typeT));
+    rp->h_group_offT = baseT;
+    WG_TRY(up(p, baseT, &rp->group_offT));
+    std::stable_sort(sc.begin(), sc.end(), [](const SC& a, const SC& b) {
+      return a.src != b.src ? a.src < b.src : a.row < b.row;
+    });
+    std::vector<int64_t> rp3(V + 1, 0);
+    std::vector<int32_t> idx3(sc.size());
+    for (size_t i = 0; i < sc.size(); ++i) { rp3[sc[i].src + 1]++; idx3[i] = (int32_t)sc[i].row; }
+    for (int64_t v = 0; v < V; ++v) rp3[v + 1] += rp3[v];
+    WG_TRY(build_exec(p, rp3, idx3, nullptr, nullptr, g->E_max, &rp->b3));
+  }
+  // ---- buffers
+  const int s = dsize(d.dtype);
+  const int64_t rows_o = rup(d.f_out, 16), rows_i = rup(d.f_in, 16);
+  const int64_t pl = rup(std::max(d.f_in, d.f_out), 8);
+  Layout& S = p->saved;
+  Layout& W = p->ws;
+  S = Layout();
+  W = Layout();
+  S.add("none", 1);
+  W.add("wt", (size_t)R * rows_o * p->pi * s);          // stacked W_r^T
+  W.add("w", (size_t)R * rows_i * p->po * s);           // stacked W_r
+  W.add("w0t", (size_t)rows_o * p->pi * s);
+  W.add("w0", (size_t)rows_i * p->po * s);
+  W.add("a1", (size_t)rp->n1 * p->pi * s);
+  W.add("t1", (size_t)rp->n1 * p->po * s);
+  W.add("self", (size_t)V * p->po * s);
+  W.add("part", sizeof(float) * std::max({1, rp->f1.n_slots, rp->f3.n_slots, rp->b1.n_slots, rp->b3.n_slots,
+                                           rp->bg.n_slots}) * pl);
+  W.add("dt", (size_t)V * p->po * s);
+  W.add("gt", (size_t)rp->n1T * p->po * s);
+  W.add("dxt", (size_t)rp->n1T * p->pi * s);
+  W.add("xg", (size_t)rp->n1T * p->pi * s);
+  W.add("dxs", (size_t)V * p->pi * s);
+  W.add("colsum", bias_grad_scratch(V, (int)p->po));
+  W.add("tn", std::max(gemm_tn_scratch(V, d.f_in, d.f_out), gemm_tn_grouped_scratch(R, d.f_in, d.f_out)));
+  // the forward gTask work items are not used by RGCN (stage CSRs replace them)
+  return WG_OK;
+}
+
+void rgcn_plan_free(wg_plan_s* p) {
+  delete static_cast<RgcnPlan*>(p->rg);
+  p->rg = nullptr;
+}
+
+// ----------------------------------------------------------------- forward
+wg_status rgcn_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cudaStream_t st) {
+  const wg_conv_desc& d = p->d;
+  wg_graph_s* g = p->g;
+  auto* rp = static_cast<RgcnPlan*>(p->rg);
+  const wg_dtype dt = d.dtype;
+  const int s = dsize(dt), R = rp->R;
+  WG_REQ(P->W && A->x && A->y && A->workspace, WG_ERR_INVALID, "RGCN forward: null argument");
+  WG_REQ(!d.self_loop || P->W_self, WG_ERR_INVALID, "self_loop needs W_self");
+  const Layout& L = p->ws;
+  void* ws = A->workspace;
+  const int64_t V = g->V, rows_o = rup(d.f_out, 16), pl = rup(std::max(d.f_in, d.f_out), 8);
+  ProfScope ps(PK_RGCN, st, 0.0, 0.0);
+  void* wt = L.at<void>(ws, "wt");
+  WG_TRY(prep_weight_batched(dt, P->W, R, d.f_in, d.f_out, 1, wt, p->pi, (int)rows_o, st));
+  // stage 1: segment sums (EDGE gTasks) and unique-source copies (VERTEX gTasks)
+  void* a1 = L.at<void>(ws, "a1");
+  {
+    AggArgs a = exec_args(rp->f1, g->E_max);
+    a.table = A->x; a.ld_tab = A->ldx;
+    a.out = a1; a.ld_out = p->pi;
+    a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
+    a.F = d.f_in;
+    WG_TRY(run(dt, a, rp->f1, st));
+  }
+  // stage 2: grouped GEMM  T1[group r] = A1[group r] W_r
+  void* t1 = L.at<void>(ws, "t1");
+  {
+    GemmPart part{a1, p->pi, wt, p->pi, d.f_in, d.f_out};
+    part.tile_group = rp->tile_type; part.group_rows = (int)rows_o; part.groups = R;
+    GemmEpi e;
+    e.D = t1; e.ldd = p->po;
+    WG_TRY(gemm_nt(dt, rp->n1, (int)rup(d.f_out, 16 / s), &part, 1, e, nullptr, 0, st));
+  }
+  // self loop x W_0
+  void* self = nullptr;
+  if (d.self_loop) {
+    void* w0t = L.at<void>(ws, "w0t");
+    WG_TRY(prep_weight(dt, P->W_self, d.f_in, d.f_out, 1, w0t, p->pi, (int)rows_o, st));
+    self = L.at<void>(ws, "self");
+    GemmPart part{A->x, A->ldx, w0t, p->pi, d.f_in, (int)rows_o};
+    GemmEpi e;
+    e.D = self; e.ldd = p->po;
+    WG_TRY(gemm_nt(dt, V, (int)rup(d.f_out, 16 / s), &part, 1, e, nullptr, 0, st));
+  }
+  // stage 3: y[v] = sum of contributions (+ self + bias), ReLU
+  {
+    AggArgs a = exec_args(rp->f3, g->E_max);
+    a.table = t1; a.ld_tab = p->po;
+    a.self_tab = self; a.ld_self = p->po;
+    a.bias = d.bias ? P->bias : nullptr;
+    a.relu = d.fuse_relu;
+    a.out = A->y; a.ld_out = A->ldy;
+    a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
+    a.F = d.f_out;
+    WG_TRY(run(dt, a, rp->f3, st));
+  }
+  return WG_OK;
+}
+
+// ---------------------------------------------------------------- backward
+wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, const wg_grads* G, cudaStream_t st) {
+  const wg_conv_desc& d = p->d;
+  wg_graph_s* g = p->g;
+  auto* rp = static_cast<RgcnPlan*>(p->rg);
+  const wg_dtype dt = d.dtype;
+  const int s = dsize(dt), R = rp->R;
+  WG_REQ(P->W && A->dy && A->x && A->workspace, WG_ERR_INVALID, "RGCN backward: null argument");
+  WG_REQ(!d.fuse_relu || A->y, WG_ERR_INVALID, "fuse_relu backward needs y");
+  WG_REQ(!d.need_dx || A->dx, WG_ERR_INVALID, "need_dx but dx is NULL");
+  const Layout& L = p->ws;
+  void* ws = A->workspace;
+  const int64_t V = g->V, rows_i = rup(d.f_in, 16), pl = rup(std::max(d.f_in, d.f_out), 8);
+  ProfScope ps(PK_RGCN, st, 0.0, 0.0);
+  // dT = dy masked by the fused ReLU; db
+  const void* dT = A->dy;
+  int64_t lddT = A->lddy;
+  if (d.fuse_relu) { dT = L.at<void>(ws, "dt"); lddT = p->po; }
+  WG_TRY(bias_grad_mask(dt, V, d.f_out, A->dy, A->lddy, d.fuse_relu ? A->y : nullptr, A->ldy,
+                        d.fuse_relu ? const_cast<void*>(dT) : nullptr, lddT, (G && d.bias) ? G->bias : nullptr,
+                        L.at<float>(ws, "colsum"), st));
+  // stage 1T: G_(u,r) = sum_{e: src u, type r} c_e dT[dst_e]
+  void* gt = L.at<void>(ws, "gt");
+  {
+    AggArgs a = exec_args(rp->b1, g->E_max);
+    a.table = dT; a.ld_tab = lddT;
+    a.out = gt; a.ld_out = p->po;
+    a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
+    a.F = d.f_out;
+    WG_TRY(run(dt, a, rp->b1, st));
+  }
+  // dW_r = X_g[group r]^T G[group r]
+  if (G && G->W) {
+    void* xg = L.at<void>(ws, "xg");
+    AggArgs a = exec_args(rp->bg, g->E_max);
+    a.table = A->x; a.ld_tab = A->ldx;
+    a.out = xg; a.ld_out = p->pi;
+    a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
+    a.F = d.f_in;
+    WG_TRY(run(dt, a, rp->bg, st));
+    WG_TRY(gemm_tn_grouped(dt, R, rp->group_offT, d.f_in, d.f_out, xg, p->pi, gt, p->po, G->W,
+                           L.at<void>(ws, "tn"), st));
+  }
+  if (d.self_loop && G && G->W_self)
+    WG_TRY(gemm_tn(dt, V, d.f_in, d.f_out, A->x, A->ldx, dT, lddT, G->W_self, L.at<void>(ws, "tn"), st));
+  if (!d.need_dx) return WG_OK;
+  // stage 2T: dX_(u,r) = G_(u,r) W_r^T (grouped)
+  void* w = L.at<void>(ws, "w");
+  WG_TRY(prep_weight_batched(dt, P->W, R, d.f_in, d.f_out, 0, w, p->po, (int)rows_i, st));
+  void* dxt = L.at<void>(ws, "dxt");
+  {
+    GemmPart part{gt, p->po, w, p->po, d.f_out, d.f_in};
+    part.tile_group = rp->tile_typeT; part.group_rows = (int)rows_i; part.groups = R;
+    GemmEpi e;
+    e.D = dxt; e.ldd = p->pi;
+    WG_TRY(gemm_nt(dt, rp->n1T, (int)rup(d.f_in, 16 / s), &part, 1, e, nullptr, 0, st));
+  }
+  void* dxs = nullptr;
+  if (d.self_loop) {
+    void* w0 = L.at<void>(ws, "w0");
+    WG_TRY(prep_weight(dt, P->W_self, d.f_in, d.f_out, 0, w0, p->po, (int)rows_i, st));
+    dxs = L.at<void>(ws, "dxs");
+    GemmPart part{dT, lddT, w0, p->po, d.f_out, (int)rows_i};
+    GemmEpi e;
+    e.D = dxs; e.ldd = p->pi;
+    WG_TRY(gemm_nt(dt, V, (int)rup(d.f_in, 16 / s), &part, 1, e, nullptr, 0, st));
+  }
+  // stage 3T: dx[u] = sum_r dX_(u,r) (+ dT W_0^T)
+  {
+    AggArgs a = exec_args(rp->b3, g->E_max);
+    a.table = dxt; a.ld_tab = p->pi;
+    a.self_tab = dxs; a.ld_self = p->pi;
+    a.out = A->dx; a.ld_out = A->lddx;
+    a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
+    a.F = d.f_in;
+    WG_TRY(run(dt, a, rp->b3, st));
+  }
+  return WG_OK;
+}
+
 }  // namespace wg

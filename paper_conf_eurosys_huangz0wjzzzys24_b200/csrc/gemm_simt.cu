@@ -39,6 +39,7 @@ __global__ void __launch_bounds__(256) k_gemm_nt(NTArgs a) {
     const GemmPart P = a.parts[p];
     const T* A = static_cast<const T*>(P.A);
     const T* B = static_cast<const T*>(P.B);
+    if (P.tile_group) B += (int64_t)P.tile_group[m0 / 128] * P.group_rows * P.ldb;
     for (int k0 = 0; k0 < P.K; k0 += BK) {
       for (int t = threadIdx.x; t < BM * BK; t += 256) {
         int mm = t / BK, kk = t % BK;
@@ -126,6 +127,60 @@ __global__ void __launch_bounds__(256) k_gemm_tn(int64_t K, int M, int N, const 
   }
 }
 
+// grouped: part[g*splits + z] = sum over the z-th K chunk of group g
+template <typename T>
+__global__ void __launch_bounds__(256) k_gemm_tn_grouped(const int64_t* off, int splits, int M, int N, const T* A,
+                                                         int64_t lda, const T* B, int64_t ldb, float* part) {
+  __shared__ float As[BK][BM + 4];
+  __shared__ float Bs[BK][BN + 4];
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  const int m0 = blockIdx.x * BM, n0 = blockIdx.y * BN;
+  const int g = blockIdx.z / splits, z = blockIdx.z % splits;
+  const int64_t g0 = off[g], g1 = off[g + 1], len = g1 - g0;
+  const int64_t kb = g0 + len * z / splits, ke = g0 + len * (z + 1) / splits;
+  float acc[4][4] = {};
+  for (int64_t k0 = kb; k0 < ke; k0 += BK) {
+    for (int t = threadIdx.x; t < BM * BK; t += 256) {
+      int kk = t / BM, mm = t % BM;
+      int64_t k = k0 + kk;
+      As[kk][mm] = (k < ke && m0 + mm < M) ? tof<T>(A[k * lda + m0 + mm]) : 0.f;
+      Bs[kk][mm] = (k < ke && n0 + mm < N) ? tof<T>(B[k * ldb + n0 + mm]) : 0.f;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int kk = 0; kk < BK; ++kk) {
+      float av[4], bv[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) { av[i] = As[kk][ty * 4 + i]; bv[i] = Bs[kk][tx * 4 + i]; }
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+  float* P = part + (int64_t)blockIdx.z * M * N;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    int m = m0 + ty * 4 + i;
+    if (m >= M) continue;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      int n = n0 + tx * 4 + j;
+      if (n < N) P[(int64_t)m * N + n] = acc[i][j];
+    }
+  }
+}
+
+__global__ void k_group_reduce(const float* part, int groups, int splits, int64_t MN, float* D) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= MN * groups) return;
+  const int64_t g = i / MN, e = i % MN;
+  float s = 0.f;
+  for (int z = 0; z < splits; ++z) s += part[(g * splits + z) * MN + e];
+  D[i] = s;
+}
+
 __global__ void k_split_reduce(const float* part, int splits, int64_t MN, float* D, int acc) {
   int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= MN) return;
@@ -159,6 +214,29 @@ wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_pa
   dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN));
   if (dt == WG_BF16) WG_LAUNCH(k_gemm_nt<__nv_bfloat16>, grid, 256, 0, s, a);
   else WG_LAUNCH(k_gemm_nt<float>, grid, 256, 0, s, a);
+  return WG_OK;
+}
+
+constexpr int GROUP_SPLITS = 4;
+
+size_t gemm_tn_grouped_scratch(int groups, int M, int N) {
+  return sizeof(float) * (size_t)groups * GROUP_SPLITS * M * N;
+}
+
+wg_status gemm_tn_grouped(wg_dtype dt, int groups, const int64_t* d_off, int M, int N, const void* A, int64_t lda,
+                          const void* B, int64_t ldb, float* D, void* scratch, cudaStream_t s) {
+  if (groups == 0 || M == 0 || N == 0) return WG_OK;
+  float* part = static_cast<float*>(scratch);
+  dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN), (unsigned)(groups * GROUP_SPLITS));
+  ProfScope ps(PK_SIMT, s, 0.0, 0.0);
+  if (dt == WG_BF16)
+    WG_LAUNCH(k_gemm_tn_grouped<__nv_bfloat16>, grid, 256, 0, s, d_off, GROUP_SPLITS, M, N, (const __nv_bfloat16*)A,
+              lda, (const __nv_bfloat16*)B, ldb, part);
+  else
+    WG_LAUNCH(k_gemm_tn_grouped<float>, grid, 256, 0, s, d_off, GROUP_SPLITS, M, N, (const float*)A, lda,
+              (const float*)B, ldb, part);
+  const int64_t MN = (int64_t)M * N;
+  WG_LAUNCH(k_group_reduce, (unsigned)cdiv(MN * groups, 256), 256, 0, s, part, groups, GROUP_SPLITS, MN, D);
   return WG_OK;
 }
 

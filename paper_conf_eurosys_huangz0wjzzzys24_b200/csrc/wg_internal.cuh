@@ -131,6 +131,7 @@ struct AggArgs {
   const void* table;          // gathered table [.. x ld_tab]
   int64_t ld_tab;
   const float* gscale;        // per gathered row (nullable)
+  const float* escale;        // per entry / edge position (nullable; not combined with gscale)
   const float* rscale;        // per output row, indexed by GLOBAL row (local + row_base) (nullable)
   int64_t row_base;           // local row -> global row offset (for rscale / self rows)
   const void* self_tab;       // self term rows (local row indexing) (nullable)
@@ -184,6 +185,11 @@ struct GemmPart {
   const void* B; int64_t ldb;   // row-major [nb x K]; rows >= nb read as 0
   int K;
   int nb;
+  // grouped GEMM (RGCN relation weights): 128-row tile t of A uses the B rows
+  // [tile_group[t] * group_rows, +nb) of a stacked [groups x group_rows x ldb] B
+  const int32_t* tile_group = nullptr;
+  int group_rows = 0;
+  int groups = 1;
 };
 struct GemmEpi {
   const float* rscale = nullptr;      // per row
@@ -204,6 +210,14 @@ size_t gemm_tn_scratch(int64_t K, int M, int N);
 wg_status gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda,
                   const void* B, int64_t ldb, float* D, void* scratch, cudaStream_t s, int acc = 0);
 
+// grouped weight gradient: D[g] (fp32 [M x N]) = sum_{k in [off[g], off[g+1])} A[k]^T B[k]
+size_t gemm_tn_grouped_scratch(int groups, int M, int N);
+wg_status gemm_tn_grouped(wg_dtype dt, int groups, const int64_t* d_off, int M, int N, const void* A, int64_t lda,
+                          const void* B, int64_t ldb, float* D, void* scratch, cudaStream_t s);
+// batched weight prep: `batch` matrices of [rows x cols] (fp32, contiguous) into
+// consecutive [out_rows x ldo] blocks
+wg_status prep_weight_batched(wg_dtype dt, const float* W, int batch, int rows, int cols, int transpose, void* out,
+                              int64_t ldo, int out_rows, cudaStream_t s);
 // weight prep: fp32 [rows x cols] -> dtype, optionally transposed, into [out_rows x ldo]
 wg_status prep_weight(wg_dtype dt, const float* W, int rows, int cols, int transpose,
                       void* out, int64_t ldo, int out_rows, cudaStream_t s);

@@ -1,0 +1,90 @@
+"""RGCN (Eq. (1)) forward + backward through the C ABI == oracle.
+
+Every per-gTask plan policy (EDGE = (dst, relation) segment sums, VERTEX =
+gTask-local unique-source transforms, mixed) must give the same result;
+small-integer inputs are bit-exact; SPLIT chunks (small E_max) are merged."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from tests.util import TOL, f64, q, rel_err
+
+pytestmark = pytest.mark.gpu
+
+
+def wg():
+    import paper_conf_eurosys_huangz0wjzzzys24_b200 as m
+    return m
+
+
+def run(dtype=torch.float32, policy="auto", norm="none", self_loop=False, bias=False, R=5, V=1500, E=20000, fi=24,
+        fo=16, E_max=0, seed=0, ints=False, relu=False, alpha=0.6):
+    m = wg()
+    src, dst, et = synth.make_graph(V, E, seed=seed, alpha=alpha, R=R)
+    g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V,
+                etype=torch.from_numpy(et).cuda(), num_types=R, max_task_edges=E_max)
+    conv = m.Conv(g, "rgcn", fi, fo, dtype=dtype, policy=policy, seed=seed, norm=norm, self_loop=self_loop,
+                  bias=bias, fuse_relu=relu)
+    params = m.init_params("rgcn", fi, fo, R=R, self_loop=self_loop, bias=bias, seed=seed)
+    if ints:
+        params = {k: torch.from_numpy(synth.small_ints(tuple(v.shape), seed=seed + 3 + i)).cuda()
+                  for i, (k, v) in enumerate(params.items())}
+        x = torch.from_numpy(synth.small_ints((V, fi), seed=seed + 1)).to(dtype)
+        dy = torch.from_numpy(synth.small_ints((V, fo), seed=seed + 2)).to(dtype)
+    else:
+        gen = torch.Generator(device="cuda").manual_seed(seed)
+        params = {k: v + 0.1 * torch.randn(v.shape, generator=gen, device="cuda") for k, v in params.items()}
+        x = torch.from_numpy(synth.make_features(V, fi, seed=seed + 1)).to(dtype)
+        dy = torch.from_numpy(synth.normal((V, fo), seed=seed + 2, std=0.25)).to(dtype)
+    xd = m.pad_to(x.cuda())
+    y, saved = conv.forward_raw(xd, params)
+    dx, grads = conv.backward_raw(m.pad_to(dy.cuda()), xd, y, saved, params)
+    torch.cuda.synchronize()
+    Wq = {k: q(v, dtype) for k, v in params.items()}
+    yo = oracle.rgcn_forward(src, dst, et, V, f64(x), Wq["W"], Wq.get("W_self"), Wq.get("bias"), norm=norm)
+    dyo = f64(dy)
+    if relu:
+        dyo = dyo * (f64(y) > 0)
+        yo = np.maximum(yo, 0)
+    dxo, dWo, dW0o, dbo = oracle.rgcn_backward(src, dst, et, V, f64(x), Wq["W"], dyo, Wq.get("W_self"), norm=norm)
+    errs = {"y": rel_err(f64(y), yo), "dx": rel_err(f64(dx), dxo), "dW": rel_err(f64(grads["W"]), dWo)}
+    if self_loop:
+        errs["dW0"] = rel_err(f64(grads["W_self"]), dW0o)
+    if bias:
+        errs["db"] = rel_err(f64(grads["bias"]), dbo)
+    return errs, conv
+
+
+@pytest.mark.parametrize("policy", ["auto", "edge", "vertex", "random"])
+@pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
+def test_rgcn_plan_invariance(policy, dtype):
+    errs, conv = run(dtype, policy)
+    if policy == "random":
+        assert conv.n_edge_tasks > 0 and conv.n_vertex_tasks > 0
+    assert all(v <= TOL[dtype] for v in errs.values()), str(errs)
+
+
+@pytest.mark.parametrize("policy", ["edge", "vertex"])
+def test_rgcn_norm_selfloop_bias_relu_split(policy):
+    errs, conv = run(torch.float32, policy, norm="right", self_loop=True, bias=True, relu=True, E_max=16, seed=3,
+                     alpha=0.8)
+    assert all(v <= 1e-4 for v in errs.values()), str(errs)
+
+
+@pytest.mark.parametrize("policy", ["edge", "vertex", "random"])
+def test_rgcn_integer_bit_exact(policy):
+    errs, _ = run(torch.float32, policy, ints=True, self_loop=True, seed=5, V=800, E=6000, fi=8, fo=8, alpha=0.3)
+    assert all(v == 0.0 for v in errs.values()), str(errs)
+
+
+def test_rgcn_single_relation():
+    errs, _ = run(torch.float32, "auto", R=1, seed=7)
+    assert all(v <= 1e-4 for v in errs.values()), str(errs)
+
+
+def test_rgcn_c3_shape_sampled():
+    """C3 layer shape (128 -> 64, R = 128 Zipf relations) at reduced V / E."""
+    errs, _ = run(torch.float32, "auto", R=128, V=20000, E=220000, fi=128, fo=64, seed=9, alpha=0.5)
+    assert all(v <= 1e-4 for v in errs.values()), str(errs)
