@@ -302,13 +302,13 @@ __global__ void k_gat_s(int64_t rows, int64_t row_base, GatArgs a, float* s) {
 // sum dt_e, dt_e written at the edge's forward position.
 template <typename T, int NV>
 __global__ void __launch_bounds__(256) k_gat_bwd_src(GatArgs a, int64_t row_base) {
-  constexpr int EPV = GV<T>::EPV;
+  constexpr int EPV = 4;                       // G is kept in fp32 (4 columns per 16-byte vector)
   const int lane = threadIdx.x & 31;
   const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (w >= a.n_chunks) return;
   const RowChunk ch = a.chunks[w];
   const int64_t u = row_base + ch.row;
-  const T* G = static_cast<const T*>(a.G);
+  const float* G = static_cast<const float*>(a.G);
   const T* DY = static_cast<const T*>(a.dy);
   int hd[NV];
   float gu[NV][EPV], elu[NV], acc[NV][EPV], dl[NV];
@@ -316,7 +316,7 @@ __global__ void __launch_bounds__(256) k_gat_bwd_src(GatArgs a, int64_t row_base
   for (int q = 0; q < NV; ++q) {
     const int vi = lane + 32 * q;
     hd[q] = vi < a.VPR ? (vi * EPV) / a.Fo : 0;
-    if (vi < a.VPR) GV<T>::unpack(ld16(G + u * a.ldg + vi * EPV), gu[q]);
+    if (vi < a.VPR) GV<float>::unpack(ld16(G + u * a.ldg + vi * EPV), gu[q]);
     else {
 #pragma unroll
       for (int i = 0; i < EPV; ++i) gu[q][i] = 0.f;
@@ -337,7 +337,8 @@ __global__ void __launch_bounds__(256) k_gat_bwd_src(GatArgs a, int64_t row_base
       if (vi < a.VPR) {
         const int c0 = vi * EPV;
         const int cc = a.concat ? c0 : (c0 % a.Fo);
-        GV<T>::unpack(ld16(DY + dd * a.lddy + cc), dyv[q]);
+#pragma unroll
+        for (int i = 0; i < EPV; ++i) dyv[q][i] = (c0 + i < a.HF) ? (float)DY[dd * a.lddy + cc + i] : 0.f;
 #pragma unroll
         for (int i = 0; i < EPV; ++i) {
           dyv[q][i] = (c0 + i < a.HF) ? dyv[q][i] * dys : 0.f;
@@ -425,7 +426,7 @@ __global__ void k_gat_dG(int64_t rows, int64_t row_base, GatArgs a, const float*
                          const float* der, T* dG, T* dGlo, int64_t ld_dG, float* part, int64_t rows_per_blk) {
   // thread per column c (HF <= 1024), rows of this block
   const int64_t r0 = blockIdx.x * rows_per_blk, r1 = min(rows, r0 + rows_per_blk);
-  const T* G = static_cast<const T*>(a.G);
+  const float* G = static_cast<const float*>(a.G);
   for (int c = threadIdx.x; c < a.HF; c += blockDim.x) {
     const int h = c / a.Fo;
     float sl = 0.f, sr = 0.f;
@@ -494,7 +495,10 @@ void gat_layout(wg_plan_s* p) {
   Layout& W = p->ws;
   S = Layout();
   W = Layout();
-  S.add("G", (size_t)V * p->po * s);
+  // g = x W is kept in fp32 for both dtypes: the attention logits and the
+  // ill-conditioned der / da_r sums (the softmax gradient cancels exactly
+  // for LeakyReLU slope 1) need its full accumulator precision
+  S.add("G", sizeof(float) * (size_t)V * pitch(HF, WG_F32));
   S.add("agg", sizeof(float) * (size_t)nr * rup(HF, 4));   // fp32: s = dy.agg feeds a cancellation (dt)
   S.add("el", sizeof(float) * V * H);
   S.add("er", sizeof(float) * V * H);
@@ -536,37 +540,37 @@ static wg_status gat_fwd_t(wg_plan_s* p, const wg_params* P, const wg_fwd_args* 
   void* ws = A->workspace;
   const int s = dsize(d.dtype);
   GatArgs a{};
-  a.H = H; a.Fo = Fo; a.HF = HF; a.VPR = (int)cdiv(HF, EPV); a.slope = d.neg_slope;
-  a.G = S.at<void>(A->saved, "G"); a.ldg = p->po;
+  a.H = H; a.Fo = Fo; a.HF = HF; a.VPR = (int)cdiv(HF, 4); a.slope = d.neg_slope;
+  a.G = S.at<void>(A->saved, "G"); a.ldg = pitch(HF, WG_F32);
   a.el = S.at<float>(A->saved, "el"); a.er = S.at<float>(A->saved, "er");
   a.m = S.at<float>(A->saved, "m"); a.l = S.at<float>(A->saved, "l");
   a.agg = S.at<void>(A->saved, "agg"); a.ld_agg = rup(HF, 4);
   a.part = L.at<float>(ws, "part"); a.part_ld = HF + 2 * H + 8;
   a.concat = d.concat_heads;
-  // G = x W  (vertex-level transform, tcgen05 for bf16)
+  // G = x W  (vertex-level transform, tcgen05 for bf16; fp32 accumulator kept)
   void* wt = L.at<void>(ws, "wt");
   WG_TRY(prep_weight(d.dtype, P->W, d.f_in, HF, 1, wt, p->pi, (int)rup(HF, 16), st));
   {
     GemmPart part{A->x, A->ldx, wt, p->pi, d.f_in, (int)rup(HF, 16)};
     GemmEpi e;
-    e.D = const_cast<void*>(a.G); e.ldd = a.ldg;
-    WG_TRY(gemm_nt(d.dtype, V, (int)rup(HF, 16 / s), &part, 1, e, nullptr, 0, st));
+    e.D = const_cast<void*>(a.G); e.ldd = a.ldg; e.d_f32 = 1;
+    WG_TRY(gemm_nt(d.dtype, V, (int)rup(HF, 8), &part, 1, e, nullptr, 0, st));
   }
-  const int NV = nv_for<T>(a.VPR);
-  ProfScope ps(PK_GAT, st, (double)g->fwd.E * (HF * s + 4.0 * H + 4) + (double)V * HF * s * 3, 0.0);
+  const int NV = nv_for<float>(a.VPR);
+  ProfScope ps(PK_GAT, st, (double)g->fwd.E * (HF * 4.0 + 4.0 * H + 4) + (double)V * HF * (4.0 + s) * 2, 0.0);
   const unsigned wb = (unsigned)cdiv(V * 32, 256);
-  if (NV == 1) WG_LAUNCH((k_gat_logits<T, 1>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
-  else if (NV == 2) WG_LAUNCH((k_gat_logits<T, 2>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
-  else WG_LAUNCH((k_gat_logits<T, 4>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
+  if (NV == 1) WG_LAUNCH((k_gat_logits<float, 1>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
+  else if (NV == 2) WG_LAUNCH((k_gat_logits<float, 2>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
+  else WG_LAUNCH((k_gat_logits<float, 4>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
   a.idx = g->fwd.idx;
   a.chunks = gp->fwd; a.n_chunks = gp->n_fwd;
   if (gp->n_fwd) {
     const unsigned cbk = (unsigned)cdiv((int64_t)gp->n_fwd * 32, 256);
-    if (NV == 1) WG_LAUNCH((k_gat_fwd<T, 1, 4>), cbk, 256, 0, st, a, vb);
-    else if (NV == 2) WG_LAUNCH((k_gat_fwd<T, 2, 4>), cbk, 256, 0, st, a, vb);
-    else WG_LAUNCH((k_gat_fwd<T, 4, 2>), cbk, 256, 0, st, a, vb);
+    if (NV == 1) WG_LAUNCH((k_gat_fwd<float, 1, 4>), cbk, 256, 0, st, a, vb);
+    else if (NV == 2) WG_LAUNCH((k_gat_fwd<float, 2, 4>), cbk, 256, 0, st, a, vb);
+    else WG_LAUNCH((k_gat_fwd<float, 4, 2>), cbk, 256, 0, st, a, vb);
   }
-  if (gp->n_fsplit) WG_LAUNCH(k_gat_fwd_combine<T>, gp->n_fsplit, 128, 0, st, a, gp->fsplit, vb);
+  if (gp->n_fsplit) WG_LAUNCH(k_gat_fwd_combine<float>, gp->n_fsplit, 128, 0, st, a, gp->fsplit, vb);
   const int FO = d.concat_heads ? HF : Fo;
   WG_LAUNCH(k_gat_out<T>, 1184, 256, 0, st, nr, a, d.bias ? P->bias : nullptr, d.fuse_relu, A->y, A->ldy, FO);
   return WG_OK;
@@ -588,13 +592,14 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
   const int s = dsize(d.dtype);
   const int FO = d.concat_heads ? HF : Fo;
   GatArgs a{};
-  a.H = H; a.Fo = Fo; a.HF = HF; a.VPR = (int)cdiv(HF, EPV); a.slope = d.neg_slope;
-  a.G = S.at<void>(A->saved, "G"); a.ldg = p->po;
+  a.H = H; a.Fo = Fo; a.HF = HF; a.VPR = (int)cdiv(HF, 4); a.slope = d.neg_slope;
+  a.G = S.at<void>(A->saved, "G"); a.ldg = pitch(HF, WG_F32);
   a.el = S.at<float>(A->saved, "el"); a.er = S.at<float>(A->saved, "er");
   a.m = S.at<float>(A->saved, "m"); a.l = S.at<float>(A->saved, "l");
   a.agg = S.at<void>(A->saved, "agg"); a.ld_agg = rup(HF, 4);
   a.part = L.at<float>(ws, "part"); a.part_ld = HF + 2 * H + 8;
   a.concat = d.concat_heads;
+  (void)EPV;
   // dT = dy (masked by the fused ReLU) ; db
   const void* dT = A->dy;
   int64_t lddT = A->lddy;
@@ -613,7 +618,7 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
   a.dg = L.at<float>(ws, "dg"); a.ld_dg = HF;
   a.del = L.at<float>(ws, "del");
   a.chunks = gp->bwd; a.n_chunks = gp->n_bwd;
-  const int NV = nv_for<T>(a.VPR);
+  const int NV = nv_for<float>(a.VPR);
   if (gp->n_bwd) {
     const unsigned cbk = (unsigned)cdiv((int64_t)gp->n_bwd * 32, 256);
     if (NV == 1) WG_LAUNCH((k_gat_bwd_src<T, 1>), cbk, 256, 0, st, a, vb);

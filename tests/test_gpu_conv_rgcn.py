@@ -24,7 +24,7 @@ def run(dtype=torch.float32, policy="auto", norm="none", self_loop=False, bias=F
     m = wg()
     src, dst, et = synth.make_graph(V, E, seed=seed, alpha=alpha, R=R)
     g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V,
-                etype=torch.from_numpy(et).cuda(), num_types=R, max_task_edges=E_max)
+                etype=None if et is None else torch.from_numpy(et).cuda(), num_types=R, max_task_edges=E_max)
     conv = m.Conv(g, "rgcn", fi, fo, dtype=dtype, policy=policy, seed=seed, norm=norm, self_loop=self_loop,
                   bias=bias, fuse_relu=relu)
     params = m.init_params("rgcn", fi, fo, R=R, self_loop=self_loop, bias=bias, seed=seed)
