@@ -25,10 +25,15 @@ class GNNStack:
     """L gTask layers (hidden ReLU fused into the layer epilogue) + CE loss + Adam."""
 
     def __init__(self, graph: Graph, model: str, dims, *, dtype=torch.bfloat16, heads: int = 1, policy="auto",
-                 seed: int = 0, lr: float = 1e-3, group=None, block: int | None = None, R: int = 1):
+                 seed: int = 0, lr: float = 1e-3, group=None, block: int | None = None, R: int = 1,
+                 conv_factory=None, device=None):
+        # conv_factory / device: injection points for the multi-process CPU test
+        # of this orchestration (tests/test_dist_gloo.py); the product path uses
+        # Conv (libwg.so) on the graph's CUDA device.
+        Conv_ = conv_factory or Conv
         self.g, self.model, self.dims, self.dtype = graph, model, list(dims), dtype
         self.L = len(dims) - 1
-        self.dev = torch.device("cuda", graph.device)
+        self.dev = device if device is not None else torch.device("cuda", graph.device)
         self.group = group
         self.dist = group is not None and torch.distributed.get_world_size(group) > 1
         self.world = torch.distributed.get_world_size(group) if group is not None else 1
@@ -44,11 +49,11 @@ class GNNStack:
             if model == "gat":
                 kw.update(heads=heads, concat=not last)
             pol = policy
-            conv = Conv(graph, model, dims[i], dims[i + 1], policy=pol, **kw)
+            conv = Conv_(graph, model, dims[i], dims[i + 1], policy=pol, **kw)
             if self.dist and conv.n_edge_tasks and conv.n_vertex_tasks:   # uniform plan per layer when distributed
                 pol = "vertex" if conv.n_vertex_tasks > conv.n_edge_tasks else "edge"
                 conv.close()
-                conv = Conv(graph, model, dims[i], dims[i + 1], policy=pol, **kw)
+                conv = Conv_(graph, model, dims[i], dims[i + 1], policy=pol, **kw)
             self.convs.append(conv)
             fo = dims[i + 1] if model != "gat" else (heads * dims[i + 1] if not last else dims[i + 1])
             self.params.append(init_params(model, dims[i], dims[i + 1], heads=heads, concat=not last, R=R,
