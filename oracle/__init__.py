@@ -159,14 +159,16 @@ def sage_forward(src, dst, V, x, Ws, Wn, b=None, rows=None):
     return y
 
 
-def sage_backward(src, dst, V, x, Ws, Wn, dy, rows=None):
+def sage_backward(src, dst, V, x, Ws, Wn, dy, rows=None, grads=True):
+    """grads=False: only dx (of `rows`) is computed (weight-gradient loops skipped)."""
     x, Ws, Wn, dy = _f64(x), _f64(Ws), _f64(Wn), _f64(dy)
     fi, fo = Ws.shape
     dx, dWs, dWn, db = np.zeros((V, fi)), np.zeros((fi, fo)), np.zeros((fi, fo)), np.zeros(fo)
     s, d = _i32(src), _i32(dst)
     m = _mask(V, rows)
     _L().wgo_sage_backward(V, s.shape[0], _p(s), _p(d), fi, fo, _p(x), _p(Ws), _p(Wn), _p(dy), _p(m),
-                           _p(dx), _p(dWs), _p(dWn), _p(db))
+                           _p(dx), _p(dWs) if grads else None, _p(dWn) if grads else None,
+                           _p(db) if grads else None)
     return dx, dWs, dWn, db
 
 
@@ -202,7 +204,8 @@ def rgcn_forward(src, dst, etype, V, x, W, W0=None, b=None, norm="none", rows=No
     return y
 
 
-def rgcn_backward(src, dst, etype, V, x, W, dy, W0=None, norm="none", rows=None):
+def rgcn_backward(src, dst, etype, V, x, W, dy, W0=None, norm="none", rows=None, grads=True):
+    """grads=False: only dx (of `rows`) is computed (weight-gradient loops skipped)."""
     x, W, W0, dy = _f64(x), _f64(W), _f64(W0), _f64(dy)
     R, fi, fo = W.shape
     dx, dW, db = np.zeros((V, fi)), np.zeros((R, fi, fo)), np.zeros(fo)
@@ -210,7 +213,8 @@ def rgcn_backward(src, dst, etype, V, x, W, dy, W0=None, norm="none", rows=None)
     s, d, t = _i32(src), _i32(dst), _i32(etype)
     m = _mask(V, rows)
     _L().wgo_rgcn_backward(V, s.shape[0], _p(s), _p(d), _p(t), R, NORM[norm], fi, fo, _p(x), _p(W), _p(W0), _p(dy),
-                           _p(m), _p(dx), _p(dW), _p(dW0), _p(db))
+                           _p(m), _p(dx), _p(dW) if grads else None, _p(dW0) if grads else None,
+                           _p(db) if grads else None)
     return dx, dW, dW0, db
 
 

@@ -181,6 +181,7 @@ static void add_msg(int fi, int fo, double c, const double* x, const double* W, 
 /* dx[0..fi) += c * (dy[0..fo) . W^T) ; dW += c * x^T dy  (exact gradients of add_msg) */
 static void add_msg_grad(int fi, int fo, double c, const double* x, const double* W,
                          const double* dy, double* dx, double* dW) {
+    if (!dx && !dW) return;   /* nothing requested for this edge (sampled-row checks) */
     for (int k = 0; k < fi; ++k) {
         double s = 0.0;
         for (int j = 0; j < fo; ++j) s += dy[j] * W[(int64_t)k * fo + j];
