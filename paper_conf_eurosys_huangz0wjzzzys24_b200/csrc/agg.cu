@@ -342,7 +342,16 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
     if (cb < ce) {
       // ---- producer state: next round to issue starts at `prod`
       int64_t prod = cb;
-      int pidx = (prod + l < ce && l < RS) ? a.idx[prod + l] : 0;
+      // source ids of the next NQ rounds, prefetched so the producer never waits
+      // on an index load (rounds are RS-aligned from cb)
+      constexpr int NQ = 3;
+      int pq[NQ];
+#pragma unroll
+      for (int k = 0; k < NQ; ++k) {
+        const int64_t e = prod + (int64_t)k * RS + l;
+        pq[k] = (e < ce && l < RS) ? a.idx[e] : 0;
+      }
+      int pidx = pq[0];
       int round_issued = 0;
       auto issue = [&]() {
         const int n = (int)min((int64_t)RS, ce - prod);
@@ -368,7 +377,13 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
         cp_async_commit();
         prod += n;
         ++round_issued;
-        pidx = (prod + l < ce && l < RS) ? a.idx[prod + l] : 0;
+#pragma unroll
+        for (int k = 0; k < NQ - 1; ++k) pq[k] = pq[k + 1];
+        {
+          const int64_t e = prod + (int64_t)(NQ - 1) * RS + l;
+          pq[NQ - 1] = (e < ce && l < RS) ? a.idx[e] : 0;
+        }
+        pidx = pq[0];
       };
 #pragma unroll 1
       for (int r = 0; r < NR; ++r) {

@@ -174,19 +174,25 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
   if (p->n_vert_tasks > 0) {
     ytab = A->xchg ? A->xchg : L.at<void>(ws, "y");
     ldY = A->xchg ? A->ld_xchg : c.po;
-    if (pre) {
+    if (pre && sage && all_vertex) {
+      // [Y | S] = x [W_n | W_s] in one GEMM (x read once); S = self term
+      void* wys = L.at<void>(ws, "wys");
+      WG_TRY(prep_weight(c.dt, P->W, c.fi, c.fo, 1, wys, c.pi, (int)c.po, st));
+      WG_TRY(prep_weight(c.dt, P->W_self, c.fi, c.fo, 1, off(wys, c.po, c.pi, c.s), c.pi, (int)c.po, st));
+      GemmPart part{x_own, A->ldx, wys, c.pi, c.fi, (int)(2 * c.po)};
+      GemmEpi e;
+      e.D = off(ytab, c.vb, ldY, c.s);
+      e.ldd = ldY;
+      e.D2 = L.at<void>(ws, "s");
+      e.ldd2 = c.po;
+      e.n_split = (int)c.po;
+      WG_TRY(gemm_nt(c.dt, c.nr, (int)(2 * c.po), &part, 1, e, nullptr, 0, st));
+    } else if (pre) {
       GemmPart part{x_own, A->ldx, wt, c.pi, c.fi, (int)c.wrows_o};
       GemmEpi e;
       e.D = off(ytab, c.vb, ldY, c.s);
       e.ldd = ldY;
       WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), &part, 1, e, nullptr, 0, st));
-      if (sage && all_vertex) {  // S = x W_s (self term of the VERTEX plan)
-        GemmPart ps{x_own, A->ldx, wst, c.pi, c.fi, (int)c.wrows_o};
-        GemmEpi es;
-        es.D = L.at<void>(ws, "s");
-        es.ldd = c.po;
-        WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), &ps, 1, es, nullptr, 0, st));
-      }
     }
   }
   if (!post) return WG_OK;
@@ -334,17 +340,21 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
     if (pre) {
       if (G && G->W) WG_TRY(gemm_tn(c.dt, c.nr, c.fi, c.fo, agg, c.pi, dTT, lddTT, G->W, tn, st));
       if (sage && G && G->W_self) WG_TRY(gemm_tn(c.dt, c.nr, c.fi, c.fo, x_own, A->ldx, dT, lddT, G->W_self, tn, st));
-      if (d.need_dx) {
+      if (d.need_dx && sage) {
+        // [dAgg | dXs] = dT [W_n ; W_s]^T in one GEMM (dT read once)
+        void* wbs = L.at<void>(ws, "wbs");
+        WG_TRY(prep_weight(c.dt, P->W, c.fi, c.fo, 0, wbs, c.po, (int)c.pi, st));
+        WG_TRY(prep_weight(c.dt, P->W_self, c.fi, c.fo, 0, off(wbs, c.pi, c.po, c.s), c.po, (int)c.pi, st));
+        GemmPart part{dT, lddT, wbs, c.po, c.fo, (int)(2 * c.pi)};
+        GemmEpi e;
+        e.D = off(dtab, c.vb, ldd, c.s); e.ldd = ldd;
+        e.D2 = L.at<void>(ws, "dxs"); e.ldd2 = c.pi; e.n_split = (int)c.pi;
+        WG_TRY(gemm_nt(c.dt, c.nr, (int)(2 * c.pi), &part, 1, e, nullptr, 0, st));
+      } else if (d.need_dx) {
         GemmPart part{dTT, lddTT, w, c.po, c.fo, (int)c.wrows_i};
         GemmEpi e;
         e.D = off(dtab, c.vb, ldd, c.s); e.ldd = ldd;
         WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), &part, 1, e, nullptr, 0, st));
-        if (sage) {  // dXs = dT W_s^T (self term)
-          GemmPart ps{dT, lddT, wsb, c.po, c.fo, (int)c.wrows_i};
-          GemmEpi es;
-          es.D = L.at<void>(ws, "dxs"); es.ldd = c.pi;
-          WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), &ps, 1, es, nullptr, 0, st));
-        }
       }
     }
     if (post && d.need_dx) {

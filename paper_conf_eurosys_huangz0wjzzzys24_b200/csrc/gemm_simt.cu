@@ -78,8 +78,11 @@ __global__ void __launch_bounds__(256) k_gemm_nt(NTArgs a) {
       if (e.bias) v += e.bias[n];
       if (e.relu) v = fmaxf(v, 0.f);
       if (e.mask_ref && !(tof<T>(static_cast<const T*>(e.mask_ref)[m * e.ld_mask + n]) > 0.f)) v = 0.f;
-      if (e.d_f32) static_cast<float*>(e.D)[m * e.ldd + n] = v;
-      else static_cast<T*>(e.D)[m * e.ldd + n] = (T)v;
+      void* Dp = e.D;
+      int64_t ld = e.ldd, nn = n;
+      if (e.D2 && n >= e.n_split) { Dp = e.D2; ld = e.ldd2; nn = n - e.n_split; }
+      if (e.d_f32) static_cast<float*>(Dp)[m * ld + nn] = v;
+      else static_cast<T*>(Dp)[m * ld + nn] = (T)v;
     }
   }
 }

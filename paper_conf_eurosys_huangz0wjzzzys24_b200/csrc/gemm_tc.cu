@@ -35,6 +35,7 @@ struct TcParams {
   int BN;         // MMA N (multiple of 16, <= 256)
   int stages;
   int nparts;
+  int n_tiles;
   int kblocks[3];
   int64_t k_base; // TN: first K row of split z = blockIdx.z * k_span
   int64_t k_span;
@@ -170,8 +171,9 @@ __global__ void __launch_bounds__(128, 1)
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   const uint32_t tmem = *tmem_slot;
 
-  const int64_t m0 = (int64_t)blockIdx.x * BM;
-  const int n0 = blockIdx.y * BN;
+  // NT: 1-D grid, N tiles of one M tile adjacent (the A tile is re-read from L2)
+  const int64_t m0 = MN ? (int64_t)blockIdx.x * BM : (int64_t)(blockIdx.x / p.n_tiles) * BM;
+  const int n0 = MN ? blockIdx.y * BN : (int)(blockIdx.x % p.n_tiles) * BN;
   int total_kb = 0;
   for (int i = 0; i < p.nparts; ++i) total_kb += p.kblocks[i];
   const int64_t kz = MN ? p.k_base + (int64_t)blockIdx.z * p.k_span : 0;
@@ -276,12 +278,15 @@ __global__ void __launch_bounds__(128, 1)
 #pragma unroll
         for (int i = 0; i < 8; ++i) f[i] = t[i] > 0.f ? f[i] : 0.f;
       }
+      void* Dp = e.D;
+      int64_t ld = e.ldd, nn = n;
+      if (e.D2 && n >= e.n_split) { Dp = e.D2; ld = e.ldd2; nn = n - e.n_split; }
       if (e.d_f32) {
-        float* o = static_cast<float*>(e.D) + m * e.ldd + n;
+        float* o = static_cast<float*>(Dp) + m * ld + nn;
 #pragma unroll
         for (int i = 0; i < 8; ++i) o[i] = f[i];
       } else {
-        *reinterpret_cast<int4*>(static_cast<__nv_bfloat16*>(e.D) + m * e.ldd + n) = bf16x8_pack(f);
+        *reinterpret_cast<int4*>(static_cast<__nv_bfloat16*>(Dp) + m * ld + nn) = bf16x8_pack(f);
       }
     }
   }
@@ -364,7 +369,7 @@ bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_part
   CUtensorMap maps[6];
   memset(maps, 0, sizeof(maps));
   TcParams p{};
-  p.M = M; p.N = N; p.BN = BN; p.nparts = n_parts; p.epi = epi;
+  p.M = M; p.N = N; p.BN = BN; p.nparts = n_parts; p.epi = epi; p.n_tiles = n_tiles;
   for (int i = 0; i < n_parts; ++i) {
     const GemmPart& q = parts[i];
     if (!make_map(&maps[2 * i], q.A, (uint64_t)q.K, (uint64_t)M, (uint64_t)q.lda * 2, BK, BM)) return false;
@@ -377,7 +382,7 @@ bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_part
   int stages = 4;
   while (stages > 2 && smem_bytes(false, BN, stages) > 110 * 1024) --stages;
   p.stages = stages;
-  dim3 grid((unsigned)cdiv(M, BM), (unsigned)n_tiles, 1);
+  dim3 grid((unsigned)(cdiv(M, BM) * n_tiles), 1, 1);
   double kt = 0;
   for (int i = 0; i < n_parts; ++i) kt += parts[i].K;
   ProfScope ps(PK_TC_NT, s, (double)M * (kt + N + (epi.addend ? N : 0) + (epi.mask_ref ? N : 0)) * 2.0,

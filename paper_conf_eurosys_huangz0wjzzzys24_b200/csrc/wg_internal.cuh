@@ -201,6 +201,8 @@ struct GemmEpi {
   int64_t ld_mask = 0;
   void* D = nullptr; int64_t ldd = 0; // output (conv dtype unless d_f32)
   int d_f32 = 0;
+  // split output: columns >= n_split go to D2 (column n - n_split); n_split % 16 == 0
+  void* D2 = nullptr; int64_t ldd2 = 0; int n_split = 0;
 };
 wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts,
                   const GemmEpi& epi, void* scratch, size_t scratch_bytes, cudaStream_t s);

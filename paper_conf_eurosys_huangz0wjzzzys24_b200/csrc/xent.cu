@@ -63,6 +63,47 @@ __global__ void __launch_bounds__(256) k_xent(int64_t M, int C, const T* x, int6
   }
 }
 
+// small C: one thread per row (the row is one contiguous <= 256-byte read; no shuffles)
+template <typename T, int CMAX>
+__global__ void __launch_bounds__(256) k_xent_row(int64_t M, int C, const T* x, int64_t ld, const int64_t* labels,
+                                                  float scale, T* dx, int64_t ldd, float* part) {
+  __shared__ float wsum[8];
+  const int Cpad = (C + 7) / 8 * 8;
+  float lsum = 0.f;
+  for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < M; r += (int64_t)gridDim.x * blockDim.x) {
+    float v[CMAX];
+    float m = -INFINITY;
+#pragma unroll
+    for (int j = 0; j < CMAX; ++j) {
+      v[j] = j < C ? ld_f<T>(x + r * ld + j) : -INFINITY;
+      m = fmaxf(m, v[j]);
+    }
+    const int64_t lab = labels[r];
+    float s = 0.f, t_lab = 0.f;
+#pragma unroll
+    for (int j = 0; j < CMAX; ++j) {
+      const float t = j < C ? v[j] - m : 0.f;
+      if (j == lab) t_lab = t;
+      v[j] = j < C ? __expf(t) : 0.f;
+      s += v[j];
+    }
+    const float inv = 1.f / s;
+#pragma unroll
+    for (int j = 0; j < CMAX; ++j)
+      if (j < Cpad) dx[r * ldd + j] = (T)(j < C ? scale * (v[j] * inv - (j == lab ? 1.f : 0.f)) : 0.f);
+    lsum += scale * (logf(s) - t_lab);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) lsum += __shfl_xor_sync(0xffffffffu, lsum, o);
+  if ((threadIdx.x & 31) == 0) wsum[threadIdx.x >> 5] = lsum;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float t = 0.f;
+    for (int w = 0; w < 8; ++w) t += wsum[w];
+    part[blockIdx.x] = t;
+  }
+}
+
 __global__ void k_sum(const float* part, int n, float* out) {
   if (threadIdx.x == 0 && blockIdx.x == 0) {
     float t = 0.f;
@@ -94,6 +135,17 @@ extern "C" wg_status wg_softmax_xent(wg_dtype dtype, int64_t M, int32_t C, const
   ProfScope ps(PK_MISC, s, (double)M * C * (dtype == WG_BF16 ? 4.0 : 8.0) + M * 8.0, 0.0);
   float* part = static_cast<float*>(scratch);
   const int per = (C + 31) / 32;
+  if (C <= 64) {
+    const unsigned nb = (unsigned)std::min<int64_t>(XENT_BLKS, std::max<int64_t>(1, cdiv(M, 256)));
+    if (dtype == WG_BF16)
+      WG_LAUNCH((k_xent_row<__nv_bfloat16, 64>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld, labels, scale,
+                (__nv_bfloat16*)dlogits, ldd, part);
+    else
+      WG_LAUNCH((k_xent_row<float, 64>), nb, 256, 0, s, M, C, (const float*)logits, ld, labels, scale,
+                (float*)dlogits, ldd, part);
+    WG_LAUNCH(k_sum, 1, 32, 0, s, part, (int)nb, loss_out);
+    return WG_OK;
+  }
   if (dtype == WG_BF16) {
     if (per <= 2) return run<__nv_bfloat16, 2>(M, C, logits, ld, labels, scale, dlogits, ldd, loss_out, part, s);
     if (per <= 8) return run<__nv_bfloat16, 8>(M, C, logits, ld, labels, scale, dlogits, ldd, loss_out, part, s);
