@@ -320,6 +320,7 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
   float* part_smem = reinterpret_cast<float*>(ring + (size_t)D * NV * WARPS * 32);  // [W][2][SLOTF]
   int* key_ring = reinterpret_cast<int*>(part_smem + (size_t)W * 2 * SLOTF);       // [W][D]
   float* sc_ring = reinterpret_cast<float*>(key_ring + W * D);                      // [W][D]
+  int* idx_ring = reinterpret_cast<int*>(sc_ring + W * D);                          // [NR+1][256]
   __shared__ int slot_row[W][2];
 
   const WorkItem it = a.items[blockIdx.x];
@@ -342,20 +343,23 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
     if (cb < ce) {
       // ---- producer state: next round to issue starts at `prod`
       int64_t prod = cb;
-      // source ids of the next NQ rounds, prefetched so the producer never waits
-      // on an index load (rounds are RS-aligned from cb)
-      constexpr int NQ = 3;
-      int pq[NQ];
-#pragma unroll
-      for (int k = 0; k < NQ; ++k) {
-        const int64_t e = prod + (int64_t)k * RS + l;
-        pq[k] = (e < ce && l < RS) ? a.idx[e] : 0;
-      }
-      int pidx = pq[0];
+      // Source ids ride the same cp.async pipeline NR rounds ahead of the row
+      // copies (per-lane ring of NR+1 rounds; rounds are RS-aligned from cb):
+      // the producer never waits on a synchronous index load.
+      auto iload = [&](int round) {
+        const int64_t e = cb + (int64_t)round * RS + l;
+        const bool ok = l < RS && e < ce;
+        cp_async4(idx_ring + (round % (NR + 1)) * (WARPS * 32) + threadIdx.x, a.idx + (ok ? e : cb), ok);
+      };
+#pragma unroll 1
+      for (int r = 0; r < NR; ++r) iload(r);
+      cp_async_commit();
+      cp_async_wait<0>();
       int round_issued = 0;
       auto issue = [&]() {
         const int n = (int)min((int64_t)RS, ce - prod);
         const int slot0 = (round_issued % NR) * RS;
+        const int pidx = idx_ring[(round_issued % (NR + 1)) * (WARPS * 32) + threadIdx.x];
 #pragma unroll
         for (int u = 0; u < RS; ++u) {
           const int s = __shfl_sync(gmask, pidx, u, LPE);
@@ -374,16 +378,10 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
           if (a.gscale) cp_async4(sr + slot0 + l, a.gscale + pidx, ok);
           else if (a.escale) cp_async4(sr + slot0 + l, a.escale + (ok ? prod + l : eb), ok);
         }
+        iload(round_issued + NR);
         cp_async_commit();
         prod += n;
         ++round_issued;
-#pragma unroll
-        for (int k = 0; k < NQ - 1; ++k) pq[k] = pq[k + 1];
-        {
-          const int64_t e = prod + (int64_t)(NQ - 1) * RS + l;
-          pq[NQ - 1] = (e < ce && l < RS) ? a.idx[e] : 0;
-        }
-        pidx = pq[0];
       };
 #pragma unroll 1
       for (int r = 0; r < NR; ++r) {
@@ -535,7 +533,7 @@ wg_status launch_cp(const AggArgs& a, int VPR, cudaStream_t s) {
   constexpr int EPV = VT<T>::EPV;
   constexpr int W = WARPS * (32 / LPE), D = NR * RS;
   const size_t smem = (size_t)D * NV * WARPS * 32 * 16 + (size_t)W * 2 * LPE * NV * EPV * sizeof(float) +
-                      (size_t)W * D * 8;
+                      (size_t)W * D * 8 + (size_t)(NR + 1) * WARPS * 32 * 4;
   static bool done = false;
   if (!done) {
     cudaFuncSetAttribute(k_agg_cp<T, LPE, NV, RS, NR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);

@@ -63,35 +63,47 @@ __global__ void __launch_bounds__(256) k_xent(int64_t M, int C, const T* x, int6
   }
 }
 
-// small C: one thread per row (the row is one contiguous <= 256-byte read; no shuffles)
-template <typename T, int CMAX>
+// small C: groups of 8 lanes per row (4 rows per warp in flight), lane j holds
+// columns j, j+8, ..., reductions are 3-step shuffles inside the group
+template <typename T, int PER>
 __global__ void __launch_bounds__(256) k_xent_row(int64_t M, int C, const T* x, int64_t ld, const int64_t* labels,
                                                   float scale, T* dx, int64_t ldd, float* part) {
   __shared__ float wsum[8];
   const int Cpad = (C + 7) / 8 * 8;
+  const int lane = threadIdx.x & 31, g = lane >> 3, l = lane & 7;
+  const unsigned gm = 0xffu << (g * 8);
   float lsum = 0.f;
-  for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < M; r += (int64_t)gridDim.x * blockDim.x) {
-    float v[CMAX];
+  const int64_t rows_per_iter = (int64_t)gridDim.x * (blockDim.x / 8);
+  for (int64_t r = blockIdx.x * (int64_t)(blockDim.x / 8) + (threadIdx.x >> 3); r < M; r += rows_per_iter) {
+    float v[PER];
     float m = -INFINITY;
 #pragma unroll
-    for (int j = 0; j < CMAX; ++j) {
-      v[j] = j < C ? ld_f<T>(x + r * ld + j) : -INFINITY;
-      m = fmaxf(m, v[j]);
+    for (int k = 0; k < PER; ++k) {
+      const int j = l + 8 * k;
+      v[k] = j < C ? ld_f<T>(x + r * ld + j) : -INFINITY;
+      m = fmaxf(m, v[k]);
     }
+#pragma unroll
+    for (int o = 4; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(gm, m, o, 8));
     const int64_t lab = labels[r];
     float s = 0.f, t_lab = 0.f;
 #pragma unroll
-    for (int j = 0; j < CMAX; ++j) {
-      const float t = j < C ? v[j] - m : 0.f;
+    for (int k = 0; k < PER; ++k) {
+      const int j = l + 8 * k;
+      const float t = j < C ? v[k] - m : 0.f;
       if (j == lab) t_lab = t;
-      v[j] = j < C ? __expf(t) : 0.f;
-      s += v[j];
+      v[k] = j < C ? __expf(t) : 0.f;
+      s += v[k];
     }
+#pragma unroll
+    for (int o = 4; o; o >>= 1) s += __shfl_xor_sync(gm, s, o, 8);
     const float inv = 1.f / s;
 #pragma unroll
-    for (int j = 0; j < CMAX; ++j)
-      if (j < Cpad) dx[r * ldd + j] = (T)(j < C ? scale * (v[j] * inv - (j == lab ? 1.f : 0.f)) : 0.f);
-    lsum += scale * (logf(s) - t_lab);
+    for (int k = 0; k < PER; ++k) {
+      const int j = l + 8 * k;
+      if (j < Cpad) dx[r * ldd + j] = (T)(j < C ? scale * (v[k] * inv - (j == lab ? 1.f : 0.f)) : 0.f);
+      if (j == lab) lsum += scale * (logf(s) - t_lab);
+    }
   }
 #pragma unroll
   for (int o = 16; o; o >>= 1) lsum += __shfl_xor_sync(0xffffffffu, lsum, o);
@@ -136,12 +148,12 @@ extern "C" wg_status wg_softmax_xent(wg_dtype dtype, int64_t M, int32_t C, const
   float* part = static_cast<float*>(scratch);
   const int per = (C + 31) / 32;
   if (C <= 64) {
-    const unsigned nb = (unsigned)std::min<int64_t>(XENT_BLKS, std::max<int64_t>(1, cdiv(M, 256)));
+    const unsigned nb = (unsigned)std::min<int64_t>(XENT_BLKS, std::max<int64_t>(1, cdiv(M, 32)));
     if (dtype == WG_BF16)
-      WG_LAUNCH((k_xent_row<__nv_bfloat16, 64>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld, labels, scale,
+      WG_LAUNCH((k_xent_row<__nv_bfloat16, 8>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld, labels, scale,
                 (__nv_bfloat16*)dlogits, ldd, part);
     else
-      WG_LAUNCH((k_xent_row<float, 64>), nb, 256, 0, s, M, C, (const float*)logits, ld, labels, scale,
+      WG_LAUNCH((k_xent_row<float, 8>), nb, 256, 0, s, M, C, (const float*)logits, ld, labels, scale,
                 (float*)dlogits, ldd, part);
     WG_LAUNCH(k_sum, 1, 32, 0, s, part, (int)nb, loss_out);
     return WG_OK;
