@@ -337,65 +337,76 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
   int* kr = key_ring + worker * D;
   float* sr = sc_ring + worker * D;
 
+  // Every worker of the CTA runs the same number of rounds (chunk lengths
+  // differ by at most one edge): control flow is warp-uniform, so all warp
+  // primitives use the full mask, and ring slots advance by wrap-around
+  // counters (no divisions in the loop).
+  const int64_t maxlen = (len + W - 1) / W;
+  const int nrounds = (int)((maxlen + RS - 1) / RS);
+  const int irb = (int)rb;
+  const int lbase = grp * LPE;
+  constexpr int TPB = WARPS * 32;
+  constexpr int RSTRIDE = NV * TPB;            // int4 per ring slot (one edge)
+  int4* my_ring = ring + threadIdx.x;
+  int* my_iring = idx_ring + threadIdx.x;
+  const bool scaled = a.gscale || a.escale;
+  (void)gmask;
+
   for (int cv0 = 0; cv0 < VPR; cv0 += CW) {
     const int nvec = min(CW, VPR - cv0);
     if (l == 0) { slot_row[worker][0] = -1; slot_row[worker][1] = -1; }
-    if (cb < ce) {
-      // ---- producer state: next round to issue starts at `prod`
-      int64_t prod = cb;
+    if (nrounds > 0) {
       // Source ids ride the same cp.async pipeline NR rounds ahead of the row
-      // copies (per-lane ring of NR+1 rounds; rounds are RS-aligned from cb):
-      // the producer never waits on a synchronous index load.
-      auto iload = [&](int round) {
+      // copies (per-lane ring of NR+1 rounds; rounds are RS-aligned from cb).
+      auto iload = [&](int round, int islot) {
         const int64_t e = cb + (int64_t)round * RS + l;
         const bool ok = l < RS && e < ce;
-        cp_async4(idx_ring + (round % (NR + 1)) * (WARPS * 32) + threadIdx.x, a.idx + (ok ? e : cb), ok);
+        cp_async4(my_iring + islot * TPB, a.idx + (ok ? e : eb), ok);
       };
 #pragma unroll 1
-      for (int r = 0; r < NR; ++r) iload(r);
+      for (int r = 0; r < NR; ++r) iload(r, r);
       cp_async_commit();
       cp_async_wait<0>();
-      int round_issued = 0;
+      int islot_w = NR, islot_r = 0, pslot = 0, issued = 0;
+      int64_t prod = cb;
       auto issue = [&]() {
-        const int n = (int)min((int64_t)RS, ce - prod);
-        const int slot0 = (round_issued % NR) * RS;
-        const int pidx = idx_ring[(round_issued % (NR + 1)) * (WARPS * 32) + threadIdx.x];
+        const int n = (int)max((int64_t)0, min((int64_t)RS, ce - prod));
+        const int pidx = my_iring[islot_r * TPB];
 #pragma unroll
         for (int u = 0; u < RS; ++u) {
-          const int s = __shfl_sync(gmask, pidx, u, LPE);
+          const int s = __shfl_sync(0xffffffffu, pidx, lbase + u);
           const T* row = tab + (int64_t)s * a.ld_tab + (int64_t)cv0 * EPV;
 #pragma unroll
           for (int q = 0; q < NV; ++q) {
             const int vi = l + q * LPE;
-            cp_async16(ring + ((size_t)(slot0 + u) * NV + q) * (WARPS * 32) + threadIdx.x, row + vi * EPV,
-                       u < n && vi < nvec);
+            cp_async16(my_ring + (pslot + u) * RSTRIDE + q * TPB, row + vi * EPV, u < n && vi < nvec);
           }
         }
         if (l < RS) {
           const bool ok = l < n;
-          if (split) { if (ok) kr[slot0 + l] = (int)(it.row_lo + rb); }
-          else cp_async4(kr + slot0 + l, a.key + (ok ? prod + l : eb), ok);
-          if (a.gscale) cp_async4(sr + slot0 + l, a.gscale + pidx, ok);
-          else if (a.escale) cp_async4(sr + slot0 + l, a.escale + (ok ? prod + l : eb), ok);
+          if (split) { if (ok) kr[pslot + l] = (int)(it.row_lo + rb); }
+          else cp_async4(kr + pslot + l, a.key + (ok ? prod + l : eb), ok);
+          if (a.gscale) cp_async4(sr + pslot + l, a.gscale + pidx, ok);
+          else if (a.escale) cp_async4(sr + pslot + l, a.escale + (ok ? prod + l : eb), ok);
         }
-        iload(round_issued + NR);
+        iload(issued + NR, islot_w);
         cp_async_commit();
-        prod += n;
-        ++round_issued;
+        islot_w = islot_w == NR ? 0 : islot_w + 1;
+        islot_r = islot_r == NR ? 0 : islot_r + 1;
+        pslot = pslot + RS == D ? 0 : pslot + RS;
+        prod += RS;
+        ++issued;
       };
 #pragma unroll 1
-      for (int r = 0; r < NR; ++r) {
-        if (prod < ce) issue();
-        else { cp_async_commit(); ++round_issued; }
-      }
+      for (int r = 0; r < NR; ++r) issue();
       float acc[NV][EPV];
 #pragma unroll
       for (int q = 0; q < NV; ++q)
 #pragma unroll
         for (int i = 0; i < EPV; ++i) acc[q][i] = 0.f;
-      int cur = split ? it.row_lo : (int)(a.key[cb] - rb);
+      int cur = cb < ce ? (split ? it.row_lo : (int)(a.key[cb] - rb)) : -1;
       bool first = true;
-      const bool first_cont = split ? (cb > eb) : (a.row_ptr[cur] < cb);
+      const bool first_cont = cb < ce && (split ? (cb > eb) : (a.row_ptr[cur] < cb));
       auto flush = [&](int row, bool as_cont, bool as_owner) {
         if (as_cont || as_owner) {
           const int s = as_cont ? 0 : 1;
@@ -413,44 +424,40 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
           }
         }
       };
-      int64_t cons = cb;
-      int round = 0;
+      int cslot = 0;
 #pragma unroll 1
-      while (cons < ce) {
+      for (int r = 0; r < nrounds; ++r) {
         cp_async_wait<NR - 1>();
-        __syncwarp(gmask);
-        const int n = (int)min((int64_t)RS, ce - cons);
-        const int slot0 = (round % NR) * RS;
+        __syncwarp();
+        const int n = (int)max((int64_t)0, min((int64_t)RS, ce - (cb + (int64_t)r * RS)));
 #pragma unroll
         for (int u = 0; u < RS; ++u) {
-          if (u >= n) break;
-          const int rk = split ? it.row_lo : kr[slot0 + u] - (int)rb;
-          const float sc = (a.gscale || a.escale) ? sr[slot0 + u] : 1.f;
-          if (rk != cur) {
-            flush(cur, first && first_cont, false);
-            first = false;
-            cur = rk;
+          if (u < n) {
+            const int rk = split ? it.row_lo : kr[cslot + u] - irb;
+            const float sc = scaled ? sr[cslot + u] : 1.f;
+            if (rk != cur) {
+              flush(cur, first && first_cont, false);
+              first = false;
+              cur = rk;
 #pragma unroll
-            for (int q = 0; q < NV; ++q)
+              for (int q = 0; q < NV; ++q)
 #pragma unroll
-              for (int i = 0; i < EPV; ++i) acc[q][i] = 0.f;
-          }
+                for (int i = 0; i < EPV; ++i) acc[q][i] = 0.f;
+            }
 #pragma unroll
-          for (int q = 0; q < NV; ++q) {
-            const int4 v = ring[((size_t)(slot0 + u) * NV + q) * (WARPS * 32) + threadIdx.x];
-            VT<T>::add(acc[q], v, sc);
+            for (int q = 0; q < NV; ++q) VT<T>::add(acc[q], my_ring[(cslot + u) * RSTRIDE + q * TPB], sc);
           }
         }
-        cons += n;
-        ++round;
-        __syncwarp(gmask);
-        if (prod < ce) issue();
-        else { cp_async_commit(); ++round_issued; }
+        cslot = cslot + RS == D ? 0 : cslot + RS;
+        __syncwarp();
+        issue();
       }
       cp_async_wait<0>();
-      const bool last_open = split ? (ce < ee) : (a.row_ptr[cur + 1] > ce);
-      if (first && first_cont) flush(cur, true, false);
-      else flush(cur, false, last_open);
+      if (cb < ce) {
+        const bool last_open = split ? (ce < ee) : (a.row_ptr[cur + 1] > ce);
+        if (first && first_cont) flush(cur, true, false);
+        else flush(cur, false, last_open);
+      }
     }
     __syncthreads();
     if (cb < ce && slot_row[worker][1] >= 0) {

@@ -23,3 +23,8 @@ if [[ $mode == ncu || $mode == all ]]; then
       python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_gemm_run.log 2>&1
   ls -la gpurun_out/*.ncu-rep
 fi
+if [[ $mode == ncuagg ]]; then
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_agg_cp -s 5 -c 1 -o gpurun_out/prof_agg1 -f \
+      python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_agg1.log 2>&1
+  ls -la gpurun_out/prof_agg1.ncu-rep
+fi

@@ -18,8 +18,8 @@ def main(path):
     out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(out.splitlines()))
     hdr, units = rows[0], rows[1]
-    stall_cols = [i for i, h in enumerate(hdr) if h.startswith("smsp__average_warp_latency_issue_stalled_") or
-                  (h.startswith("smsp__warp_issue_stalled_") and h.endswith("_per_warp_active.pct"))]
+    stall_cols = [i for i, h in enumerate(hdr) if h.startswith("smsp__average_warps_issue_stalled_") and
+                  h.endswith("_per_issue_active.ratio")]
     for r in rows[2:]:
         print("----")
         for w in WANT:
