@@ -430,6 +430,16 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
         cp_async_wait<NR - 1>();
         __syncwarp();
         const int n = (int)max((int64_t)0, min((int64_t)RS, ce - (cb + (int64_t)r * RS)));
+        // fast path: a full round inside the current row (edges are sorted by
+        // row, so first == last == cur implies all) -> branch-free accumulate
+        if (n == RS && (split || (kr[cslot] - irb == cur && kr[cslot + RS - 1] - irb == cur))) {
+#pragma unroll
+          for (int u = 0; u < RS; ++u) {
+            const float sc = scaled ? sr[cslot + u] : 1.f;
+#pragma unroll
+            for (int q = 0; q < NV; ++q) VT<T>::add(acc[q], my_ring[(cslot + u) * RSTRIDE + q * TPB], sc);
+          }
+        } else {
 #pragma unroll
         for (int u = 0; u < RS; ++u) {
           if (u < n) {
@@ -447,6 +457,7 @@ __global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
 #pragma unroll
             for (int q = 0; q < NV; ++q) VT<T>::add(acc[q], my_ring[(cslot + u) * RSTRIDE + q * TPB], sc);
           }
+        }
         }
         cslot = cslot + RS == D ? 0 : cslot + RS;
         __syncwarp();
@@ -566,7 +577,19 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
   if (VPR <= 1) return launch_cfg<T, 1, 1, 1>(a, VPR, s);
   if (VPR <= 2) return launch_cfg<T, 2, 1, 2>(a, VPR, s);
   if (VPR <= 4) return launch_cfg<T, 4, 1, 4>(a, VPR, s);
-  if (!use_v2()) {
+  static int cfg = -1;
+  if (cfg < 0) {
+    const char* e = getenv("WG_AGG_CFG");
+    cfg = e ? atoi(e) : 0;
+  }
+  if (!use_v2() && cfg == 1) {   // finer rounds
+    if (VPR <= 8) return launch_cp<T, 8, 1, 4, 6>(a, VPR, s);
+    if (VPR <= 16) return launch_cp<T, 16, 1, 4, 6>(a, VPR, s);
+    if (VPR <= 32) return launch_cp<T, 32, 1, 4, 6>(a, VPR, s);
+  } else if (!use_v2() && cfg == 2) {   // 2 vectors per lane for wide rows
+    if (VPR <= 8) return launch_cp<T, 8, 1, 7, 3>(a, VPR, s);
+    if (VPR <= 32) return launch_cp<T, 16, 2, 4, 3>(a, VPR, s);
+  } else if (!use_v2()) {
     if (VPR <= 8) return launch_cp<T, 8, 1, 7, 3>(a, VPR, s);
     if (VPR <= 16) return launch_cp<T, 16, 1, 7, 3>(a, VPR, s);
     if (VPR <= 32) return launch_cp<T, 32, 1, 7, 3>(a, VPR, s);
