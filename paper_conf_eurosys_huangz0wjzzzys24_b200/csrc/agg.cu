@@ -582,13 +582,14 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
     const char* e = getenv("WG_AGG_CFG");
     cfg = e ? atoi(e) : 0;
   }
-  if (!use_v2() && cfg == 1) {   // finer rounds
-    if (VPR <= 8) return launch_cp<T, 8, 1, 4, 6>(a, VPR, s);
-    if (VPR <= 16) return launch_cp<T, 16, 1, 4, 6>(a, VPR, s);
-    if (VPR <= 32) return launch_cp<T, 32, 1, 4, 6>(a, VPR, s);
-  } else if (!use_v2() && cfg == 2) {   // 2 vectors per lane for wide rows
-    if (VPR <= 8) return launch_cp<T, 8, 1, 7, 3>(a, VPR, s);
-    if (VPR <= 32) return launch_cp<T, 16, 2, 4, 3>(a, VPR, s);
+  if (!use_v2() && cfg == 1) {   // coarser rounds, double buffered
+    if (VPR <= 8) return launch_cp<T, 8, 1, 8, 2>(a, VPR, s);
+    if (VPR <= 16) return launch_cp<T, 16, 1, 10, 2>(a, VPR, s);
+    if (VPR <= 32) return launch_cp<T, 32, 1, 10, 2>(a, VPR, s);
+  } else if (!use_v2() && cfg == 2) {   // deep ring, one CTA per SM
+    if (VPR <= 8) return launch_cp<T, 8, 1, 8, 4>(a, VPR, s);
+    if (VPR <= 16) return launch_cp<T, 16, 1, 14, 3>(a, VPR, s);
+    if (VPR <= 32) return launch_cp<T, 32, 1, 14, 3>(a, VPR, s);
   } else if (!use_v2()) {
     if (VPR <= 8) return launch_cp<T, 8, 1, 7, 3>(a, VPR, s);
     if (VPR <= 16) return launch_cp<T, 16, 1, 7, 3>(a, VPR, s);
