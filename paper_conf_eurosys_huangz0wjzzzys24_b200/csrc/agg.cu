@@ -306,8 +306,8 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
-template <typename T, int LPE, int NV, int RS, int NR>
-__global__ void __launch_bounds__(WARPS * 32, 2) k_agg_cp(AggArgs a, int VPR) {
+template <typename T, int LPE, int NV, int RS, int NR, int MINB = 2>
+__global__ void __launch_bounds__(WARPS * 32, MINB) k_agg_cp(AggArgs a, int VPR) {
   constexpr int EPV = VT<T>::EPV;
   constexpr int G = 32 / LPE;
   constexpr int W = WARPS * G;
@@ -546,7 +546,7 @@ wg_status launch_cfg(const AggArgs& a, int VPR, cudaStream_t s) {
   return WG_OK;
 }
 
-template <typename T, int LPE, int NV, int RS, int NR>
+template <typename T, int LPE, int NV, int RS, int NR, int MINB = 2>
 wg_status launch_cp(const AggArgs& a, int VPR, cudaStream_t s) {
   constexpr int EPV = VT<T>::EPV;
   constexpr int W = WARPS * (32 / LPE), D = NR * RS;
@@ -554,10 +554,10 @@ wg_status launch_cp(const AggArgs& a, int VPR, cudaStream_t s) {
                       (size_t)W * D * 8 + (size_t)(NR + 1) * WARPS * 32 * 4;
   static bool done = false;
   if (!done) {
-    cudaFuncSetAttribute(k_agg_cp<T, LPE, NV, RS, NR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(k_agg_cp<T, LPE, NV, RS, NR, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     done = true;
   }
-  WG_LAUNCH((k_agg_cp<T, LPE, NV, RS, NR>), a.n_items, WARPS * 32, smem, s, a, VPR);
+  WG_LAUNCH((k_agg_cp<T, LPE, NV, RS, NR, MINB>), a.n_items, WARPS * 32, smem, s, a, VPR);
   return WG_OK;
 }
 
@@ -582,14 +582,14 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
     const char* e = getenv("WG_AGG_CFG");
     cfg = e ? atoi(e) : 0;
   }
-  if (!use_v2() && cfg == 1) {   // coarser rounds, double buffered
-    if (VPR <= 8) return launch_cp<T, 8, 1, 8, 2>(a, VPR, s);
-    if (VPR <= 16) return launch_cp<T, 16, 1, 10, 2>(a, VPR, s);
-    if (VPR <= 32) return launch_cp<T, 32, 1, 10, 2>(a, VPR, s);
-  } else if (!use_v2() && cfg == 2) {   // deep ring, one CTA per SM
-    if (VPR <= 8) return launch_cp<T, 8, 1, 8, 4>(a, VPR, s);
-    if (VPR <= 16) return launch_cp<T, 16, 1, 14, 3>(a, VPR, s);
-    if (VPR <= 32) return launch_cp<T, 32, 1, 14, 3>(a, VPR, s);
+  if (!use_v2() && cfg == 1) {   // 3 CTAs / SM, ring 6 x 2
+    if (VPR <= 8) return launch_cp<T, 8, 1, 6, 2, 3>(a, VPR, s);
+    if (VPR <= 16) return launch_cp<T, 16, 1, 6, 2, 3>(a, VPR, s);
+    if (VPR <= 32) return launch_cp<T, 32, 1, 6, 2, 3>(a, VPR, s);
+  } else if (!use_v2() && cfg == 2) {   // 3 CTAs / SM, ring 4 x 3
+    if (VPR <= 8) return launch_cp<T, 8, 1, 4, 3, 3>(a, VPR, s);
+    if (VPR <= 16) return launch_cp<T, 16, 1, 4, 3, 3>(a, VPR, s);
+    if (VPR <= 32) return launch_cp<T, 32, 1, 4, 3, 3>(a, VPR, s);
   } else if (!use_v2()) {
     if (VPR <= 8) return launch_cp<T, 8, 1, 7, 3>(a, VPR, s);
     if (VPR <= 16) return launch_cp<T, 16, 1, 7, 3>(a, VPR, s);
