@@ -582,18 +582,20 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
     const char* e = getenv("WG_AGG_CFG");
     cfg = e ? atoi(e) : 0;
   }
-  if (!use_v2() && cfg == 1) {   // 3 CTAs / SM, ring 6 x 2
+  if (!use_v2() && cfg == 1) {   // 3 CTAs / SM, ring 5 x 2
+    if (VPR <= 8) return launch_cp<T, 8, 1, 5, 2, 3>(a, VPR, s);
+    if (VPR <= 16) return launch_cp<T, 16, 1, 5, 2, 3>(a, VPR, s);
+    if (VPR <= 32) return launch_cp<T, 32, 1, 5, 2, 3>(a, VPR, s);
+  } else if (!use_v2() && cfg == 2) {   // 4 CTAs / SM, ring 4 x 2
+    if (VPR <= 8) return launch_cp<T, 8, 1, 4, 2, 4>(a, VPR, s);
+    if (VPR <= 16) return launch_cp<T, 16, 1, 4, 2, 4>(a, VPR, s);
+    if (VPR <= 32) return launch_cp<T, 32, 1, 4, 2, 4>(a, VPR, s);
+  } else if (!use_v2()) {
+    // default: 3 CTAs (24 warps) per SM, 12 edges in flight per worker
+    // (A/B on C4: 7x3 @ 2 CTAs/SM 72 %, 6x2 @ 3 CTAs/SM 82 % of HBM)
     if (VPR <= 8) return launch_cp<T, 8, 1, 6, 2, 3>(a, VPR, s);
     if (VPR <= 16) return launch_cp<T, 16, 1, 6, 2, 3>(a, VPR, s);
     if (VPR <= 32) return launch_cp<T, 32, 1, 6, 2, 3>(a, VPR, s);
-  } else if (!use_v2() && cfg == 2) {   // 3 CTAs / SM, ring 4 x 3
-    if (VPR <= 8) return launch_cp<T, 8, 1, 4, 3, 3>(a, VPR, s);
-    if (VPR <= 16) return launch_cp<T, 16, 1, 4, 3, 3>(a, VPR, s);
-    if (VPR <= 32) return launch_cp<T, 32, 1, 4, 3, 3>(a, VPR, s);
-  } else if (!use_v2()) {
-    if (VPR <= 8) return launch_cp<T, 8, 1, 7, 3>(a, VPR, s);
-    if (VPR <= 16) return launch_cp<T, 16, 1, 7, 3>(a, VPR, s);
-    if (VPR <= 32) return launch_cp<T, 32, 1, 7, 3>(a, VPR, s);
   } else {
     if (VPR <= 8) return launch_cfg<T, 8, 1, 4>(a, VPR, s);
     if (VPR <= 16) return launch_cfg<T, 16, 1, 4>(a, VPR, s);
