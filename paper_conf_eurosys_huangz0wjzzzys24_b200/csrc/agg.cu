@@ -591,11 +591,12 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
     if (VPR <= 16) return launch_cp<T, 16, 1, 4, 2, 4>(a, VPR, s);
     if (VPR <= 32) return launch_cp<T, 32, 1, 4, 2, 4>(a, VPR, s);
   } else if (!use_v2()) {
-    // default: 3 CTAs (24 warps) per SM, 12 edges in flight per worker
-    // (A/B on C4: 7x3 @ 2 CTAs/SM 72 %, 6x2 @ 3 CTAs/SM 82 % of HBM)
-    if (VPR <= 8) return launch_cp<T, 8, 1, 6, 2, 3>(a, VPR, s);
-    if (VPR <= 16) return launch_cp<T, 16, 1, 6, 2, 3>(a, VPR, s);
-    if (VPR <= 32) return launch_cp<T, 32, 1, 6, 2, 3>(a, VPR, s);
+    // default: 3 CTAs (24 warps) per SM, 10 edges in flight per worker
+    // (A/B on C4: 7x3 @ 2 CTAs/SM 72 %, 6x2 @ 3/SM 83 %, 5x2 @ 3/SM 84.5 %,
+    //  4x2 @ 4/SM 82 % of HBM)
+    if (VPR <= 8) return launch_cp<T, 8, 1, 5, 2, 3>(a, VPR, s);
+    if (VPR <= 16) return launch_cp<T, 16, 1, 5, 2, 3>(a, VPR, s);
+    if (VPR <= 32) return launch_cp<T, 32, 1, 5, 2, 3>(a, VPR, s);
   } else {
     if (VPR <= 8) return launch_cfg<T, 8, 1, 4>(a, VPR, s);
     if (VPR <= 16) return launch_cfg<T, 16, 1, 4>(a, VPR, s);
