@@ -196,6 +196,14 @@ typedef struct {
   void* workspace;
   void* xchg;
   int64_t ld_xchg;
+  /* Fusion of adjacent layers (optional, NULL / 0 = off):
+   * dx_mask: dx is written already multiplied by [dx_mask > 0] (the ReLU of
+   *          the layer that produced x), row-major [owned rows x ld_dx_mask];
+   * dy_masked: dy already carries this layer's fused-ReLU mask (as produced
+   *          by the next layer's dx_mask), so y is not read.               */
+  const void* dx_mask;
+  int64_t ld_dx_mask;
+  int32_t dy_masked;
 } wg_bwd_args;
 
 wg_status wg_conv_forward(wg_plan p, const wg_params* params, const wg_fwd_args* a, wg_stream stream);

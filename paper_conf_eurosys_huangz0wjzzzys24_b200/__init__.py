@@ -241,7 +241,9 @@ class Conv:
         return y, saved
 
     def backward_raw(self, dy, x, y, saved, params: dict, dx=None, phase=C.PHASE_ALL, xchg=None, stream=None,
-                     grads: dict | None = None):
+                     grads: dict | None = None, dx_mask=None, dy_masked: bool = False):
+        """dx_mask: write dx already multiplied by [dx_mask > 0] (fusing the previous
+        layer's ReLU backward); dy_masked: dy already carries this layer's ReLU mask."""
         dev = dy.device
         if grads is None:
             grads = {n: torch.empty_like(params[n], dtype=torch.float32) for n in PARAM_NAMES
@@ -252,7 +254,8 @@ class Conv:
         gr = C.Grads(*[_ptr(grads.get(n)) for n in PARAM_NAMES])
         a = C.BwdArgs(phase, _ptr(dy), ld_of(dy), _ptr(x), ld_of(x), _ptr(y), ld_of(y) if y is not None else 0,
                       _ptr(saved), _ptr(dx), ld_of(dx) if dx is not None else 0, _ptr(self.workspace),
-                      _ptr(xchg), ld_of(xchg) if xchg is not None else 0)
+                      _ptr(xchg), ld_of(xchg) if xchg is not None else 0,
+                      _ptr(dx_mask), ld_of(dx_mask) if dx_mask is not None else 0, int(dy_masked))
         C.check(C.lib().wg_conv_backward(self._h, ctypes.byref(pr), ctypes.byref(a), ctypes.byref(gr),
                                          _stream(stream)), "wg_conv_backward")
         return dx, grads

@@ -68,7 +68,8 @@ class FwdArgs(ctypes.Structure):
 
 class BwdArgs(ctypes.Structure):
     _fields_ = [("phase", i32), ("dy", P), ("lddy", i64), ("x", P), ("ldx", i64), ("y", P), ("ldy", i64),
-                ("saved", P), ("dx", P), ("lddx", i64), ("workspace", P), ("xchg", P), ("ld_xchg", i64)]
+                ("saved", P), ("dx", P), ("lddx", i64), ("workspace", P), ("xchg", P), ("ld_xchg", i64),
+                ("dx_mask", P), ("ld_dx_mask", i64), ("dy_masked", i32)]
 
 
 class WGError(RuntimeError):

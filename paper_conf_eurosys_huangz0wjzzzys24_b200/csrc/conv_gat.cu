@@ -651,6 +651,7 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
                          GemmPart{dGlo, p->po, w, p->po, HF, (int)rup(d.f_in, 16)}};
     GemmEpi e;
     e.D = A->dx; e.ldd = A->lddx;
+    e.mask_ref = A->dx_mask; e.ld_mask = A->ld_dx_mask;
     WG_TRY(gemm_nt(d.dtype, nr, (int)rup(d.f_in, 16 / s), parts, dGlo ? 2 : 1, e, nullptr, 0, st));
   }
   return WG_OK;

@@ -266,9 +266,11 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   const bool sage = d.model == WG_SAGE, gin = d.model == WG_GIN;
   const bool pre = A->phase != WG_PHASE_POST, post = A->phase != WG_PHASE_PRE;
   WG_REQ(P && P->W && A->dy && A->x && A->workspace, WG_ERR_INVALID, "backward: null argument");
-  WG_REQ(!d.fuse_relu || A->y, WG_ERR_INVALID, "fuse_relu backward needs y");
+  WG_REQ(!d.fuse_relu || A->y || A->dy_masked, WG_ERR_INVALID, "fuse_relu backward needs y");
   WG_REQ(!d.need_dx || A->dx, WG_ERR_INVALID, "need_dx but dx is NULL");
   WG_REQ(p->n_edge_tasks == 0 || A->saved, WG_ERR_INVALID, "saved is NULL");
+  // dy already masked by the next layer (dx_mask fusion): no mask pass here
+  const bool mask_dy = d.fuse_relu && !A->dy_masked;
   const bool dist = c.nr != c.Vg;
   void* ws = A->workspace;
   const Layout& L = p->ws;
@@ -296,11 +298,11 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   void* dt_buf = nullptr;
   int64_t ld_dtb = c.po;
   if (gpath_lin && xchg) { dt_buf = off(xchg, c.vb, A->ld_xchg, c.s); ld_dtb = A->ld_xchg; }
-  else if (d.fuse_relu) { dt_buf = off(L.at<void>(ws, "dt"), c.vb, c.po, c.s); ld_dtb = c.po; }
+  else if (mask_dy) { dt_buf = off(L.at<void>(ws, "dt"), c.vb, c.po, c.s); ld_dtb = c.po; }
   if (pre) {
     float* db = gin ? (G ? G->b2 : nullptr) : (G ? G->bias : nullptr);
     if (dt_buf || db)
-      WG_TRY(bias_grad_mask(c.dt, c.nr, c.fo, A->dy, A->lddy, d.fuse_relu ? A->y : nullptr, A->ldy, dt_buf, ld_dtb,
+      WG_TRY(bias_grad_mask(c.dt, c.nr, c.fo, A->dy, A->lddy, mask_dy ? A->y : nullptr, A->ldy, dt_buf, ld_dtb,
                             db, colsum, st));
   }
   const void* dT = dt_buf ? dt_buf : A->dy;
@@ -364,6 +366,7 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
       if (sage) { a.self_tab = L.at<void>(ws, "dxs"); a.ld_self = c.pi; a.self_coef = 1.f; }
       if (gin) { a.self_tab = off(dtab, c.vb, ldd, c.s); a.ld_self = ldd; a.self_coef = 1.f + d.gin_eps; }
       a.out = A->dx; a.ld_out = A->lddx;
+      a.mask_ref = A->dx_mask; a.ld_mask = A->ld_dx_mask;
       a.partial = L.at<float>(ws, "partT"); a.ld_part = pl;
       a.F = c.fi;
       WG_TRY(run_agg(c, a, p->bt, st));
@@ -392,6 +395,7 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
     if (sage) parts[np++] = GemmPart{dT, lddT, wsb, c.po, c.fo, (int)c.wrows_i};
     GemmEpi e;
     e.D = A->dx; e.ldd = A->lddx;
+    e.mask_ref = A->dx_mask; e.ld_mask = A->ld_dx_mask;
     WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), parts, np, e, nullptr, 0, st));
   }
   return WG_OK;

@@ -544,6 +544,7 @@ wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, 
     a.table = dxt; a.ld_tab = p->pi;
     a.self_tab = dxs; a.ld_self = p->pi;
     a.out = A->dx; a.ld_out = A->lddx;
+    a.mask_ref = A->dx_mask; a.ld_mask = A->ld_dx_mask;
     a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
     a.F = d.f_in;
     WG_TRY(run(dt, a, rp->b3, st));

@@ -104,23 +104,29 @@ class GNNStack:
         self.x = x
         return self._own(self.h[self.L])
 
+    fuse_masks = True
+
     def backward(self, dlogits):
         g = dlogits
+        masked = False
         for i in reversed(range(self.L)):
             c = self.convs[i]
             xin = self.x if i == 0 else self.h[i]
             dx = self._own(self.dx[i]) if i > 0 else None
             y = self._own(self.h[i + 1])
+            # fuse layer i-1's ReLU backward into layer i's dx epilogue
+            fuse = self.fuse_masks and i > 0 and getattr(self.convs[i - 1], "fuse_relu", False)
+            kw = dict(grads=self.grads[i], dy_masked=masked,
+                      dx_mask=self._own(self.h[i]) if fuse else None)
             if self.dist:
                 xb = self.xchg_b[i]
-                c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, phase=C.PHASE_PRE, xchg=xb,
-                               grads=self.grads[i])
+                c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, phase=C.PHASE_PRE, xchg=xb, **kw)
                 self._allgather(xb)
-                c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, phase=C.PHASE_POST, xchg=xb,
-                               grads=self.grads[i])
+                c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, phase=C.PHASE_POST, xchg=xb, **kw)
             else:
-                c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, grads=self.grads[i])
+                c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, **kw)
             g = dx
+            masked = fuse
         if self.dist:
             flat = torch.cat([v.reshape(-1) for gr in self.grads for v in gr.values()])
             torch.distributed.all_reduce(flat, group=self.group)

@@ -79,7 +79,14 @@ class FakeSage:
         return y, saved
 
     @torch.no_grad()
-    def backward_raw(self, dy, x, y, saved, params, dx=None, phase=0, xchg=None, grads=None, stream=None):
+    def backward_raw(self, dy, x, y, saved, params, dx=None, phase=0, xchg=None, grads=None, stream=None,
+                     dx_mask=None, dy_masked=False):
+        dx, grads = self._backward(dy, x, y, saved, params, dx, phase, xchg, grads)
+        if dx is not None and dx_mask is not None and phase != 1:
+            dx *= (dx_mask > 0)
+        return dx, grads
+
+    def _backward(self, dy, x, y, saved, params, dx, phase, xchg, grads):
         Ws, Wn = params["W_self"].double(), params["W"].double()
         xo = x[self.vb:self.ve]
         dT = dy * (y > 0) if self.fuse_relu else dy

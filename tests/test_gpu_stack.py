@@ -103,6 +103,30 @@ def test_1d_partition_phases_match_single(model, policy, P):
         assert rel_err(f64(tot), f64(gr1[k])) < 1e-5, k
 
 
+def test_stack_relu_fusion_is_exact():
+    """dx_mask / dy_masked fusion (adjacent layers) changes no value."""
+    m = wg()
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack
+    V, E = 3000, 40000
+    src, dst, _ = synth.make_graph(V, E, seed=43, alpha=0.6, symmetric=True)
+    g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V)
+    x = m.padded(V, 24, torch.bfloat16)
+    x.copy_(torch.from_numpy(synth.make_features(V, 24, seed=44)))
+    dl = m.padded(V, 6, torch.bfloat16)
+    dl.copy_(torch.from_numpy(synth.normal((V, 6), seed=45)))
+    out = []
+    for fuse in (False, True):
+        st = GNNStack(g, "sage", [24, 40, 40, 6], dtype=torch.bfloat16, seed=5)
+        st.fuse_masks = fuse
+        st.forward(x)
+        st.backward(dl)
+        torch.cuda.synchronize()
+        out.append([{k: v.clone() for k, v in gr.items()} for gr in st.grads])
+    for a, b in zip(*out):
+        for k in a:
+            assert torch.equal(a[k], b[k]), k
+
+
 def test_stack_training_decreases_loss():
     m = wg()
     from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack
