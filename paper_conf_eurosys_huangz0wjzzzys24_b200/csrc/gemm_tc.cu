@@ -358,11 +358,20 @@ wg_status launch(dim3 grid, size_t smem, const CUtensorMap* maps, const TcParams
 
 }  // namespace
 
+bool tc_make_map(CUtensorMap* m, const void* ptr, uint64_t inner, uint64_t outer, uint64_t ld_bytes, uint32_t box_in,
+                 uint32_t box_out) {
+  return make_map(m, ptr, inner, outer, ld_bytes, box_in, box_out);
+}
+
+bool tc_gemm_nt_persistent(int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi, cudaStream_t s,
+                           wg_status* st);
+
 bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi,
                 cudaStream_t s, wg_status* st) {
   if (dt != WG_BF16 || !tc_enabled() || n_parts > 3 || M <= 0) return false;
   for (int i = 0; i < n_parts; ++i)
     if (parts[i].tile_group) return false;   // grouped B: CUDA-core path (TODO: per-tile B coordinate)
+  if (tc_gemm_nt_persistent(M, N, parts, n_parts, epi, s, st)) return true;
   const int n_tiles = (int)cdiv(N, 256);
   const int BN = (int)rup(cdiv(N, n_tiles), 16);
   if (BN > 256) return false;
