@@ -331,9 +331,10 @@ bool tc_gemm_nt_persistent(int64_t M, int N, const GemmPart* parts, int n_parts,
     disabled = (e && e[0] == '1') ? 1 : 0;
   }
   if (disabled || epi.d_f32 || n_parts > 3 || M <= 0) return false;
+  // several N tiles: BN = 256 so every 64-column store box stays inside its
+  // tile (the ragged end is clipped by the tensor map); one tile: BN = N
   const int n_tiles = (int)cdiv(N, 256);
-  const int BN = (int)rup(cdiv(N, n_tiles), 16);
-  if (BN > 256) return false;
+  const int BN = n_tiles > 1 ? 256 : (int)rup(N, 16);
   if (epi.D2 && (epi.n_split % BN != 0)) return false;   // split must fall on a tile boundary
   CUtensorMap maps[10];
   memset(maps, 0, sizeof(maps));
