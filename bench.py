@@ -11,6 +11,11 @@ all-reduce (N > 1), Adam step.  value = layers * E / step time (whole job).
 
     python bench.py [--gpus N --steps K --warmup W] [--impl reference]
     torchrun --nproc-per-node N bench.py --gpus N        (1-D dst partition)
+    python bench.py --config C1|C2|C3 [--model ...]      (the other configs' models:
+        C1 GCN fp32, C2 GAT 4 heads fp32, C3 RGCN R=128 fp32, C4 --model gin)
+
+The default line (no flags) is the driver's: C4 SAGE.  The other configs are
+the parity cases of BASELINE.json, measured the same way (profiles/r01/).
 
 Timing: CUDA events on the compute stream, barrier + synchronize on both sides,
 max over ranks; inputs (features 490 MB, tables >= 1.2 GB) exceed the 126 MB
@@ -52,7 +57,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C4")
-    ap.add_argument("--model", default="sage", choices=["sage", "gin", "gcn"])
+    ap.add_argument("--model", default=None, choices=["sage", "gin", "gcn", "gat", "rgcn"],
+                    help="default: the config's model (C4: sage)")
     ap.add_argument("--policy", default="auto")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
@@ -60,21 +66,36 @@ def parse():
     return ap.parse_args()
 
 
+def conv_options(c, model):
+    """Per-model layer options of the workload (readings Q1-Q6)."""
+    if model == "rgcn":     # the usual R-GCN layer: 1/|N_v^r| normalisation, self-loop W_0, bias (Q2 options)
+        return {"norm": "right", "self_loop": True}
+    return {}
+
+
 def workload(cfg_name, model):
     import synth
     c = synth.CONFIGS[cfg_name]
-    return c, {"workload": f"{cfg_name}: {model} {len(c.dims) - 1}-layer {'-'.join(map(str, c.dims))} on synthetic "
-                           f"{c.note.split(',')[0]} ({c.V} V, {c.E} E)",
-               "V": c.V, "E": c.E, "dims": list(c.dims), "model": model, "alpha": c.alpha,
-               "symmetric": c.symmetric, "seed": c.seed}
+    model = model or c.model
+    extra = {}
+    if model == "gat":
+        extra["heads"] = c.heads
+    if model == "rgcn":
+        extra.update(R=c.R, zipf_s=c.zipf_s, **conv_options(c, model))
+    return c, model, {"workload": f"{cfg_name}: {model} {len(c.dims) - 1}-layer {'-'.join(map(str, c.dims))} on "
+                                  f"synthetic {c.note.split(',')[0]} ({c.V} V, {c.E} E)",
+                      "V": c.V, "E": c.E, "dims": list(c.dims), "model": model, "alpha": c.alpha,
+                      "symmetric": c.symmetric, "seed": c.seed, "features": c.xdist, **extra}
 
 
-def make_inputs(c):
+def make_inputs(c, model):
     import synth
-    src, dst, _ = synth.make_graph(c.V, c.E, seed=c.seed * 16, alpha=c.alpha, symmetric=c.symmetric)
-    x = synth.make_features(c.V, c.dims[0], seed=c.seed * 16 + 2)
+    R = c.R if model == "rgcn" else 1
+    src, dst, et = synth.make_graph(c.V, c.E, seed=c.seed * 16, alpha=c.alpha, symmetric=c.symmetric, R=R,
+                                    zipf_s=c.zipf_s)
+    x = synth.make_features(c.V, c.dims[0], seed=c.seed * 16 + 2, dist=c.xdist, p=c.xp)
     labels = np.random.Generator(np.random.Philox(c.seed * 16 + 5)).integers(0, c.dims[-1], c.V).astype(np.int64)
-    return src, dst, x, labels
+    return src, dst, et, x, labels
 
 
 class Clocks:
@@ -117,7 +138,14 @@ class Clocks:
                 "samples": len(sm)}
 
 
-def cpu_baseline(c, src, dst, x, model, budget_s):
+def layer_shapes(c, model):
+    """(f_in, f_out, concat) of each layer: GAT hidden layers read heads * dims[i] columns."""
+    L = len(c.dims) - 1
+    return [((c.heads * c.dims[i] if (model == "gat" and i > 0) else c.dims[i]), c.dims[i + 1], i < L - 1)
+            for i in range(L)]
+
+
+def cpu_baseline(c, model, src, dst, et, budget_s):
     """The oracle (plain C, fp64, 1 thread) on a bounded sample: every in-edge
     of a seeded random sample of destination rows (its induced star graph),
     one forward + backward per layer shape of the workload."""
@@ -125,8 +153,9 @@ def cpu_baseline(c, src, dst, x, model, budget_s):
     rng = np.random.Generator(np.random.Philox(c.seed * 16 + 9))
     order = np.argsort(dst, kind="stable")
     indptr = np.concatenate([[0], np.cumsum(np.bincount(dst, minlength=c.V))])
-    dims = c.dims
-    per_edge = sum(dims[i] * dims[i + 1] for i in range(len(dims) - 1)) * 2 * 3  # fwd+bwd flops per edge
+    shapes = layer_shapes(c, model)
+    H = c.heads if model == "gat" else 1
+    per_edge = sum(fi * fo * H for fi, fo, _ in shapes) * 2 * 3      # ~ fwd+bwd flops per edge (per-edge messages)
     target_edges = max(200, int(budget_s * 1.2e9 / per_edge))
     rows, n = [], 0
     for v in rng.permutation(c.V):
@@ -141,23 +170,34 @@ def cpu_baseline(c, src, dst, x, model, budget_s):
     s, d = src[eids], dst[eids]
     verts, inv = np.unique(np.concatenate([s, d]), return_inverse=True)
     s2, d2 = inv[:len(s)].astype(np.int32), inv[len(s):].astype(np.int32)
+    t2 = et[eids].astype(np.int32) if (model == "rgcn" and et is not None) else None
     Vs = len(verts)
     t_total = 0.0
-    for i in range(len(dims) - 1):
-        fi, fo = dims[i], dims[i + 1]
-        xs = np.random.default_rng(i).standard_normal((Vs, fi))
-        W1 = np.random.default_rng(10 + i).standard_normal((fi, fo)) * 0.05
-        W2 = np.random.default_rng(20 + i).standard_normal((fi, fo)) * 0.05
-        dy = np.random.default_rng(30 + i).standard_normal((Vs, fo))
+    for i, (fi, fo, concat) in enumerate(shapes):
+        r = lambda k, *sh: np.random.default_rng(10 * k + i).standard_normal(sh)
+        xs = r(0, Vs, fi)
         t0 = time.perf_counter()
         if model == "sage":
-            oracle.sage_forward(s2, d2, Vs, xs, W2, W1, np.zeros(fo))
-            oracle.sage_backward(s2, d2, Vs, xs, W2, W1, dy)
+            oracle.sage_forward(s2, d2, Vs, xs, 0.05 * r(1, fi, fo), 0.05 * r(2, fi, fo), np.zeros(fo))
+            oracle.sage_backward(s2, d2, Vs, xs, 0.05 * r(1, fi, fo), 0.05 * r(2, fi, fo), r(3, Vs, fo))
+        elif model == "gcn":
+            oracle.gcn_forward(s2, d2, Vs, xs, 0.05 * r(1, fi, fo), np.zeros(fo))
+            oracle.gcn_backward(s2, d2, Vs, xs, 0.05 * r(1, fi, fo), r(3, Vs, fo))
+        elif model == "gin":
+            W1, W2 = 0.05 * r(1, fi, fo), 0.05 * r(2, fo, fo)
+            oracle.gin_forward(s2, d2, Vs, xs, W1, np.zeros(fo), W2, np.zeros(fo))
+            oracle.gin_backward(s2, d2, Vs, xs, W1, np.zeros(fo), W2, r(3, Vs, fo))
+        elif model == "gat":
+            W, al, ar = 0.05 * r(1, fi, H * fo), 0.1 * r(2, H, fo), 0.1 * r(4, H, fo)
+            oracle.gat_forward(s2, d2, Vs, xs, W, al, ar, None, heads=H, concat=concat)
+            oracle.gat_backward(s2, d2, Vs, xs, W, al, ar, r(3, Vs, H * fo if concat else fo), heads=H,
+                                concat=concat)
         else:
-            oracle.gcn_forward(s2, d2, Vs, xs, W1, np.zeros(fo))
-            oracle.gcn_backward(s2, d2, Vs, xs, W1, dy)
+            W, W0 = 0.05 * r(1, c.R, fi, fo), 0.05 * r(2, fi, fo)
+            oracle.rgcn_forward(s2, d2, t2, Vs, xs, W, W0, np.zeros(fo), norm="right")
+            oracle.rgcn_backward(s2, d2, t2, Vs, xs, W, r(3, Vs, fo), W0, norm="right")
         t_total += time.perf_counter() - t0
-    L = len(dims) - 1
+    L = len(shapes)
     return {"value": L * len(eids) / t_total, "unit": "edges/s", "cores": 1, "kind": "oracle",
             "sample": f"all {len(eids)} in-edges of {len(rows)} random dst rows (induced star graph, {Vs} V), "
                       f"fwd+bwd of each of the {L} layer shapes, {t_total:.1f} s",
@@ -168,12 +208,12 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    c, cfg = workload(args.config, args.model)
-    src, dst, x, _ = make_inputs(c)
+    c, model, cfg = workload(args.config, args.model)
+    src, dst, et, _, _ = make_inputs(c, model)
     vals = []
     per = max(2.0, 60.0 / max(1, args.steps + args.warmup))
     for i in range(args.warmup + args.steps):
-        r = cpu_baseline(c, src, dst, x, args.model, per)
+        r = cpu_baseline(c, model, src, dst, et, per)
         if i >= args.warmup:
             vals.append(r)
     v = statistics.median([r["value"] for r in vals])
@@ -203,23 +243,28 @@ def main():
     import paper_conf_eurosys_huangz0wjzzzys24_b200 as wg
     from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack, partition_1d
 
-    c, cfg = workload(args.config, args.model)
+    c, model, cfg = workload(args.config, args.model)
     t0 = time.perf_counter()
-    src, dst, x_np, labels_np = make_inputs(c)
+    src, dst, et, x_np, labels_np = make_inputs(c, model)
     t_gen = time.perf_counter() - t0
     dev = torch.device("cuda", local)
+    if world > 1 and model in ("gat", "rgcn"):
+        raise SystemExit("the 1-D multi-GPU partition covers GCN / SAGE / GIN (DESIGN.md §7)")
     block, bounds = partition_1d(c.V, world)
     vb, ve = bounds[rank] if world > 1 else (0, c.V)
     torch.cuda.synchronize()
     t0 = time.perf_counter()
+    R = c.R if model == "rgcn" else 1
     g = wg.Graph(torch.from_numpy(src).to(dev), torch.from_numpy(dst).to(dev), num_vertices=c.V,
+                 etype=torch.from_numpy(et).to(dev) if R > 1 else None, num_types=R,
                  v_begin=vb if world > 1 else 0, v_end=ve if world > 1 else 0)
     torch.cuda.synchronize()
     t_part = time.perf_counter() - t0
     dtype = torch.bfloat16 if c.dtype == "bf16" else torch.float32
     t0 = time.perf_counter()
-    stack = GNNStack(g, args.model, c.dims, dtype=dtype, policy=args.policy, group=group,
-                     block=block if world > 1 else None)
+    stack = GNNStack(g, model, c.dims, dtype=dtype, policy=args.policy, group=group,
+                     block=block if world > 1 else None, heads=c.heads if model == "gat" else 1, R=R,
+                     conv_kw=conv_options(c, model))
     t_plan = time.perf_counter() - t0
     Vtab = stack.Vtab
     x = wg.padded(Vtab, c.dims[0], dtype, dev)
@@ -291,17 +336,22 @@ def main():
                "d2h_bytes_per_step": 4}
 
     pk, pk_src = peaks()
-    agg = prof["gather_reduce"]
+    # dominant kernel class: the most time among classes that report algorithmic bytes
+    # (gather_reduce = k_agg_cp / k_agg, a6 + a10; gat = the GAT edge kernels)
+    dom = max((k for k in prof if prof[k]["bytes"] > 0), key=lambda k: prof[k]["ms"])
+    agg = prof[dom]
     achieved = agg["bytes"] / (agg["ms"] / 1e3) / 1e9 if agg["ms"] > 0 else 0.0
     traffic = None
     tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tf):
         try:
-            traffic = json.load(open(tf)).get(f"{args.config}:{args.model}:gather_reduce")
+            traffic = json.load(open(tf)).get(f"{args.config}:{model}:{dom}")
         except Exception:
             traffic = None
-    step_ms_sum = sum(v["ms"] for v in prof.values()) / args.steps
-    roofline = {"bound": "hbm", "kernel": "k_agg (gather + segment-reduce, a6/a10)", "achieved": achieved,
+    names = {"gather_reduce": "k_agg_cp / k_agg (gather + segment-reduce, a6/a10)",
+             "gat": "GAT edge kernels (logits + online softmax + gather, a6/a10)",
+             "tc_gemm_nt": "tcgen05 GEMM-NT (a5/a7/a9)", "tc_gemm_tn": "tcgen05 GEMM-TN (a11)"}
+    roofline = {"bound": "hbm", "kernel": names.get(dom, dom), "class": dom, "achieved": achieved,
                 "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": achieved / pk["hbm_gbs"], "traffic": traffic,
                 "peak_source": f"{pk_src} (MEASURED_PEAKS.json hbm_gbs)" if pk_src == "measured" else "fallback",
                 "bytes_per_launch": agg["bytes"] / max(1, agg["launches"]),
@@ -312,6 +362,7 @@ def main():
         if v["launches"] == 0:
             continue
         kernels[k] = {"ms_per_step": v["ms"] / args.steps, "launches_per_step": v["launches"] / args.steps,
+                      "enclosing_scope": v["bytes"] == 0 and k in ("rgcn",),
                       "GB/s": v["bytes"] / (v["ms"] / 1e3) / 1e9 if v["ms"] else None,
                       "TFLOP/s": v["flops"] / (v["ms"] / 1e3) / 1e12 if v["ms"] else None}
     line = {"metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": world, "steps": args.steps,
@@ -327,7 +378,7 @@ def main():
             "one_off": {"partition_s": t_part, "plan_s": t_plan, "synth_s": t_gen},
             "clocks": clk, "loss": float(loss.item()), "e2e": e2e}
     if rank == 0 and world == 1 and not args.no_cpu:
-        line["cpu_baseline"] = cpu_baseline(c, src, dst, x_np, args.model, args.cpu_seconds)
+        line["cpu_baseline"] = cpu_baseline(c, model, src, dst, et, args.cpu_seconds)
     elif rank == 0:
         line["cpu_baseline"] = None
     if rank == 0:

@@ -130,6 +130,9 @@ typedef struct {
   int32_t need_dx;          /* backward produces dx (0 for the input layer)      */
 } wg_conv_desc;
 
+/* Errors: WG_ERR_INVALID (bad sizes / model / dtype), WG_ERR_UNSUPPORTED
+ * (typed graph with a non-RGCN model; GAT / RGCN on a graph that owns only
+ * a row block -- the 1-D partition covers GCN / SAGE / GIN).               */
 wg_status wg_plan_create(wg_graph g, const wg_conv_desc* desc, wg_plan* out);
 /* Bytes of the caller-owned `saved` (forward -> backward) and `workspace`
  * buffers; both 256-byte aligned device memory.                            */
@@ -167,7 +170,9 @@ typedef struct {
 /* Phases for the 1-D multi-GPU layer (§8(e)).  Single GPU: WG_PHASE_ALL.
  * PRE computes this rank's rows of the exchange table into
  * `xchg + row_offset * ld_xchg`; the caller all-gathers `xchg` (in place);
- * POST consumes the gathered table.                                        */
+ * POST consumes the gathered table.  GAT and RGCN plans accept only
+ * WG_PHASE_ALL (and only on a full graph, see wg_plan_create):
+ * other phases return WG_ERR_UNSUPPORTED.                                  */
 typedef enum { WG_PHASE_ALL = 0, WG_PHASE_PRE = 1, WG_PHASE_POST = 2 } wg_phase;
 
 typedef struct {

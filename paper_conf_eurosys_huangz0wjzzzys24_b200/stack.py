@@ -26,7 +26,8 @@ class GNNStack:
 
     def __init__(self, graph: Graph, model: str, dims, *, dtype=torch.bfloat16, heads: int = 1, policy="auto",
                  seed: int = 0, lr: float = 1e-3, group=None, block: int | None = None, R: int = 1,
-                 conv_factory=None, device=None):
+                 conv_kw: dict | None = None, conv_factory=None, device=None):
+        # conv_kw: extra Conv options for every layer (e.g. RGCN norm / self_loop).
         # conv_factory / device: injection points for the multi-process CPU test
         # of this orchestration (tests/test_dist_gloo.py); the product path uses
         # Conv (libwg.so) on the graph's CUDA device.
@@ -43,25 +44,30 @@ class GNNStack:
         self.block = block if block is not None else self.rows
         self.Vtab = self.block * self.world if self.dist else graph.V
         self.convs, self.params = [], []
+        # layer i reads a table of width f_in(i): dims[0], then the previous
+        # layer's output width (heads * dims[i] for concatenated GAT heads)
+        self.f_in = [dims[0]] + [heads * dims[i] if model == "gat" else dims[i] for i in range(1, self.L)]
         for i in range(self.L):
             last = i == self.L - 1
-            kw = dict(dtype=dtype, fuse_relu=not last, need_dx=i > 0, seed=seed + i)
+            kw = dict(dtype=dtype, fuse_relu=not last, need_dx=i > 0, seed=seed + i, **(conv_kw or {}))
             if model == "gat":
                 kw.update(heads=heads, concat=not last)
             pol = policy
-            conv = Conv_(graph, model, dims[i], dims[i + 1], policy=pol, **kw)
+            fi = self.f_in[i]
+            conv = Conv_(graph, model, fi, dims[i + 1], policy=pol, **kw)
             if self.dist and conv.n_edge_tasks and conv.n_vertex_tasks:   # uniform plan per layer when distributed
                 pol = "vertex" if conv.n_vertex_tasks > conv.n_edge_tasks else "edge"
                 conv.close()
-                conv = Conv_(graph, model, dims[i], dims[i + 1], policy=pol, **kw)
+                conv = Conv_(graph, model, fi, dims[i + 1], policy=pol, **kw)
             self.convs.append(conv)
-            fo = dims[i + 1] if model != "gat" else (heads * dims[i + 1] if not last else dims[i + 1])
-            self.params.append(init_params(model, dims[i], dims[i + 1], heads=heads, concat=not last, R=R,
+            self.params.append(init_params(model, fi, dims[i + 1], heads=heads, concat=not last, R=R,
+                                           self_loop=bool((conv_kw or {}).get("self_loop", False)),
+                                           bias=bool((conv_kw or {}).get("bias", True)),
                                            device=self.dev, seed=seed + 100 + i))
         # activation tables: h[0] = input, h[i+1] = output of layer i (global rows when distributed)
         self.h = [None] + [padded(self.Vtab, c.out_dim, dtype, self.dev) for c in self.convs]
         self.saved = [c.new_saved() for c in self.convs]
-        self.dx = [None] + [padded(self.Vtab if self.dist else self.rows, dims[i], dtype, self.dev)
+        self.dx = [None] + [padded(self.Vtab if self.dist else self.rows, self.f_in[i], dtype, self.dev)
                             for i in range(1, self.L)]
         self.grads = [{k: torch.zeros_like(v) for k, v in p.items()} for p in self.params]
         self.xchg_f, self.xchg_b = [], []

@@ -127,14 +127,21 @@ def test_stack_relu_fusion_is_exact():
             assert torch.equal(a[k], b[k]), k
 
 
-def test_stack_training_decreases_loss():
+@pytest.mark.parametrize("model", ["sage", "gcn", "gin", "gat", "rgcn"])
+def test_stack_training_decreases_loss(model):
     m = wg()
     from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack
     V, E = 4000, 60000
-    src, dst, _ = synth.make_graph(V, E, seed=41, alpha=0.5, symmetric=True)
-    g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V)
+    R = 6 if model == "rgcn" else 1
+    src, dst, et = synth.make_graph(V, E, seed=41, alpha=0.5, symmetric=R == 1, R=R)
+    g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V,
+                etype=torch.from_numpy(et).cuda() if R > 1 else None, num_types=R)
     dims = [32, 64, 64, 8]
-    st = GNNStack(g, "sage", dims, dtype=torch.bfloat16, lr=1e-2)
+    kw = dict(heads=3) if model == "gat" else dict(R=R, conv_kw={"norm": "right", "self_loop": True}) \
+        if model == "rgcn" else {}
+    st = GNNStack(g, model, dims, dtype=torch.bfloat16, lr=1e-2, **kw)
+    if model == "gat":     # hidden GAT layers read heads * dims[i] columns
+        assert [c.f_in for c in st.convs] == [32, 192, 192] and st.h[1].shape[1] >= 192
     x = m.padded(V, 32, torch.bfloat16)
     x.copy_(torch.from_numpy(synth.make_features(V, 32, seed=42)))
     labels = torch.from_numpy(np.random.default_rng(1).integers(0, 8, V)).cuda()
