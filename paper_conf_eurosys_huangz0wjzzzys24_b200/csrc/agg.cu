@@ -636,14 +636,17 @@ wg_status launch_combine(wg_dtype dt, const CombineArgs& a, cudaStream_t s) {
 namespace {
 
 template <typename T>
-__global__ void k_prep_weight(const float* W, int rows, int cols, int transpose, T* out, int64_t ldo, int out_rows) {
-  // out is [out_rows x ldo]; element (i, j) = transpose ? W[j][i] : W[i][j], 0 outside
-  int64_t n = (int64_t)out_rows * ldo;
+__global__ void k_prep_weight(const float* W, int batch, int rows, int cols, int transpose, T* out, int64_t ldo,
+                              int out_rows) {
+  // out is batch x [out_rows x ldo]; element (b, i, j) = transpose ? W[b][j][i] : W[b][i][j], 0 outside
+  const int64_t n = (int64_t)batch * out_rows * ldo;
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
-    int i = (int)(t / ldo), j = (int)(t % ldo);
+    const int64_t bi = t / ldo;
+    const int b = (int)(bi / out_rows), i = (int)(bi % out_rows), j = (int)(t % ldo);
+    const float* Wb = W + (int64_t)b * rows * cols;
     float v = 0.f;
-    if (transpose) { if (i < cols && j < rows) v = W[(int64_t)j * cols + i]; }
-    else { if (i < rows && j < cols) v = W[(int64_t)i * cols + j]; }
+    if (transpose) { if (i < cols && j < rows) v = Wb[(int64_t)j * cols + i]; }
+    else { if (i < rows && j < cols) v = Wb[(int64_t)i * cols + j]; }
     out[t] = (T)v;
   }
 }
@@ -699,26 +702,23 @@ constexpr int COLSUM_BLKS = 1184;  // 8 x 148 SMs
 
 }  // namespace
 
-wg_status prep_weight(wg_dtype dt, const float* W, int rows, int cols, int transpose, void* out, int64_t ldo,
-                      int out_rows, cudaStream_t s) {
-  int64_t n = (int64_t)out_rows * ldo;
-  unsigned grid = (unsigned)std::min<int64_t>(cdiv(n, 256), 1184);
-  ProfScope ps(PK_MISC, s, (double)rows * cols * 4.0 + (double)n * (dt == WG_BF16 ? 2.0 : 4.0), 0.0);
+wg_status prep_weight_batched(wg_dtype dt, const float* W, int batch, int rows, int cols, int transpose, void* out,
+                              int64_t ldo, int out_rows, cudaStream_t s) {
+  const int64_t n = (int64_t)batch * out_rows * ldo;
+  const unsigned grid = (unsigned)std::min<int64_t>(cdiv(n, 256), 1184);
+  ProfScope ps(PK_MISC, s, (double)batch * rows * cols * 4.0 + (double)n * (dt == WG_BF16 ? 2.0 : 4.0), 0.0);
   if (grid == 0) return WG_OK;
   if (dt == WG_BF16)
-    WG_LAUNCH(k_prep_weight<__nv_bfloat16>, grid, 256, 0, s, W, rows, cols, transpose, (__nv_bfloat16*)out, ldo, out_rows);
+    WG_LAUNCH(k_prep_weight<__nv_bfloat16>, grid, 256, 0, s, W, batch, rows, cols, transpose, (__nv_bfloat16*)out, ldo,
+              out_rows);
   else
-    WG_LAUNCH(k_prep_weight<float>, grid, 256, 0, s, W, rows, cols, transpose, (float*)out, ldo, out_rows);
+    WG_LAUNCH(k_prep_weight<float>, grid, 256, 0, s, W, batch, rows, cols, transpose, (float*)out, ldo, out_rows);
   return WG_OK;
 }
 
-wg_status prep_weight_batched(wg_dtype dt, const float* W, int batch, int rows, int cols, int transpose, void* out,
-                              int64_t ldo, int out_rows, cudaStream_t s) {
-  const int es = dt == WG_BF16 ? 2 : 4;
-  for (int b = 0; b < batch; ++b)
-    WG_TRY(prep_weight(dt, W + (int64_t)b * rows * cols, rows, cols, transpose,
-                       static_cast<char*>(out) + (int64_t)b * out_rows * ldo * es, ldo, out_rows, s));
-  return WG_OK;
+wg_status prep_weight(wg_dtype dt, const float* W, int rows, int cols, int transpose, void* out, int64_t ldo,
+                      int out_rows, cudaStream_t s) {
+  return prep_weight_batched(dt, W, 1, rows, cols, transpose, out, ldo, out_rows, s);
 }
 
 size_t bias_grad_scratch(int64_t M, int N) { return sizeof(float) * (size_t)COLSUM_BLKS * N; }

@@ -48,8 +48,8 @@ struct RgcnPlan {
   CsrExec f1, f3, b1, b3, bg;
   int32_t* tile_type = nullptr;      // [n1 / 128]
   int32_t* tile_typeT = nullptr;     // [n1T / 128]
-  int64_t* group_offT = nullptr;     // device [R+1] transposed group row offsets
-  std::vector<int64_t> h_group_offT;
+  std::vector<int64_t> h_group_offT; // [R+1] transposed group row offsets
+  TnUnits tn;                        // dW_r work units over the transposed groups
 };
 
 template <typename T>
@@ -367,7 +367,18 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
       for (int64_t t = baseT[r] / TILE_M; t < baseT[r + 1] / TILE_M; ++t) tt[t] = r;
     WG_TRY(up(p, tt, &rp->tile_typeT));
     rp->h_group_offT = baseT;
-    WG_TRY(up(p, baseT, &rp->group_offT));
+    {
+      std::vector<int4> units;
+      std::vector<int32_t> uoff;
+      const int64_t tiles = cdiv(d.f_in, 128) * cdiv(d.f_out, d.dtype == WG_F32 ? 128 : 256);
+      make_tn_units(baseT, std::max<int64_t>(R, 4 * 148 / tiles), 128 / dsize(d.dtype), &units, &uoff);
+      int4* du = nullptr;
+      int32_t* duo = nullptr;
+      WG_TRY(up(p, units, &du));
+      WG_TRY(up(p, uoff, &duo));
+      rp->tn.units = du; rp->tn.unit_off = duo;
+      rp->tn.n_units = (int)units.size(); rp->tn.groups = R; rp->tn.align = TILE_M; rp->tn.k_total = baseT[R];
+    }
     std::stable_sort(sc.begin(), sc.end(), [](const SC& a, const SC& b) {
       return a.src != b.src ? a.src < b.src : a.row < b.row;
     });
@@ -401,7 +412,7 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
   W.add("xg", (size_t)rp->n1T * p->pi * s);
   W.add("dxs", (size_t)V * p->pi * s);
   W.add("colsum", bias_grad_scratch(V, (int)p->po));
-  W.add("tn", std::max(gemm_tn_scratch(V, d.f_in, d.f_out), gemm_tn_grouped_scratch(R, d.f_in, d.f_out)));
+  W.add("tn", std::max(gemm_tn_scratch(V, d.f_in, d.f_out), gemm_tn_grouped_scratch(rp->tn.n_units, d.f_in, d.f_out)));
   // the forward gTask work items are not used by RGCN (stage CSRs replace them)
   return WG_OK;
 }
@@ -511,7 +522,7 @@ wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, 
     a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
     a.F = d.f_in;
     WG_TRY(run(dt, a, rp->bg, st));
-    WG_TRY(gemm_tn_grouped(dt, R, rp->group_offT, d.f_in, d.f_out, xg, p->pi, gt, p->po, G->W,
+    WG_TRY(gemm_tn_grouped(dt, rp->tn, d.f_in, d.f_out, xg, p->pi, gt, p->po, G->W,
                            L.at<void>(ws, "tn"), st));
   }
   if (d.self_loop && G && G->W_self)

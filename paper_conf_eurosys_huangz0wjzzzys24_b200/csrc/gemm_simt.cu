@@ -1,6 +1,6 @@
-// CUDA-core (FFMA) GEMMs.  Used for the fp32 path (tf32 tensor cores alone
-// cannot meet the 1e-4 fp32 tolerance) and as the bf16
-// fallback for shapes the tcgen05 kernel does not take.
+// CUDA-core (FFMA) GEMMs: the fallback for shapes / alignments the tcgen05
+// kernels (bf16, and fp32 through 3xTF32) do not take.  Dispatch: gemm_nt /
+// gemm_tn / gemm_tn_grouped try the tensor-core path first.
 #include <algorithm>
 
 #include "wg_internal.cuh"
@@ -9,7 +9,9 @@ namespace wg {
 
 bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi,
                 cudaStream_t s, wg_status* st);
-bool tc_gemm_tn(int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb, float* D,
+bool tc_gemm_tn_grouped(wg_dtype dt, const TnUnits& U, int M, int N, const void* A, int64_t lda, const void* B,
+                        int64_t ldb, float* D, float* part, cudaStream_t s, wg_status* st);
+bool tc_gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb, float* D,
                 float* part, cudaStream_t s, wg_status* st, int acc);
 
 namespace {
@@ -130,17 +132,16 @@ __global__ void __launch_bounds__(256) k_gemm_tn(int64_t K, int M, int N, const 
   }
 }
 
-// grouped: part[g*splits + z] = sum over the z-th K chunk of group g
+// grouped: part[u] = the product over unit u's K rows [u.x, u.x + u.y * kb_rows)
 template <typename T>
-__global__ void __launch_bounds__(256) k_gemm_tn_grouped(const int64_t* off, int splits, int M, int N, const T* A,
-                                                         int64_t lda, const T* B, int64_t ldb, float* part) {
+__global__ void __launch_bounds__(256) k_gemm_tn_units(const int4* units, int kb_rows, int M, int N, const T* A,
+                                                       int64_t lda, const T* B, int64_t ldb, float* part) {
   __shared__ float As[BK][BM + 4];
   __shared__ float Bs[BK][BN + 4];
   const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
   const int m0 = blockIdx.x * BM, n0 = blockIdx.y * BN;
-  const int g = blockIdx.z / splits, z = blockIdx.z % splits;
-  const int64_t g0 = off[g], g1 = off[g + 1], len = g1 - g0;
-  const int64_t kb = g0 + len * z / splits, ke = g0 + len * (z + 1) / splits;
+  const int4 u = units[blockIdx.z];
+  const int64_t kb = u.x, ke = (int64_t)u.x + (int64_t)u.y * kb_rows;
   float acc[4][4] = {};
   for (int64_t k0 = kb; k0 < ke; k0 += BK) {
     for (int t = threadIdx.x; t < BM * BK; t += 256) {
@@ -175,12 +176,12 @@ __global__ void __launch_bounds__(256) k_gemm_tn_grouped(const int64_t* off, int
   }
 }
 
-__global__ void k_group_reduce(const float* part, int groups, int splits, int64_t MN, float* D) {
-  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+__global__ void k_units_reduce(const float* part, const int32_t* unit_off, int groups, int64_t MN, float* D) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= MN * groups) return;
   const int64_t g = i / MN, e = i % MN;
   float s = 0.f;
-  for (int z = 0; z < splits; ++z) s += part[(g * splits + z) * MN + e];
+  for (int u = unit_off[g]; u < unit_off[g + 1]; ++u) s += part[(int64_t)u * MN + e];
   D[i] = s;
 }
 
@@ -207,7 +208,7 @@ wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_pa
   if (M == 0 || N == 0) return WG_OK;
   WG_REQ(n_parts >= 1 && n_parts <= 3, WG_ERR_INVALID, "gemm_nt: 1..3 parts");
   wg_status st = WG_OK;
-  if (dt == WG_BF16 && tc_gemm_nt(dt, M, N, parts, n_parts, epi, s, &st)) return st;
+  if (tc_gemm_nt(dt, M, N, parts, n_parts, epi, s, &st)) return st;
   NTArgs a{};
   a.M = M; a.N = N; a.n_parts = n_parts; a.epi = epi;
   double kt = 0;
@@ -220,26 +221,48 @@ wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_pa
   return WG_OK;
 }
 
-constexpr int GROUP_SPLITS = 4;
-
-size_t gemm_tn_grouped_scratch(int groups, int M, int N) {
-  return sizeof(float) * (size_t)groups * GROUP_SPLITS * M * N;
+void make_tn_units(const std::vector<int64_t>& h_off, int64_t target_units, int kb_rows, std::vector<int4>* units,
+                   std::vector<int32_t>* unit_off) {
+  const int groups = (int)h_off.size() - 1;
+  const int64_t total = h_off.back();
+  const int64_t span = std::max<int64_t>(kb_rows, rup(cdiv(std::max<int64_t>(total, 1), target_units), kb_rows));
+  units->clear();
+  unit_off->assign(groups + 1, 0);
+  for (int g = 0; g < groups; ++g) {
+    (*unit_off)[g] = (int32_t)units->size();
+    for (int64_t k = h_off[g]; k < h_off[g + 1]; k += span) {
+      const int64_t rows = std::min(span, h_off[g + 1] - k);
+      units->push_back(make_int4((int)k, (int)cdiv(rows, kb_rows), g, 0));
+    }
+  }
+  (*unit_off)[groups] = (int32_t)units->size();
 }
 
-wg_status gemm_tn_grouped(wg_dtype dt, int groups, const int64_t* d_off, int M, int N, const void* A, int64_t lda,
-                          const void* B, int64_t ldb, float* D, void* scratch, cudaStream_t s) {
-  if (groups == 0 || M == 0 || N == 0) return WG_OK;
+size_t gemm_tn_grouped_scratch(int n_units, int M, int N) {
+  return sizeof(float) * (size_t)std::max(n_units, 1) * M * N;
+}
+
+wg_status gemm_tn_grouped(wg_dtype dt, const TnUnits& U, int M, int N, const void* A, int64_t lda, const void* B,
+                          int64_t ldb, float* D, void* scratch, cudaStream_t s) {
+  if (U.groups == 0 || M == 0 || N == 0) return WG_OK;
   float* part = static_cast<float*>(scratch);
-  dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN), (unsigned)(groups * GROUP_SPLITS));
-  ProfScope ps(PK_SIMT, s, 0.0, 0.0);
-  if (dt == WG_BF16)
-    WG_LAUNCH(k_gemm_tn_grouped<__nv_bfloat16>, grid, 256, 0, s, d_off, GROUP_SPLITS, M, N, (const __nv_bfloat16*)A,
-              lda, (const __nv_bfloat16*)B, ldb, part);
-  else
-    WG_LAUNCH(k_gemm_tn_grouped<float>, grid, 256, 0, s, d_off, GROUP_SPLITS, M, N, (const float*)A, lda,
-              (const float*)B, ldb, part);
   const int64_t MN = (int64_t)M * N;
-  WG_LAUNCH(k_group_reduce, (unsigned)cdiv(MN * groups, 256), 256, 0, s, part, groups, GROUP_SPLITS, MN, D);
+  if (U.n_units == 0) {
+    WG_CK(cudaMemsetAsync(D, 0, sizeof(float) * MN * U.groups, s));
+    return WG_OK;
+  }
+  wg_status st = WG_OK;
+  if (tc_gemm_tn_grouped(dt, U, M, N, A, lda, B, ldb, D, part, s, &st)) return st;
+  dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN), (unsigned)U.n_units);
+  ProfScope ps(PK_SIMT, s, (double)U.k_total * (M + N) * (dt == WG_BF16 ? 2.0 : 4.0), 2.0 * U.k_total * M * N);
+  const int kb_rows = 128 / (dt == WG_BF16 ? 2 : 4);
+  if (dt == WG_BF16)
+    WG_LAUNCH(k_gemm_tn_units<__nv_bfloat16>, grid, 256, 0, s, U.units, kb_rows, M, N, (const __nv_bfloat16*)A, lda,
+              (const __nv_bfloat16*)B, ldb, part);
+  else
+    WG_LAUNCH(k_gemm_tn_units<float>, grid, 256, 0, s, U.units, kb_rows, M, N, (const float*)A, lda, (const float*)B,
+              ldb, part);
+  WG_LAUNCH(k_units_reduce, (unsigned)cdiv(MN * U.groups, 256), 256, 0, s, part, U.unit_off, U.groups, MN, D);
   return WG_OK;
 }
 
@@ -257,7 +280,7 @@ wg_status gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t l
   float* part = static_cast<float*>(scratch);
   int splits = tn_splits(K, M, N);
   wg_status st = WG_OK;
-  if (dt == WG_BF16 && tc_gemm_tn(K, M, N, A, lda, B, ldb, D, part, s, &st, acc)) return st;
+  if (tc_gemm_tn(dt, K, M, N, A, lda, B, ldb, D, part, s, &st, acc)) return st;
   const int64_t kchunk = rup(cdiv(K, splits), BK);
   splits = (int)cdiv(K, kchunk);
   ProfScope ps(PK_SIMT, s, (double)K * (M + N) * (dt == WG_BF16 ? 2.0 : 4.0), 2.0 * K * M * N);

@@ -40,6 +40,7 @@ struct TcParams {
   int64_t k_base; // TN: first K row of split z = blockIdx.z * k_span
   int64_t k_span;
   int64_t K;      // TN total K
+  const int4* units;  // grouped TN: per blockIdx.z {first K row, k-blocks, -, -}
   GemmEpi epi;
   float* part;    // TN partial output [splits x M x N]
 };
@@ -76,14 +77,16 @@ __device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map
 }
 
 // UMMA shared-memory descriptor (sm100): start>>4 [0,14), LBO>>4 [16,30),
-// SBO>>4 [32,46), version 1 [46,48), layout SWIZZLE_128B = 2 [61,64)
-__device__ __forceinline__ uint64_t umma_desc(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+// SBO>>4 [32,46), version 1 [46,48), layout [61,64): SWIZZLE_128B = 2,
+// SWIZZLE_128B_BASE32B = 1 (the only MN-major layout for 32-bit operands:
+// 32-byte granules, 4-row atoms; TMA CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)
+__device__ __forceinline__ uint64_t umma_desc(uint32_t addr, uint32_t lbo, uint32_t sbo, uint32_t layout = 2) {
   uint64_t d = 0;
   d |= (uint64_t)((addr >> 4) & 0x3FFF);
   d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
   d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;
   d |= (uint64_t)1 << 46;
-  d |= (uint64_t)2 << 61;
+  d |= (uint64_t)layout << 61;
   return d;
 }
 
@@ -133,22 +136,57 @@ __device__ __forceinline__ int4 bf16x8_pack(const float* f) {
   return make_int4((int)w[0], (int)w[1], (int)w[2], (int)w[3]);
 }
 
-template <bool MN>
-__global__ void __launch_bounds__(128, 1)
+__device__ __forceinline__ void umma_tf32(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                          uint32_t accumulate) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n"
+      "}\n" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
+}
+
+__device__ __forceinline__ void mbar_arrive1(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+
+// 3xTF32 operand split: hi = x with the 13 low mantissa bits cleared, lo = x - hi
+__device__ __forceinline__ void split_tf32(uint4& x, uint4& lo) {
+  uint32_t* v = reinterpret_cast<uint32_t*>(&x);
+  uint32_t* l = reinterpret_cast<uint32_t*>(&lo);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t h = v[i] & 0xffffe000u;
+    l[i] = __float_as_uint(__uint_as_float(v[i]) - __uint_as_float(h));
+    v[i] = h;
+  }
+}
+
+// MN: TN variant (both operands MN-major, fp32 partial output).  T = float:
+// 3xTF32 with two extra converter warps (threads 128..191) that split each
+// landed stage into hi (in place) and lo (twin buffer after the stage).
+// Stage depth: 128 / sizeof(T) K elements (one 128-byte swizzle row).
+template <bool MN, typename T>
+__global__ void __launch_bounds__(sizeof(T) == 4 ? 192 : 128, 1)
     k_tc_gemm(const __grid_constant__ CUtensorMap tA0, const __grid_constant__ CUtensorMap tB0,
               const __grid_constant__ CUtensorMap tA1, const __grid_constant__ CUtensorMap tB1,
               const __grid_constant__ CUtensorMap tA2, const __grid_constant__ CUtensorMap tB2, TcParams p) {
+  constexpr bool TF32 = sizeof(T) == 4;
+  constexpr int BKE = 128 / sizeof(T);      // K elements per stage
+  constexpr int CHE = 128 / sizeof(T);      // MN elements per 128-byte chunk
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int BN = p.BN, S = p.stages;
-  const int b_stage = MN ? ((BN + 63) / 64) * BK * 128 : BN * 128;
-  uint8_t* a_smem = smem;
-  uint8_t* b_smem = smem + S * A_STAGE;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(b_smem + S * b_stage);
+  const int b_stage = MN ? ((BN + CHE - 1) / CHE) * BKE * 128 : BN * 128;
+  const int stage = (A_STAGE + b_stage) * (TF32 ? 2 : 1);
+  uint8_t* ring = smem;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(ring + S * stage);
   uint64_t* full = bars;
   uint64_t* empty = bars + 4;
-  uint64_t* accf = bars + 8;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 9);
+  uint64_t* conv = bars + 8;
+  uint64_t* accf = bars + 12;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 13);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   uint32_t tcols = 32;
   while ((int)tcols < BN) tcols <<= 1;
@@ -157,6 +195,7 @@ __global__ void __launch_bounds__(128, 1)
     for (int s = 0; s < S; ++s) {
       mbar_init(smem_u32(&full[s]), 1);
       mbar_init(smem_u32(&empty[s]), 1);
+      mbar_init(smem_u32(&conv[s]), 64);
     }
     mbar_init(smem_u32(accf), 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -176,7 +215,12 @@ __global__ void __launch_bounds__(128, 1)
   const int n0 = MN ? blockIdx.y * BN : (int)(blockIdx.x % p.n_tiles) * BN;
   int total_kb = 0;
   for (int i = 0; i < p.nparts; ++i) total_kb += p.kblocks[i];
-  const int64_t kz = MN ? p.k_base + (int64_t)blockIdx.z * p.k_span : 0;
+  int64_t kz = MN ? p.k_base + (int64_t)blockIdx.z * p.k_span : 0;
+  if (MN && p.units) {          // grouped TN: unit z = {first K row, k-blocks}
+    const int4 u = p.units[blockIdx.z];
+    kz = u.x;
+    total_kb = u.y;
+  }
 
   if (threadIdx.x == 0) {
     // ---------------- TMA producer
@@ -188,105 +232,136 @@ __global__ void __launch_bounds__(128, 1)
       mbar_wait(smem_u32(&empty[s]), ph ^ 1);
       mbar_expect_tx(smem_u32(&full[s]), tx);
       const uint32_t fb = smem_u32(&full[s]);
-      const uint32_t ad = smem_u32(a_smem + s * A_STAGE), bd = smem_u32(b_smem + s * b_stage);
+      const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE;
       if (MN) {
-        const int krow = (int)(kz + (int64_t)kb * BK);
-        tma_load_2d(ad, &tA0, (int)m0, krow, fb);
-        tma_load_2d(ad + BK * 128, &tA0, (int)m0 + 64, krow, fb);
-        for (int j = 0; j * 64 < BN; ++j) tma_load_2d(bd + j * BK * 128, &tB0, n0 + 64 * j, krow, fb);
+        const int krow = (int)(kz + (int64_t)kb * BKE);
+#pragma unroll
+        for (int j = 0; j < BM / CHE; ++j) tma_load_2d(ad + j * BKE * 128, &tA0, (int)m0 + CHE * j, krow, fb);
+        for (int j = 0; j * CHE < BN; ++j) tma_load_2d(bd + j * BKE * 128, &tB0, n0 + CHE * j, krow, fb);
       } else {
         const CUtensorMap* ta = part == 0 ? &tA0 : (part == 1 ? &tA1 : &tA2);
         const CUtensorMap* tb = part == 0 ? &tB0 : (part == 1 ? &tB1 : &tB2);
-        tma_load_2d(ad, ta, kk * BK, (int)m0, fb);
-        tma_load_2d(bd, tb, kk * BK, n0, fb);
+        tma_load_2d(ad, ta, kk * BKE, (int)m0, fb);
+        tma_load_2d(bd, tb, kk * BKE, n0, fb);
         if (++kk == p.kblocks[part]) { kk = 0; ++part; }
       }
     }
   } else if (threadIdx.x == 32) {
     // ---------------- MMA issuer
-    // instruction descriptor: D f32 [4,6)=1, A bf16 [7,10)=1, B bf16 [10,13)=1,
-    // A/B major [15],[16], N>>3 [17,23), M>>4 [24,29)
-    const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((MN ? 1u : 0u) << 15) | ((MN ? 1u : 0u) << 16) |
+    // instruction descriptor: D f32 [4,6)=1, A / B format [7,10) / [10,13)
+    // (bf16 = 1, tf32 = 2), A/B major [15],[16], N>>3 [17,23), M>>4 [24,29)
+    const uint32_t fmt = TF32 ? 2u : 1u;
+    const uint32_t idesc = (1u << 4) | (fmt << 7) | (fmt << 10) | ((MN ? 1u : 0u) << 15) | ((MN ? 1u : 0u) << 16) |
                            ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
     for (int kb = 0; kb < total_kb; ++kb) {
       const int s = kb % S;
       const uint32_t ph = (kb / S) & 1;
-      mbar_wait(smem_u32(&full[s]), ph);
+      mbar_wait(smem_u32(TF32 ? &conv[s] : &full[s]), ph);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-      const uint32_t ad = smem_u32(a_smem + s * A_STAGE), bd = smem_u32(b_smem + s * b_stage);
+      const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE;
+      const uint32_t al = bd + b_stage, bl = al + A_STAGE;
 #pragma unroll
-      for (int k = 0; k < BK / 16; ++k) {
-        uint64_t adesc, bdesc;
-        if (MN) {  // MN-major SW128: LBO = next 64-wide MN chunk, SBO = next 8 K rows
-          adesc = umma_desc(ad + k * 16 * 128, BK * 128, 1024);
-          bdesc = umma_desc(bd + k * 16 * 128, BK * 128, 1024);
-        } else {   // K-major SW128: K step of 16 elements = +32 bytes inside the atom
-          adesc = umma_desc(ad + k * 32, 16, 1024);
-          bdesc = umma_desc(bd + k * 32, 16, 1024);
+      for (int k = 0; k < 4; ++k) {   // 4 MMAs of 32 bytes of K (16 bf16 / 8 tf32)
+        // MN-major: LBO = next 128-byte MN chunk, SBO = next K atom (8 rows
+        // SW128 / 4 rows SW128_BASE32B for tf32); K-major SW128: K step =
+        // +32 bytes inside the atom
+        const uint32_t step = MN ? (uint32_t)(k * (32 / sizeof(T)) * 128) : (uint32_t)(k * 32);
+        const uint32_t lbo = MN ? BKE * 128 : 16;
+        const uint32_t sbo = (MN && TF32) ? 512 : 1024;
+        const uint32_t lay = (MN && TF32) ? 1 : 2;
+        const uint32_t on = (kb | k) != 0 ? 1u : 0u;
+        if constexpr (TF32) {
+          umma_tf32(tmem, umma_desc(ad + step, lbo, sbo, lay), umma_desc(bd + step, lbo, sbo, lay), idesc, on);
+          umma_tf32(tmem, umma_desc(ad + step, lbo, sbo, lay), umma_desc(bl + step, lbo, sbo, lay), idesc, 1u);
+          umma_tf32(tmem, umma_desc(al + step, lbo, sbo, lay), umma_desc(bd + step, lbo, sbo, lay), idesc, 1u);
+        } else {
+          umma_bf16(tmem, umma_desc(ad + step, lbo, sbo, lay), umma_desc(bd + step, lbo, sbo, lay), idesc, on);
         }
-        umma_bf16(tmem, adesc, bdesc, idesc, (kb | k) != 0 ? 1u : 0u);
       }
       umma_commit(smem_u32(&empty[s]));
     }
     umma_commit(smem_u32(accf));
+  } else if (TF32 && warp >= 4) {
+    // ---------------- hi / lo converters
+    const int ct = threadIdx.x - 128;
+    const int n16 = (A_STAGE + b_stage) / 16;
+    for (int kb = 0; kb < total_kb; ++kb) {
+      const int s = kb % S;
+      mbar_wait(smem_u32(&full[s]), (kb / S) & 1);
+      uint4* x = reinterpret_cast<uint4*>(ring + s * stage);
+      uint4* lo = x + n16;
+#pragma unroll 4
+      for (int i = ct; i < n16; i += 64) {
+        uint4 v = x[i], l;
+        split_tf32(v, l);
+        x[i] = v;
+        lo[i] = l;
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      mbar_arrive1(smem_u32(&conv[s]));
+    }
   }
   __syncwarp();
-  // ---------------- epilogue: warp w owns TMEM lanes / tile rows 32w..32w+31
-  mbar_wait(smem_u32(accf), 0);
-  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-  const int r = warp * 32 + lane;
-  const int64_t m = m0 + r;
-  const GemmEpi& e = p.epi;
-  const float rs = (!MN && e.rscale && m < p.M) ? e.rscale[m] : 1.f;
-  for (int c0 = 0; c0 < BN; c0 += 16) {
-    float v[16];
-    tmem_ld16(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0, v);
-    if (m >= p.M) continue;
-    if (MN) {
-      float* out = p.part + (int64_t)blockIdx.z * p.M * p.N + m * p.N;
+  if (warp < 4) {
+    // ---------------- epilogue: warp w owns TMEM lanes / tile rows 32w..32w+31
+    mbar_wait(smem_u32(accf), 0);
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const int r = warp * 32 + lane;
+    const int64_t m = m0 + r;
+    const GemmEpi& e = p.epi;
+    const float rs = (!MN && e.rscale && m < p.M) ? e.rscale[m] : 1.f;
+    for (int c0 = 0; c0 < BN; c0 += 16) {
+      float v[16];
+      tmem_ld16(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0, v);
+      if (m >= p.M) continue;
+      if (MN) {
+        float* out = p.part + (int64_t)blockIdx.z * p.M * p.N + m * p.N;
 #pragma unroll
-      for (int i = 0; i < 16; ++i) {
-        const int n = n0 + c0 + i;
-        if (n < p.N) out[n] = v[i];
+        for (int i = 0; i < 16; ++i) {
+          const int n = n0 + c0 + i;
+          if (n < p.N) out[n] = v[i];
+        }
+        continue;
       }
-      continue;
-    }
+      if constexpr (!TF32) {
 #pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const int n = n0 + c0 + 8 * h;
-      if (n >= p.N) continue;
-      float* f = v + 8 * h;
+        for (int h = 0; h < 2; ++h) {
+          const int n = n0 + c0 + 8 * h;
+          if (n >= p.N) continue;
+          float* f = v + 8 * h;
 #pragma unroll
-      for (int i = 0; i < 8; ++i) f[i] *= rs;
-      if (e.addend) {
-        float t[8];
-        bf16x8_unpack(*reinterpret_cast<const int4*>(static_cast<const __nv_bfloat16*>(e.addend) + m * e.ld_add + n), t);
+          for (int i = 0; i < 8; ++i) f[i] *= rs;
+          if (e.addend) {
+            float t[8];
+            bf16x8_unpack(*reinterpret_cast<const int4*>(static_cast<const __nv_bfloat16*>(e.addend) + m * e.ld_add + n), t);
 #pragma unroll
-        for (int i = 0; i < 8; ++i) f[i] += t[i];
-      }
-      if (e.bias) {
+            for (int i = 0; i < 8; ++i) f[i] += t[i];
+          }
+          if (e.bias) {
 #pragma unroll
-        for (int i = 0; i < 8; ++i) f[i] += (n + i < p.N) ? e.bias[n + i] : 0.f;
-      }
-      if (e.relu) {
+            for (int i = 0; i < 8; ++i) f[i] += (n + i < p.N) ? e.bias[n + i] : 0.f;
+          }
+          if (e.relu) {
 #pragma unroll
-        for (int i = 0; i < 8; ++i) f[i] = fmaxf(f[i], 0.f);
-      }
-      if (e.mask_ref) {
-        float t[8];
-        bf16x8_unpack(*reinterpret_cast<const int4*>(static_cast<const __nv_bfloat16*>(e.mask_ref) + m * e.ld_mask + n), t);
+            for (int i = 0; i < 8; ++i) f[i] = fmaxf(f[i], 0.f);
+          }
+          if (e.mask_ref) {
+            float t[8];
+            bf16x8_unpack(*reinterpret_cast<const int4*>(static_cast<const __nv_bfloat16*>(e.mask_ref) + m * e.ld_mask + n), t);
 #pragma unroll
-        for (int i = 0; i < 8; ++i) f[i] = t[i] > 0.f ? f[i] : 0.f;
-      }
-      void* Dp = e.D;
-      int64_t ld = e.ldd, nn = n;
-      if (e.D2 && n >= e.n_split) { Dp = e.D2; ld = e.ldd2; nn = n - e.n_split; }
-      if (e.d_f32) {
-        float* o = static_cast<float*>(Dp) + m * ld + nn;
+            for (int i = 0; i < 8; ++i) f[i] = t[i] > 0.f ? f[i] : 0.f;
+          }
+          void* Dp = e.D;
+          int64_t ld = e.ldd, nn = n;
+          if (e.D2 && n >= e.n_split) { Dp = e.D2; ld = e.ldd2; nn = n - e.n_split; }
+          if (e.d_f32) {
+            float* o = static_cast<float*>(Dp) + m * ld + nn;
 #pragma unroll
-        for (int i = 0; i < 8; ++i) o[i] = f[i];
-      } else {
-        *reinterpret_cast<int4*>(static_cast<__nv_bfloat16*>(Dp) + m * ld + nn) = bf16x8_pack(f);
+            for (int i = 0; i < 8; ++i) o[i] = f[i];
+          } else {
+            *reinterpret_cast<int4*>(static_cast<__nv_bfloat16*>(Dp) + m * ld + nn) = bf16x8_pack(f);
+          }
+        }
       }
     }
   }
@@ -316,9 +391,10 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
-// 2-D bf16 tensor map, 128-byte swizzle; dims {inner, outer}, row pitch ld_bytes
-bool make_map(CUtensorMap* m, const void* ptr, uint64_t inner, uint64_t outer, uint64_t ld_bytes, uint32_t box_in,
-              uint32_t box_out) {
+// 2-D tensor map, 128-byte swizzle; dims {inner, outer}, row pitch ld_bytes
+bool make_map_t(CUtensorMap* m, CUtensorMapDataType ty, const void* ptr, uint64_t inner, uint64_t outer,
+                uint64_t ld_bytes, uint32_t box_in, uint32_t box_out,
+                CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B) {
   auto fn = encode_fn();
   if (!fn) return false;
   if ((reinterpret_cast<uintptr_t>(ptr) & 15) || (ld_bytes & 15)) return false;
@@ -326,9 +402,13 @@ bool make_map(CUtensorMap* m, const void* ptr, uint64_t inner, uint64_t outer, u
   cuuint64_t strides[1] = {ld_bytes};
   cuuint32_t box[2] = {box_in, box_out};
   cuuint32_t estr[2] = {1, 1};
-  return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box, estr,
-            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+  return fn(m, ty, 2, const_cast<void*>(ptr), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swz,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+bool make_map(CUtensorMap* m, const void* ptr, uint64_t inner, uint64_t outer, uint64_t ld_bytes, uint32_t box_in,
+              uint32_t box_out) {
+  return make_map_t(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, ptr, inner, outer, ld_bytes, box_in, box_out);
 }
 
 int g_tc_disabled = -1;
@@ -340,38 +420,41 @@ bool tc_enabled() {
   return !g_tc_disabled;
 }
 
-size_t smem_bytes(bool mn, int BN, int stages) {
-  const int b_stage = mn ? ((BN + 63) / 64) * BK * 128 : BN * 128;
-  return 1024 + (size_t)stages * (A_STAGE + b_stage) + 128;
+size_t smem_bytes(bool mn, int BN, int stages, int es = 2) {
+  const int che = 128 / es, bke = 128 / es;
+  const int b_stage = mn ? ((BN + che - 1) / che) * bke * 128 : BN * 128;
+  return 1024 + (size_t)stages * (A_STAGE + b_stage) * (es == 4 ? 2 : 1) + 128;
 }
 
-template <bool MN>
+template <bool MN, typename T>
 wg_status launch(dim3 grid, size_t smem, const CUtensorMap* maps, const TcParams& p, cudaStream_t s) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_tc_gemm<MN>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(k_tc_gemm<MN, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr = true;
   }
-  WG_LAUNCH(k_tc_gemm<MN>, grid, 128, smem, s, maps[0], maps[1], maps[2], maps[3], maps[4], maps[5], p);
+  WG_LAUNCH((k_tc_gemm<MN, T>), grid, sizeof(T) == 4 ? 192 : 128, smem, s, maps[0], maps[1], maps[2], maps[3], maps[4],
+            maps[5], p);
   return WG_OK;
 }
 
 }  // namespace
 
-bool tc_make_map(CUtensorMap* m, const void* ptr, uint64_t inner, uint64_t outer, uint64_t ld_bytes, uint32_t box_in,
-                 uint32_t box_out) {
-  return make_map(m, ptr, inner, outer, ld_bytes, box_in, box_out);
+bool tc_make_map_t(CUtensorMap* m, CUtensorMapDataType ty, const void* ptr, uint64_t inner, uint64_t outer,
+                   uint64_t ld_bytes, uint32_t box_in, uint32_t box_out) {
+  return make_map_t(m, ty, ptr, inner, outer, ld_bytes, box_in, box_out);
 }
 
-bool tc_gemm_nt_persistent(int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi, cudaStream_t s,
-                           wg_status* st);
+bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi,
+                           cudaStream_t s, wg_status* st);
 
 bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi,
                 cudaStream_t s, wg_status* st) {
-  if (dt != WG_BF16 || !tc_enabled() || n_parts > 3 || M <= 0) return false;
+  if (!tc_enabled() || n_parts > 3 || M <= 0) return false;
+  if (tc_gemm_nt_persistent(dt, M, N, parts, n_parts, epi, s, st)) return true;
+  if (dt != WG_BF16) return false;
   for (int i = 0; i < n_parts; ++i)
-    if (parts[i].tile_group) return false;   // grouped B: CUDA-core path (TODO: per-tile B coordinate)
-  if (tc_gemm_nt_persistent(M, N, parts, n_parts, epi, s, st)) return true;
+    if (parts[i].tile_group) return false;   // grouped B: persistent kernel only
   const int n_tiles = (int)cdiv(N, 256);
   const int BN = (int)rup(cdiv(N, n_tiles), 16);
   if (BN > 256) return false;
@@ -396,41 +479,100 @@ bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_part
   for (int i = 0; i < n_parts; ++i) kt += parts[i].K;
   ProfScope ps(PK_TC_NT, s, (double)M * (kt + N + (epi.addend ? N : 0) + (epi.mask_ref ? N : 0)) * 2.0,
                2.0 * M * N * kt);
-  *st = launch<false>(grid, smem_bytes(false, BN, stages), maps, p, s);
+  *st = launch<false, __nv_bfloat16>(grid, smem_bytes(false, BN, stages), maps, p, s);
   return true;
 }
 
-bool tc_gemm_tn(int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb, float* D,
-                float* part, cudaStream_t s, wg_status* st, int acc) {
-  if (!tc_enabled() || K <= 0) return false;
-  const int n_tiles = (int)cdiv(N, 256);
-  const int BN = (int)rup(cdiv(N, n_tiles), 16);
-  const int m_tiles = (int)cdiv(M, BM);
+namespace {
+// TN map pair + launch geometry shared by the plain and grouped TN GEMMs
+struct TnSetup {
   CUtensorMap maps[6];
-  memset(maps, 0, sizeof(maps));
-  if (!make_map(&maps[0], A, (uint64_t)M, (uint64_t)K, (uint64_t)lda * 2, 64, BK)) return false;
-  if (!make_map(&maps[1], B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb * 2, 64, BK)) return false;
-  for (int i = 2; i < 6; ++i) maps[i] = maps[i & 1];
+  int BN, n_tiles, m_tiles, stages, es;
+  size_t smem;
+};
+
+bool tn_setup(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb,
+              TnSetup* t) {
+  t->es = dt == WG_F32 ? 4 : 2;
+  const CUtensorMapDataType ty = dt == WG_F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16;
+  const int che = 128 / t->es, bke = 128 / t->es;
+  const int bn_max = dt == WG_F32 ? 128 : 256;
+  t->n_tiles = (int)cdiv(N, bn_max);
+  t->BN = (int)rup(cdiv(N, t->n_tiles), 16);
+  t->m_tiles = (int)cdiv(M, BM);
+  memset(t->maps, 0, sizeof(t->maps));
+  // MN-major 32-bit operands: the 32-byte-granule 128-byte swizzle (see umma_desc)
+  const CUtensorMapSwizzle swz = dt == WG_F32 ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B;
+  if (!make_map_t(&t->maps[0], ty, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda * t->es, che, bke, swz)) return false;
+  if (!make_map_t(&t->maps[1], ty, B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb * t->es, che, bke, swz)) return false;
+  for (int i = 2; i < 6; ++i) t->maps[i] = t->maps[i & 1];
+  t->stages = 4;
+  while (t->stages > 2 && smem_bytes(true, t->BN, t->stages, t->es) > 200 * 1024) --t->stages;
+  t->smem = smem_bytes(true, t->BN, t->stages, t->es);
+  return t->smem <= 227 * 1024;
+}
+
+wg_status tn_launch(wg_dtype dt, const TnSetup& t, dim3 grid, const TcParams& p, cudaStream_t s) {
+  return dt == WG_F32 ? launch<true, float>(grid, t.smem, t.maps, p, s)
+                      : launch<true, __nv_bfloat16>(grid, t.smem, t.maps, p, s);
+}
+
+}  // namespace
+
+bool tc_gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda, const void* B, int64_t ldb,
+                float* D, float* part, cudaStream_t s, wg_status* st, int acc) {
+  if (!tc_enabled() || K <= 0) return false;
+  TnSetup t;
+  if (!tn_setup(dt, K, M, N, A, lda, B, ldb, &t)) return false;
+  const int bke = 128 / t.es;
   // split K so that the grid covers the SMs twice
-  const int tiles = m_tiles * n_tiles;
+  const int tiles = t.m_tiles * t.n_tiles;
   int64_t splits = std::max<int64_t>(1, (148 * 2) / tiles);
-  splits = std::min<int64_t>(splits, cdiv(K, BK));
+  splits = std::min<int64_t>(splits, cdiv(K, bke));
   splits = std::min<int64_t>(splits, 160);
-  const int64_t span = rup(cdiv(K, splits), BK);
+  const int64_t span = rup(cdiv(K, splits), bke);
   splits = cdiv(K, span);
   TcParams p{};
-  p.M = M; p.N = N; p.BN = BN; p.nparts = 1; p.kblocks[0] = (int)(span / BK);
-  p.k_base = 0; p.k_span = span; p.K = K; p.part = part;
-  int stages = 4;
-  while (stages > 2 && smem_bytes(true, BN, stages) > 200 * 1024) --stages;
-  p.stages = stages;
-  dim3 grid((unsigned)m_tiles, (unsigned)n_tiles, (unsigned)splits);
-  ProfScope ps(PK_TC_TN, s, (double)K * (M + N) * 2.0 + (double)M * N * 4.0, 2.0 * K * M * N);
-  *st = launch<true>(grid, smem_bytes(true, BN, stages), maps, p, s);
+  p.M = M; p.N = N; p.BN = t.BN; p.nparts = 1; p.kblocks[0] = (int)(span / bke);
+  p.k_base = 0; p.k_span = span; p.K = K; p.part = part; p.stages = t.stages;
+  dim3 grid((unsigned)t.m_tiles, (unsigned)t.n_tiles, (unsigned)splits);
+  ProfScope ps(PK_TC_TN, s, (double)K * (M + N) * t.es + (double)M * N * 4.0, 2.0 * K * M * N);
+  *st = tn_launch(dt, t, grid, p, s);
   if (*st != WG_OK) return true;
   const int64_t MN = (int64_t)M * N;
-  cudaStream_t ss = s;
-  k_split_reduce_tc<<<(unsigned)cdiv(MN, 256), 256, 0, ss>>>(part, (int)splits, MN, D, acc);
+  k_split_reduce_tc<<<(unsigned)cdiv(MN, 256), 256, 0, s>>>(part, (int)splits, MN, D, acc);
+  ++launch_counter();
+  if (cudaGetLastError() != cudaSuccess) *st = WG_ERR_CUDA;
+  return true;
+}
+
+namespace {
+// D[g] = sum of the partials of group g's units, in unit order (deterministic)
+__global__ void k_unit_reduce(const float* part, const int32_t* unit_off, int groups, int64_t MN, float* D) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= MN * groups) return;
+  const int64_t g = i / MN, e = i % MN;
+  float s = 0.f;
+  for (int u = unit_off[g]; u < unit_off[g + 1]; ++u) s += part[(int64_t)u * MN + e];
+  D[i] = s;
+}
+}  // namespace
+
+bool tc_gemm_tn_grouped(wg_dtype dt, const TnUnits& U, int M, int N, const void* A, int64_t lda, const void* B,
+                        int64_t ldb, float* D, float* part, cudaStream_t s, wg_status* st) {
+  if (!tc_enabled() || U.n_units <= 0 || U.align % (128 / (dt == WG_F32 ? 4 : 2)) != 0) return false;
+  TnSetup t;
+  if (!tn_setup(dt, U.k_total, M, N, A, lda, B, ldb, &t)) return false;
+  TcParams p{};
+  p.M = M; p.N = N; p.BN = t.BN; p.nparts = 1; p.K = U.k_total; p.part = part; p.stages = t.stages;
+  p.units = U.units;
+  dim3 grid((unsigned)t.m_tiles, (unsigned)t.n_tiles, (unsigned)U.n_units);
+  ProfScope ps(PK_TC_TN, s, (double)U.k_total * (M + N) * t.es + (double)U.n_units * M * N * 4.0,
+               2.0 * U.k_total * M * N);
+  *st = tn_launch(dt, t, grid, p, s);
+  if (*st != WG_OK) return true;
+  const int64_t MN = (int64_t)M * N;
+  k_unit_reduce<<<(unsigned)cdiv(MN * U.groups, 256), 256, 0, s>>>(part, U.unit_off, U.groups, MN, D);
   ++launch_counter();
   if (cudaGetLastError() != cudaSuccess) *st = WG_ERR_CUDA;
   return true;

@@ -1,6 +1,16 @@
-// Persistent, warp-specialized tcgen05 GEMM (NT, bf16) with a TMA epilogue.
+// Persistent, warp-specialized tcgen05 GEMM (NT) with a TMA epilogue.
 //
 //   D[M x N] = sum_p A_p[M x K_p] B_p[N x K_p]^T  (+ row scale, bias, addend, ReLU, ReLU-mask)
+//
+// bf16: kind::f16.  fp32: 3xTF32 (kind::tf32): every operand x = hi + lo with
+// hi = x with its 13 low mantissa bits cleared and lo = x - hi (exact), and
+// D += A_hi B_hi + A_hi B_lo + A_lo B_hi (the dropped lo*lo term is ~2^-22
+// relative), so fp32 layers keep fp32-level accuracy on tensor cores.  The
+// split runs in shared memory: two converter warps rewrite each landed stage
+// (hi in place, lo into a twin buffer) before the MMA warp consumes it.
+//
+// Grouped B (RGCN relation weights, GemmPart::tile_group): the B rows of
+// 128-row tile t start at tile_group[t] * group_rows.
 //
 // These layer transforms are HBM-bound (K <= 512), so what matters is keeping
 // loads, MMAs and the output stream overlapped across tiles:
@@ -12,8 +22,9 @@
 //   warp 6      epilogue loader: TMA loads of the addend / mask tiles, 64
 //               columns at a time, into a 2-deep buffer;
 //   warps 2-5   epilogue: tcgen05.ld (warp w drains TMEM lanes 32*(w%4)..),
-//               fused epilogue math, bf16 pack into a 128-byte-swizzled staging
-//               tile, TMA store (bulk_group, 2-deep) -- coalesced writes.
+//               fused epilogue math, pack into a 128-byte-swizzled staging
+//               tile, TMA store (bulk_group, 2-deep) -- coalesced writes;
+//   warps 7-8   (fp32 only) hi / lo converters.
 // One CTA per SM loops over 128 x BN tiles (N fastest, so A tiles of the N
 // tiles of one row block are adjacent in time).
 #include <cuda.h>
@@ -27,22 +38,34 @@
 
 namespace wg {
 
-bool tc_make_map(CUtensorMap* m, const void* ptr, uint64_t inner, uint64_t outer, uint64_t ld_bytes, uint32_t box_in,
-                 uint32_t box_out);
-bool tc_enabled_pub();
+bool tc_make_map_t(CUtensorMap* m, CUtensorMapDataType ty, const void* ptr, uint64_t inner, uint64_t outer,
+                   uint64_t ld_bytes, uint32_t box_in, uint32_t box_out);
 
 namespace {
 
-constexpr int BM = 128, BK = 64, CH = 64;          // CH: epilogue column chunk (one 128-B swizzle box)
-constexpr int A_STAGE = BM * BK * 2;               // 16 KB
-constexpr int CHUNK_BYTES = BM * CH * 2;           // 16 KB
-constexpr int NTHREADS = 224;                      // 7 warps
+// Every stage row and every epilogue chunk row is one 128-byte swizzle span:
+// BKE = 128 / sizeof(T) K elements per stage, CHE = 128 / sizeof(T) columns
+// per epilogue chunk.
+constexpr int BM = 128;
+constexpr int A_STAGE = BM * 128;                  // 16 KB
+constexpr int CHUNK_BYTES = BM * 128;              // 16 KB
+
+template <typename T> struct Cfg {
+  static constexpr bool TF32 = sizeof(T) == 4;
+  static constexpr int ES = sizeof(T);
+  static constexpr int BKE = 128 / ES;
+  static constexpr int CHE = 128 / ES;
+  static constexpr int EPV = 16 / ES;              // elements per 16-byte unit
+  static constexpr int NTHREADS = TF32 ? 288 : 224;
+};
 
 struct P2 {
   int64_t M;
   int N, BN, n_tiles, stages, nparts, n_split;
   int64_t num_tiles;
   int kblocks[3];
+  const int32_t* tile_group[3];
+  int group_rows[3];
   const float* rscale;
   const float* bias;
   int relu, has_add, has_mask;
@@ -96,6 +119,22 @@ __device__ __forceinline__ void mma(uint32_t tmem, uint64_t a, uint64_t b, uint3
       "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\ntcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem),
       "l"(a), "l"(b), "r"(idesc), "r"(acc));
 }
+__device__ __forceinline__ void mma_tf32(uint32_t tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\ntcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+// x = hi + lo, hi = x with the 13 low mantissa bits cleared (exactly a TF32 value)
+__device__ __forceinline__ void split_tf32(uint4& x, uint4& lo) {
+  uint32_t* v = reinterpret_cast<uint32_t*>(&x);
+  uint32_t* l = reinterpret_cast<uint32_t*>(&lo);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t h = v[i] & 0xffffe000u;
+    l[i] = __float_as_uint(__uint_as_float(v[i]) - __uint_as_float(h));
+    v[i] = h;
+  }
+}
 __device__ __forceinline__ void mma_commit(uint32_t bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
 }
@@ -107,39 +146,87 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* r) {
       : "r"(taddr));
 }
 
-// element offset of (row r, col c) inside a [128 x 64] bf16 tile with 128-byte swizzle
-__device__ __forceinline__ uint32_t sw_off(int r, int c) {
-  return (uint32_t)(r * 128 + ((((c >> 3) ^ (r & 7))) << 4) + ((c & 7) << 1));
+// byte offset of 16-byte unit k of row r inside a [128 x 128 B] tile with 128-byte swizzle
+__device__ __forceinline__ uint32_t sw_off(int r, int k) { return (uint32_t)(r * 128 + ((k ^ (r & 7)) << 4)); }
+
+template <typename T> __device__ __forceinline__ void unpack16(const int4& q, float* f);
+template <> __device__ __forceinline__ void unpack16<__nv_bfloat16>(const int4& q, float* f) {
+  const uint32_t w[4] = {(uint32_t)q.x, (uint32_t)q.y, (uint32_t)q.z, (uint32_t)q.w};
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    f[2 * i] = __uint_as_float(w[i] << 16);
+    f[2 * i + 1] = __uint_as_float(w[i] & 0xffff0000u);
+  }
+}
+template <> __device__ __forceinline__ void unpack16<float>(const int4& q, float* f) {
+  f[0] = __int_as_float(q.x); f[1] = __int_as_float(q.y); f[2] = __int_as_float(q.z); f[3] = __int_as_float(q.w);
+}
+template <typename T> __device__ __forceinline__ int4 pack16(const float* f);
+template <> __device__ __forceinline__ int4 pack16<__nv_bfloat16>(const float* f) {
+  uint32_t pk[4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(f[2 * i], f[2 * i + 1]);
+    pk[i] = *reinterpret_cast<uint32_t*>(&h);
+  }
+  return make_int4((int)pk[0], (int)pk[1], (int)pk[2], (int)pk[3]);
+}
+template <> __device__ __forceinline__ int4 pack16<float>(const float* f) {
+  return make_int4(__float_as_int(f[0]), __float_as_int(f[1]), __float_as_int(f[2]), __float_as_int(f[3]));
 }
 
-__global__ void __launch_bounds__(NTHREADS, 1)
+// shared-memory plan (bytes from the 1024-aligned base), identical on host and device
+struct SmemPlan {
+  int stage, ring, stg, add, mask, bars, total;
+};
+__host__ __device__ inline SmemPlan smem_plan(bool tf32, int BN, int S, bool has_add, bool has_mask) {
+  SmemPlan q;
+  q.stage = (A_STAGE + BN * 128) * (tf32 ? 2 : 1);   // [A | B] (+ [A_lo | B_lo])
+  q.ring = S * q.stage;
+  q.stg = q.ring;
+  q.add = q.stg + 2 * CHUNK_BYTES;
+  q.mask = q.add + (has_add ? 2 * CHUNK_BYTES : 0);
+  q.bars = q.mask + (has_mask ? 2 * CHUNK_BYTES : 0);
+  q.total = q.bars + 256;
+  return q;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
     k_gemm_nt_p(const __grid_constant__ CUtensorMap tA0, const __grid_constant__ CUtensorMap tB0,
                 const __grid_constant__ CUtensorMap tA1, const __grid_constant__ CUtensorMap tB1,
                 const __grid_constant__ CUtensorMap tA2, const __grid_constant__ CUtensorMap tB2,
                 const __grid_constant__ CUtensorMap tD, const __grid_constant__ CUtensorMap tD2,
                 const __grid_constant__ CUtensorMap tAdd, const __grid_constant__ CUtensorMap tMask, P2 p) {
+  using C = Cfg<T>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int BN = p.BN, S = p.stages;
-  const int b_stage = BN * 128;
-  uint8_t* a_sm = smem;
-  uint8_t* b_sm = a_sm + S * A_STAGE;
-  uint8_t* st_sm = b_sm + S * b_stage;             // 2 x 16 KB output staging
-  uint8_t* ad_sm = st_sm + 2 * CHUNK_BYTES;        // 2 x 16 KB addend
-  uint8_t* mk_sm = ad_sm + 2 * CHUNK_BYTES;        // 2 x 16 KB mask
-  uint64_t* bars = reinterpret_cast<uint64_t*>(mk_sm + 2 * CHUNK_BYTES);
-  uint64_t* full = bars;            // [4]
-  uint64_t* empty = bars + 4;       // [4]
+  const int b_bytes = BN * 128;
+  const SmemPlan L = smem_plan(C::TF32, BN, S, p.has_add, p.has_mask);
+  // stage s: A at s*stage, B at +A_STAGE; fp32: A_lo at +A_STAGE+b_bytes, B_lo after it
+  uint8_t* ring = smem;
+  uint8_t* st_sm = smem + L.stg;                   // 2 x 16 KB output staging
+  uint8_t* ad_sm = smem + L.add;                   // 2 x 16 KB addend
+  uint8_t* mk_sm = smem + L.mask;                  // 2 x 16 KB mask
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
+  uint64_t* full = bars;            // [4] TMA landed
+  uint64_t* empty = bars + 4;       // [4] MMA done with the stage
   uint64_t* tfull = bars + 8;       // [2]
   uint64_t* tempty = bars + 10;     // [2]
   uint64_t* efull = bars + 12;      // [2]
   uint64_t* eempty = bars + 14;     // [2]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 16);
+  uint64_t* conv = bars + 16;       // [4] fp32: hi / lo split done
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 20);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int nchunk = (BN + CH - 1) / CH;
+  const int nchunk = (BN + C::CHE - 1) / C::CHE;
 
   if (threadIdx.x == 0) {
-    for (int s = 0; s < S; ++s) { mbar_init(su32(&full[s]), 1); mbar_init(su32(&empty[s]), 1); }
+    for (int s = 0; s < S; ++s) {
+      mbar_init(su32(&full[s]), 1);
+      mbar_init(su32(&empty[s]), 1);
+      mbar_init(su32(&conv[s]), 64);
+    }
     for (int b = 0; b < 2; ++b) {
       mbar_init(su32(&tfull[b]), 1);
       mbar_init(su32(&tempty[b]), 128);
@@ -162,20 +249,28 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   if (warp == 0) {
     if (lane == 0) {
       // ------------------------------------------------ TMA producer
-      const uint32_t tx = A_STAGE + b_stage;
+      const uint32_t tx = A_STAGE + b_bytes;
       int s = 0;
       uint32_t ph = 0;
       for (int64_t t = blockIdx.x; t < p.num_tiles; t += gridDim.x) {
-        const int m0 = (int)((t / p.n_tiles) * BM), n0 = (int)((t % p.n_tiles) * BN);
+        const int64_t mt = t / p.n_tiles;
+        const int m0 = (int)(mt * BM), n0 = (int)((t % p.n_tiles) * BN);
         int part = 0, kk = 0;
+        int brow = n0 + (p.tile_group[0] ? p.tile_group[0][mt] * p.group_rows[0] : 0);
         for (int kb = 0; kb < total_kb; ++kb) {
           mbar_wait(su32(&empty[s]), ph ^ 1);
           mbar_expect_tx(su32(&full[s]), tx);
           const CUtensorMap* ta = part == 0 ? &tA0 : (part == 1 ? &tA1 : &tA2);
           const CUtensorMap* tb = part == 0 ? &tB0 : (part == 1 ? &tB1 : &tB2);
-          tma_load(su32(a_sm + s * A_STAGE), ta, kk * BK, m0, su32(&full[s]));
-          tma_load(su32(b_sm + s * b_stage), tb, kk * BK, n0, su32(&full[s]));
-          if (++kk == p.kblocks[part]) { kk = 0; ++part; }
+          uint8_t* st = ring + s * L.stage;
+          tma_load(su32(st), ta, kk * C::BKE, m0, su32(&full[s]));
+          tma_load(su32(st + A_STAGE), tb, kk * C::BKE, brow, su32(&full[s]));
+          if (++kk == p.kblocks[part]) {
+            kk = 0;
+            ++part;
+            if (part < p.nparts)
+              brow = n0 + (p.tile_group[part] ? p.tile_group[part][mt] * p.group_rows[part] : 0);
+          }
           if (++s == S) { s = 0; ph ^= 1; }
         }
       }
@@ -183,7 +278,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
   } else if (warp == 1) {
     if (lane == 0) {
       // ------------------------------------------------ MMA issuer
-      const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(BN >> 3) << 17) |
+      // idesc: D f32 [4,6), A / B format [7,10) / [10,13) (bf16 = 1, tf32 = 2), N>>3, M>>4
+      const uint32_t fmt = C::TF32 ? 2u : 1u;
+      const uint32_t idesc = (1u << 4) | (fmt << 7) | (fmt << 10) | ((uint32_t)(BN >> 3) << 17) |
                              ((uint32_t)(BM >> 4) << 24);
       int s = 0;
       uint32_t ph = 0;
@@ -194,12 +291,21 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t acc = tmem + (uint32_t)(buf * 256);
         for (int kb = 0; kb < total_kb; ++kb) {
-          mbar_wait(su32(&full[s]), ph);
+          mbar_wait(su32(C::TF32 ? &conv[s] : &full[s]), ph);
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          const uint32_t ad = su32(a_sm + s * A_STAGE), bd = su32(b_sm + s * b_stage);
+          const uint32_t ad = su32(ring + s * L.stage), bd = ad + A_STAGE;
 #pragma unroll
-          for (int k = 0; k < BK / 16; ++k)
-            mma(acc, desc_sw128(ad + k * 32), desc_sw128(bd + k * 32), idesc, (kb | k) != 0 ? 1u : 0u);
+          for (int k = 0; k < 4; ++k) {     // 4 MMAs of 32 bytes of K (16 bf16 / 8 tf32)
+            const uint32_t on = (kb | k) != 0 ? 1u : 0u;
+            if constexpr (C::TF32) {
+              const uint32_t al = bd + b_bytes, bl = al + A_STAGE;
+              mma_tf32(acc, desc_sw128(ad + k * 32), desc_sw128(bd + k * 32), idesc, on);
+              mma_tf32(acc, desc_sw128(ad + k * 32), desc_sw128(bl + k * 32), idesc, 1u);
+              mma_tf32(acc, desc_sw128(al + k * 32), desc_sw128(bd + k * 32), idesc, 1u);
+            } else {
+              mma(acc, desc_sw128(ad + k * 32), desc_sw128(bd + k * 32), idesc, on);
+            }
+          }
           mma_commit(su32(&empty[s]));
           if (++s == S) { s = 0; ph ^= 1; }
         }
@@ -217,8 +323,33 @@ __global__ void __launch_bounds__(NTHREADS, 1)
           const int b = g & 1;
           mbar_wait(su32(&eempty[b]), ((g >> 1) & 1) ^ 1);
           mbar_expect_tx(su32(&efull[b]), tx);
-          if (p.has_add) tma_load(su32(ad_sm + b * CHUNK_BYTES), &tAdd, n0 + c * CH, m0, su32(&efull[b]));
-          if (p.has_mask) tma_load(su32(mk_sm + b * CHUNK_BYTES), &tMask, n0 + c * CH, m0, su32(&efull[b]));
+          if (p.has_add) tma_load(su32(ad_sm + b * CHUNK_BYTES), &tAdd, n0 + c * C::CHE, m0, su32(&efull[b]));
+          if (p.has_mask) tma_load(su32(mk_sm + b * CHUNK_BYTES), &tMask, n0 + c * C::CHE, m0, su32(&efull[b]));
+        }
+      }
+    }
+  } else if (warp >= 7) {
+    if constexpr (C::TF32) {
+      // ------------------------------------------------ hi / lo converters (64 threads)
+      const int ct = threadIdx.x - 224;
+      const int n16 = (A_STAGE + b_bytes) / 16;
+      int s = 0;
+      uint32_t ph = 0;
+      for (int64_t t = blockIdx.x; t < p.num_tiles; t += gridDim.x) {
+        for (int kb = 0; kb < total_kb; ++kb) {
+          mbar_wait(su32(&full[s]), ph);
+          uint4* x = reinterpret_cast<uint4*>(ring + s * L.stage);
+          uint4* lo = x + n16;
+#pragma unroll 4
+          for (int i = ct; i < n16; i += 64) {
+            uint4 v = x[i], l;
+            split_tf32(v, l);
+            x[i] = v;
+            lo[i] = l;
+          }
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          mbar_arrive(su32(&conv[s]));
+          if (++s == S) { s = 0; ph ^= 1; }
         }
       }
     }
@@ -242,11 +373,9 @@ __global__ void __launch_bounds__(NTHREADS, 1)
       for (int c = 0; c < nchunk; ++c, ++g) {
         const int b = g & 1;
         uint32_t u[64];
-        const uint32_t taddr = tmem + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(buf * 256 + c * CH);
-        tmem_ld16(taddr, u);
-        tmem_ld16(taddr + 16, u + 16);
-        tmem_ld16(taddr + 32, u + 32);
-        tmem_ld16(taddr + 48, u + 48);
+        const uint32_t taddr = tmem + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(buf * 256 + c * C::CHE);
+#pragma unroll
+        for (int q = 0; q < C::CHE / 16; ++q) tmem_ld16(taddr + 16 * q, u + 16 * q);
         asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
         if (epi_loads) mbar_wait(su32(&efull[b]), (g >> 1) & 1);
         // the staging buffer b was last read by the TMA store issued two chunks ago
@@ -256,52 +385,40 @@ __global__ void __launch_bounds__(NTHREADS, 1)
         const uint8_t* adp = ad_sm + b * CHUNK_BYTES;
         const uint8_t* mkp = mk_sm + b * CHUNK_BYTES;
 #pragma unroll
-        for (int k = 0; k < 8; ++k) {           // 8 columns (one 16-byte chunk) at a time
-          float f[8];
-          const int nc = n0 + c * CH + k * 8;
+        for (int k = 0; k < 8; ++k) {           // one 16-byte unit (EPV columns) at a time
+          float f[C::EPV];
+          const int nc = n0 + c * C::CHE + k * C::EPV;
 #pragma unroll
-          for (int i = 0; i < 8; ++i) f[i] = rs * __uint_as_float(u[k * 8 + i]);
+          for (int i = 0; i < C::EPV; ++i) f[i] = rs * __uint_as_float(u[k * C::EPV + i]);
           if (p.has_add) {
-            const int4 q = *reinterpret_cast<const int4*>(adp + sw_off(r, k * 8));
-            const uint32_t w[4] = {(uint32_t)q.x, (uint32_t)q.y, (uint32_t)q.z, (uint32_t)q.w};
+            float a[C::EPV];
+            unpack16<T>(*reinterpret_cast<const int4*>(adp + sw_off(r, k)), a);
 #pragma unroll
-            for (int i = 0; i < 4; ++i) {
-              f[2 * i] += __uint_as_float(w[i] << 16);
-              f[2 * i + 1] += __uint_as_float(w[i] & 0xffff0000u);
-            }
+            for (int i = 0; i < C::EPV; ++i) f[i] += a[i];
           }
           if (p.bias) {
 #pragma unroll
-            for (int i = 0; i < 8; ++i) f[i] += (nc + i < p.N) ? p.bias[nc + i] : 0.f;
+            for (int i = 0; i < C::EPV; ++i) f[i] += (nc + i < p.N) ? p.bias[nc + i] : 0.f;
           }
           if (p.relu) {
 #pragma unroll
-            for (int i = 0; i < 8; ++i) f[i] = fmaxf(f[i], 0.f);
+            for (int i = 0; i < C::EPV; ++i) f[i] = fmaxf(f[i], 0.f);
           }
           if (p.has_mask) {
-            const int4 q = *reinterpret_cast<const int4*>(mkp + sw_off(r, k * 8));
-            const uint32_t w[4] = {(uint32_t)q.x, (uint32_t)q.y, (uint32_t)q.z, (uint32_t)q.w};
+            float a[C::EPV];
+            unpack16<T>(*reinterpret_cast<const int4*>(mkp + sw_off(r, k)), a);
 #pragma unroll
-            for (int i = 0; i < 4; ++i) {
-              if (!(__uint_as_float(w[i] << 16) > 0.f)) f[2 * i] = 0.f;
-              if (!(__uint_as_float(w[i] & 0xffff0000u) > 0.f)) f[2 * i + 1] = 0.f;
-            }
+            for (int i = 0; i < C::EPV; ++i) if (!(a[i] > 0.f)) f[i] = 0.f;
           }
 #pragma unroll
-          for (int i = 0; i < 8; ++i) if (nc + i >= p.N) f[i] = 0.f;
-          uint32_t pk[4];
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            __nv_bfloat162 h = __floats2bfloat162_rn(f[2 * i], f[2 * i + 1]);
-            pk[i] = *reinterpret_cast<uint32_t*>(&h);
-          }
-          *reinterpret_cast<int4*>(stg + sw_off(r, k * 8)) = make_int4((int)pk[0], (int)pk[1], (int)pk[2], (int)pk[3]);
+          for (int i = 0; i < C::EPV; ++i) if (nc + i >= p.N) f[i] = 0.f;
+          *reinterpret_cast<int4*>(stg + sw_off(r, k)) = pack16<T>(f);
         }
         if (epi_loads) mbar_arrive(su32(&eempty[b]));
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         epi_bar();
         if (et == 0) {
-          tma_store(td, ncol0 + c * CH, m0, su32(stg));
+          tma_store(td, ncol0 + c * C::CHE, m0, su32(stg));
           bulk_commit();
         }
       }
@@ -316,25 +433,35 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 
 int g_sms = 0;
 
-}  // namespace
-
-size_t gemm_nt_p_smem(int BN, int stages) {
-  return 1024 + (size_t)stages * (A_STAGE + BN * 128) + 6 * CHUNK_BYTES + 256;
+template <typename T>
+void set_smem_attr() {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_gemm_nt_p<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    attr = true;
+  }
 }
 
+}  // namespace
+
 // returns false when the shape / epilogue is not handled (caller falls back)
-bool tc_gemm_nt_persistent(int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi, cudaStream_t s,
-                           wg_status* st) {
+bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi,
+                           cudaStream_t s, wg_status* st) {
   static int disabled = -1;
   if (disabled < 0) {
     const char* e = getenv("WG_GEMM_V1");
     disabled = (e && e[0] == '1') ? 1 : 0;
   }
-  if (disabled || epi.d_f32 || n_parts > 3 || M <= 0) return false;
-  // several N tiles: BN = 256 so every 64-column store box stays inside its
-  // tile (the ragged end is clipped by the tensor map); one tile: BN = N
-  const int n_tiles = (int)cdiv(N, 256);
-  const int BN = n_tiles > 1 ? 256 : (int)rup(N, 16);
+  const bool f32 = dt == WG_F32;
+  if (disabled || (epi.d_f32 && !f32) || n_parts > 3 || M <= 0) return false;
+  const int es = f32 ? 4 : 2, che = 128 / es;
+  const CUtensorMapDataType ty = f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16;
+  // several N tiles: BN = 256 (bf16) / 128 (fp32, the lo twins double the
+  // stage) so every store box stays inside its tile (the ragged end is
+  // clipped by the tensor map); one tile: BN = N
+  const int bn_max = f32 ? 128 : 256;
+  const int n_tiles = (int)cdiv(N, bn_max);
+  const int BN = n_tiles > 1 ? bn_max : (int)rup(N, 16);
   if (epi.D2 && (epi.n_split % BN != 0)) return false;   // split must fall on a tile boundary
   CUtensorMap maps[10];
   memset(maps, 0, sizeof(maps));
@@ -343,53 +470,63 @@ bool tc_gemm_nt_persistent(int64_t M, int N, const GemmPart* parts, int n_parts,
   p.num_tiles = cdiv(M, BM) * n_tiles;
   for (int i = 0; i < n_parts; ++i) {
     const GemmPart& q = parts[i];
-    if (q.tile_group) return false;
-    if (!tc_make_map(&maps[2 * i], q.A, (uint64_t)q.K, (uint64_t)M, (uint64_t)q.lda * 2, BK, BM)) return false;
-    if (!tc_make_map(&maps[2 * i + 1], q.B, (uint64_t)q.K, (uint64_t)q.nb, (uint64_t)q.ldb * 2, BK, BN)) return false;
-    p.kblocks[i] = (int)cdiv(q.K, BK);
+    const uint64_t brows = q.tile_group ? (uint64_t)q.groups * q.group_rows : (uint64_t)q.nb;
+    if (q.tile_group && BN > q.group_rows) return false;
+    if (!tc_make_map_t(&maps[2 * i], ty, q.A, (uint64_t)q.K, (uint64_t)M, (uint64_t)q.lda * es, che, BM)) return false;
+    if (!tc_make_map_t(&maps[2 * i + 1], ty, q.B, (uint64_t)q.K, brows, (uint64_t)q.ldb * es, che, BN)) return false;
+    p.kblocks[i] = (int)cdiv(q.K, che);
+    p.tile_group[i] = q.tile_group;
+    p.group_rows[i] = q.group_rows;
   }
   for (int i = n_parts; i < 3; ++i) { maps[2 * i] = maps[0]; maps[2 * i + 1] = maps[1]; }
   const int n1 = epi.D2 ? epi.n_split : N;
-  if (!tc_make_map(&maps[6], epi.D, (uint64_t)n1, (uint64_t)M, (uint64_t)epi.ldd * 2, CH, BM)) return false;
+  if (!tc_make_map_t(&maps[6], ty, epi.D, (uint64_t)n1, (uint64_t)M, (uint64_t)epi.ldd * es, che, BM)) return false;
   maps[7] = maps[6];
   if (epi.D2) {
     p.n_split = epi.n_split;
-    if (!tc_make_map(&maps[7], epi.D2, (uint64_t)(N - epi.n_split), (uint64_t)M, (uint64_t)epi.ldd2 * 2, CH, BM))
+    if (!tc_make_map_t(&maps[7], ty, epi.D2, (uint64_t)(N - epi.n_split), (uint64_t)M, (uint64_t)epi.ldd2 * es, che,
+                       BM))
       return false;
   }
   maps[8] = maps[9] = maps[6];
   if (epi.addend) {
-    if (!tc_make_map(&maps[8], epi.addend, (uint64_t)N, (uint64_t)M, (uint64_t)epi.ld_add * 2, CH, BM)) return false;
+    if (!tc_make_map_t(&maps[8], ty, epi.addend, (uint64_t)N, (uint64_t)M, (uint64_t)epi.ld_add * es, che, BM))
+      return false;
     p.has_add = 1;
   }
   if (epi.mask_ref) {
-    if (!tc_make_map(&maps[9], epi.mask_ref, (uint64_t)N, (uint64_t)M, (uint64_t)epi.ld_mask * 2, CH, BM)) return false;
+    if (!tc_make_map_t(&maps[9], ty, epi.mask_ref, (uint64_t)N, (uint64_t)M, (uint64_t)epi.ld_mask * es, che, BM))
+      return false;
     p.has_mask = 1;
   }
   p.rscale = epi.rscale;
   p.bias = epi.bias;
   p.relu = epi.relu;
+  const int limit = 227 * 1024 - 1024;
   int stages = 4;
-  while (stages > 2 && gemm_nt_p_smem(BN, stages) > 227 * 1024) --stages;
-  if (gemm_nt_p_smem(BN, stages) > 227 * 1024) return false;
+  while (stages > 2 && smem_plan(f32, BN, stages, p.has_add, p.has_mask).total > limit) --stages;
+  if (smem_plan(f32, BN, stages, p.has_add, p.has_mask).total > limit) return false;
   p.stages = stages;
   if (!g_sms) {
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
   }
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(k_gemm_nt_p, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-    attr = true;
-  }
   const unsigned grid = (unsigned)std::min<int64_t>(p.num_tiles, g_sms);
+  const size_t smem = 1024 + (size_t)smem_plan(f32, BN, stages, p.has_add, p.has_mask).total;
   double kt = 0;
   for (int i = 0; i < n_parts; ++i) kt += parts[i].K;
-  ProfScope ps(PK_TC_NT, s, (double)M * (kt + N + (epi.addend ? N : 0) + (epi.mask_ref ? N : 0)) * 2.0,
+  ProfScope ps(PK_TC_NT, s, (double)M * (kt + N + (epi.addend ? N : 0) + (epi.mask_ref ? N : 0)) * es,
                2.0 * M * N * kt);
-  k_gemm_nt_p<<<grid, NTHREADS, gemm_nt_p_smem(BN, stages), s>>>(maps[0], maps[1], maps[2], maps[3], maps[4],
-                                                                 maps[5], maps[6], maps[7], maps[8], maps[9], p);
+  if (f32) {
+    set_smem_attr<float>();
+    k_gemm_nt_p<float><<<grid, Cfg<float>::NTHREADS, smem, s>>>(maps[0], maps[1], maps[2], maps[3], maps[4], maps[5],
+                                                               maps[6], maps[7], maps[8], maps[9], p);
+  } else {
+    set_smem_attr<__nv_bfloat16>();
+    k_gemm_nt_p<__nv_bfloat16><<<grid, Cfg<__nv_bfloat16>::NTHREADS, smem, s>>>(
+        maps[0], maps[1], maps[2], maps[3], maps[4], maps[5], maps[6], maps[7], maps[8], maps[9], p);
+  }
   ++launch_counter();
   cudaError_t e = cudaGetLastError();
   *st = e == cudaSuccess ? WG_OK : WG_ERR_CUDA;

@@ -206,6 +206,19 @@ struct GemmEpi {
 };
 wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts,
                   const GemmEpi& epi, void* scratch, size_t scratch_bytes, cudaStream_t s);
+// Grouped TN work units (RGCN dW_r): group g owns K rows [off[g], off[g+1]),
+// cut into units of <= span rows (multiples of `align`); unit u = {first K
+// row, k-blocks of 128 / sizeof(dtype) rows, group, -}, units of a group are
+// consecutive, unit_off[g] .. unit_off[g+1].  Built once per plan.
+struct TnUnits {
+  const int4* units = nullptr;
+  const int32_t* unit_off = nullptr;
+  int n_units = 0, groups = 0, align = 0;
+  int64_t k_total = 0;
+};
+// host: unit table for group offsets h_off (size groups + 1); kb_rows = rows per k-block
+void make_tn_units(const std::vector<int64_t>& h_off, int64_t target_units, int kb_rows, std::vector<int4>* units,
+                   std::vector<int32_t>* unit_off);
 // dW[M x N] (fp32, exact shape, ld = N) = A[K x M]^T * B[K x N] (split-K, deterministic)
 size_t gemm_tn_scratch(int64_t K, int M, int N);
 // acc != 0: D += A^T B (fixed order: the previous D is added after the split sums)
@@ -213,8 +226,8 @@ wg_status gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t l
                   const void* B, int64_t ldb, float* D, void* scratch, cudaStream_t s, int acc = 0);
 
 // grouped weight gradient: D[g] (fp32 [M x N]) = sum_{k in [off[g], off[g+1])} A[k]^T B[k]
-size_t gemm_tn_grouped_scratch(int groups, int M, int N);
-wg_status gemm_tn_grouped(wg_dtype dt, int groups, const int64_t* d_off, int M, int N, const void* A, int64_t lda,
+size_t gemm_tn_grouped_scratch(int n_units, int M, int N);
+wg_status gemm_tn_grouped(wg_dtype dt, const TnUnits& U, int M, int N, const void* A, int64_t lda,
                           const void* B, int64_t ldb, float* D, void* scratch, cudaStream_t s);
 // batched weight prep: `batch` matrices of [rows x cols] (fp32, contiguous) into
 // consecutive [out_rows x ldo] blocks

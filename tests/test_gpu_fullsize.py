@@ -46,7 +46,7 @@ def entry_probe(src, dst, coef, x, dy, i, j):
 def c4():
     import bench
     c = synth.CONFIGS["C4"]
-    src, dst, x, labels = bench.make_inputs(c)
+    src, dst, _, x, labels = bench.make_inputs(c, "sage")
     m = wg()
     g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=c.V)
     return c, src, dst, g
