@@ -103,10 +103,12 @@ struct GatArgs {
   // forward outputs
   void* agg; int64_t ld_agg;           // per-head aggregation (pre-bias)
   float* m; float* l;                  // [V x H] softmax max / denominator
+  void* y; int64_t ldy; int FO;        // layer output (conv dtype): concat -> HF columns, mean -> Fo
+  const float* bias; int relu;
   float* part; int part_ld;            // partial slots [slots x part_ld]: HF acc + H m + H l
   // backward
   const void* dy; int64_t lddy; int concat;
-  const float* s;                      // [V x H]  dy_k . agg_k
+  const float4* bs;                    // [V x H] {er, m + log l, s, 0}: per-destination backward stats
   const int64_t* fwdpos;               // transposed position -> forward position
   float* dt;                           // [E x H] (forward order)
   float* dg; int64_t ld_dg;            // [V x HF] fp32 (sum alpha dy)
@@ -148,11 +150,49 @@ __global__ void k_gat_logits(int64_t V, GatArgs a, const float* al, const float*
   }
 }
 
+// y row of destination `row` from its per-head aggregate row `o` (fp32, HF
+// values, shared memory): concat -> o + b, mean over heads -> mean_k o_k + b;
+// optional ReLU; pad columns up to a multiple of 8 written as 0.  Threads
+// t = 0..nt-1 of the caller each write 4 columns at a time.
+template <typename TO>
+__device__ __forceinline__ void gat_write_y(const GatArgs& a, int64_t row, const float* o, int t, int nt) {
+  const int wcols = ((a.FO + 7) / 8) * 8;
+  for (int c = 4 * t; c < wcols; c += 4 * nt) {
+    float v[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int cc = c + i;
+      float x = 0.f;
+      if (cc < a.FO) {
+        if (a.concat) x = o[cc];
+        else {
+          for (int h = 0; h < a.H; ++h) x += o[h * a.Fo + cc];
+          x /= (float)a.H;
+        }
+        if (a.bias) x += a.bias[cc];
+        if (a.relu) x = fmaxf(x, 0.f);
+      }
+      v[i] = x;
+    }
+    TO* yp = static_cast<TO*>(a.y) + row * a.ldy + c;
+    if constexpr (sizeof(TO) == 4) {
+      *reinterpret_cast<float4*>(yp) = make_float4(v[0], v[1], v[2], v[3]);
+    } else {
+      __nv_bfloat162 h0 = __floats2bfloat162_rn(v[0], v[1]), h1 = __floats2bfloat162_rn(v[2], v[3]);
+      uint2 u;
+      u.x = *reinterpret_cast<uint32_t*>(&h0);
+      u.y = *reinterpret_cast<uint32_t*>(&h1);
+      *reinterpret_cast<uint2*>(yp) = u;
+    }
+  }
+}
+
 // ------------------------------------------------- forward online softmax
 // one warp per row chunk (destination row, in-edges [e_lo, e_hi))
-template <typename T, int NV, int U>
+template <typename T, typename TO, int NV, int U>
 __global__ void __launch_bounds__(256) k_gat_fwd(GatArgs a, int64_t row_base) {
   constexpr int EPV = GV<T>::EPV;
+  __shared__ float orow[8][NV * 32 * EPV];          // per-warp aggregate row (y epilogue)
   const int lane = threadIdx.x & 31;
   const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (w >= a.n_chunks) return;
@@ -224,85 +264,111 @@ __global__ void __launch_bounds__(256) k_gat_fwd(GatArgs a, int64_t row_base) {
       for (int i = 0; i < EPV; ++i) o[i] = (c0 + i < a.HF) ? acc[q][i] * inv : 0.f;
       float* ag = static_cast<float*>(a.agg) + (int64_t)ch.row * a.ld_agg + c0;
 #pragma unroll
-      for (int i = 0; i < EPV; ++i) ag[i] = o[i];
+      for (int i = 0; i < EPV; ++i) { ag[i] = o[i]; orow[threadIdx.x >> 5][c0 + i] = o[i]; }
       if (head_lead) { a.m[d * a.H + hd[q]] = m[q]; a.l[d * a.H + hd[q]] = l[q]; }
     }
   }
+  if (ch.slot < 0) {                               // warp-uniform
+    __syncwarp();
+    gat_write_y<TO>(a, ch.row, orow[threadIdx.x >> 5], lane, 32);
+  }
 }
 
-// flash-style merge of the (m, l, acc) partials of split rows, chunk order
-template <typename T>
-__global__ void k_gat_fwd_combine(GatArgs a, const SplitRow* rows, int64_t row_base) {
-  constexpr int EPV = GV<T>::EPV;
+// flash-style merge of the (m, l, acc) partials of split rows, chunk order:
+// M = max_k m_k, then l = sum_k l_k e^{m_k - M}, o = sum_k acc_k e^{m_k - M}
+// (independent loads, fixed order); writes agg, m, l and the y row
+template <typename TO>
+__global__ void __launch_bounds__(256) k_gat_fwd_combine(GatArgs a, const SplitRow* rows, int64_t row_base) {
+  __shared__ float orow[1024];
   const SplitRow sr = rows[blockIdx.x];
   const int64_t d = row_base + sr.row;
-  for (int c = threadIdx.x; c < a.VPR * EPV; c += blockDim.x) {
-    const int h = min(c / a.Fo, a.H - 1);
-    float m = -INFINITY, l = 0.f, o = 0.f;
+  for (int c = threadIdx.x; c < a.HF; c += blockDim.x) {
+    const int h = c / a.Fo;
+    const float* p0 = a.part + (int64_t)sr.first_slot * a.part_ld;
+    float M = -INFINITY;
     for (int k = 0; k < sr.n_slots; ++k) {
-      const float* pp = a.part + (int64_t)(sr.first_slot + k) * a.part_ld;
-      const float mk = pp[a.HF + h], lk = pp[a.HF + a.H + h];
-      if (lk <= 0.f) continue;
-      const float mn = fmaxf(m, mk);
-      const float s0 = __expf(m - mn), s1 = __expf(mk - mn);
-      l = l * s0 + lk * s1;
-      o = o * s0 + (c < a.HF ? pp[c] : 0.f) * s1;
-      m = mn;
+      const float* pp = p0 + (int64_t)k * a.part_ld;
+      if (pp[a.HF + a.H + h] > 0.f) M = fmaxf(M, pp[a.HF + h]);
     }
-    const float val = (c < a.HF && l > 0.f) ? o / l : 0.f;
-    static_cast<float*>(a.agg)[(int64_t)sr.row * a.ld_agg + c] = val;
-    if (c < a.HF && c % a.Fo == 0) { a.m[d * a.H + h] = m; a.l[d * a.H + h] = l; }
-  }
-}
-
-// y = concat(agg) + b or mean_k(agg_k) + b, optional ReLU; also s = dy . agg (backward)
-template <typename T>
-__global__ void k_gat_out(int64_t rows, GatArgs a, const float* bias, int relu, void* y, int64_t ldy, int FO) {
-  const int64_t n = rows * (int64_t)ldy;
-  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t r = t / ldy;
-    const int c = (int)(t % ldy);
-    float v = 0.f;
-    if (c < FO) {
-      const float* ag = static_cast<const float*>(a.agg) + r * a.ld_agg;
-      if (a.concat) v = ag[c];
-      else {
-        for (int h = 0; h < a.H; ++h) v += (float)ag[h * a.Fo + c];
-        v /= (float)a.H;
-      }
-      if (bias) v += bias[c];
-      if (relu) v = fmaxf(v, 0.f);
-    }
-    if (c < ((FO + 7) / 8) * 8) static_cast<T*>(y)[r * ldy + c] = (T)v;
-  }
-}
-
-// s[v,h] = dy_k[v] . agg_k[v]   (= sum_{e in in(v)} alpha_e dalpha_e)
-template <typename T>
-__global__ void k_gat_s(int64_t rows, int64_t row_base, GatArgs a, float* s) {
-  const int lane = threadIdx.x & 31;
-  const int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  if (r >= rows) return;
-  const float* ag = static_cast<const float*>(a.agg) + r * a.ld_agg;
-  const T* dy = static_cast<const T*>(a.dy) + r * a.lddy;
-  for (int h = 0; h < a.H; ++h) {
-    float acc = 0.f;
-    for (int j = lane; j < a.Fo; j += 32) {
-      const float g = a.concat ? (float)dy[h * a.Fo + j] : (float)dy[j] / (float)a.H;
-      acc += g * (float)ag[h * a.Fo + j];
-    }
+    float l = 0.f, o = 0.f;
+    int k = 0;
+    for (; k + 4 <= sr.n_slots; k += 4) {
+      float lk[4], mk[4], ok[4];
 #pragma unroll
-    for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-    if (lane == 0) s[(row_base + r) * a.H + h] = acc;
+      for (int j = 0; j < 4; ++j) {
+        const float* pp = p0 + (int64_t)(k + j) * a.part_ld;
+        lk[j] = pp[a.HF + a.H + h]; mk[j] = pp[a.HF + h]; ok[j] = pp[c];
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        if (lk[j] <= 0.f) continue;
+        const float sc = __expf(mk[j] - M);
+        l += lk[j] * sc;
+        o += ok[j] * sc;
+      }
+    }
+    for (; k < sr.n_slots; ++k) {
+      const float* pp = p0 + (int64_t)k * a.part_ld;
+      const float lk = pp[a.HF + a.H + h];
+      if (lk <= 0.f) continue;
+      const float sc = __expf(pp[a.HF + h] - M);
+      l += lk * sc;
+      o += pp[c] * sc;
+    }
+    const float val = l > 0.f ? o / l : 0.f;
+    static_cast<float*>(a.agg)[(int64_t)sr.row * a.ld_agg + c] = val;
+    orow[c] = val;
+    if (c % a.Fo == 0) { a.m[d * a.H + h] = M; a.l[d * a.H + h] = l; }
+  }
+  __syncthreads();
+  gat_write_y<TO>(a, sr.row, orow, threadIdx.x, blockDim.x);
+}
+
+// dy columns [c, c+4) of destination row dd as fp32 (16-byte or 8-byte load)
+template <typename T> __device__ __forceinline__ void ld_dy4(const T* p, float* f);
+template <> __device__ __forceinline__ void ld_dy4<float>(const float* p, float* f) {
+  const int4 v = ld16(p);
+  f[0] = __int_as_float(v.x); f[1] = __int_as_float(v.y); f[2] = __int_as_float(v.z); f[3] = __int_as_float(v.w);
+}
+template <> __device__ __forceinline__ void ld_dy4<__nv_bfloat16>(const __nv_bfloat16* p, float* f) {
+  const uint2 v = __ldg(reinterpret_cast<const uint2*>(p));
+  f[0] = __uint_as_float(v.x << 16); f[1] = __uint_as_float(v.x & 0xffff0000u);
+  f[2] = __uint_as_float(v.y << 16); f[3] = __uint_as_float(v.y & 0xffff0000u);
+}
+
+// per-head sum of a lane value: SEG > 0: heads are aligned groups of SEG
+// lanes (SEG = Fo / 4, a power of two <= 32); SEG == 0: generic (any Fo)
+template <int NV, int SEG>
+__device__ __forceinline__ void head_sums(const float* part, const int* hd, int H, float* out) {
+  if constexpr (SEG > 0) {
+#pragma unroll
+    for (int q = 0; q < NV; ++q) {
+      float v = part[q];
+#pragma unroll
+      for (int o = SEG / 2; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+      out[q] = v;
+    }
+  } else {
+#pragma unroll
+    for (int q = 0; q < NV; ++q) out[q] = 0.f;
+    for (int h = 0; h < H; ++h) {
+      float sh = 0.f;
+#pragma unroll
+      for (int q = 0; q < NV; ++q) if (hd[q] == h) sh += part[q];
+#pragma unroll
+      for (int o = 16; o; o >>= 1) sh += __shfl_xor_sync(0xffffffffu, sh, o);
+#pragma unroll
+      for (int q = 0; q < NV; ++q) if (hd[q] == h) out[q] = sh;
+    }
   }
 }
 
-// ---------------------------------------------- backward, source-major pass
-// warp per (source row, out-edge chunk): dg[u] += sum alpha dy_k[d], del[u] +=
-// sum dt_e, dt_e written at the edge's forward position.
-template <typename T, int NV>
-__global__ void __launch_bounds__(256) k_gat_bwd_src(GatArgs a, int64_t row_base) {
-  constexpr int EPV = 4;                       // G is kept in fp32 (4 columns per 16-byte vector)
+// Source-major backward pass, U out-edges in flight per warp: per out-edge e
+// = (u -> dd): dalpha = dy_k[dd] . g_k[u], alpha = exp(lrelu(t) - lse[dd]),
+// dt_e = alpha (dalpha - s[dd]) lrelu'(t); dg[u] += alpha dy_k[dd]; del[u] += dt_e.
+template <typename T, int NV, int U, int SEG>
+__global__ void __launch_bounds__(256, 2) k_gat_bwd_src2(GatArgs a, int64_t row_base) {
+  constexpr int EPV = 4;                       // G is fp32: 4 columns per 16-byte vector
   const int lane = threadIdx.x & 31;
   const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (w >= a.n_chunks) return;
@@ -310,13 +376,19 @@ __global__ void __launch_bounds__(256) k_gat_bwd_src(GatArgs a, int64_t row_base
   const int64_t u = row_base + ch.row;
   const float* G = static_cast<const float*>(a.G);
   const T* DY = static_cast<const T*>(a.dy);
-  int hd[NV];
+  int hd[NV], cc[NV];
+  bool on[NV], lead[NV];
   float gu[NV][EPV], elu[NV], acc[NV][EPV], dl[NV];
+  const float dys = a.concat ? 1.f : 1.f / (float)a.H;
 #pragma unroll
   for (int q = 0; q < NV; ++q) {
     const int vi = lane + 32 * q;
-    hd[q] = vi < a.VPR ? (vi * EPV) / a.Fo : 0;
-    if (vi < a.VPR) GV<float>::unpack(ld16(G + u * a.ldg + vi * EPV), gu[q]);
+    on[q] = vi < a.VPR;
+    const int c0 = vi * EPV;
+    hd[q] = on[q] ? c0 / a.Fo : 0;
+    cc[q] = a.concat ? c0 : c0 % a.Fo;
+    lead[q] = on[q] && (c0 % a.Fo) == 0;
+    if (on[q]) GV<float>::unpack(ld16(G + u * a.ldg + c0), gu[q]);
     else {
 #pragma unroll
       for (int i = 0; i < EPV; ++i) gu[q][i] = 0.f;
@@ -326,69 +398,140 @@ __global__ void __launch_bounds__(256) k_gat_bwd_src(GatArgs a, int64_t row_base
 #pragma unroll
     for (int i = 0; i < EPV; ++i) acc[q][i] = 0.f;
   }
-  const float dys = a.concat ? 1.f : 1.f / (float)a.H;
-  for (int64_t e = ch.e_lo; e < ch.e_hi; ++e) {
-    const int64_t dd = a.idx[e];
-    float dyv[NV][EPV], part[NV];
+  for (int64_t base = ch.e_lo; base < ch.e_hi; base += 32) {
+    const int n = (int)min((int64_t)32, ch.e_hi - base);
+    const int my = lane < n ? a.idx[base + lane] : 0;
+    const int64_t myp = lane < n ? a.fwdpos[base + lane] : 0;
+    for (int j = 0; j < n; j += U) {
+      float dyv[U][NV][EPV];
+      float4 st[U][NV];
 #pragma unroll
-    for (int q = 0; q < NV; ++q) {
-      const int vi = lane + 32 * q;
-      part[q] = 0.f;
-      if (vi < a.VPR) {
-        const int c0 = vi * EPV;
-        const int cc = a.concat ? c0 : (c0 % a.Fo);
+      for (int k = 0; k < U; ++k) {
+        const int64_t dd = __shfl_sync(0xffffffffu, my, j + k < n ? j + k : 0);
 #pragma unroll
-        for (int i = 0; i < EPV; ++i) dyv[q][i] = (c0 + i < a.HF) ? (float)DY[dd * a.lddy + cc + i] : 0.f;
+        for (int q = 0; q < NV; ++q) {
+          if (on[q] && j + k < n) {
+            ld_dy4<T>(DY + dd * a.lddy + cc[q], dyv[k][q]);
+            st[k][q] = __ldg(a.bs + dd * a.H + hd[q]);
+          } else {
 #pragma unroll
-        for (int i = 0; i < EPV; ++i) {
-          dyv[q][i] = (c0 + i < a.HF) ? dyv[q][i] * dys : 0.f;
-          part[q] += dyv[q][i] * gu[q][i];
+            for (int i = 0; i < EPV; ++i) dyv[k][q][i] = 0.f;
+            st[k][q] = make_float4(0.f, 0.f, 0.f, 0.f);
+          }
         }
-      } else {
-#pragma unroll
-        for (int i = 0; i < EPV; ++i) dyv[q][i] = 0.f;
       }
-    }
-    // dalpha per head: segmented (by head) warp reduction
-    float dal[NV];
 #pragma unroll
-    for (int q = 0; q < NV; ++q) dal[q] = 0.f;
-    for (int h = 0; h < a.H; ++h) {
-      float sh = 0.f;
+      for (int k = 0; k < U; ++k) {
+        if (j + k >= n) break;                 // warp-uniform
+        float part[NV], dal[NV];
 #pragma unroll
-      for (int q = 0; q < NV; ++q) if (hd[q] == h) sh += part[q];
+        for (int q = 0; q < NV; ++q) {
+          part[q] = 0.f;
 #pragma unroll
-      for (int o = 16; o; o >>= 1) sh += __shfl_xor_sync(0xffffffffu, sh, o);
+          for (int i = 0; i < EPV; ++i) {
+            dyv[k][q][i] *= dys;
+            part[q] += dyv[k][q][i] * gu[q][i];
+          }
+        }
+        head_sums<NV, SEG>(part, hd, a.H, dal);
+        const int64_t fp = __shfl_sync(0xffffffffu, myp, j + k);
 #pragma unroll
-      for (int q = 0; q < NV; ++q) if (hd[q] == h) dal[q] = sh;
-    }
+        for (int q = 0; q < NV; ++q) {
+          const float t = elu[q] + st[k][q].x;
+          const float alpha = __expf(lrelu(t, a.slope) - st[k][q].y);
+          const float dtv = alpha * (dal[q] - st[k][q].z) * (t > 0.f ? 1.f : a.slope);
 #pragma unroll
-    for (int q = 0; q < NV; ++q) {
-      const int vi = lane + 32 * q;
-      const int h = hd[q];
-      const float t = elu[q] + a.er[dd * a.H + h];
-      const float alpha = __expf(lrelu(t, a.slope) - a.m[dd * a.H + h]) / a.l[dd * a.H + h];
-      const float dtv = alpha * (dal[q] - a.s[dd * a.H + h]) * (t > 0.f ? 1.f : a.slope);
-#pragma unroll
-      for (int i = 0; i < EPV; ++i) acc[q][i] += alpha * dyv[q][i];
-      if (vi < a.VPR && (vi * EPV) % a.Fo == 0) {
-        dl[q] += dtv;
-        a.dt[a.fwdpos[e] * a.H + h] = dtv;
+          for (int i = 0; i < EPV; ++i) acc[q][i] += alpha * dyv[k][q][i];
+          if (lead[q]) {
+            dl[q] += dtv;
+            a.dt[fp * a.H + hd[q]] = dtv;
+          }
+        }
       }
     }
   }
 #pragma unroll
   for (int q = 0; q < NV; ++q) {
-    const int vi = lane + 32 * q;
-    if (vi >= a.VPR) continue;
-    const int c0 = vi * EPV;
+    if (!on[q]) continue;
+    const int c0 = (lane + 32 * q) * EPV;
     float* out = ch.slot >= 0 ? a.part + (int64_t)ch.slot * a.part_ld : a.dg + u * a.ld_dg;
-#pragma unroll
-    for (int i = 0; i < EPV; ++i) out[c0 + i] = acc[q][i];
-    if (c0 % a.Fo == 0) {
+    *reinterpret_cast<float4*>(out + c0) = make_float4(acc[q][0], acc[q][1], acc[q][2], acc[q][3]);
+    if (lead[q]) {
       if (ch.slot >= 0) out[a.HF + hd[q]] = dl[q];
       else a.del[u * a.H + hd[q]] = dl[q];
     }
+  }
+}
+
+// per destination row and head: s = dy_k . agg_k (fp32 agg), and the packed
+// backward stats bs = {er, m + log l, s, 0}
+template <typename T, int NV, int SEG>
+__global__ void __launch_bounds__(256) k_gat_s2(int64_t rows, int64_t row_base, GatArgs a, float4* bs) {
+  constexpr int EPV = 4;
+  const int lane = threadIdx.x & 31;
+  const int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (r >= rows) return;
+  const int64_t v = row_base + r;
+  const float* ag = static_cast<const float*>(a.agg) + r * a.ld_agg;
+  const T* dy = static_cast<const T*>(a.dy) + r * a.lddy;
+  const float dys = a.concat ? 1.f : 1.f / (float)a.H;
+  float part[NV], sums[NV];
+  int hd[NV];
+  bool lead[NV];
+#pragma unroll
+  for (int q = 0; q < NV; ++q) {
+    const int vi = lane + 32 * q;
+    const int c0 = vi * EPV;
+    part[q] = 0.f;
+    hd[q] = vi < a.VPR ? c0 / a.Fo : 0;
+    lead[q] = vi < a.VPR && (c0 % a.Fo) == 0;
+    if (vi < a.VPR) {
+      float g[EPV], d[EPV];
+      GV<float>::unpack(ld16(ag + c0), g);
+      ld_dy4<T>(dy + (a.concat ? c0 : c0 % a.Fo), d);
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) part[q] += d[i] * dys * g[i];
+    }
+  }
+  head_sums<NV, SEG>(part, hd, a.H, sums);
+#pragma unroll
+  for (int q = 0; q < NV; ++q) {
+    if (!lead[q]) continue;
+    const int64_t k = v * a.H + hd[q];
+    const float l = a.l[k];
+    bs[k] = make_float4(a.er[k], l > 0.f ? a.m[k] + __logf(l) : 0.f, sums[q], 0.f);
+  }
+}
+
+// der[v,h] = sum_{e in in(v)} dt_e (forward order: contiguous per row), warp per row
+template <int H>
+__global__ void k_gat_der2(int64_t rows, int64_t row_base, const int64_t* row_ptr, const float* dt, float* der) {
+  const int lane = threadIdx.x & 31;
+  const int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (r >= rows) return;
+  float s[H];
+#pragma unroll
+  for (int h = 0; h < H; ++h) s[h] = 0.f;
+  const int64_t e1 = row_ptr[r + 1];
+  for (int64_t e = row_ptr[r] + lane; e < e1; e += 32) {
+    if constexpr (H == 4) {
+      const float4 v = __ldg(reinterpret_cast<const float4*>(dt) + e);
+      s[0] += v.x; s[1] += v.y; s[2] += v.z; s[3] += v.w;
+    } else {
+#pragma unroll
+      for (int h = 0; h < H; ++h) s[h] += dt[e * H + h];
+    }
+  }
+#pragma unroll
+  for (int h = 0; h < H; ++h) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s[h] += __shfl_xor_sync(0xffffffffu, s[h], o);
+  }
+  if (lane < H) {
+    float o = s[0];
+#pragma unroll
+    for (int h = 1; h < H; ++h) if (lane == h) o = s[h];
+    der[(row_base + r) * H + lane] = o;
   }
 }
 
@@ -424,22 +567,35 @@ __global__ void k_gat_der(int64_t rows, int64_t row_base, const int64_t* row_ptr
 template <typename T>
 __global__ void k_gat_dG(int64_t rows, int64_t row_base, GatArgs a, const float* al, const float* ar,
                          const float* der, T* dG, T* dGlo, int64_t ld_dG, float* part, int64_t rows_per_blk) {
-  // thread per column c (HF <= 1024), rows of this block
+  // thread per column c (HF <= 1024), rows of this block, 4 rows in flight
+  constexpr int RB = 4;
   const int64_t r0 = blockIdx.x * rows_per_blk, r1 = min(rows, r0 + rows_per_blk);
   const float* G = static_cast<const float*>(a.G);
   for (int c = threadIdx.x; c < a.HF; c += blockDim.x) {
     const int h = c / a.Fo;
+    const float alc = al[c], arc = ar[c];
     float sl = 0.f, sr = 0.f;
-    for (int64_t r = r0; r < r1; ++r) {
-      const int64_t v = row_base + r;
-      const float dlv = a.del[v * a.H + h], drv = der[v * a.H + h];
-      const float val = a.dg[v * a.ld_dg + c] + dlv * al[c] + drv * ar[c];
-      const T hi = (T)val;
-      dG[r * ld_dG + c] = hi;
-      if (dGlo) dGlo[r * ld_dG + c] = (T)(val - (float)hi);
-      const float g = (float)G[v * a.ldg + c];
-      sl += dlv * g;
-      sr += drv * g;
+    for (int64_t rb = r0; rb < r1; rb += RB) {
+      float dlv[RB], drv[RB], dgv[RB], gv[RB];
+#pragma unroll
+      for (int i = 0; i < RB; ++i) {
+        const int64_t v = row_base + min(rb + i, r1 - 1);
+        dlv[i] = a.del[v * a.H + h];
+        drv[i] = der[v * a.H + h];
+        dgv[i] = a.dg[v * a.ld_dg + c];
+        gv[i] = G[v * a.ldg + c];
+      }
+#pragma unroll
+      for (int i = 0; i < RB; ++i) {
+        if (rb + i >= r1) break;
+        const int64_t r = rb + i;
+        const float val = dgv[i] + dlv[i] * alc + drv[i] * arc;
+        const T hi = (T)val;
+        dG[r * ld_dG + c] = hi;
+        if (dGlo) dGlo[r * ld_dG + c] = (T)(val - (float)hi);
+        sl += dlv[i] * gv[i];
+        sr += drv[i] * gv[i];
+      }
     }
     part[(int64_t)blockIdx.x * 2 * a.HF + c] = sl;
     part[(int64_t)blockIdx.x * 2 * a.HF + a.HF + c] = sr;
@@ -456,6 +612,8 @@ __global__ void k_pair_reduce(const float* part, int nblk, int n, float* out0, f
 }
 
 constexpr int DG_BLKS = 592;
+
+unsigned gs_grid(int64_t threads) { return (unsigned)std::max<int64_t>(1, cdiv(threads, 256)); }
 
 template <typename T>
 int nv_for(int VPR) { return VPR <= 32 ? 1 : (VPR <= 64 ? 2 : 4); }
@@ -506,9 +664,9 @@ void gat_layout(wg_plan_s* p) {
   S.add("l", sizeof(float) * V * H);
   W.add("wt", (size_t)rup(HF, 16) * p->pi * s);
   W.add("w", (size_t)rup(d.f_in, 16) * p->po * s);
-  W.add("part", sizeof(float) * std::max(1, std::max(gp->n_fslots, gp->n_bslots)) * (HF + 2 * H + 8));
+  W.add("part", sizeof(float) * std::max(1, std::max(gp->n_fslots, gp->n_bslots)) * rup(HF + 2 * H + 8, 4));
   W.add("dt", sizeof(float) * std::max<int64_t>(1, g->fwd.E) * H);
-  W.add("s", sizeof(float) * V * H);
+  W.add("bs", sizeof(float4) * V * H);
   W.add("del", sizeof(float) * V * H);
   W.add("der", sizeof(float) * V * H);
   W.add("dg", sizeof(float) * V * HF);
@@ -535,6 +693,7 @@ static wg_status gat_fwd_t(wg_plan_s* p, const wg_params* P, const wg_fwd_args* 
   const int64_t V = g->V, nr = g->ve - g->vb, vb = g->vb;
   WG_REQ(nr == V, WG_ERR_UNSUPPORTED, "GAT with a 1-D partition is not implemented");
   WG_REQ(Fo % EPV == 0, WG_ERR_UNSUPPORTED, "GAT: per-head width must be a multiple of 16 bytes");
+  WG_REQ(HF <= 512, WG_ERR_UNSUPPORTED, "GAT: heads * f_out must be <= 512");
   WG_REQ(P->W && P->attn_l && P->attn_r, WG_ERR_INVALID, "GAT needs W, attn_l, attn_r");
   const Layout &S = p->saved, &L = p->ws;
   void* ws = A->workspace;
@@ -545,8 +704,10 @@ static wg_status gat_fwd_t(wg_plan_s* p, const wg_params* P, const wg_fwd_args* 
   a.el = S.at<float>(A->saved, "el"); a.er = S.at<float>(A->saved, "er");
   a.m = S.at<float>(A->saved, "m"); a.l = S.at<float>(A->saved, "l");
   a.agg = S.at<void>(A->saved, "agg"); a.ld_agg = rup(HF, 4);
-  a.part = L.at<float>(ws, "part"); a.part_ld = HF + 2 * H + 8;
+  a.part = L.at<float>(ws, "part"); a.part_ld = (int)rup(HF + 2 * H + 8, 4);   // 16-byte rows (float4 partial stores)
   a.concat = d.concat_heads;
+  a.y = A->y; a.ldy = A->ldy; a.FO = d.concat_heads ? HF : Fo;
+  a.bias = d.bias ? P->bias : nullptr; a.relu = d.fuse_relu;
   // G = x W  (vertex-level transform, tcgen05 for bf16; fp32 accumulator kept)
   void* wt = L.at<void>(ws, "wt");
   WG_TRY(prep_weight(d.dtype, P->W, d.f_in, HF, 1, wt, p->pi, (int)rup(HF, 16), st));
@@ -557,22 +718,23 @@ static wg_status gat_fwd_t(wg_plan_s* p, const wg_params* P, const wg_fwd_args* 
     WG_TRY(gemm_nt(d.dtype, V, (int)rup(HF, 8), &part, 1, e, nullptr, 0, st));
   }
   const int NV = nv_for<float>(a.VPR);
-  ProfScope ps(PK_GAT, st, (double)g->fwd.E * (HF * 4.0 + 4.0 * H + 4) + (double)V * HF * (4.0 + s) * 2, 0.0);
-  const unsigned wb = (unsigned)cdiv(V * 32, 256);
+  // algorithmic bytes: logits (G row), per edge the gathered G row + el + index,
+  // per row the aggregate (saved) and y
+  ProfScope ps(PK_GAT, st,
+               (double)g->fwd.E * (HF * 4.0 + 4.0 * H + 4) + (double)V * HF * 8.0 + (double)V * a.FO * s, 0.0);
+  const unsigned wb = gs_grid(V * 32);
   if (NV == 1) WG_LAUNCH((k_gat_logits<float, 1>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
   else if (NV == 2) WG_LAUNCH((k_gat_logits<float, 2>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
   else WG_LAUNCH((k_gat_logits<float, 4>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
   a.idx = g->fwd.idx;
   a.chunks = gp->fwd; a.n_chunks = gp->n_fwd;
   if (gp->n_fwd) {
-    const unsigned cbk = (unsigned)cdiv((int64_t)gp->n_fwd * 32, 256);
-    if (NV == 1) WG_LAUNCH((k_gat_fwd<float, 1, 4>), cbk, 256, 0, st, a, vb);
-    else if (NV == 2) WG_LAUNCH((k_gat_fwd<float, 2, 4>), cbk, 256, 0, st, a, vb);
-    else WG_LAUNCH((k_gat_fwd<float, 4, 2>), cbk, 256, 0, st, a, vb);
+    const unsigned cbk = gs_grid((int64_t)gp->n_fwd * 32);
+    if (NV == 1) WG_LAUNCH((k_gat_fwd<float, T, 1, 4>), cbk, 256, 0, st, a, vb);
+    else if (NV == 2) WG_LAUNCH((k_gat_fwd<float, T, 2, 4>), cbk, 256, 0, st, a, vb);
+    else WG_LAUNCH((k_gat_fwd<float, T, 4, 2>), cbk, 256, 0, st, a, vb);
   }
-  if (gp->n_fsplit) WG_LAUNCH(k_gat_fwd_combine<float>, gp->n_fsplit, 128, 0, st, a, gp->fsplit, vb);
-  const int FO = d.concat_heads ? HF : Fo;
-  WG_LAUNCH(k_gat_out<T>, 1184, 256, 0, st, nr, a, d.bias ? P->bias : nullptr, d.fuse_relu, A->y, A->ldy, FO);
+  if (gp->n_fsplit) WG_LAUNCH(k_gat_fwd_combine<T>, gp->n_fsplit, 256, 0, st, a, gp->fsplit, vb);
   return WG_OK;
 }
 
@@ -597,7 +759,7 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
   a.el = S.at<float>(A->saved, "el"); a.er = S.at<float>(A->saved, "er");
   a.m = S.at<float>(A->saved, "m"); a.l = S.at<float>(A->saved, "l");
   a.agg = S.at<void>(A->saved, "agg"); a.ld_agg = rup(HF, 4);
-  a.part = L.at<float>(ws, "part"); a.part_ld = HF + 2 * H + 8;
+  a.part = L.at<float>(ws, "part"); a.part_ld = (int)rup(HF + 2 * H + 8, 4);   // 16-byte rows (float4 partial stores)
   a.concat = d.concat_heads;
   (void)EPV;
   // dT = dy (masked by the fused ReLU) ; db
@@ -608,30 +770,61 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
                         d.fuse_relu ? const_cast<void*>(dT) : nullptr, lddT, Gr ? Gr->bias : nullptr,
                         L.at<float>(ws, "colsum"), st));
   a.dy = dT; a.lddy = lddT;
-  float* sbuf = L.at<float>(ws, "s");
-  a.s = sbuf;
-  ProfScope ps(PK_GAT, st, (double)g->bwd.E * (FO * s + 16.0 * H + 12) + (double)V * HF * (s + 12), 0.0);
-  WG_LAUNCH(k_gat_s<T>, (unsigned)cdiv(nr * 32, 256), 256, 0, st, nr, vb, a, sbuf);
+  float4* bs = L.at<float4>(ws, "bs");
+  a.bs = bs;
+  void* dG = L.at<void>(ws, "dG");
+  void* dGlo = d.dtype == WG_BF16 ? L.at<void>(ws, "dGlo") : nullptr;
+  {
+  // algorithmic bytes: s/bs (agg, dy rows), per out-edge the gathered dy row +
+  // stats + index + fwdpos + dt, per row G and dg; der (dt again); dG
+  ProfScope ps(PK_GAT, st,
+               (double)g->bwd.E * (HF * s + 16.0 * H + 12 + 8.0 * H) +
+                   (double)V * HF * (4.0 + s + 4.0 + 4.0 + 4.0 + 4.0 + s * (d.dtype == WG_BF16 ? 2 : 1)), 0.0);
+  const int NV = nv_for<float>(a.VPR);
+  const int vph = Fo / 4;                      // fp32 G vectors per head
+  const int SEG = (vph == 8 || vph == 16 || vph == 32) ? vph : 0;
+  const unsigned rbk = gs_grid(nr * 32);
+#define WG_GAT_S(NV_, SEG_) WG_LAUNCH((k_gat_s2<T, NV_, SEG_>), rbk, 256, 0, st, nr, vb, a, bs)
+#define WG_GAT_SEG(M, NV_)                      \
+  do {                                          \
+    if (SEG == 8) M(NV_, 8);                    \
+    else if (SEG == 16) M(NV_, 16);             \
+    else if (SEG == 32) M(NV_, 32);             \
+    else M(NV_, 0);                             \
+  } while (0)
+  if (NV == 1) WG_GAT_SEG(WG_GAT_S, 1);
+  else if (NV == 2) WG_GAT_SEG(WG_GAT_S, 2);
+  else WG_GAT_SEG(WG_GAT_S, 4);
   a.idx = g->bwd.idx;
   a.fwdpos = g->fwdpos;
   a.dt = L.at<float>(ws, "dt");
   a.dg = L.at<float>(ws, "dg"); a.ld_dg = HF;
   a.del = L.at<float>(ws, "del");
   a.chunks = gp->bwd; a.n_chunks = gp->n_bwd;
-  const int NV = nv_for<float>(a.VPR);
   if (gp->n_bwd) {
-    const unsigned cbk = (unsigned)cdiv((int64_t)gp->n_bwd * 32, 256);
-    if (NV == 1) WG_LAUNCH((k_gat_bwd_src<T, 1>), cbk, 256, 0, st, a, vb);
-    else if (NV == 2) WG_LAUNCH((k_gat_bwd_src<T, 2>), cbk, 256, 0, st, a, vb);
-    else WG_LAUNCH((k_gat_bwd_src<T, 4>), cbk, 256, 0, st, a, vb);
+    const unsigned cbk = gs_grid((int64_t)gp->n_bwd * 32);
+#define WG_GAT_B1(NV_, SEG_) WG_LAUNCH((k_gat_bwd_src2<T, NV_, 8, SEG_>), cbk, 256, 0, st, a, vb)
+#define WG_GAT_B2(NV_, SEG_) WG_LAUNCH((k_gat_bwd_src2<T, NV_, 4, SEG_>), cbk, 256, 0, st, a, vb)
+#define WG_GAT_B4(NV_, SEG_) WG_LAUNCH((k_gat_bwd_src2<T, NV_, 2, SEG_>), cbk, 256, 0, st, a, vb)
+    if (NV == 1) WG_GAT_SEG(WG_GAT_B1, 1);
+    else if (NV == 2) WG_GAT_SEG(WG_GAT_B2, 2);
+    else WG_GAT_SEG(WG_GAT_B4, 4);
+#undef WG_GAT_B1
+#undef WG_GAT_B2
+#undef WG_GAT_B4
   }
+#undef WG_GAT_S
+#undef WG_GAT_SEG
   // rows without out-edges have no chunk: their dg / del are zero
   // (chunks cover every row, including empty ones -- see build_chunks)
   if (gp->n_bsplit) WG_LAUNCH(k_gat_bwd_combine, gp->n_bsplit, 128, 0, st, a, gp->bsplit, vb);
   float* der = L.at<float>(ws, "der");
-  WG_LAUNCH(k_gat_der, (unsigned)cdiv(nr * 32, 256), 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, H, der);
-  void* dG = L.at<void>(ws, "dG");
-  void* dGlo = d.dtype == WG_BF16 ? L.at<void>(ws, "dGlo") : nullptr;
+  const unsigned tbk = gs_grid(nr * 32);
+  if (H == 4) WG_LAUNCH(k_gat_der2<4>, tbk, 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, der);
+  else if (H == 1) WG_LAUNCH(k_gat_der2<1>, tbk, 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, der);
+  else if (H == 2) WG_LAUNCH(k_gat_der2<2>, tbk, 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, der);
+  else if (H == 8) WG_LAUNCH(k_gat_der2<8>, tbk, 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, der);
+  else WG_LAUNCH(k_gat_der, (unsigned)cdiv(nr * 32, 256), 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, H, der);
   const int64_t rpb = std::max<int64_t>(1, cdiv(nr, DG_BLKS));
   const int nblk = (int)cdiv(nr, rpb);
   float* dgp = L.at<float>(ws, "dgp");
@@ -639,6 +832,7 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
             rpb);
   WG_LAUNCH(k_pair_reduce, (unsigned)cdiv(2 * HF, 128), 128, 0, st, dgp, nblk, HF, Gr ? Gr->attn_l : nullptr,
             Gr ? Gr->attn_r : nullptr);
+  }
   // dW = x^T dG ; dx = dG W^T   (dG = hi + lo for bf16)
   if (Gr && Gr->W) {
     WG_TRY(gemm_tn(d.dtype, nr, d.f_in, HF, A->x, A->ldx, dG, p->po, Gr->W, L.at<void>(ws, "tn"), st));

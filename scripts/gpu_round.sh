@@ -19,7 +19,7 @@ if [[ $mode == ncu || $mode == all ]]; then
       python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_launch_run.log 2>&1
   timeout 1200 ncu --set full --clock-control none --import-source on -k regex:k_agg -s 6 -c 3 -o gpurun_out/prof_agg -f \
       python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_full_run.log 2>&1
-  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:k_tc_gemm -s 4 -c 2 -o gpurun_out/prof_gemm -f \
+  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:k_gemm_nt_p -s 4 -c 3 -o gpurun_out/prof_gemm -f \
       python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_gemm_run.log 2>&1
   ls -la gpurun_out/*.ncu-rep
 fi
@@ -27,4 +27,9 @@ if [[ $mode == ncuagg ]]; then
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_agg_cp -s 5 -c 1 -o gpurun_out/prof_agg1 -f \
       python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_agg1.log 2>&1
   ls -la gpurun_out/prof_agg1.ncu-rep
+fi
+if [[ $mode == ncugemm ]]; then
+  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:"k_gemm_nt_p|k_tc_gemm" -s 4 -c 6 -o gpurun_out/prof_gemm -f \
+      python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_gemm_run.log 2>&1
+  ls -la gpurun_out/prof_gemm.ncu-rep
 fi
