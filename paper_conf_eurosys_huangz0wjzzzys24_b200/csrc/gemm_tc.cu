@@ -151,24 +151,56 @@ __device__ __forceinline__ void mbar_arrive1(uint32_t bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
 
-// 3xTF32 operand split: hi = x with the 13 low mantissa bits cleared, lo = x - hi
-__device__ __forceinline__ void split_tf32(uint4& x, uint4& lo) {
-  uint32_t* v = reinterpret_cast<uint32_t*>(&x);
-  uint32_t* l = reinterpret_cast<uint32_t*>(&lo);
+// 3xTF32 stage split in shared memory: n16 16-byte units at `base` become hi
+// (in place) and lo (at base + n16 * 16); threads ct = 0..nct-1, explicit
+// shared-space vector loads / stores, 4 units in flight per thread
+__device__ __forceinline__ void tf32_split_stage(uint32_t base, int n16, int ct, int nct) {
+  const uint32_t lo = base + (uint32_t)n16 * 16u;
+  int i = ct;
+  for (; i + 3 * nct < n16; i += 4 * nct) {
+    uint32_t v[4][4];
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const uint32_t h = v[i] & 0xffffe000u;
-    l[i] = __float_as_uint(__uint_as_float(v[i]) - __uint_as_float(h));
-    v[i] = h;
+    for (int u = 0; u < 4; ++u)
+      asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(v[u][0]), "=r"(v[u][1]), "=r"(v[u][2]), "=r"(v[u][3])
+                   : "r"(base + (uint32_t)(i + u * nct) * 16u));
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      uint32_t h[4], l[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        h[k] = v[u][k] & 0xffffe000u;
+        l[k] = __float_as_uint(__uint_as_float(v[u][k]) - __uint_as_float(h[k]));
+      }
+      const uint32_t off = (uint32_t)(i + u * nct) * 16u;
+      asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(base + off), "r"(h[0]), "r"(h[1]), "r"(h[2]), "r"(h[3])
+                   : "memory");
+      asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(lo + off), "r"(l[0]), "r"(l[1]), "r"(l[2]), "r"(l[3])
+                   : "memory");
+    }
+  }
+  for (; i < n16; i += nct) {
+    uint32_t v[4], h[4], l[4];
+    asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3])
+                 : "r"(base + (uint32_t)i * 16u));
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      h[k] = v[k] & 0xffffe000u;
+      l[k] = __float_as_uint(__uint_as_float(v[k]) - __uint_as_float(h[k]));
+    }
+    asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(base + (uint32_t)i * 16u), "r"(h[0]), "r"(h[1]), "r"(h[2]),
+                 "r"(h[3]) : "memory");
+    asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(lo + (uint32_t)i * 16u), "r"(l[0]), "r"(l[1]), "r"(l[2]),
+                 "r"(l[3]) : "memory");
   }
 }
 
 // MN: TN variant (both operands MN-major, fp32 partial output).  T = float:
-// 3xTF32 with two extra converter warps (threads 128..191) that split each
+// 3xTF32 with four extra converter warps (threads 128..255) that split each
 // landed stage into hi (in place) and lo (twin buffer after the stage).
 // Stage depth: 128 / sizeof(T) K elements (one 128-byte swizzle row).
 template <bool MN, typename T>
-__global__ void __launch_bounds__(sizeof(T) == 4 ? 192 : 128, 1)
+__global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
     k_tc_gemm(const __grid_constant__ CUtensorMap tA0, const __grid_constant__ CUtensorMap tB0,
               const __grid_constant__ CUtensorMap tA1, const __grid_constant__ CUtensorMap tB1,
               const __grid_constant__ CUtensorMap tA2, const __grid_constant__ CUtensorMap tB2, TcParams p) {
@@ -195,7 +227,7 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 192 : 128, 1)
     for (int s = 0; s < S; ++s) {
       mbar_init(smem_u32(&full[s]), 1);
       mbar_init(smem_u32(&empty[s]), 1);
-      mbar_init(smem_u32(&conv[s]), 64);
+      mbar_init(smem_u32(&conv[s]), 128);
     }
     mbar_init(smem_u32(accf), 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -288,15 +320,7 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 192 : 128, 1)
     for (int kb = 0; kb < total_kb; ++kb) {
       const int s = kb % S;
       mbar_wait(smem_u32(&full[s]), (kb / S) & 1);
-      uint4* x = reinterpret_cast<uint4*>(ring + s * stage);
-      uint4* lo = x + n16;
-#pragma unroll 4
-      for (int i = ct; i < n16; i += 64) {
-        uint4 v = x[i], l;
-        split_tf32(v, l);
-        x[i] = v;
-        lo[i] = l;
-      }
+      tf32_split_stage(smem_u32(ring + s * stage), n16, ct, 128);
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       mbar_arrive1(smem_u32(&conv[s]));
     }
@@ -433,7 +457,7 @@ wg_status launch(dim3 grid, size_t smem, const CUtensorMap* maps, const TcParams
     cudaFuncSetAttribute(k_tc_gemm<MN, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr = true;
   }
-  WG_LAUNCH((k_tc_gemm<MN, T>), grid, sizeof(T) == 4 ? 192 : 128, smem, s, maps[0], maps[1], maps[2], maps[3], maps[4],
+  WG_LAUNCH((k_tc_gemm<MN, T>), grid, sizeof(T) == 4 ? 256 : 128, smem, s, maps[0], maps[1], maps[2], maps[3], maps[4],
             maps[5], p);
   return WG_OK;
 }

@@ -6,7 +6,7 @@
 // hi = x with its 13 low mantissa bits cleared and lo = x - hi (exact), and
 // D += A_hi B_hi + A_hi B_lo + A_lo B_hi (the dropped lo*lo term is ~2^-22
 // relative), so fp32 layers keep fp32-level accuracy on tensor cores.  The
-// split runs in shared memory: two converter warps rewrite each landed stage
+// split runs in shared memory: four converter warps rewrite each landed stage
 // (hi in place, lo into a twin buffer) before the MMA warp consumes it.
 //
 // Grouped B (RGCN relation weights, GemmPart::tile_group): the B rows of
@@ -24,7 +24,7 @@
 //   warps 2-5   epilogue: tcgen05.ld (warp w drains TMEM lanes 32*(w%4)..),
 //               fused epilogue math, pack into a 128-byte-swizzled staging
 //               tile, TMA store (bulk_group, 2-deep) -- coalesced writes;
-//   warps 7-8   (fp32 only) hi / lo converters.
+//   warps 7-10  (fp32 only) hi / lo converters.
 // One CTA per SM loops over 128 x BN tiles (N fastest, so A tiles of the N
 // tiles of one row block are adjacent in time).
 #include <cuda.h>
@@ -56,7 +56,7 @@ template <typename T> struct Cfg {
   static constexpr int BKE = 128 / ES;
   static constexpr int CHE = 128 / ES;
   static constexpr int EPV = 16 / ES;              // elements per 16-byte unit
-  static constexpr int NTHREADS = TF32 ? 288 : 224;
+  static constexpr int NTHREADS = TF32 ? 352 : 224;   // fp32: + 4 converter warps
 };
 
 struct P2 {
@@ -124,17 +124,50 @@ __device__ __forceinline__ void mma_tf32(uint32_t tmem, uint64_t a, uint64_t b, 
       "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\ntcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem),
       "l"(a), "l"(b), "r"(idesc), "r"(acc));
 }
-// x = hi + lo, hi = x with the 13 low mantissa bits cleared (exactly a TF32 value)
-__device__ __forceinline__ void split_tf32(uint4& x, uint4& lo) {
-  uint32_t* v = reinterpret_cast<uint32_t*>(&x);
-  uint32_t* l = reinterpret_cast<uint32_t*>(&lo);
+// 3xTF32 stage split in shared memory: n16 16-byte units at `base` become hi
+// (in place) and lo (at base + n16 * 16); threads ct = 0..nct-1, explicit
+// shared-space vector loads / stores, 4 units in flight per thread
+__device__ __forceinline__ void tf32_split_stage(uint32_t base, int n16, int ct, int nct) {
+  const uint32_t lo = base + (uint32_t)n16 * 16u;
+  int i = ct;
+  for (; i + 3 * nct < n16; i += 4 * nct) {
+    uint32_t v[4][4];
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const uint32_t h = v[i] & 0xffffe000u;
-    l[i] = __float_as_uint(__uint_as_float(v[i]) - __uint_as_float(h));
-    v[i] = h;
+    for (int u = 0; u < 4; ++u)
+      asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(v[u][0]), "=r"(v[u][1]), "=r"(v[u][2]), "=r"(v[u][3])
+                   : "r"(base + (uint32_t)(i + u * nct) * 16u));
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      uint32_t h[4], l[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        h[k] = v[u][k] & 0xffffe000u;
+        l[k] = __float_as_uint(__uint_as_float(v[u][k]) - __uint_as_float(h[k]));
+      }
+      const uint32_t off = (uint32_t)(i + u * nct) * 16u;
+      asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(base + off), "r"(h[0]), "r"(h[1]), "r"(h[2]), "r"(h[3])
+                   : "memory");
+      asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(lo + off), "r"(l[0]), "r"(l[1]), "r"(l[2]), "r"(l[3])
+                   : "memory");
+    }
+  }
+  for (; i < n16; i += nct) {
+    uint32_t v[4], h[4], l[4];
+    asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3])
+                 : "r"(base + (uint32_t)i * 16u));
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      h[k] = v[k] & 0xffffe000u;
+      l[k] = __float_as_uint(__uint_as_float(v[k]) - __uint_as_float(h[k]));
+    }
+    asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(base + (uint32_t)i * 16u), "r"(h[0]), "r"(h[1]), "r"(h[2]),
+                 "r"(h[3]) : "memory");
+    asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(lo + (uint32_t)i * 16u), "r"(l[0]), "r"(l[1]), "r"(l[2]),
+                 "r"(l[3]) : "memory");
   }
 }
+
 __device__ __forceinline__ void mma_commit(uint32_t bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
 }
@@ -225,7 +258,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
     for (int s = 0; s < S; ++s) {
       mbar_init(su32(&full[s]), 1);
       mbar_init(su32(&empty[s]), 1);
-      mbar_init(su32(&conv[s]), 64);
+      mbar_init(su32(&conv[s]), 128);
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(su32(&tfull[b]), 1);
@@ -330,7 +363,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
     }
   } else if (warp >= 7) {
     if constexpr (C::TF32) {
-      // ------------------------------------------------ hi / lo converters (64 threads)
+      // ------------------------------------------------ hi / lo converters (128 threads)
       const int ct = threadIdx.x - 224;
       const int n16 = (A_STAGE + b_bytes) / 16;
       int s = 0;
@@ -338,15 +371,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
       for (int64_t t = blockIdx.x; t < p.num_tiles; t += gridDim.x) {
         for (int kb = 0; kb < total_kb; ++kb) {
           mbar_wait(su32(&full[s]), ph);
-          uint4* x = reinterpret_cast<uint4*>(ring + s * L.stage);
-          uint4* lo = x + n16;
-#pragma unroll 4
-          for (int i = ct; i < n16; i += 64) {
-            uint4 v = x[i], l;
-            split_tf32(v, l);
-            x[i] = v;
-            lo[i] = l;
-          }
+          tf32_split_stage(su32(ring + s * L.stage), n16, ct, 128);
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           mbar_arrive(su32(&conv[s]));
           if (++s == S) { s = 0; ph ^= 1; }
