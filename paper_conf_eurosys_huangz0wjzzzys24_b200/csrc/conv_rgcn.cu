@@ -7,18 +7,24 @@
 //   EDGE   (gather-then-transform): one stage-1 row per (dst, relation)
 //          segment, S = sum_e c_e x[src_e]; the row is transformed by W_r and
 //          contributes once to y[dst];
-//   VERTEX (transform-before-gather): one stage-1 row per unique source of the
-//          gTask (T1 unique extraction: src-id_unique / src-id_map),
-//          transformed once by W_r (T2 indexing swapping, Index-2D A[B] x C[D] =
-//          (A x C)[B, D]); every edge contributes c_e Y[map(e)].
-// Stage-1 rows of all gTasks are laid out grouped by relation (each group padded
-// to 128 rows), so one grouped GEMM applies W_r to every row of group r
-// ("a batch of K src rows becomes a matrix-matrix product");
-// stage 3 is the contribution-list gather-reduce into destination rows.
-// Backward mirrors this on the transposed partition (source tile x relation):
-// G = sum over (src, relation) segments of c_e dy[dst], dX = G W_r^T (grouped),
-// dx = sum over a source's segments; dW_r = X_g^T G over group r.
-// Round-1 scope: unfused (stage buffers round-trip HBM); DESIGN.md "RGCN".
+//   VERTEX (transform-before-gather): one Y row per unique (source, relation)
+//          pair over all VERTEX gTasks of the relation (T1 unique extraction,
+//          src-id_unique / src-id_map), Y = x[src] W_r computed
+//          once (T2 indexing swapping, Index-2D A[B] x C[D] = (A x C)[B, D],
+//          P:L1867-1876); every edge contributes c_e Y[map(e)].  The GEMM
+//          gathers its A rows straight from x (TMA tile::gather4): the unique
+//          rows are never materialised.
+// Y rows and EDGE segment rows are laid out grouped by relation (each group
+// padded to 128 rows), so one grouped GEMM per block applies W_r to every row
+// of group r ("a batch of K src rows becomes a matrix-matrix product",
+// P:L2159-2189); stage 3 is the contribution-list gather-reduce into
+// destination rows.  Backward mirrors this on the transposed partition
+// (source tile x relation): G = sum over (src, relation) segments of c_e
+// dy[dst], dX = G W_r^T (grouped), dx = sum over a source's segments;
+// dW_r = X_g^T G over group r, X_g = x[src] of every (src, relation) row
+// (a gather copy: a TMA gather4 K-row load of 32-bit MN-major tiles measured
+// 2.5x slower than this copy + tile loads).
+// Stage buffers (segment sums, Y, G, dX) round-trip HBM; DESIGN.md "RGCN".
 #include <algorithm>
 #include <numeric>
 #include <random>
@@ -44,10 +50,13 @@ struct CsrExec {
 
 struct RgcnPlan {
   int R = 1;
-  int64_t n1 = 0, n1T = 0;           // stage-1 typed rows (padded), forward / transposed
-  CsrExec f1, f3, b1, b3, bg;
-  int32_t* tile_type = nullptr;      // [n1 / 128]
+  int64_t n1v = 0, n1e = 0, n1T = 0; // Y rows, EDGE segment rows, transposed rows (each padded per relation)
+  CsrExec f1, f3, b1, b3;
+  int32_t* ysrc = nullptr;           // [n1v] source vertex of each Y row (0 in padding)
+  int32_t* tile_type_v = nullptr;    // [n1v / 128]
+  int32_t* tile_type_e = nullptr;    // [n1e / 128]
   int32_t* tile_typeT = nullptr;     // [n1T / 128]
+  CsrExec bg;                        // transposed rows -> their source vertex (X_g gather copy)
   std::vector<int64_t> h_group_offT; // [R+1] transposed group row offsets
   TnUnits tn;                        // dW_r work units over the transposed groups
 };
@@ -234,13 +243,21 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
     p->n_vert_tasks = std::count(p->plan_bits.begin(), p->plan_bits.end(), 1);
     p->n_edge_tasks = nt - p->n_vert_tasks;
   }
-  // ---- forward stage-1 rows, grouped by relation
+  // ---- forward rows: EDGE segment rows and VERTEX unique (src, relation) rows, grouped by relation
   struct Row1 { int64_t ent_b, ent_e; float rs; };
   std::vector<std::vector<Row1>> rows1(R);
-  std::vector<std::vector<int32_t>> ents(R);                 // per-type stage-1 entries (source ids)
-  struct Contrib { int32_t dst; int32_t type; int64_t row; float c; };
+  std::vector<std::vector<int32_t>> ents(R);                 // per-type EDGE stage-1 entries (source ids)
+  std::vector<std::vector<int32_t>> uniq(R);                 // per-type VERTEX sources (sorted, unique)
+  struct Contrib { int32_t dst; int32_t type; int64_t row; float c; bool vert; };
   std::vector<Contrib> contrib;
   contrib.reserve(E);
+  for (int64_t t = 0; t < nt; ++t)
+    if (p->plan_bits[t] == 1)
+      for (int64_t i = tasks[t].e_begin; i < tasks[t].e_end; ++i) uniq[tasks[t].type].push_back(fi_[i]);
+  for (int r = 0; r < R; ++r) {
+    std::sort(uniq[r].begin(), uniq[r].end());
+    uniq[r].erase(std::unique(uniq[r].begin(), uniq[r].end()), uniq[r].end());
+  }
   int64_t open_seg_dst = -1, open_seg_type = -1;           // EDGE segment continuing across SPLIT tasks
   for (int64_t t = 0; t < nt; ++t) {
     const wg_task& k = tasks[t];
@@ -253,7 +270,7 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
         if (!cont) {
           const float rs = d.norm == WG_NORM_RIGHT ? 1.f / (float)seg_len_at[i] : 1.f;
           rows1[r].push_back(Row1{(int64_t)ents[r].size(), (int64_t)ents[r].size(), rs});
-          contrib.push_back(Contrib{fk[i], r, (int64_t)rows1[r].size() - 1, 1.f});
+          contrib.push_back(Contrib{fk[i], r, (int64_t)rows1[r].size() - 1, 1.f, false});
         }
         for (int64_t q = i; q < j; ++q) ents[r].push_back(fi_[q]);
         rows1[r].back().ent_e = (int64_t)ents[r].size();
@@ -263,30 +280,34 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
       }
     } else {
       open_seg_dst = -1;
-      std::vector<int32_t> us(fi_.begin() + k.e_begin, fi_.begin() + k.e_end);
-      std::sort(us.begin(), us.end());
-      us.erase(std::unique(us.begin(), us.end()), us.end());
-      const int64_t base = (int64_t)rows1[r].size();
-      for (int32_t u : us) {
-        rows1[r].push_back(Row1{(int64_t)ents[r].size(), (int64_t)ents[r].size() + 1, 1.f});
-        ents[r].push_back(u);
-      }
       for (int64_t i = k.e_begin; i < k.e_end; ++i) {
-        const int64_t m = std::lower_bound(us.begin(), us.end(), fi_[i]) - us.begin();
-        contrib.push_back(Contrib{fk[i], r, base + m, coef_eid[fperm[i]]});
+        const int64_t m = std::lower_bound(uniq[r].begin(), uniq[r].end(), fi_[i]) - uniq[r].begin();
+        contrib.push_back(Contrib{fk[i], r, m, coef_eid[fperm[i]], true});
       }
     }
   }
-  // typed layout: group r at base1[r], padded to 128 rows
-  std::vector<int64_t> base1(R + 1, 0);
-  for (int r = 0; r < R; ++r) base1[r + 1] = base1[r] + rup((int64_t)rows1[r].size(), TILE_M);
-  rp->n1 = base1[R];
+  // Y block: group r at base_v[r]; EDGE block: group r at base_e[r]; each padded to 128 rows
+  std::vector<int64_t> base_v(R + 1, 0), base_e(R + 1, 0);
+  for (int r = 0; r < R; ++r) {
+    base_v[r + 1] = base_v[r] + rup((int64_t)uniq[r].size(), TILE_M);
+    base_e[r + 1] = base_e[r] + rup((int64_t)rows1[r].size(), TILE_M);
+  }
+  rp->n1v = base_v[R];
+  rp->n1e = base_e[R];
   {
-    std::vector<int64_t> rpv(rp->n1 + 1, 0);
+    std::vector<int32_t> ys(rp->n1v, 0), tt(rp->n1v / TILE_M);
+    for (int r = 0; r < R; ++r) {
+      std::copy(uniq[r].begin(), uniq[r].end(), ys.begin() + base_v[r]);
+      for (int64_t t = base_v[r] / TILE_M; t < base_v[r + 1] / TILE_M; ++t) tt[t] = r;
+    }
+    WG_TRY(up(p, ys, &rp->ysrc));
+    WG_TRY(up(p, tt, &rp->tile_type_v));
+  }
+  {
+    std::vector<int64_t> rpv(rp->n1e + 1, 0);
     std::vector<int32_t> idx;
-    std::vector<float> rs(rp->n1, 1.f);
+    std::vector<float> rs(rp->n1e, 1.f);
     bool any_rs = false;
-    idx.reserve(E);
     int64_t row = 0;
     for (int r = 0; r < R; ++r) {
       for (const Row1& w : rows1[r]) {
@@ -295,17 +316,18 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
         any_rs |= w.rs != 1.f;
         rpv[++row] = (int64_t)idx.size();
       }
-      while (row < base1[r + 1]) rpv[++row] = (int64_t)idx.size();
+      while (row < base_e[r + 1]) rpv[++row] = (int64_t)idx.size();
     }
     WG_TRY(build_exec(p, rpv, idx, nullptr, any_rs ? &rs : nullptr, g->E_max, &rp->f1));
-    std::vector<int32_t> tt(rp->n1 / TILE_M);
+    std::vector<int32_t> tt(rp->n1e / TILE_M);
     for (int r = 0; r < R; ++r)
-      for (int64_t t = base1[r] / TILE_M; t < base1[r + 1] / TILE_M; ++t) tt[t] = r;
-    WG_TRY(up(p, tt, &rp->tile_type));
+      for (int64_t t = base_e[r] / TILE_M; t < base_e[r + 1] / TILE_M; ++t) tt[t] = r;
+    WG_TRY(up(p, tt, &rp->tile_type_e));
   }
-  // stage 3: contributions per destination row (sorted by dst, then typed row)
+  // stage 3: contributions per destination row (sorted by dst, then stage row);
+  // stage rows: [Y block | EDGE block]
   {
-    for (auto& c : contrib) c.row += base1[c.type];
+    for (auto& c : contrib) c.row += c.vert ? base_v[c.type] : rp->n1v + base_e[c.type];
     std::stable_sort(contrib.begin(), contrib.end(), [](const Contrib& a, const Contrib& b) {
       return a.dst != b.dst ? a.dst < b.dst : a.row < b.row;
     });
@@ -401,15 +423,15 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
   W.add("w", (size_t)R * rows_i * p->po * s);           // stacked W_r
   W.add("w0t", (size_t)rows_o * p->pi * s);
   W.add("w0", (size_t)rows_i * p->po * s);
-  W.add("a1", (size_t)rp->n1 * p->pi * s);
-  W.add("t1", (size_t)rp->n1 * p->po * s);
+  W.add("a1", (size_t)std::max<int64_t>(rp->n1e, 1) * p->pi * s);
+  W.add("t1", (size_t)std::max<int64_t>(rp->n1v + rp->n1e, 1) * p->po * s);
   W.add("self", (size_t)V * p->po * s);
   W.add("part", sizeof(float) * std::max({1, rp->f1.n_slots, rp->f3.n_slots, rp->b1.n_slots, rp->b3.n_slots,
                                            rp->bg.n_slots}) * pl);
+  W.add("xg", (size_t)rp->n1T * p->pi * s);
   W.add("dt", (size_t)V * p->po * s);
   W.add("gt", (size_t)rp->n1T * p->po * s);
   W.add("dxt", (size_t)rp->n1T * p->pi * s);
-  W.add("xg", (size_t)rp->n1T * p->pi * s);
   W.add("dxs", (size_t)V * p->pi * s);
   W.add("colsum", bias_grad_scratch(V, (int)p->po));
   W.add("tn", std::max(gemm_tn_scratch(V, d.f_in, d.f_out), gemm_tn_grouped_scratch(rp->tn.n_units, d.f_in, d.f_out)));
@@ -437,9 +459,9 @@ wg_status rgcn_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, c
   ProfScope ps(PK_RGCN, st, 0.0, 0.0);
   void* wt = L.at<void>(ws, "wt");
   WG_TRY(prep_weight_batched(dt, P->W, R, d.f_in, d.f_out, 1, wt, p->pi, (int)rows_o, st));
-  // stage 1: segment sums (EDGE gTasks) and unique-source copies (VERTEX gTasks)
+  // stage 1 (EDGE gTasks): segment sums S = sum c_e x[src] into the EDGE block rows
   void* a1 = L.at<void>(ws, "a1");
-  {
+  if (rp->n1e) {
     AggArgs a = exec_args(rp->f1, g->E_max);
     a.table = A->x; a.ld_tab = A->ldx;
     a.out = a1; a.ld_out = p->pi;
@@ -447,14 +469,23 @@ wg_status rgcn_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, c
     a.F = d.f_in;
     WG_TRY(run(dt, a, rp->f1, st));
   }
-  // stage 2: grouped GEMM  T1[group r] = A1[group r] W_r
+  // stage 2: grouped GEMMs  T1[Y block, group r] = x[ysrc] W_r (A rows gathered
+  // from x) and T1[EDGE block, group r] = S W_r
   void* t1 = L.at<void>(ws, "t1");
-  {
-    GemmPart part{a1, p->pi, wt, p->pi, d.f_in, d.f_out};
-    part.tile_group = rp->tile_type; part.group_rows = (int)rows_o; part.groups = R;
+  if (rp->n1v) {
+    GemmPart part{A->x, A->ldx, wt, p->pi, d.f_in, d.f_out};
+    part.tile_group = rp->tile_type_v; part.group_rows = (int)rows_o; part.groups = R;
+    part.a_rows = rp->ysrc; part.a_table_rows = V;
     GemmEpi e;
     e.D = t1; e.ldd = p->po;
-    WG_TRY(gemm_nt(dt, rp->n1, (int)rup(d.f_out, 16 / s), &part, 1, e, nullptr, 0, st));
+    WG_TRY(gemm_nt(dt, rp->n1v, (int)rup(d.f_out, 16 / s), &part, 1, e, nullptr, 0, st));
+  }
+  if (rp->n1e) {
+    GemmPart part{a1, p->pi, wt, p->pi, d.f_in, d.f_out};
+    part.tile_group = rp->tile_type_e; part.group_rows = (int)rows_o; part.groups = R;
+    GemmEpi e;
+    e.D = static_cast<char*>(t1) + (size_t)rp->n1v * p->po * s; e.ldd = p->po;
+    WG_TRY(gemm_nt(dt, rp->n1e, (int)rup(d.f_out, 16 / s), &part, 1, e, nullptr, 0, st));
   }
   // self loop x W_0
   void* self = nullptr;
@@ -522,8 +553,7 @@ wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, 
     a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
     a.F = d.f_in;
     WG_TRY(run(dt, a, rp->bg, st));
-    WG_TRY(gemm_tn_grouped(dt, rp->tn, d.f_in, d.f_out, xg, p->pi, gt, p->po, G->W,
-                           L.at<void>(ws, "tn"), st));
+    WG_TRY(gemm_tn_grouped(dt, rp->tn, d.f_in, d.f_out, xg, p->pi, gt, p->po, G->W, L.at<void>(ws, "tn"), st));
   }
   if (d.self_loop && G && G->W_self)
     WG_TRY(gemm_tn(dt, V, d.f_in, d.f_out, A->x, A->ldx, dT, lddT, G->W_self, L.at<void>(ws, "tn"), st));

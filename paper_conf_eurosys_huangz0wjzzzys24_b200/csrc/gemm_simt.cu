@@ -47,7 +47,8 @@ __global__ void __launch_bounds__(256) k_gemm_nt(NTArgs a) {
         int mm = t / BK, kk = t % BK;
         int64_t m = m0 + mm;
         int k = k0 + kk;
-        As[kk][mm] = (m < a.M && k < P.K) ? tof<T>(A[m * P.lda + k]) : 0.f;
+        const int64_t am = P.a_rows ? (m < a.M ? (int64_t)P.a_rows[m] : 0) : m;   // row-gathered A
+        As[kk][mm] = (m < a.M && k < P.K) ? tof<T>(A[am * P.lda + k]) : 0.f;
         int n = n0 + mm;
         Bs[kk][mm] = (n < a.N && n < P.nb && k < P.K) ? tof<T>(B[(int64_t)n * P.ldb + k]) : 0.f;
       }

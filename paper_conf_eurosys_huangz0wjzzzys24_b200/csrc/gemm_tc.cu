@@ -478,7 +478,7 @@ bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_part
   if (tc_gemm_nt_persistent(dt, M, N, parts, n_parts, epi, s, st)) return true;
   if (dt != WG_BF16) return false;
   for (int i = 0; i < n_parts; ++i)
-    if (parts[i].tile_group) return false;   // grouped B: persistent kernel only
+    if (parts[i].tile_group || parts[i].a_rows) return false;   // grouped B / gathered A: persistent kernel only
   const int n_tiles = (int)cdiv(N, 256);
   const int BN = (int)rup(cdiv(N, n_tiles), 16);
   if (BN > 256) return false;

@@ -66,6 +66,7 @@ struct P2 {
   int kblocks[3];
   const int32_t* tile_group[3];
   int group_rows[3];
+  const int32_t* a_rows[3];
   const float* rscale;
   const float* bias;
   int relu, has_add, has_mask;
@@ -91,6 +92,15 @@ __device__ __forceinline__ void tma_load(uint32_t dst, const CUtensorMap* m, int
   asm volatile(
       "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::
           "r"(dst), "l"(reinterpret_cast<uint64_t>(m)), "r"(c0), "r"(c1), "r"(bar)
+      : "memory");
+}
+// TMA tile::gather4: rows r0..r3 of a 2-D map (box {inner, 1}) at column c0 -> 4 consecutive smem rows
+__device__ __forceinline__ void tma_gather4(uint32_t dst, const CUtensorMap* m, int c0, int r0, int r1, int r2, int r3,
+                                            uint32_t bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, "
+      "%4, %5, %6}], [%7];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(m)), "r"(c0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(bar)
       : "memory");
 }
 __device__ __forceinline__ void tma_store(const CUtensorMap* m, int c0, int c1, uint32_t src) {
@@ -280,32 +290,42 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
   for (int i = 0; i < p.nparts; ++i) total_kb += p.kblocks[i];
 
   if (warp == 0) {
-    if (lane == 0) {
-      // ------------------------------------------------ TMA producer
-      const uint32_t tx = A_STAGE + b_bytes;
-      int s = 0;
-      uint32_t ph = 0;
-      for (int64_t t = blockIdx.x; t < p.num_tiles; t += gridDim.x) {
-        const int64_t mt = t / p.n_tiles;
-        const int m0 = (int)(mt * BM), n0 = (int)((t % p.n_tiles) * BN);
-        int part = 0, kk = 0;
-        int brow = n0 + (p.tile_group[0] ? p.tile_group[0][mt] * p.group_rows[0] : 0);
-        for (int kb = 0; kb < total_kb; ++kb) {
+    // ------------------------------------------------ TMA producer (lane 0;
+    // row-gathered A parts: every lane issues the gather4 of its 4 tile rows)
+    const uint32_t tx = A_STAGE + b_bytes;
+    int s = 0;
+    uint32_t ph = 0;
+    for (int64_t t = blockIdx.x; t < p.num_tiles; t += gridDim.x) {
+      const int64_t mt = t / p.n_tiles;
+      const int m0 = (int)(mt * BM), n0 = (int)((t % p.n_tiles) * BN);
+      int part = 0, kk = 0;
+      int brow = n0 + (p.tile_group[0] ? p.tile_group[0][mt] * p.group_rows[0] : 0);
+      int4 gi = make_int4(0, 0, 0, 0);
+      if (p.a_rows[0]) gi = __ldg(reinterpret_cast<const int4*>(p.a_rows[0] + m0) + lane);
+      for (int kb = 0; kb < total_kb; ++kb) {
+        const CUtensorMap* ta = part == 0 ? &tA0 : (part == 1 ? &tA1 : &tA2);
+        const CUtensorMap* tb = part == 0 ? &tB0 : (part == 1 ? &tB1 : &tB2);
+        uint8_t* st = ring + s * L.stage;
+        if (lane == 0) {
           mbar_wait(su32(&empty[s]), ph ^ 1);
           mbar_expect_tx(su32(&full[s]), tx);
-          const CUtensorMap* ta = part == 0 ? &tA0 : (part == 1 ? &tA1 : &tA2);
-          const CUtensorMap* tb = part == 0 ? &tB0 : (part == 1 ? &tB1 : &tB2);
-          uint8_t* st = ring + s * L.stage;
-          tma_load(su32(st), ta, kk * C::BKE, m0, su32(&full[s]));
-          tma_load(su32(st + A_STAGE), tb, kk * C::BKE, brow, su32(&full[s]));
-          if (++kk == p.kblocks[part]) {
-            kk = 0;
-            ++part;
-            if (part < p.nparts)
-              brow = n0 + (p.tile_group[part] ? p.tile_group[part][mt] * p.group_rows[part] : 0);
-          }
-          if (++s == S) { s = 0; ph ^= 1; }
         }
+        __syncwarp();
+        if (p.a_rows[part]) {
+          tma_gather4(su32(st) + lane * 512, ta, kk * C::BKE, gi.x, gi.y, gi.z, gi.w, su32(&full[s]));
+        } else if (lane == 0) {
+          tma_load(su32(st), ta, kk * C::BKE, m0, su32(&full[s]));
+        }
+        if (lane == 0) tma_load(su32(st + A_STAGE), tb, kk * C::BKE, brow, su32(&full[s]));
+        if (++kk == p.kblocks[part]) {
+          kk = 0;
+          ++part;
+          if (part < p.nparts) {
+            brow = n0 + (p.tile_group[part] ? p.tile_group[part][mt] * p.group_rows[part] : 0);
+            if (p.a_rows[part]) gi = __ldg(reinterpret_cast<const int4*>(p.a_rows[part] + m0) + lane);
+          }
+        }
+        if (++s == S) { s = 0; ph ^= 1; }
       }
     }
   } else if (warp == 1) {
@@ -497,7 +517,14 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
     const GemmPart& q = parts[i];
     const uint64_t brows = q.tile_group ? (uint64_t)q.groups * q.group_rows : (uint64_t)q.nb;
     if (q.tile_group && BN > q.group_rows) return false;
-    if (!tc_make_map_t(&maps[2 * i], ty, q.A, (uint64_t)q.K, (uint64_t)M, (uint64_t)q.lda * es, che, BM)) return false;
+    if (q.a_rows) {   // gather4 map: box {che, 1} over the whole table
+      if ((reinterpret_cast<uintptr_t>(q.a_rows) & 15) != 0) return false;
+      if (!tc_make_map_t(&maps[2 * i], ty, q.A, (uint64_t)q.K, (uint64_t)q.a_table_rows, (uint64_t)q.lda * es, che, 1))
+        return false;
+    } else if (!tc_make_map_t(&maps[2 * i], ty, q.A, (uint64_t)q.K, (uint64_t)M, (uint64_t)q.lda * es, che, BM)) {
+      return false;
+    }
+    p.a_rows[i] = q.a_rows;
     if (!tc_make_map_t(&maps[2 * i + 1], ty, q.B, (uint64_t)q.K, brows, (uint64_t)q.ldb * es, che, BN)) return false;
     p.kblocks[i] = (int)cdiv(q.K, che);
     p.tile_group[i] = q.tile_group;

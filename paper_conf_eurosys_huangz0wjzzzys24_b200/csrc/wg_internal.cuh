@@ -190,6 +190,11 @@ struct GemmPart {
   const int32_t* tile_group = nullptr;
   int group_rows = 0;
   int groups = 1;
+  // row-gathered A (tcgen05 path only, TMA tile::gather4): row m of A is row
+  // a_rows[m] of the [a_table_rows x lda] table A; a_rows holds rup(M, 128)
+  // valid indices
+  const int32_t* a_rows = nullptr;
+  int64_t a_table_rows = 0;
 };
 struct GemmEpi {
   const float* rscale = nullptr;      // per row
