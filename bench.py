@@ -401,11 +401,13 @@ def main():
     dom = max((k for k in prof if prof[k]["bytes"] > 0), key=lambda k: prof[k]["ms"])
     agg = prof[dom]
     achieved = agg["bytes"] / (agg["ms"] / 1e3) / 1e9 if agg["ms"] > 0 else 0.0
-    traffic = None
+    traffic, traffic_src = None, None
     tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tf):
         try:
-            traffic = json.load(open(tf)).get(f"{args.config}:{model}:{dom}")
+            tr = json.load(open(tf)).get(f"{args.config}:{model}:{dom}")
+            traffic = tr["bytes_per_launch"] if tr else None
+            traffic_src = tr["source"] if tr else None
         except Exception:
             traffic = None
     names = {"gather_reduce": "k_agg_cp / k_agg (gather + segment-reduce, a6/a10)",
@@ -413,6 +415,7 @@ def main():
              "tc_gemm_nt": "tcgen05 GEMM-NT (a5/a7/a9)", "tc_gemm_tn": "tcgen05 GEMM-TN (a11)"}
     roofline = {"bound": "hbm", "kernel": names.get(dom, dom), "class": dom, "achieved": achieved,
                 "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": achieved / pk["hbm_gbs"], "traffic": traffic,
+                "traffic_source": f"profiles/ncu_traffic.json: {traffic_src}" if traffic else None,
                 "peak_source": f"{pk_src} (MEASURED_PEAKS.json hbm_gbs)" if pk_src == "measured" else "fallback",
                 "bytes_per_launch": agg["bytes"] / max(1, agg["launches"]),
                 "launches_per_step": agg["launches"] / args.steps,
