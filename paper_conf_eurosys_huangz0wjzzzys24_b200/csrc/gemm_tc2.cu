@@ -19,12 +19,16 @@
 //   warp 1      TMEM allocator + MMA issuer: tcgen05.mma (M=128, N=BN, K=16)
 //               into one of TWO accumulator buffers (2 x BN TMEM columns), so
 //               tile i+1's MMAs run while tile i is drained;
-//   warp 6      epilogue loader: TMA loads of the addend / mask tiles, 64
-//               columns at a time, into a 2-deep buffer;
-//   warps 2-5   epilogue: tcgen05.ld (warp w drains TMEM lanes 32*(w%4)..),
-//               fused epilogue math, pack into a 128-byte-swizzled staging
-//               tile, TMA store (bulk_group, 2-deep) -- coalesced writes;
-//   warps 7-10  (fp32 only) hi / lo converters.
+//   warps 2-9   epilogue, two groups of four warps (one warp per TMEM lane
+//               quarter in each group; warp w drains lanes 32*(w%4)..): the
+//               groups take alternate 128-byte-wide output chunks, so one
+//               group's tcgen05.ld / math overlaps the other's staging and TMA
+//               store.  Per chunk: tcgen05.ld, fused epilogue math, pack into
+//               a 128-byte-swizzled staging tile, TMA store (bulk_group) --
+//               coalesced writes;
+//   warp 10     epilogue loader: TMA loads of the addend / mask chunks into a
+//               2-deep buffer (buffer b feeds epilogue group b);
+//   warps 11-14 (fp32 only) hi / lo converters.
 // One CTA per SM loops over 128 x BN tiles (N fastest, so A tiles of the N
 // tiles of one row block are adjacent in time).
 #include <cuda.h>
@@ -33,6 +37,7 @@
 #include <algorithm>
 #include <cstring>
 #include <mutex>
+#include <type_traits>
 
 #include "wg_internal.cuh"
 
@@ -56,7 +61,8 @@ template <typename T> struct Cfg {
   static constexpr int BKE = 128 / ES;
   static constexpr int CHE = 128 / ES;
   static constexpr int EPV = 16 / ES;              // elements per 16-byte unit
-  static constexpr int NTHREADS = TF32 ? 352 : 224;   // fp32: + 4 converter warps
+  static constexpr int NTHREADS = TF32 ? 480 : 352;   // fp32: + 4 converter warps
+  static constexpr int CONV0 = 352;                   // first converter thread
 };
 
 struct P2 {
@@ -69,7 +75,7 @@ struct P2 {
   const int32_t* a_rows[3];
   const float* rscale;
   const float* bias;
-  int relu, has_add, has_mask;
+  int relu, has_add, has_mask, bias_vec;
 };
 
 __device__ __forceinline__ uint32_t su32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
@@ -113,7 +119,7 @@ __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.comm
 template <int N>
 __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
-__device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+__device__ __forceinline__ void epi_bar(int grp) { asm volatile("bar.sync %0, 128;" ::"r"(grp + 1) : "memory"); }
 
 __device__ __forceinline__ uint64_t desc_sw128(uint32_t addr) {
   uint64_t d = 0;
@@ -234,7 +240,11 @@ __host__ __device__ inline SmemPlan smem_plan(bool tf32, int BN, int S, bool has
   return q;
 }
 
-template <typename T>
+// FL: compile-time epilogue operands (EP_ADD addend, EP_MASK ReLU mask, EP_BIAS
+// bias), so the per-chunk epilogue code carries no predicated dead paths
+constexpr int EP_ADD = 1, EP_MASK = 2, EP_BIAS = 4;
+
+template <typename T, int FL>
 __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
     k_gemm_nt_p(const __grid_constant__ CUtensorMap tA0, const __grid_constant__ CUtensorMap tB0,
                 const __grid_constant__ CUtensorMap tA1, const __grid_constant__ CUtensorMap tB1,
@@ -272,7 +282,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(su32(&tfull[b]), 1);
-      mbar_init(su32(&tempty[b]), 128);
+      mbar_init(su32(&tempty[b]), 256);
       mbar_init(su32(&efull[b]), 1);
       mbar_init(su32(&eempty[b]), 128);
     }
@@ -365,8 +375,8 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
         mma_commit(su32(&tfull[buf]));
       }
     }
-  } else if (warp == 6) {
-    if (lane == 0 && (p.has_add || p.has_mask)) {
+  } else if (warp == 10) {
+    if (lane == 0 && (FL & (EP_ADD | EP_MASK)) != 0) {
       // ------------------------------------------------ epilogue loader
       const uint32_t tx = (p.has_add ? CHUNK_BYTES : 0) + (p.has_mask ? CHUNK_BYTES : 0);
       int g = 0;
@@ -381,10 +391,10 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
         }
       }
     }
-  } else if (warp >= 7) {
+  } else if (warp >= 11) {
     if constexpr (C::TF32) {
       // ------------------------------------------------ hi / lo converters (128 threads)
-      const int ct = threadIdx.x - 224;
+      const int ct = threadIdx.x - C::CONV0;
       const int n16 = (A_STAGE + b_bytes) / 16;
       int s = 0;
       uint32_t ph = 0;
@@ -399,11 +409,16 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
       }
     }
   } else {
-    // ------------------------------------------------ epilogue (warps 2..5)
-    const int et = threadIdx.x - 64;               // 0..127
+    // ------------------------------------------------ epilogue (warps 2..9)
+    const int grp = (warp - 2) >> 2;               // epilogue group: chunks g with g % 2 == grp
+    const int et = (threadIdx.x - 64) & 127;       // 0..127 inside the group
     const int quarter = warp & 3;                  // TMEM lane quarter this warp may access
     const int r = quarter * 32 + lane;             // tile row
-    const bool epi_loads = p.has_add || p.has_mask;
+    constexpr bool epi_loads = (FL & (EP_ADD | EP_MASK)) != 0;
+    const float lo_clamp = p.relu ? 0.f : -INFINITY;
+    uint8_t* stg = st_sm + grp * CHUNK_BYTES;      // this group's staging tile
+    const uint8_t* adp = ad_sm + grp * CHUNK_BYTES;
+    const uint8_t* mkp = mk_sm + grp * CHUNK_BYTES;
     int j = 0, g = 0;
     for (int64_t t = blockIdx.x; t < p.num_tiles; t += gridDim.x, ++j) {
       const int m0 = (int)((t / p.n_tiles) * BM), n0 = (int)((t % p.n_tiles) * BN);
@@ -416,52 +431,64 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
       mbar_wait(su32(&tfull[buf]), (j >> 1) & 1);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       for (int c = 0; c < nchunk; ++c, ++g) {
-        const int b = g & 1;
+        if ((g & 1) != grp) continue;              // the other group's chunk
         uint32_t u[64];
         const uint32_t taddr = tmem + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(buf * 256 + c * C::CHE);
 #pragma unroll
         for (int q = 0; q < C::CHE / 16; ++q) tmem_ld16(taddr + 16 * q, u + 16 * q);
         asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-        if (epi_loads) mbar_wait(su32(&efull[b]), (g >> 1) & 1);
-        // the staging buffer b was last read by the TMA store issued two chunks ago
-        if (et == 0) bulk_wait_read<1>();
-        epi_bar();
-        uint8_t* stg = st_sm + b * CHUNK_BYTES;
-        const uint8_t* adp = ad_sm + b * CHUNK_BYTES;
-        const uint8_t* mkp = mk_sm + b * CHUNK_BYTES;
+        if (epi_loads) mbar_wait(su32(&efull[grp]), (g >> 1) & 1);
+        // the staging tile was last read by this group's previous TMA store
+        if (et == 0) bulk_wait_read<0>();
+        epi_bar(grp);
+        const int nc0 = n0 + c * C::CHE;
+        // one 16-byte output unit (EPV columns) at a time; FULL: every column < N
+        auto units = [&](auto full_t) {
+          constexpr bool FULL = decltype(full_t)::value;
 #pragma unroll
-        for (int k = 0; k < 8; ++k) {           // one 16-byte unit (EPV columns) at a time
-          float f[C::EPV];
-          const int nc = n0 + c * C::CHE + k * C::EPV;
+          for (int k = 0; k < 8; ++k) {
+            float f[C::EPV];
+            const int nc = nc0 + k * C::EPV;
 #pragma unroll
-          for (int i = 0; i < C::EPV; ++i) f[i] = rs * __uint_as_float(u[k * C::EPV + i]);
-          if (p.has_add) {
-            float a[C::EPV];
-            unpack16<T>(*reinterpret_cast<const int4*>(adp + sw_off(r, k)), a);
+            for (int i = 0; i < C::EPV; ++i) f[i] = rs * __uint_as_float(u[k * C::EPV + i]);
+            if constexpr ((FL & EP_ADD) != 0) {
+              float a[C::EPV];
+              unpack16<T>(*reinterpret_cast<const int4*>(adp + sw_off(r, k)), a);
 #pragma unroll
-            for (int i = 0; i < C::EPV; ++i) f[i] += a[i];
+              for (int i = 0; i < C::EPV; ++i) f[i] += a[i];
+            }
+            if constexpr ((FL & EP_BIAS) != 0) {
+              if constexpr (FULL) {
+#pragma unroll
+                for (int i = 0; i < C::EPV; i += 4) {
+                  const float4 b4 = __ldg(reinterpret_cast<const float4*>(p.bias + nc + i));
+                  f[i] += b4.x; f[i + 1] += b4.y; f[i + 2] += b4.z; f[i + 3] += b4.w;
+                }
+              } else {
+#pragma unroll
+                for (int i = 0; i < C::EPV; ++i) f[i] += (nc + i < p.N) ? p.bias[nc + i] : 0.f;
+              }
+            }
+#pragma unroll
+            for (int i = 0; i < C::EPV; ++i) f[i] = fmaxf(f[i], lo_clamp);   // ReLU (or -inf: none)
+            if constexpr ((FL & EP_MASK) != 0) {
+              float a[C::EPV];
+              unpack16<T>(*reinterpret_cast<const int4*>(mkp + sw_off(r, k)), a);
+#pragma unroll
+              for (int i = 0; i < C::EPV; ++i) if (!(a[i] > 0.f)) f[i] = 0.f;
+            }
+            if constexpr (!FULL) {
+#pragma unroll
+              for (int i = 0; i < C::EPV; ++i) if (nc + i >= p.N) f[i] = 0.f;
+            }
+            *reinterpret_cast<int4*>(stg + sw_off(r, k)) = pack16<T>(f);
           }
-          if (p.bias) {
-#pragma unroll
-            for (int i = 0; i < C::EPV; ++i) f[i] += (nc + i < p.N) ? p.bias[nc + i] : 0.f;
-          }
-          if (p.relu) {
-#pragma unroll
-            for (int i = 0; i < C::EPV; ++i) f[i] = fmaxf(f[i], 0.f);
-          }
-          if (p.has_mask) {
-            float a[C::EPV];
-            unpack16<T>(*reinterpret_cast<const int4*>(mkp + sw_off(r, k)), a);
-#pragma unroll
-            for (int i = 0; i < C::EPV; ++i) if (!(a[i] > 0.f)) f[i] = 0.f;
-          }
-#pragma unroll
-          for (int i = 0; i < C::EPV; ++i) if (nc + i >= p.N) f[i] = 0.f;
-          *reinterpret_cast<int4*>(stg + sw_off(r, k)) = pack16<T>(f);
-        }
-        if (epi_loads) mbar_arrive(su32(&eempty[b]));
+        };
+        if (nc0 + C::CHE <= p.N && p.bias_vec) units(std::true_type{});
+        else units(std::false_type{});
+        if (epi_loads) mbar_arrive(su32(&eempty[grp]));
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        epi_bar();
+        epi_bar(grp);
         if (et == 0) {
           tma_store(td, ncol0 + c * C::CHE, m0, su32(stg));
           bulk_commit();
@@ -478,12 +505,28 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
 
 int g_sms = 0;
 
-template <typename T>
-void set_smem_attr() {
+template <typename T, int FL>
+void launch_p(unsigned grid, size_t smem, cudaStream_t s, const CUtensorMap* maps, const P2& p) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_gemm_nt_p<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(k_gemm_nt_p<T, FL>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr = true;
+  }
+  k_gemm_nt_p<T, FL><<<grid, Cfg<T>::NTHREADS, smem, s>>>(maps[0], maps[1], maps[2], maps[3], maps[4], maps[5],
+                                                          maps[6], maps[7], maps[8], maps[9], p);
+}
+
+template <typename T>
+void launch_fl(int fl, unsigned grid, size_t smem, cudaStream_t s, const CUtensorMap* maps, const P2& p) {
+  switch (fl) {
+    case 0: launch_p<T, 0>(grid, smem, s, maps, p); break;
+    case 1: launch_p<T, 1>(grid, smem, s, maps, p); break;
+    case 2: launch_p<T, 2>(grid, smem, s, maps, p); break;
+    case 3: launch_p<T, 3>(grid, smem, s, maps, p); break;
+    case 4: launch_p<T, 4>(grid, smem, s, maps, p); break;
+    case 5: launch_p<T, 5>(grid, smem, s, maps, p); break;
+    case 6: launch_p<T, 6>(grid, smem, s, maps, p); break;
+    default: launch_p<T, 7>(grid, smem, s, maps, p); break;
   }
 }
 
@@ -553,6 +596,7 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
   }
   p.rscale = epi.rscale;
   p.bias = epi.bias;
+  p.bias_vec = (reinterpret_cast<uintptr_t>(epi.bias) & 15) == 0;
   p.relu = epi.relu;
   const int limit = 227 * 1024 - 1024;
   int stages = 4;
@@ -570,15 +614,9 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
   for (int i = 0; i < n_parts; ++i) kt += parts[i].K;
   ProfScope ps(PK_TC_NT, s, (double)M * (kt + N + (epi.addend ? N : 0) + (epi.mask_ref ? N : 0)) * es,
                2.0 * M * N * kt);
-  if (f32) {
-    set_smem_attr<float>();
-    k_gemm_nt_p<float><<<grid, Cfg<float>::NTHREADS, smem, s>>>(maps[0], maps[1], maps[2], maps[3], maps[4], maps[5],
-                                                               maps[6], maps[7], maps[8], maps[9], p);
-  } else {
-    set_smem_attr<__nv_bfloat16>();
-    k_gemm_nt_p<__nv_bfloat16><<<grid, Cfg<__nv_bfloat16>::NTHREADS, smem, s>>>(
-        maps[0], maps[1], maps[2], maps[3], maps[4], maps[5], maps[6], maps[7], maps[8], maps[9], p);
-  }
+  const int fl = (p.has_add ? EP_ADD : 0) | (p.has_mask ? EP_MASK : 0) | (p.bias ? EP_BIAS : 0);
+  if (f32) launch_fl<float>(fl, grid, smem, s, maps, p);
+  else launch_fl<__nv_bfloat16>(fl, grid, smem, s, maps, p);
   ++launch_counter();
   cudaError_t e = cudaGetLastError();
   *st = e == cudaSuccess ? WG_OK : WG_ERR_CUDA;
