@@ -279,8 +279,8 @@ def main():
     src, dst, et, x_np, labels_np = make_inputs(c, model)
     t_gen = time.perf_counter() - t0
     dev = torch.device("cuda", local)
-    if world > 1 and model in ("gat", "rgcn"):
-        raise SystemExit("the 1-D multi-GPU partition covers GCN / SAGE / GIN (DESIGN.md §7)")
+    if world > 1 and model == "gat":
+        raise SystemExit("the 1-D multi-GPU partition covers GCN / SAGE / GIN / RGCN (DESIGN.md §9)")
     block, bounds = partition_1d(c.V, world)
     vb, ve = bounds[rank] if world > 1 else (0, c.V)
     torch.cuda.synchronize()

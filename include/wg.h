@@ -131,8 +131,8 @@ typedef struct {
 } wg_conv_desc;
 
 /* Errors: WG_ERR_INVALID (bad sizes / model / dtype), WG_ERR_UNSUPPORTED
- * (typed graph with a non-RGCN model; GAT / RGCN on a graph that owns only
- * a row block -- the 1-D partition covers GCN / SAGE / GIN).               */
+ * (typed graph with a non-RGCN model; GAT on a graph that owns only a row
+ * block -- the 1-D partition covers GCN / SAGE / GIN / RGCN).              */
 wg_status wg_plan_create(wg_graph g, const wg_conv_desc* desc, wg_plan* out);
 /* Bytes of the caller-owned `saved` (forward -> backward) and `workspace`
  * buffers; both 256-byte aligned device memory.                            */
@@ -170,9 +170,11 @@ typedef struct {
 /* Phases for the 1-D multi-GPU layer (§8(e)).  Single GPU: WG_PHASE_ALL.
  * PRE computes this rank's rows of the exchange table into
  * `xchg + row_offset * ld_xchg`; the caller all-gathers `xchg` (in place);
- * POST consumes the gathered table.  GAT and RGCN plans accept only
- * WG_PHASE_ALL (and only on a full graph, see wg_plan_create):
- * other phases return WG_ERR_UNSUPPORTED.                                  */
+ * POST consumes the gathered table.  RGCN: the forward has no exchange
+ * (x must hold all rows: PRE does nothing, POST = ALL); the backward
+ * exchange table is dT = dy (masked by the fused ReLU), f_out wide.  GAT
+ * plans accept only WG_PHASE_ALL (and only on a full graph, see
+ * wg_plan_create): other phases return WG_ERR_UNSUPPORTED.                  */
 typedef enum { WG_PHASE_ALL = 0, WG_PHASE_PRE = 1, WG_PHASE_POST = 2 } wg_phase;
 
 typedef struct {

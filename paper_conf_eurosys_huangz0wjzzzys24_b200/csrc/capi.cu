@@ -91,8 +91,8 @@ wg_status wg_conv_forward(wg_plan p, const wg_params* params, const wg_fwd_args*
   WG_REQ(p && params && a, WG_ERR_INVALID, "wg_conv_forward: null argument");
   WG_REQ(a->phase == WG_PHASE_ALL || a->phase == WG_PHASE_PRE || a->phase == WG_PHASE_POST, WG_ERR_INVALID,
          "wg_conv_forward: bad phase");
-  WG_REQ(a->phase == WG_PHASE_ALL || (p->d.model != WG_GAT && p->d.model != WG_RGCN), WG_ERR_UNSUPPORTED,
-         "wg_conv_forward: PRE / POST phases are for GCN / SAGE / GIN");
+  WG_REQ(a->phase == WG_PHASE_ALL || p->d.model != WG_GAT, WG_ERR_UNSUPPORTED,
+         "wg_conv_forward: PRE / POST phases are for GCN / SAGE / GIN / RGCN");
   WG_CK(cudaSetDevice(p->g->device));
   WG_CK(cudaGetLastError());
   cudaStream_t s = (cudaStream_t)stream;
@@ -109,8 +109,8 @@ wg_status wg_conv_backward(wg_plan p, const wg_params* params, const wg_bwd_args
   WG_REQ(p && params && a, WG_ERR_INVALID, "wg_conv_backward: null argument");
   WG_REQ(a->phase == WG_PHASE_ALL || a->phase == WG_PHASE_PRE || a->phase == WG_PHASE_POST, WG_ERR_INVALID,
          "wg_conv_backward: bad phase");
-  WG_REQ(a->phase == WG_PHASE_ALL || (p->d.model != WG_GAT && p->d.model != WG_RGCN), WG_ERR_UNSUPPORTED,
-         "wg_conv_backward: PRE / POST phases are for GCN / SAGE / GIN");
+  WG_REQ(a->phase == WG_PHASE_ALL || p->d.model != WG_GAT, WG_ERR_UNSUPPORTED,
+         "wg_conv_backward: PRE / POST phases are for GCN / SAGE / GIN / RGCN");
   WG_CK(cudaSetDevice(p->g->device));
   WG_CK(cudaGetLastError());
   cudaStream_t s = (cudaStream_t)stream;

@@ -180,43 +180,54 @@ wg_status run(wg_dtype dt, const AggArgs& a, const CsrExec& X, cudaStream_t s) {
 wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
   wg_graph_s* g = p->g;
   const wg_conv_desc& d = p->d;
-  WG_REQ(g->vb == 0 && g->ve == g->V, WG_ERR_UNSUPPORTED, "RGCN with a 1-D partition is not implemented");
+  // 1-D partition: this rank owns rows [vb, ve); its forward
+  // side holds their in-edges, its transposed side their out-edges; x / dT
+  // tables are read with global row ids (replicated / all-gathered), outputs
+  // are written for the owned rows only.
   const int R = g->by_type ? g->R : 1;
-  const int64_t E = g->fwd.E, V = g->V;
+  const int64_t E = g->fwd.E, Eb = g->bwd.E, V = g->V, vb = g->vb, nr = g->ve - g->vb;
   auto* rp = new RgcnPlan();
   rp->R = R;
   p->rg = rp;
   p->pi = pitch(d.f_in, d.dtype);
   p->po = pitch(d.f_out, d.dtype);
+  p->bwd_path = 1;    // the backward exchange table is dT (f_out wide)
   // ---- host copies of the forward / transposed sorted edge arrays
   std::vector<int32_t> fk, fi_, ft, fperm, bk, bi, bt, bperm;
   WG_TRY(down(g->fwd.key, E, fk));
   WG_TRY(down(g->fwd.idx, E, fi_));
   WG_TRY(down(g->fwd.perm, E, fperm));
-  WG_TRY(down(g->bwd.key, E, bk));
-  WG_TRY(down(g->bwd.idx, E, bi));
-  WG_TRY(down(g->bwd.perm, E, bperm));
+  WG_TRY(down(g->bwd.key, Eb, bk));
+  WG_TRY(down(g->bwd.idx, Eb, bi));
+  WG_TRY(down(g->bwd.perm, Eb, bperm));
   if (g->by_type) {
     WG_TRY(down(g->fwd.type, E, ft));
-    WG_TRY(down(g->bwd.type, E, bt));
+    WG_TRY(down(g->bwd.type, Eb, bt));
   } else {
     ft.assign(E, 0);
-    bt.assign(E, 0);
+    bt.assign(Eb, 0);
+  }
+  // per-edge coefficient c_e (forward / transposed order): 1 or 1/|in_r(dst)|
+  // (global counts, graph.cu rel_counts)
+  std::vector<float> coef_f(E, 1.f), coef_b(Eb, 1.f);
+  if (d.norm == WG_NORM_RIGHT) {
+    std::vector<int32_t> cnt;
+    if (g->by_type) {
+      WG_TRY(down(g->rel_cnt, g->E_total, cnt));
+    } else {   // one relation: |in_r(v)| = deg_in(v)
+      std::vector<int32_t> din;
+      WG_TRY(down(g->deg_in, V, din));
+      cnt.resize(1);
+      for (int64_t i = 0; i < E; ++i) coef_f[i] = 1.f / (float)std::max(1, din[fk[i]]);
+      for (int64_t i = 0; i < Eb; ++i) coef_b[i] = 1.f / (float)std::max(1, din[bi[i]]);
+    }
+    if (g->by_type) {
+      for (int64_t i = 0; i < E; ++i) coef_f[i] = 1.f / (float)cnt[fperm[i]];
+      for (int64_t i = 0; i < Eb; ++i) coef_b[i] = 1.f / (float)cnt[bperm[i]];
+    }
   }
   const auto& tasks = g->fwd.h_tasks;
   const int64_t nt = (int64_t)tasks.size();
-  // per-edge coefficient c_e (by global edge id): 1 or 1/|in_r(dst)|
-  std::vector<float> coef_eid(E, 1.f);
-  // segment runs in the forward order: (dst, type) constant
-  std::vector<int64_t> seg_len_at(E, 0);   // length of the segment each position belongs to
-  for (int64_t i = 0; i < E;) {
-    int64_t j = i;
-    while (j < E && fk[j] == fk[i] && ft[j] == ft[i]) ++j;
-    for (int64_t k = i; k < j; ++k) seg_len_at[k] = j - i;
-    i = j;
-  }
-  if (d.norm == WG_NORM_RIGHT)
-    for (int64_t i = 0; i < E; ++i) coef_eid[fperm[i]] = 1.f / (float)seg_len_at[i];
   // ---- plan bits (a4)
   p->plan_bits.assign(nt, 0);
   {
@@ -268,9 +279,9 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
         while (j < k.e_end && fk[j] == fk[i]) ++j;
         const bool cont = (i == k.e_begin) && open_seg_dst == fk[i] && open_seg_type == r && (k.flags & WG_TASK_SPLIT);
         if (!cont) {
-          const float rs = d.norm == WG_NORM_RIGHT ? 1.f / (float)seg_len_at[i] : 1.f;
+          const float rs = coef_f[i];   // segment (dst, r): every edge has the same c_e
           rows1[r].push_back(Row1{(int64_t)ents[r].size(), (int64_t)ents[r].size(), rs});
-          contrib.push_back(Contrib{fk[i], r, (int64_t)rows1[r].size() - 1, 1.f, false});
+          contrib.push_back(Contrib{fk[i] - (int32_t)vb, r, (int64_t)rows1[r].size() - 1, 1.f, false});
         }
         for (int64_t q = i; q < j; ++q) ents[r].push_back(fi_[q]);
         rows1[r].back().ent_e = (int64_t)ents[r].size();
@@ -282,7 +293,7 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
       open_seg_dst = -1;
       for (int64_t i = k.e_begin; i < k.e_end; ++i) {
         const int64_t m = std::lower_bound(uniq[r].begin(), uniq[r].end(), fi_[i]) - uniq[r].begin();
-        contrib.push_back(Contrib{fk[i], r, m, coef_eid[fperm[i]], true});
+        contrib.push_back(Contrib{fk[i] - (int32_t)vb, r, m, coef_f[i], true});
       }
     }
   }
@@ -331,7 +342,7 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
     std::stable_sort(contrib.begin(), contrib.end(), [](const Contrib& a, const Contrib& b) {
       return a.dst != b.dst ? a.dst < b.dst : a.row < b.row;
     });
-    std::vector<int64_t> rpv(V + 1, 0);
+    std::vector<int64_t> rpv(nr + 1, 0);
     std::vector<int32_t> idx(contrib.size());
     std::vector<float> es(contrib.size());
     bool any = false;
@@ -341,16 +352,16 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
       es[i] = contrib[i].c;
       any |= es[i] != 1.f;
     }
-    for (int64_t v = 0; v < V; ++v) rpv[v + 1] += rpv[v];
+    for (int64_t v = 0; v < nr; ++v) rpv[v + 1] += rpv[v];
     WG_TRY(build_exec(p, rpv, idx, any ? &es : nullptr, nullptr, g->E_max, &rp->f3));
   }
   // ---- transposed: (src, relation) segments grouped by relation
   {
     std::vector<std::vector<std::pair<int64_t, int64_t>>> segs(R);   // [b, e) in transposed order
     std::vector<std::vector<int32_t>> seg_src(R);
-    for (int64_t i = 0; i < E;) {
+    for (int64_t i = 0; i < Eb;) {
       int64_t j = i;
-      while (j < E && bk[j] == bk[i] && bt[j] == bt[i]) ++j;
+      while (j < Eb && bk[j] == bk[i] && bt[j] == bt[i]) ++j;
       segs[bt[i]].push_back({i, j});
       seg_src[bt[i]].push_back(bk[i]);
       i = j;
@@ -361,8 +372,8 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
     std::vector<int64_t> rpv(rp->n1T + 1, 0), rpg(rp->n1T + 1, 0);
     std::vector<int32_t> idx, gidx;
     std::vector<float> es;
-    idx.reserve(E);
-    es.reserve(E);
+    idx.reserve(Eb);
+    es.reserve(Eb);
     bool any = false;
     struct SC { int32_t src; int64_t row; };
     std::vector<SC> sc;
@@ -371,7 +382,7 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
       for (size_t s = 0; s < segs[r].size(); ++s) {
         for (int64_t q = segs[r][s].first; q < segs[r][s].second; ++q) {
           idx.push_back(bi[q]);
-          const float c = coef_eid[bperm[q]];
+          const float c = coef_b[q];
           es.push_back(c);
           any |= c != 1.f;
         }
@@ -404,10 +415,10 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
     std::stable_sort(sc.begin(), sc.end(), [](const SC& a, const SC& b) {
       return a.src != b.src ? a.src < b.src : a.row < b.row;
     });
-    std::vector<int64_t> rp3(V + 1, 0);
+    std::vector<int64_t> rp3(nr + 1, 0);
     std::vector<int32_t> idx3(sc.size());
-    for (size_t i = 0; i < sc.size(); ++i) { rp3[sc[i].src + 1]++; idx3[i] = (int32_t)sc[i].row; }
-    for (int64_t v = 0; v < V; ++v) rp3[v + 1] += rp3[v];
+    for (size_t i = 0; i < sc.size(); ++i) { rp3[sc[i].src - vb + 1]++; idx3[i] = (int32_t)sc[i].row; }
+    for (int64_t v = 0; v < nr; ++v) rp3[v + 1] += rp3[v];
     WG_TRY(build_exec(p, rp3, idx3, nullptr, nullptr, g->E_max, &rp->b3));
   }
   // ---- buffers
@@ -425,16 +436,16 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
   W.add("w0", (size_t)rows_i * p->po * s);
   W.add("a1", (size_t)std::max<int64_t>(rp->n1e, 1) * p->pi * s);
   W.add("t1", (size_t)std::max<int64_t>(rp->n1v + rp->n1e, 1) * p->po * s);
-  W.add("self", (size_t)V * p->po * s);
+  W.add("self", (size_t)nr * p->po * s);
   W.add("part", sizeof(float) * std::max({1, rp->f1.n_slots, rp->f3.n_slots, rp->b1.n_slots, rp->b3.n_slots,
                                            rp->bg.n_slots}) * pl);
   W.add("xg", (size_t)rp->n1T * p->pi * s);
-  W.add("dt", (size_t)V * p->po * s);
+  W.add("dt", (size_t)nr * p->po * s);
   W.add("gt", (size_t)rp->n1T * p->po * s);
   W.add("dxt", (size_t)rp->n1T * p->pi * s);
-  W.add("dxs", (size_t)V * p->pi * s);
-  W.add("colsum", bias_grad_scratch(V, (int)p->po));
-  W.add("tn", std::max(gemm_tn_scratch(V, d.f_in, d.f_out), gemm_tn_grouped_scratch(rp->tn.n_units, d.f_in, d.f_out)));
+  W.add("dxs", (size_t)nr * p->pi * s);
+  W.add("colsum", bias_grad_scratch(nr, (int)p->po));
+  W.add("tn", std::max(gemm_tn_scratch(nr, d.f_in, d.f_out), gemm_tn_grouped_scratch(rp->tn.n_units, d.f_in, d.f_out)));
   // the forward gTask work items are not used by RGCN (stage CSRs replace them)
   return WG_OK;
 }
@@ -453,9 +464,13 @@ wg_status rgcn_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, c
   const int s = dsize(dt), R = rp->R;
   WG_REQ(P->W && A->x && A->y && A->workspace, WG_ERR_INVALID, "RGCN forward: null argument");
   WG_REQ(!d.self_loop || P->W_self, WG_ERR_INVALID, "self_loop needs W_self");
+  // 1-D partition: x holds every row (the caller all-gathers it); nothing to
+  // exchange before the forward, so PRE is a no-op and POST = ALL
+  if (A->phase == WG_PHASE_PRE) return WG_OK;
   const Layout& L = p->ws;
   void* ws = A->workspace;
-  const int64_t V = g->V, rows_o = rup(d.f_out, 16), pl = rup(std::max(d.f_in, d.f_out), 8);
+  const int64_t V = g->V, vb = g->vb, nr = g->ve - g->vb, rows_o = rup(d.f_out, 16),
+                pl = rup(std::max(d.f_in, d.f_out), 8);
   ProfScope ps(PK_RGCN, st, 0.0, 0.0);
   void* wt = L.at<void>(ws, "wt");
   WG_TRY(prep_weight_batched(dt, P->W, R, d.f_in, d.f_out, 1, wt, p->pi, (int)rows_o, st));
@@ -493,10 +508,11 @@ wg_status rgcn_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, c
     void* w0t = L.at<void>(ws, "w0t");
     WG_TRY(prep_weight(dt, P->W_self, d.f_in, d.f_out, 1, w0t, p->pi, (int)rows_o, st));
     self = L.at<void>(ws, "self");
-    GemmPart part{A->x, A->ldx, w0t, p->pi, d.f_in, (int)rows_o};
+    const char* x_own = static_cast<const char*>(A->x) + (size_t)vb * A->ldx * s;
+    GemmPart part{x_own, A->ldx, w0t, p->pi, d.f_in, (int)rows_o};
     GemmEpi e;
     e.D = self; e.ldd = p->po;
-    WG_TRY(gemm_nt(dt, V, (int)rup(d.f_out, 16 / s), &part, 1, e, nullptr, 0, st));
+    WG_TRY(gemm_nt(dt, nr, (int)rup(d.f_out, 16 / s), &part, 1, e, nullptr, 0, st));
   }
   // stage 3: y[v] = sum of contributions (+ self + bias), ReLU
   {
@@ -521,30 +537,55 @@ wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, 
   const wg_dtype dt = d.dtype;
   const int s = dsize(dt), R = rp->R;
   WG_REQ(P->W && A->dy && A->x && A->workspace, WG_ERR_INVALID, "RGCN backward: null argument");
-  WG_REQ(!d.fuse_relu || A->y, WG_ERR_INVALID, "fuse_relu backward needs y");
+  const bool mask_dy = d.fuse_relu && !A->dy_masked;
+  WG_REQ(!mask_dy || A->y, WG_ERR_INVALID, "fuse_relu backward needs y");
   WG_REQ(!d.need_dx || A->dx, WG_ERR_INVALID, "need_dx but dx is NULL");
+  const bool pre = A->phase != WG_PHASE_POST, post = A->phase != WG_PHASE_PRE;
   const Layout& L = p->ws;
   void* ws = A->workspace;
-  const int64_t V = g->V, rows_i = rup(d.f_in, 16), pl = rup(std::max(d.f_in, d.f_out), 8);
+  const int64_t vb = g->vb, nr = g->ve - g->vb, rows_i = rup(d.f_in, 16), pl = rup(std::max(d.f_in, d.f_out), 8);
+  const bool dist = nr != g->V;
+  WG_REQ(!dist || A->xchg, WG_ERR_INVALID, "RGCN backward on a 1-D partition needs the dT exchange table");
   ProfScope ps(PK_RGCN, st, 0.0, 0.0);
-  // dT = dy masked by the fused ReLU; db
-  const void* dT = A->dy;
-  int64_t lddT = A->lddy;
-  if (d.fuse_relu) { dT = L.at<void>(ws, "dt"); lddT = p->po; }
-  WG_TRY(bias_grad_mask(dt, V, d.f_out, A->dy, A->lddy, d.fuse_relu ? A->y : nullptr, A->ldy,
-                        d.fuse_relu ? const_cast<void*>(dT) : nullptr, lddT, (G && d.bias) ? G->bias : nullptr,
-                        L.at<float>(ws, "colsum"), st));
+  const char* x_own = static_cast<const char*>(A->x) + (size_t)vb * A->ldx * s;
+  // dT = dy (masked by the fused ReLU): this rank's rows; the transposed
+  // gather reads dT of every row -- the exchange table when distributed
+  void* dt_own = nullptr;                       // written rows (nullptr: dT is dy itself)
+  int64_t ld_own = p->po;
+  if (A->xchg) { dt_own = static_cast<char*>(A->xchg) + (size_t)vb * A->ld_xchg * s; ld_own = A->ld_xchg; }
+  else if (mask_dy) dt_own = L.at<void>(ws, "dt");
+  const void* dT = dt_own ? dt_own : A->dy;     // own rows
+  const int64_t lddT = dt_own ? ld_own : A->lddy;
+  const void* dT_tab = A->xchg ? A->xchg : dT;  // every row (global ids)
+  const int64_t ld_tab = A->xchg ? A->ld_xchg : lddT;
+  void* dxs = d.self_loop ? L.at<void>(ws, "dxs") : nullptr;
+  if (pre) {
+    if (dt_own || (G && d.bias))
+      WG_TRY(bias_grad_mask(dt, nr, d.f_out, A->dy, A->lddy, mask_dy ? A->y : nullptr, A->ldy, dt_own, ld_own,
+                            (G && d.bias) ? G->bias : nullptr, L.at<float>(ws, "colsum"), st));
+    if (d.self_loop && G && G->W_self)
+      WG_TRY(gemm_tn(dt, nr, d.f_in, d.f_out, x_own, A->ldx, dT, lddT, G->W_self, L.at<void>(ws, "tn"), st));
+    if (d.self_loop && d.need_dx) {   // dx self term dT W_0^T (own rows)
+      void* w0 = L.at<void>(ws, "w0");
+      WG_TRY(prep_weight(dt, P->W_self, d.f_in, d.f_out, 0, w0, p->po, (int)rows_i, st));
+      GemmPart part{dT, lddT, w0, p->po, d.f_out, (int)rows_i};
+      GemmEpi e;
+      e.D = dxs; e.ldd = p->pi;
+      WG_TRY(gemm_nt(dt, nr, (int)rup(d.f_in, 16 / s), &part, 1, e, nullptr, 0, st));
+    }
+  }
+  if (!post) return WG_OK;
   // stage 1T: G_(u,r) = sum_{e: src u, type r} c_e dT[dst_e]
   void* gt = L.at<void>(ws, "gt");
   {
     AggArgs a = exec_args(rp->b1, g->E_max);
-    a.table = dT; a.ld_tab = lddT;
+    a.table = dT_tab; a.ld_tab = ld_tab;
     a.out = gt; a.ld_out = p->po;
     a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
     a.F = d.f_out;
     WG_TRY(run(dt, a, rp->b1, st));
   }
-  // dW_r = X_g[group r]^T G[group r]
+  // dW_r = X_g[group r]^T G[group r]   (this rank's out-edges; the caller all-reduces)
   if (G && G->W) {
     void* xg = L.at<void>(ws, "xg");
     AggArgs a = exec_args(rp->bg, g->E_max);
@@ -555,8 +596,6 @@ wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, 
     WG_TRY(run(dt, a, rp->bg, st));
     WG_TRY(gemm_tn_grouped(dt, rp->tn, d.f_in, d.f_out, xg, p->pi, gt, p->po, G->W, L.at<void>(ws, "tn"), st));
   }
-  if (d.self_loop && G && G->W_self)
-    WG_TRY(gemm_tn(dt, V, d.f_in, d.f_out, A->x, A->ldx, dT, lddT, G->W_self, L.at<void>(ws, "tn"), st));
   if (!d.need_dx) return WG_OK;
   // stage 2T: dX_(u,r) = G_(u,r) W_r^T (grouped)
   void* w = L.at<void>(ws, "w");
@@ -568,16 +607,6 @@ wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, 
     GemmEpi e;
     e.D = dxt; e.ldd = p->pi;
     WG_TRY(gemm_nt(dt, rp->n1T, (int)rup(d.f_in, 16 / s), &part, 1, e, nullptr, 0, st));
-  }
-  void* dxs = nullptr;
-  if (d.self_loop) {
-    void* w0 = L.at<void>(ws, "w0");
-    WG_TRY(prep_weight(dt, P->W_self, d.f_in, d.f_out, 0, w0, p->po, (int)rows_i, st));
-    dxs = L.at<void>(ws, "dxs");
-    GemmPart part{dT, lddT, w0, p->po, d.f_out, (int)rows_i};
-    GemmEpi e;
-    e.D = dxs; e.ldd = p->pi;
-    WG_TRY(gemm_nt(dt, V, (int)rup(d.f_in, 16 / s), &part, 1, e, nullptr, 0, st));
   }
   // stage 3T: dx[u] = sum_r dX_(u,r) (+ dT W_0^T)
   {

@@ -222,6 +222,44 @@ int bits_for(uint64_t maxval) {
 
 // Partition one side.  kv = key vertex per edge (dst fwd / src transposed),
 // ov = other endpoint.  Owned key rows [vb, ve).
+// |in_r(dst_e)| per global edge id (RGCN NORM_RIGHT, Q2: c_e = 1/|N_v^r|):
+// sort the (dst, type) keys of ALL edges, count each edge's key by two binary
+// searches -- global, so a rank of a 1-D partition also has the coefficient
+// of out-edges whose destination another rank owns
+__global__ void k_rel_keys(const int32_t* dst, const int32_t* et, int64_t E, int32_t R, uint64_t* k) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < E; e += (int64_t)gridDim.x * blockDim.x)
+    k[e] = (uint64_t)dst[e] * (uint64_t)R + (uint64_t)et[e];
+}
+__global__ void k_rel_count(const uint64_t* keys, const uint64_t* sorted, int64_t E, int32_t* cnt) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < E; e += (int64_t)gridDim.x * blockDim.x) {
+    const uint64_t k = keys[e];
+    int64_t lo = 0, hi = E;
+    while (lo < hi) { const int64_t m = (lo + hi) >> 1; if (sorted[m] < k) lo = m + 1; else hi = m; }
+    int64_t lo2 = lo, hi2 = E;
+    while (lo2 < hi2) { const int64_t m = (lo2 + hi2) >> 1; if (sorted[m] <= k) lo2 = m + 1; else hi2 = m; }
+    cnt[e] = (int32_t)(lo2 - lo);
+  }
+}
+
+wg_status rel_counts(wg_graph_s* g, const int32_t* dst, const int32_t* et, cudaStream_t st) {
+  const int64_t E = g->E_total;
+  WG_TRY(dalloc(g, &g->rel_cnt, std::max<int64_t>(E, 1), st));
+  if (E == 0) return WG_OK;
+  Tmp k(st), ks(st), temp(st);
+  WG_TRY(k.get(sizeof(uint64_t) * E));
+  WG_TRY(ks.get(sizeof(uint64_t) * E));
+  const unsigned nb = (unsigned)std::min<int64_t>(nblk(E), 148 * 16);
+  WG_LAUNCH(k_rel_keys, nb, 256, 0, st, dst, et, E, g->R, k.as<uint64_t>());
+  const int nbits = bits_for((uint64_t)(g->V - 1) * g->R + (g->R - 1));
+  size_t tb = 0;
+  WG_CK(cub::DeviceRadixSort::SortKeys(nullptr, tb, k.as<uint64_t>(), ks.as<uint64_t>(), E, 0, nbits, st));
+  WG_TRY(temp.get(tb));
+  WG_CK(cub::DeviceRadixSort::SortKeys(temp.p, tb, k.as<uint64_t>(), ks.as<uint64_t>(), E, 0, nbits, st));
+  ++launch_counter();
+  WG_LAUNCH(k_rel_count, nb, 256, 0, st, k.as<uint64_t>(), ks.as<uint64_t>(), E, g->rel_cnt);
+  return WG_OK;
+}
+
 wg_status build_side(wg_graph_s* g, Side& S, const int32_t* kv, const int32_t* ov, const int32_t* et,
                      cudaStream_t st) {
   const int64_t E = g->E_total, T = g->T;
@@ -481,6 +519,7 @@ wg_status graph_create(const wg_graph_desc* d, int device, cudaStream_t st, wg_g
   if (g->by_type) {
     if ((s = dalloc(g, &g->etype_all, E, st)) != WG_OK) { free_tmp(); return fail(s); }
     cudaMemcpyAsync(g->etype_all, et, 4 * E, cudaMemcpyDeviceToDevice, st);
+    if ((s = rel_counts(g, dst, et, st)) != WG_OK) { free_tmp(); return fail(s); }
   }
   if ((s = build_side(g, g->fwd, dst, src, et, st)) != WG_OK) { free_tmp(); return fail(s); }
   if ((s = build_side(g, g->bwd, src, dst, et, st)) != WG_OK) { free_tmp(); return fail(s); }

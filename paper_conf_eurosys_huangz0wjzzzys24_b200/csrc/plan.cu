@@ -177,9 +177,9 @@ wg_status plan_create(wg_graph g, const wg_conv_desc* d, wg_plan* out) {
   if (d->model != WG_RGCN)
     WG_REQ(!g->by_type, WG_ERR_UNSUPPORTED, "typed graph (num_types > 1) is only supported by RGCN");
   if (d->model == WG_GAT) WG_REQ(d->heads >= 1, WG_ERR_INVALID, "GAT needs heads >= 1");
-  if (d->model == WG_GAT || d->model == WG_RGCN)
+  if (d->model == WG_GAT)
     WG_REQ(g->vb == 0 && g->ve == g->V, WG_ERR_UNSUPPORTED,
-           "GAT / RGCN layers need the full graph (the 1-D partition covers GCN / SAGE / GIN)");
+           "GAT layers need the full graph (the 1-D partition covers GCN / SAGE / GIN / RGCN)");
   WG_CK(cudaSetDevice(g->device));
   auto* p = new wg_plan_s();
   p->g = g;

@@ -115,6 +115,7 @@ struct wg_graph_s {
   wg::Side fwd, bwd;
   int64_t* fwdpos = nullptr;   // [E_T] (owning all rows)
   int32_t* etype_all = nullptr; // [E_total] types by global edge id (typed graphs)
+  int32_t* rel_cnt = nullptr;   // [E_total] |in_r(dst_e)| by global edge id (typed graphs)
   std::vector<void*> allocs;
   int live_plans = 0;
 };

@@ -55,7 +55,7 @@ class GNNStack:
             pol = policy
             fi = self.f_in[i]
             conv = Conv_(graph, model, fi, dims[i + 1], policy=pol, **kw)
-            if self.dist and conv.n_edge_tasks and conv.n_vertex_tasks:   # uniform plan per layer when distributed
+            if self.dist and model != "rgcn" and conv.n_edge_tasks and conv.n_vertex_tasks:   # uniform plan per layer
                 pol = "vertex" if conv.n_vertex_tasks > conv.n_edge_tasks else "edge"
                 conv.close()
                 conv = Conv_(graph, model, fi, dims[i + 1], policy=pol, **kw)
@@ -73,7 +73,7 @@ class GNNStack:
         self.xchg_f, self.xchg_b = [], []
         for c in self.convs:
             self.xchg_f.append(padded(self.Vtab, pitch(c.f_out, dtype), dtype, self.dev)
-                               if (self.dist and c.n_vertex_tasks) else None)
+                               if self._fwd_xchg(c) else None)
             wb = (c.f_out if c.bwd_path == 1 else c.f_in)
             self.xchg_b.append(padded(self.Vtab, pitch(wb, dtype), dtype, self.dev) if self.dist else None)
         for p in self.params:
@@ -82,6 +82,11 @@ class GNNStack:
         self.opt = torch.optim.Adam([v for p in self.params for v in p.values()], lr=lr)
 
     # -------------------------------------------------------------- helpers
+    def _fwd_xchg(self, c):
+        """VERTEX layers exchange Y = h W (transform before communicate); RGCN
+        (per-relation transforms) and EDGE layers gather the activation itself."""
+        return self.dist and c.n_vertex_tasks > 0 and c.model != "rgcn"
+
     def _own(self, t):
         return t[self.vb:self.vb + self.rows] if self.dist else t
 
@@ -97,15 +102,15 @@ class GNNStack:
         h = x
         for i, c in enumerate(self.convs):
             y = self._own(self.h[i + 1])
-            if self.dist and c.n_vertex_tasks:
+            if self._fwd_xchg(c):
                 xg = self.xchg_f[i]
                 c.forward_raw(h, self.params[i], y=y, saved=self.saved[i], phase=C.PHASE_PRE, xchg=xg)
                 self._allgather(xg)
                 c.forward_raw(h, self.params[i], y=y, saved=self.saved[i], phase=C.PHASE_POST, xchg=xg)
             else:
                 c.forward_raw(h, self.params[i], y=y, saved=self.saved[i])
-            if self.dist and i + 1 < self.L and not self.convs[i + 1].n_vertex_tasks:
-                self._allgather(self.h[i + 1])       # next EDGE layer gathers raw rows
+            if self.dist and i + 1 < self.L and not self._fwd_xchg(self.convs[i + 1]):
+                self._allgather(self.h[i + 1])       # next EDGE / RGCN layer gathers raw rows
             h = self.h[i + 1]
         self.x = x
         return self._own(self.h[self.L])

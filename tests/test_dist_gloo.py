@@ -4,8 +4,9 @@ GNNStack's distributed path (T-aligned equal vertex blocks, PRE / all-gather /
 POST exchange phases for forward and backward, exchanged table = activation
 for EDGE layers or Y = x W for VERTEX layers, dAgg or dT in backward, weight-
 gradient all-reduce) runs on two CPU processes over gloo.  The layer compute is
-a test-only float64 torch implementation of GraphSAGE that honours the
-library's phase contract (include/wg.h, wg_fwd_args / wg_bwd_args); the CUDA
+a test-only float64 torch implementation of GraphSAGE (and of RGCN with
+1/|N_v^r| normalisation and a self-loop: its forward reads the all-gathered
+activation, its backward exchanges dT) that honours the library's phase contract (include/wg.h, wg_fwd_args / wg_bwd_args); the CUDA
 kernels themselves are covered by tests/test_gpu_*.  Each rank's logits rows
 and the all-reduced weight gradients must equal the single-process run."""
 import os
@@ -21,7 +22,8 @@ import synth
 
 
 class FakeGraph:
-    def __init__(self, src, dst, V, vb=0, ve=None):
+    def __init__(self, src, dst, V, vb=0, ve=None, etype=None):
+        self.etype = None if etype is None else torch.from_numpy(etype).long()
         self.src, self.dst, self.V = torch.from_numpy(src).long(), torch.from_numpy(dst).long(), V
         self.v_begin, self.n_rows = vb, (V if ve is None else ve) - vb
         self.device = "cpu"
@@ -32,6 +34,7 @@ class FakeSage:
 
     def __init__(self, graph, model, fi, fo, *, policy="edge", fuse_relu=False, need_dx=True, **kw):
         self.g, self.f_in, self.f_out, self.out_dim = graph, fi, fo, fo
+        self.model = model
         self.n_vertex_tasks = 1 if policy == "vertex" else 0
         self.n_edge_tasks = 1 - self.n_vertex_tasks
         self.bwd_path = self.n_vertex_tasks
@@ -118,19 +121,84 @@ class FakeSage:
         return dx, grads
 
 
+class FakeRgcn:
+    """RGCN layer in float64 (c_e = 1/|in_r(dst)|, self-loop W_0, bias) following
+    the RGCN phase contract: forward reads all rows of x (no exchange), backward
+    PRE writes this rank's dT rows into the exchange table, POST gathers it."""
+
+    def __init__(self, graph, model, fi, fo, *, fuse_relu=False, need_dx=True, **kw):
+        self.g, self.f_in, self.f_out, self.out_dim, self.model = graph, fi, fo, fo, model
+        self.n_vertex_tasks, self.n_edge_tasks, self.bwd_path = 1, 1, 1   # mixed plans are fine for RGCN
+        self.fuse_relu, self.need_dx = fuse_relu, need_dx
+        key = graph.dst * R + graph.etype
+        cnt = torch.bincount(key, minlength=graph.V * R)
+        self.c = 1.0 / cnt[key].double()                  # global |in_r(dst_e)|
+        self.vb, self.ve = graph.v_begin, graph.v_begin + graph.n_rows
+        self.inm = (graph.dst >= self.vb) & (graph.dst < self.ve)
+        self.outm = (graph.src >= self.vb) & (graph.src < self.ve)
+
+    def new_saved(self):
+        return {}
+
+    def close(self):
+        pass
+
+    @torch.no_grad()
+    def forward_raw(self, x, params, y=None, saved=None, phase=0, xchg=None, stream=None):
+        if phase == 1:
+            return y, saved
+        W, W0, b = params["W"].double(), params["W_self"].double(), params["bias"].double()
+        m = self.inm
+        s, d, t, c = self.g.src[m], self.g.dst[m], self.g.etype[m], self.c[m]
+        msg = torch.einsum("ei,eio->eo", x[s], W[t]) * c[:, None]
+        out = x[self.vb:self.ve] @ W0 + b
+        out.index_add_(0, d - self.vb, msg)
+        y[:] = torch.relu(out) if self.fuse_relu else out
+        return y, saved
+
+    @torch.no_grad()
+    def backward_raw(self, dy, x, y, saved, params, dx=None, phase=0, xchg=None, grads=None, stream=None,
+                     dx_mask=None, dy_masked=False):
+        W, W0 = params["W"].double(), params["W_self"].double()
+        fo = self.f_out
+        dT = dy * (y > 0) if (self.fuse_relu and not dy_masked) else dy
+        if xchg is None:                          # single process: the table is local
+            xchg = torch.zeros(self.g.V, fo, dtype=torch.float64)
+        if phase in (0, 1):
+            xchg[self.vb:self.ve, :fo] = dT
+            grads["W_self"][:] = x[self.vb:self.ve].T @ dT
+            grads["bias"][:] = dT.sum(0)
+        if phase == 1:
+            return dx, grads
+        m = self.outm
+        s, d, t, c = self.g.src[m], self.g.dst[m], self.g.etype[m], self.c[m]
+        gd = xchg[d, :fo] * c[:, None]
+        dW = torch.zeros_like(W)
+        dW.index_add_(0, t, torch.einsum("ei,eo->eio", x[s], gd))
+        grads["W"][:] = dW
+        if self.need_dx:
+            out = dT @ W0.T
+            out.index_add_(0, s - self.vb, torch.einsum("eo,eio->ei", gd, W[t]))
+            dx[:] = out * (dx_mask > 0) if dx_mask is not None else out
+        return dx, grads
+
+
 def factory(graph, model, fi, fo, **kw):
+    if model == "rgcn":
+        return FakeRgcn(graph, model, fi, fo, **kw)
     kw["policy"] = "edge" if fi != 6 else "vertex"    # layer 2 of dims [8, 6, 6, 5] is a VERTEX layer
     return FakeSage(graph, model, fi, fo, **kw)
 
 
-V, E, DIMS = 700, 6000, [8, 6, 6, 5]
+V, E, DIMS, R = 700, 6000, [8, 6, 6, 5], 3
 
 
-def run_stack(graph, group, block):
+def run_stack(graph, group, block, model="sage"):
     from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack
     torch.manual_seed(0)
-    st = GNNStack(graph, "sage", DIMS, dtype=torch.float64, group=group, block=block, conv_factory=factory,
-                  device=torch.device("cpu"), seed=3)
+    kw = dict(R=R, conv_kw={"self_loop": True}) if model == "rgcn" else {}
+    st = GNNStack(graph, model, DIMS, dtype=torch.float64, group=group, block=block, conv_factory=factory,
+                  device=torch.device("cpu"), seed=3, **kw)
     x = torch.zeros(st.Vtab, DIMS[0], dtype=torch.float64)
     x[:V] = torch.from_numpy(synth.make_features(V, DIMS[0], seed=4)).double()
     logits = st.forward(x).clone()
@@ -140,15 +208,16 @@ def run_stack(graph, group, block):
     return logits, [{k: v.clone() for k, v in g.items()} for g in st.grads]
 
 
-def worker(rank, world, port, q):
+def worker(rank, world, port, q, model):
     os.environ["MASTER_ADDR"], os.environ["MASTER_PORT"] = "127.0.0.1", str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import partition_1d
-    src, dst, _ = synth.make_graph(V, E, seed=9, alpha=0.5, symmetric=True)
-    ref_logits, ref_grads = run_stack(FakeGraph(src, dst, V), None, None)
+    src, dst, et = synth.make_graph(V, E, seed=9, alpha=0.5, symmetric=model != "rgcn", R=R if model == "rgcn" else 1)
+    et = et if model == "rgcn" else None
+    ref_logits, ref_grads = run_stack(FakeGraph(src, dst, V, etype=et), None, None, model)
     block, bounds = partition_1d(V, world, T=128)
     vb, ve = bounds[rank]
-    logits, grads = run_stack(FakeGraph(src, dst, V, vb, ve), dist.group.WORLD, block)
+    logits, grads = run_stack(FakeGraph(src, dst, V, vb, ve, etype=et), dist.group.WORLD, block, model)
     ok = torch.allclose(logits, ref_logits[vb:ve], rtol=1e-10, atol=1e-12)
     for g1, g2 in zip(grads, ref_grads):      # fp32 gradients: all-reduce sums partials in another order
         for k in g1:
@@ -165,12 +234,13 @@ def free_port():
     return p
 
 
+@pytest.mark.parametrize("model", ["sage", "rgcn"])
 @pytest.mark.parametrize("world", [2])
-def test_gloo_1d_partition_matches_single(world):
+def test_gloo_1d_partition_matches_single(world, model):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = free_port()
-    procs = [ctx.Process(target=worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=worker, args=(r, world, port, q, model)) for r in range(world)]
     for p in procs:
         p.start()
     res = []
