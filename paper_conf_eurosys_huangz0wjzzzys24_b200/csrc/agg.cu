@@ -690,12 +690,31 @@ __global__ void __launch_bounds__(256) k_colsum(int64_t M, int N, const T* dy, i
   }
 }
 
-__global__ void k_colsum_reduce(const float* part, int nblk, int N, float* out) {
-  int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= N) return;
+// out[c] = sum_b part[b][c]: 32 columns per CTA, warp w sums blocks b = w mod 8
+// (4 loads in flight), then the 8 warp partials are added in warp order --
+// a fixed order, so the result is deterministic
+__global__ void __launch_bounds__(256) k_colsum_reduce(const float* part, int nblk, int N, float* out) {
+  __shared__ float red[8][33];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + lane;
   float s = 0.f;
-  for (int b = 0; b < nblk; ++b) s += part[(int64_t)b * N + c];
-  out[c] = s;
+  if (c < N) {
+    int b = warp;
+    for (; b + 24 < nblk; b += 32) {
+      const float v0 = part[(int64_t)b * N + c], v1 = part[(int64_t)(b + 8) * N + c];
+      const float v2 = part[(int64_t)(b + 16) * N + c], v3 = part[(int64_t)(b + 24) * N + c];
+      s += v0; s += v1; s += v2; s += v3;
+    }
+    for (; b < nblk; b += 8) s += part[(int64_t)b * N + c];
+  }
+  red[warp][lane] = s;
+  __syncthreads();
+  if (warp == 0 && c < N) {
+    float t = 0.f;
+#pragma unroll
+    for (int w = 0; w < 8; ++w) t += red[w][lane];
+    out[c] = t;
+  }
 }
 
 constexpr int COLSUM_BLKS = 1184;  // 8 x 148 SMs
@@ -740,7 +759,7 @@ wg_status bias_grad_mask(wg_dtype dt, int64_t M, int N, const void* dy, int64_t 
   else
     WG_LAUNCH(k_colsum<float>, nblk, threads, smem, s, M, N, (const float*)dy, lddy, (const float*)ref, ldref,
               (float*)dt_out, ldt, scratch, rpb);
-  if (db) WG_LAUNCH(k_colsum_reduce, (unsigned)cdiv(N, 128), 128, 0, s, scratch, nblk, N, db);
+  if (db) WG_LAUNCH(k_colsum_reduce, (unsigned)cdiv(N, 32), 256, 0, s, scratch, nblk, N, db);
   return WG_OK;
 }
 

@@ -274,6 +274,149 @@ __global__ void __launch_bounds__(256) k_gat_fwd(GatArgs a, int64_t row_base) {
   }
 }
 
+// Forward, chunked softmax: one warp per row chunk; the row's edges are taken
+// 32 at a time -- lane k computes the logits of edge k for every head, the
+// chunk max / exp run once per edge (not once per edge and feature), the
+// accumulator is rescaled once per 32 edges, and the gather loop is a plain
+// alpha-weighted row sum (alpha and source id broadcast through shared
+// memory).  Same outputs as k_gat_fwd (agg, m, l, y / split partials).
+constexpr int GAT_HM = 8;   // heads handled by k_gat_fwd2
+
+template <typename T, typename TO, int NV, int U, int HM>
+__global__ void __launch_bounds__(256, (HM <= 4 && NV == 2) ? 4 : 3) k_gat_fwd2(GatArgs a, int64_t row_base) {
+  constexpr int EPV = GV<T>::EPV;
+  static_assert(EPV == 4, "G is fp32 (agg rows are stored as float4)");
+  static_assert(HM <= GAT_HM, "heads");
+  __shared__ float orow[8][NV * 32 * EPV];
+  __shared__ float alp[8][32][HM + 1];       // p_e per head of the chunk's edges
+  __shared__ int sid[8][32];                  // source ids of the chunk's edges
+  __shared__ float hsc[8][3][HM];             // per head: rescale factor, m, l
+  const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
+  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (w >= a.n_chunks) return;
+  const RowChunk ch = a.chunks[w];
+  const int64_t d = row_base + ch.row;
+  const int H = a.H;
+  const T* G = static_cast<const T*>(a.G);
+  float erd[HM], m[HM], lp[HM];
+#pragma unroll
+  for (int h = 0; h < HM; ++h) {
+    erd[h] = h < H ? a.er[d * H + h] : 0.f;
+    m[h] = -INFINITY;
+    lp[h] = 0.f;
+  }
+  int hd[NV];
+  float acc[NV][EPV];
+#pragma unroll
+  for (int q = 0; q < NV; ++q) {
+    const int vi = lane + 32 * q;
+    hd[q] = vi < a.VPR ? min((vi * EPV) / a.Fo, HM - 1) : 0;
+#pragma unroll
+    for (int i = 0; i < EPV; ++i) acc[q][i] = 0.f;
+  }
+  for (int64_t base = ch.e_lo; base < ch.e_hi; base += 32) {
+    const int n = (int)min((int64_t)32, ch.e_hi - base);
+    int s = 0;
+    float lg[HM];
+    if (lane < n) {
+      s = a.idx[base + lane];
+#pragma unroll
+      for (int h = 0; h < HM; ++h) lg[h] = h < H ? lrelu(a.el[(int64_t)s * H + h] + erd[h], a.slope) : -INFINITY;
+    } else {
+#pragma unroll
+      for (int h = 0; h < HM; ++h) lg[h] = -INFINITY;
+    }
+    sid[wi][lane] = s;
+#pragma unroll
+    for (int h = 0; h < HM; ++h) {
+      if (h >= H) break;
+      float mc = lg[h];
+#pragma unroll
+      for (int o = 16; o; o >>= 1) mc = fmaxf(mc, __shfl_xor_sync(0xffffffffu, mc, o));
+      const float mn = fmaxf(m[h], mc);
+      const float sc = __expf(m[h] - mn);      // m = -inf on the first chunk: 0
+      const float p = lane < n ? __expf(lg[h] - mn) : 0.f;
+      lp[h] = lp[h] * sc + p;
+      m[h] = mn;
+      alp[wi][lane][h] = p;
+      if (lane == 0) hsc[wi][0][h] = sc;
+    }
+    __syncwarp();
+#pragma unroll
+    for (int q = 0; q < NV; ++q) {
+      const float f = hsc[wi][0][hd[q]];
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) acc[q][i] *= f;
+    }
+    for (int j = 0; j < n; j += U) {
+      int4 v[U][NV];
+      float al[U][NV];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int k = j + u;
+        const bool ok = k < n;
+        const int sk = sid[wi][ok ? k : 0];
+#pragma unroll
+        for (int q = 0; q < NV; ++q) {
+          const int vi = lane + 32 * q;
+          v[u][q] = (ok && vi < a.VPR) ? ld16(G + (int64_t)sk * a.ldg + vi * EPV) : make_int4(0, 0, 0, 0);
+          al[u][q] = ok ? alp[wi][k][hd[q]] : 0.f;
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int q = 0; q < NV; ++q) {
+          float g[EPV];
+          GV<T>::unpack(v[u][q], g);
+#pragma unroll
+          for (int i = 0; i < EPV; ++i) acc[q][i] += al[u][q] * g[i];
+        }
+    }
+    __syncwarp();
+  }
+  // per-head denominators (lane partials -> warp sums); m / l to shared memory
+#pragma unroll
+  for (int h = 0; h < HM; ++h) {
+    if (h >= H) break;
+    float l = lp[h];
+#pragma unroll
+    for (int o = 16; o; o >>= 1) l += __shfl_xor_sync(0xffffffffu, l, o);
+    if (lane == 0) { hsc[wi][1][h] = m[h]; hsc[wi][2][h] = l; }
+  }
+  __syncwarp();
+  if (ch.slot >= 0) {
+    float* pp = a.part + (int64_t)ch.slot * a.part_ld;
+#pragma unroll
+    for (int q = 0; q < NV; ++q) {
+      const int vi = lane + 32 * q;
+      if (vi >= a.VPR) continue;
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) pp[vi * EPV + i] = acc[q][i];
+    }
+    if (lane < H) { pp[a.HF + lane] = hsc[wi][1][lane]; pp[a.HF + a.H + lane] = hsc[wi][2][lane]; }
+    return;
+  }
+#pragma unroll
+  for (int q = 0; q < NV; ++q) {
+    const int vi = lane + 32 * q;
+    if (vi >= a.VPR) continue;
+    const int c0 = vi * EPV;
+    const float l = hsc[wi][2][hd[q]];
+    const float inv = l > 0.f ? 1.f / l : 0.f;
+    float o[EPV];
+#pragma unroll
+    for (int i = 0; i < EPV; ++i) o[i] = (c0 + i < a.HF) ? acc[q][i] * inv : 0.f;
+    float* ag = static_cast<float*>(a.agg) + (int64_t)ch.row * a.ld_agg + c0;
+    *reinterpret_cast<float4*>(ag) = make_float4(o[0], o[1], o[2], o[3]);
+#pragma unroll
+    for (int i = 0; i < EPV; ++i) orow[wi][c0 + i] = o[i];
+  }
+  if (lane < H) { a.m[d * H + lane] = hsc[wi][1][lane]; a.l[d * H + lane] = hsc[wi][2][lane]; }
+  __syncwarp();
+  gat_write_y<TO>(a, ch.row, orow[wi], lane, 32);
+}
+
 // flash-style merge of the (m, l, acc) partials of split rows, chunk order:
 // M = max_k m_k, then l = sum_k l_k e^{m_k - M}, o = sum_k acc_k e^{m_k - M}
 // (independent loads, fixed order); writes agg, m, l and the y row
@@ -286,8 +429,19 @@ __global__ void __launch_bounds__(256) k_gat_fwd_combine(GatArgs a, const SplitR
     const int h = c / a.Fo;
     const float* p0 = a.part + (int64_t)sr.first_slot * a.part_ld;
     float M = -INFINITY;
-    for (int k = 0; k < sr.n_slots; ++k) {
-      const float* pp = p0 + (int64_t)k * a.part_ld;
+    int k0 = 0;
+    for (; k0 + 4 <= sr.n_slots; k0 += 4) {      // 4 independent slot loads in flight
+      float lk[4], mk[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const float* pp = p0 + (int64_t)(k0 + j) * a.part_ld;
+        lk[j] = pp[a.HF + a.H + h]; mk[j] = pp[a.HF + h];
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) if (lk[j] > 0.f) M = fmaxf(M, mk[j]);
+    }
+    for (; k0 < sr.n_slots; ++k0) {
+      const float* pp = p0 + (int64_t)k0 * a.part_ld;
       if (pp[a.HF + a.H + h] > 0.f) M = fmaxf(M, pp[a.HF + h]);
     }
     float l = 0.f, o = 0.f;
@@ -503,36 +657,70 @@ __global__ void __launch_bounds__(256) k_gat_s2(int64_t rows, int64_t row_base, 
   }
 }
 
-// der[v,h] = sum_{e in in(v)} dt_e (forward order: contiguous per row), warp per row
+// der over the forward row chunks (<= GAT_CHUNK edges each, SPLIT rows cut
+// into several): eight lanes per chunk, four independent loads in flight per
+// lane, fixed-order reduction; SPLIT chunks leave H partials in their slot,
+// summed in chunk order by k_gat_der_combine
 template <int H>
-__global__ void k_gat_der2(int64_t rows, int64_t row_base, const int64_t* row_ptr, const float* dt, float* der) {
-  const int lane = threadIdx.x & 31;
-  const int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  if (r >= rows) return;
+__global__ void k_gat_der3(const RowChunk* chunks, int n, int64_t row_base, const float* dt, float* der,
+                           float* part, int part_ld) {
+  const int sub = threadIdx.x & 7;
+  const int64_t c = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 3;
   float s[H];
 #pragma unroll
   for (int h = 0; h < H; ++h) s[h] = 0.f;
-  const int64_t e1 = row_ptr[r + 1];
-  for (int64_t e = row_ptr[r] + lane; e < e1; e += 32) {
-    if constexpr (H == 4) {
-      const float4 v = __ldg(reinterpret_cast<const float4*>(dt) + e);
-      s[0] += v.x; s[1] += v.y; s[2] += v.z; s[3] += v.w;
-    } else {
+  RowChunk ch{};
+  if (c < n) {
+    ch = chunks[c];
+    auto add = [&](int64_t e) {
+      if constexpr (H == 4) {
+        const float4 v = __ldg(reinterpret_cast<const float4*>(dt) + e);
+        s[0] += v.x; s[1] += v.y; s[2] += v.z; s[3] += v.w;
+      } else {
 #pragma unroll
-      for (int h = 0; h < H; ++h) s[h] += dt[e * H + h];
+        for (int h = 0; h < H; ++h) s[h] += dt[e * H + h];
+      }
+    };
+    int64_t e = ch.e_lo + sub;
+    for (; e + 24 < ch.e_hi; e += 32) {
+      if constexpr (H == 4) {
+        const float4 v0 = __ldg(reinterpret_cast<const float4*>(dt) + e);
+        const float4 v1 = __ldg(reinterpret_cast<const float4*>(dt) + e + 8);
+        const float4 v2 = __ldg(reinterpret_cast<const float4*>(dt) + e + 16);
+        const float4 v3 = __ldg(reinterpret_cast<const float4*>(dt) + e + 24);
+        s[0] += v0.x; s[1] += v0.y; s[2] += v0.z; s[3] += v0.w;
+        s[0] += v1.x; s[1] += v1.y; s[2] += v1.z; s[3] += v1.w;
+        s[0] += v2.x; s[1] += v2.y; s[2] += v2.z; s[3] += v2.w;
+        s[0] += v3.x; s[1] += v3.y; s[2] += v3.z; s[3] += v3.w;
+      } else {
+        add(e); add(e + 8); add(e + 16); add(e + 24);
+      }
     }
+    for (; e < ch.e_hi; e += 8) add(e);
   }
 #pragma unroll
   for (int h = 0; h < H; ++h) {
 #pragma unroll
-    for (int o = 16; o; o >>= 1) s[h] += __shfl_xor_sync(0xffffffffu, s[h], o);
+    for (int o = 4; o; o >>= 1) s[h] += __shfl_xor_sync(0xffffffffu, s[h], o);
   }
-  if (lane < H) {
+  if (c < n && sub < H) {
     float o = s[0];
 #pragma unroll
-    for (int h = 1; h < H; ++h) if (lane == h) o = s[h];
-    der[(row_base + r) * H + lane] = o;
+    for (int h = 1; h < H; ++h) if (sub == h) o = s[h];
+    if (ch.slot >= 0) part[(int64_t)ch.slot * part_ld + sub] = o;
+    else der[(row_base + ch.row) * H + sub] = o;
   }
+}
+
+__global__ void k_gat_der_combine(const SplitRow* rows, int n, int64_t row_base, const float* part, int part_ld,
+                                  int H, float* der) {
+  const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (t >= (int64_t)n * H) return;
+  const SplitRow sr = rows[t / H];
+  const int h = (int)(t % H);
+  float s = 0.f;
+  for (int k = 0; k < sr.n_slots; ++k) s += part[(int64_t)(sr.first_slot + k) * part_ld + h];
+  der[(row_base + sr.row) * H + h] = s;
 }
 
 __global__ void k_gat_bwd_combine(GatArgs a, const SplitRow* rows, int64_t row_base) {
@@ -602,13 +790,24 @@ __global__ void k_gat_dG(int64_t rows, int64_t row_base, GatArgs a, const float*
   }
 }
 
-__global__ void k_pair_reduce(const float* part, int nblk, int n, float* out0, float* out1) {
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= 2 * n) return;
+// out0 / out1 = column sums of the [nblk x 2n] block partials (first / second
+// half): 32 columns per CTA, fixed-order warp split as k_colsum_reduce
+__global__ void __launch_bounds__(256) k_pair_reduce(const float* part, int nblk, int n, float* out0, float* out1) {
+  __shared__ float red[8][33];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + lane;
   float s = 0.f;
-  for (int b = 0; b < nblk; ++b) s += part[(int64_t)b * 2 * n + c];
-  if (c < n) { if (out0) out0[c] = s; }
-  else if (out1) out1[c - n] = s;
+  if (c < 2 * n)
+    for (int b = warp; b < nblk; b += 8) s += part[(int64_t)b * 2 * n + c];
+  red[warp][lane] = s;
+  __syncthreads();
+  if (warp == 0 && c < 2 * n) {
+    float t = 0.f;
+#pragma unroll
+    for (int w = 0; w < 8; ++w) t += red[w][lane];
+    if (c < n) { if (out0) out0[c] = t; }
+    else if (out1) out1[c - n] = t;
+  }
 }
 
 constexpr int DG_BLKS = 592;
@@ -730,9 +929,19 @@ static wg_status gat_fwd_t(wg_plan_s* p, const wg_params* P, const wg_fwd_args* 
   a.chunks = gp->fwd; a.n_chunks = gp->n_fwd;
   if (gp->n_fwd) {
     const unsigned cbk = gs_grid((int64_t)gp->n_fwd * 32);
-    if (NV == 1) WG_LAUNCH((k_gat_fwd<float, T, 1, 4>), cbk, 256, 0, st, a, vb);
-    else if (NV == 2) WG_LAUNCH((k_gat_fwd<float, T, 2, 4>), cbk, 256, 0, st, a, vb);
-    else WG_LAUNCH((k_gat_fwd<float, T, 4, 2>), cbk, 256, 0, st, a, vb);
+    if (H <= 4) {
+      if (NV == 1) WG_LAUNCH((k_gat_fwd2<float, T, 1, 8, 4>), cbk, 256, 0, st, a, vb);
+      else if (NV == 2) WG_LAUNCH((k_gat_fwd2<float, T, 2, 4, 4>), cbk, 256, 0, st, a, vb);
+      else WG_LAUNCH((k_gat_fwd2<float, T, 4, 2, 4>), cbk, 256, 0, st, a, vb);
+    } else if (H <= GAT_HM) {
+      if (NV == 1) WG_LAUNCH((k_gat_fwd2<float, T, 1, 8, 8>), cbk, 256, 0, st, a, vb);
+      else if (NV == 2) WG_LAUNCH((k_gat_fwd2<float, T, 2, 4, 8>), cbk, 256, 0, st, a, vb);
+      else WG_LAUNCH((k_gat_fwd2<float, T, 4, 2, 8>), cbk, 256, 0, st, a, vb);
+    } else {
+      if (NV == 1) WG_LAUNCH((k_gat_fwd<float, T, 1, 4>), cbk, 256, 0, st, a, vb);
+      else if (NV == 2) WG_LAUNCH((k_gat_fwd<float, T, 2, 4>), cbk, 256, 0, st, a, vb);
+      else WG_LAUNCH((k_gat_fwd<float, T, 4, 2>), cbk, 256, 0, st, a, vb);
+    }
   }
   if (gp->n_fsplit) WG_LAUNCH(k_gat_fwd_combine<T>, gp->n_fsplit, 256, 0, st, a, gp->fsplit, vb);
   return WG_OK;
@@ -819,18 +1028,26 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
   // (chunks cover every row, including empty ones -- see build_chunks)
   if (gp->n_bsplit) WG_LAUNCH(k_gat_bwd_combine, gp->n_bsplit, 128, 0, st, a, gp->bsplit, vb);
   float* der = L.at<float>(ws, "der");
-  const unsigned tbk = gs_grid(nr * 32);
-  if (H == 4) WG_LAUNCH(k_gat_der2<4>, tbk, 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, der);
-  else if (H == 1) WG_LAUNCH(k_gat_der2<1>, tbk, 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, der);
-  else if (H == 2) WG_LAUNCH(k_gat_der2<2>, tbk, 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, der);
-  else if (H == 8) WG_LAUNCH(k_gat_der2<8>, tbk, 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, der);
-  else WG_LAUNCH(k_gat_der, (unsigned)cdiv(nr * 32, 256), 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, H, der);
+  // (the split-row partial slots of the source-major pass were consumed by
+  // k_gat_bwd_combine above: `part` is reused for the der partials)
+  const unsigned tbk = gs_grid((int64_t)gp->n_fwd * 8), tbk32 = gs_grid(nr * 32);
+  if (H == 4 || H == 1 || H == 2 || H == 8) {
+    if (H == 4) WG_LAUNCH(k_gat_der3<4>, tbk, 256, 0, st, gp->fwd, gp->n_fwd, vb, a.dt, der, a.part, a.part_ld);
+    else if (H == 1) WG_LAUNCH(k_gat_der3<1>, tbk, 256, 0, st, gp->fwd, gp->n_fwd, vb, a.dt, der, a.part, a.part_ld);
+    else if (H == 2) WG_LAUNCH(k_gat_der3<2>, tbk, 256, 0, st, gp->fwd, gp->n_fwd, vb, a.dt, der, a.part, a.part_ld);
+    else WG_LAUNCH(k_gat_der3<8>, tbk, 256, 0, st, gp->fwd, gp->n_fwd, vb, a.dt, der, a.part, a.part_ld);
+    if (gp->n_fsplit)
+      WG_LAUNCH(k_gat_der_combine, gs_grid((int64_t)gp->n_fsplit * H), 256, 0, st, gp->fsplit, gp->n_fsplit, vb,
+                a.part, a.part_ld, H, der);
+  } else {
+    WG_LAUNCH(k_gat_der, tbk32, 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, H, der);
+  }
   const int64_t rpb = std::max<int64_t>(1, cdiv(nr, DG_BLKS));
   const int nblk = (int)cdiv(nr, rpb);
   float* dgp = L.at<float>(ws, "dgp");
   WG_LAUNCH(k_gat_dG<T>, nblk, 256, 0, st, nr, vb, a, P->attn_l, P->attn_r, der, (T*)dG, (T*)dGlo, p->po, dgp,
             rpb);
-  WG_LAUNCH(k_pair_reduce, (unsigned)cdiv(2 * HF, 128), 128, 0, st, dgp, nblk, HF, Gr ? Gr->attn_l : nullptr,
+  WG_LAUNCH(k_pair_reduce, (unsigned)cdiv(2 * HF, 32), 256, 0, st, dgp, nblk, HF, Gr ? Gr->attn_l : nullptr,
             Gr ? Gr->attn_r : nullptr);
   }
   // dW = x^T dG ; dx = dG W^T   (dG = hi + lo for bf16)
