@@ -282,8 +282,8 @@ __global__ void __launch_bounds__(256) k_gat_fwd(GatArgs a, int64_t row_base) {
 // memory).  Same outputs as k_gat_fwd (agg, m, l, y / split partials).
 constexpr int GAT_HM = 8;   // heads handled by k_gat_fwd2
 
-template <typename T, typename TO, int NV, int U, int HM>
-__global__ void __launch_bounds__(256, (HM <= 4 && NV == 2) ? 4 : 3) k_gat_fwd2(GatArgs a, int64_t row_base) {
+template <typename T, typename TO, int NV, int U, int HM, int MINB = (HM <= 4 && NV == 2) ? 4 : 3>
+__global__ void __launch_bounds__(256, MINB) k_gat_fwd2(GatArgs a, int64_t row_base) {
   constexpr int EPV = GV<T>::EPV;
   static_assert(EPV == 4, "G is fp32 (agg rows are stored as float4)");
   static_assert(HM <= GAT_HM, "heads");
@@ -610,6 +610,127 @@ __global__ void __launch_bounds__(256, 2) k_gat_bwd_src2(GatArgs a, int64_t row_
     const int c0 = (lane + 32 * q) * EPV;
     float* out = ch.slot >= 0 ? a.part + (int64_t)ch.slot * a.part_ld : a.dg + u * a.ld_dg;
     *reinterpret_cast<float4*>(out + c0) = make_float4(acc[q][0], acc[q][1], acc[q][2], acc[q][3]);
+    if (lead[q]) {
+      if (ch.slot >= 0) out[a.HF + hd[q]] = dl[q];
+      else a.del[u * a.H + hd[q]] = dl[q];
+    }
+  }
+}
+
+// Source-major backward pass, per-edge pre-pass: for each 32-edge chunk of the
+// source row, lane k evaluates edge k's per-head terms once (alpha_e,
+// alpha_e * lrelu'(t_e), s[dd]) into shared memory; the gather loop then only
+// reads dy rows, forms the per-head dot products and accumulates.  The
+// head-mean factor (last layer) is folded into g[u] and applied to dg once.
+// Same outputs as k_gat_bwd_src2 (dg, del, dt_e, split partials).
+template <typename T, int NV, int U, int SEG, int HM, int MINB = 2>
+__global__ void __launch_bounds__(256, MINB) k_gat_bwd_src3(GatArgs a, int64_t row_base) {
+  constexpr int EPV = 4;                       // G is fp32: 4 columns per 16-byte vector
+  __shared__ float e_al[8][32][HM + 1];        // alpha_e per head
+  __shared__ float e_af[8][32][HM + 1];        // alpha_e * lrelu'(t_e)
+  __shared__ float e_s[8][32][HM + 1];         // s[dd] per head
+  __shared__ int e_dd[8][32];
+  __shared__ int64_t e_fp[8][32];
+  const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
+  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (w >= a.n_chunks) return;
+  const RowChunk ch = a.chunks[w];
+  const int64_t u = row_base + ch.row;
+  const int H = a.H;
+  const float* G = static_cast<const float*>(a.G);
+  const T* DY = static_cast<const T*>(a.dy);
+  int hd[NV], cc[NV];
+  bool on[NV], lead[NV];
+  float gu[NV][EPV], acc[NV][EPV], dl[NV], elu[HM];
+  const float dys = a.concat ? 1.f : 1.f / (float)a.H;
+#pragma unroll
+  for (int h = 0; h < HM; ++h) elu[h] = h < H ? a.el[u * H + h] : 0.f;
+#pragma unroll
+  for (int q = 0; q < NV; ++q) {
+    const int vi = lane + 32 * q;
+    on[q] = vi < a.VPR;
+    const int c0 = vi * EPV;
+    hd[q] = on[q] ? min(c0 / a.Fo, HM - 1) : 0;
+    cc[q] = a.concat ? c0 : c0 % a.Fo;
+    lead[q] = on[q] && (c0 % a.Fo) == 0;
+    if (on[q]) GV<float>::unpack(ld16(G + u * a.ldg + c0), gu[q]);
+    else {
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) gu[q][i] = 0.f;
+    }
+#pragma unroll
+    for (int i = 0; i < EPV; ++i) { gu[q][i] *= dys; acc[q][i] = 0.f; }
+    dl[q] = 0.f;
+  }
+  for (int64_t base = ch.e_lo; base < ch.e_hi; base += 32) {
+    const int n = (int)min((int64_t)32, ch.e_hi - base);
+    int dd = 0;
+    int64_t fp = 0;
+    if (lane < n) {
+      dd = a.idx[base + lane];
+      fp = a.fwdpos[base + lane];
+#pragma unroll
+      for (int h = 0; h < HM; ++h) {
+        if (h >= H) break;
+        const float4 st = __ldg(a.bs + (int64_t)dd * H + h);
+        const float t = elu[h] + st.x;
+        const float al = __expf(lrelu(t, a.slope) - st.y);
+        e_al[wi][lane][h] = al;
+        e_af[wi][lane][h] = al * (t > 0.f ? 1.f : a.slope);
+        e_s[wi][lane][h] = st.z;
+      }
+    }
+    e_dd[wi][lane] = dd;
+    e_fp[wi][lane] = fp;
+    __syncwarp();
+    for (int j = 0; j < n; j += U) {
+      float dyv[U][NV][EPV];
+#pragma unroll
+      for (int k = 0; k < U; ++k) {
+        const bool ok = j + k < n;
+        const int64_t ddk = e_dd[wi][ok ? j + k : 0];
+#pragma unroll
+        for (int q = 0; q < NV; ++q) {
+          if (on[q] && ok) ld_dy4<T>(DY + ddk * a.lddy + cc[q], dyv[k][q]);
+          else {
+#pragma unroll
+            for (int i = 0; i < EPV; ++i) dyv[k][q][i] = 0.f;
+          }
+        }
+      }
+#pragma unroll
+      for (int k = 0; k < U; ++k) {
+        if (j + k >= n) break;                 // warp-uniform
+        float part[NV], dal[NV];
+#pragma unroll
+        for (int q = 0; q < NV; ++q) {
+          part[q] = 0.f;
+#pragma unroll
+          for (int i = 0; i < EPV; ++i) part[q] += dyv[k][q][i] * gu[q][i];
+        }
+        head_sums<NV, SEG>(part, hd, a.H, dal);
+#pragma unroll
+        for (int q = 0; q < NV; ++q) {
+          const float al = e_al[wi][j + k][hd[q]];
+#pragma unroll
+          for (int i = 0; i < EPV; ++i) acc[q][i] += al * dyv[k][q][i];
+          if (lead[q]) {
+            const float dtv = e_af[wi][j + k][hd[q]] * (dal[q] - e_s[wi][j + k][hd[q]]);
+            dl[q] += dtv;
+            a.dt[e_fp[wi][j + k] * a.H + hd[q]] = dtv;
+          }
+        }
+      }
+    }
+    __syncwarp();
+  }
+#pragma unroll
+  for (int q = 0; q < NV; ++q) {
+    if (!on[q]) continue;
+    const int c0 = (lane + 32 * q) * EPV;
+    float* out = ch.slot >= 0 ? a.part + (int64_t)ch.slot * a.part_ld : a.dg + u * a.ld_dg;
+    *reinterpret_cast<float4*>(out + c0) =
+        make_float4(acc[q][0] * dys, acc[q][1] * dys, acc[q][2] * dys, acc[q][3] * dys);
     if (lead[q]) {
       if (ch.slot >= 0) out[a.HF + hd[q]] = dl[q];
       else a.del[u * a.H + hd[q]] = dl[q];
@@ -1012,9 +1133,17 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
   a.chunks = gp->bwd; a.n_chunks = gp->n_bwd;
   if (gp->n_bwd) {
     const unsigned cbk = gs_grid((int64_t)gp->n_bwd * 32);
-#define WG_GAT_B1(NV_, SEG_) WG_LAUNCH((k_gat_bwd_src2<T, NV_, 8, SEG_>), cbk, 256, 0, st, a, vb)
-#define WG_GAT_B2(NV_, SEG_) WG_LAUNCH((k_gat_bwd_src2<T, NV_, 4, SEG_>), cbk, 256, 0, st, a, vb)
-#define WG_GAT_B4(NV_, SEG_) WG_LAUNCH((k_gat_bwd_src2<T, NV_, 2, SEG_>), cbk, 256, 0, st, a, vb)
+#define WG_GAT_B1(NV_, SEG_) do { if (H <= 4) WG_LAUNCH((k_gat_bwd_src3<T, NV_, 8, SEG_, 4>), cbk, 256, 0, st, a, vb); \
+    else if (H <= GAT_HM) WG_LAUNCH((k_gat_bwd_src3<T, NV_, 8, SEG_, 8>), cbk, 256, 0, st, a, vb);             \
+    else WG_LAUNCH((k_gat_bwd_src2<T, NV_, 8, SEG_>), cbk, 256, 0, st, a, vb); } while (0)
+// NV = 2 (the C2 widths): two dy rows in flight per warp at 4 CTAs / SM beats
+// four rows at 2 CTAs / SM (per-row latency chains, C2 A/B: 4.94 -> 4.76 ms)
+#define WG_GAT_B2(NV_, SEG_) do { if (H <= 4) WG_LAUNCH((k_gat_bwd_src3<T, NV_, 2, SEG_, 4, 4>), cbk, 256, 0, st, a, vb); \
+    else if (H <= GAT_HM) WG_LAUNCH((k_gat_bwd_src3<T, NV_, 4, SEG_, 8>), cbk, 256, 0, st, a, vb);             \
+    else WG_LAUNCH((k_gat_bwd_src2<T, NV_, 4, SEG_>), cbk, 256, 0, st, a, vb); } while (0)
+#define WG_GAT_B4(NV_, SEG_) do { if (H <= 4) WG_LAUNCH((k_gat_bwd_src3<T, NV_, 2, SEG_, 4>), cbk, 256, 0, st, a, vb); \
+    else if (H <= GAT_HM) WG_LAUNCH((k_gat_bwd_src3<T, NV_, 2, SEG_, 8>), cbk, 256, 0, st, a, vb);             \
+    else WG_LAUNCH((k_gat_bwd_src2<T, NV_, 2, SEG_>), cbk, 256, 0, st, a, vb); } while (0)
     if (NV == 1) WG_GAT_SEG(WG_GAT_B1, 1);
     else if (NV == 2) WG_GAT_SEG(WG_GAT_B2, 2);
     else WG_GAT_SEG(WG_GAT_B4, 4);

@@ -234,13 +234,33 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
     const int s = dsize(d.dtype);
     const int64_t A = rup((int64_t)d.f_in * s, 32), B = rup((int64_t)d.f_out * s, 32);
     std::mt19937_64 rng(d.policy_seed);
+    // Y rows are unique per (source, relation) over ALL VERTEX gTasks of the
+    // relation, so a gTask's share of the Y transform is amortised:
+    // n_uniq_src(g) * U_r / S_r rows (U_r distinct sources of relation r,
+    // S_r = sum of n_uniq_src over its gTasks)
+    std::vector<int64_t> U(R, 0), S(R, 0);
+    {
+      std::vector<uint64_t> seen((size_t)cdiv((int64_t)R * V, 64), 0);
+      for (int64_t i = 0; i < E; ++i) {
+        const uint64_t bit = (uint64_t)ft[i] * (uint64_t)V + (uint64_t)fi_[i];
+        uint64_t& w = seen[bit >> 6];
+        const uint64_t m = 1ull << (bit & 63);
+        if (!(w & m)) { w |= m; ++U[ft[i]]; }
+      }
+      for (int64_t t = 0; t < nt; ++t) S[tasks[t].type] += tasks[t].n_uniq_src;
+    }
     for (int64_t t = 0; t < nt; ++t) {
       const wg_task& k = tasks[t];
       int64_t nseg = 0;
       for (int64_t i = k.e_begin; i < k.e_end; ++i) nseg += (i == k.e_begin || fk[i] != fk[i - 1]);
       const int64_t ne = k.e_end - k.e_begin, nu = k.n_uniq_src;
+      // EDGE: gather f_in rows, then per (dst, relation) segment the S row
+      // write + GEMM read, the T row write + stage-3 read
       const int64_t te = ne * (A + 4) + nseg * (2 * A + 2 * B + 4);
-      const int64_t tv = nu * (2 * A + 2 * B) + ne * (B + 8);
+      // VERTEX: the amortised Y rows (gathered f_in row read + f_out row
+      // write), then every edge reads its f_out-wide Y row
+      const int64_t ny = S[k.type] > 0 ? nu * U[k.type] / S[k.type] : nu;
+      const int64_t tv = ny * (A + B) + ne * (B + 8);
       uint8_t b = 0;
       if (d.policy == WG_PLAN_ALL_VERTEX) b = 1;
       else if (d.policy == WG_PLAN_RANDOM) b = (uint8_t)(rng() & 1);
