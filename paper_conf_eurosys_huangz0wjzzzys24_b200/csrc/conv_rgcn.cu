@@ -73,8 +73,11 @@ wg_status up(wg_plan_s* p, const std::vector<T>& h, T** d) {
   return WG_OK;
 }
 
-// Work items over a generic CSR: consecutive rows grouped until E_max entries
-// or 128 rows; rows with more than E_max entries become SPLIT chunks.
+// Work items over a generic CSR: consecutive rows grouped until min(E_max,
+// ITEM_EDGES) entries or ITEM_ROWS rows; rows with more than E_max entries
+// become SPLIT chunks.  Stage rows are short (C3: ~1.4 edges per (dst,
+// relation) row), so items span many rows: a CTA must stream thousands of
+// edges to amortise its pipeline fill (128-row items ran at 29% of HBM).
 wg_status build_exec(wg_plan_s* p, const std::vector<int64_t>& rp, const std::vector<int32_t>& idx,
                      const std::vector<float>* es, const std::vector<float>* rs, int64_t E_max, CsrExec* X) {
   X->rows = (int64_t)rp.size() - 1;
@@ -90,6 +93,8 @@ wg_status build_exec(wg_plan_s* p, const std::vector<int64_t>& rp, const std::ve
   std::vector<std::pair<int64_t, WorkItem>> L;
   int slot = 0;
   ItemList& IL = X->items;
+  constexpr int64_t ITEM_ROWS = 4096, ITEM_EDGES = 4096;
+  const int64_t item_edges = std::min(E_max, ITEM_EDGES);
   int64_t lo = 0;
   auto close = [&](int64_t hi) {
     if (hi <= lo) return;
@@ -116,7 +121,7 @@ wg_status build_exec(wg_plan_s* p, const std::vector<int64_t>& rp, const std::ve
       lo = r + 1;
       continue;
     }
-    if (rp[r + 1] - rp[lo] > E_max || r - lo >= 128) {
+    if (rp[r + 1] - rp[lo] > item_edges || r - lo >= ITEM_ROWS) {
       close(r);
       lo = r;
     }
