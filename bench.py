@@ -60,6 +60,8 @@ def parse():
     ap.add_argument("--model", default=None, choices=["sage", "gin", "gcn", "gat", "rgcn"],
                     help="default: the config's model (C4: sage)")
     ap.add_argument("--policy", default="auto")
+    ap.add_argument("--emax", type=int, default=0,
+                    help="gTask edge limit E_max (0: the Q13 rule); SURVEY §8(f) f1 K sweeps")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
@@ -288,7 +290,7 @@ def main():
     R = c.R if model == "rgcn" else 1
     g = wg.Graph(torch.from_numpy(src).to(dev), torch.from_numpy(dst).to(dev), num_vertices=c.V,
                  etype=torch.from_numpy(et).to(dev) if R > 1 else None, num_types=R,
-                 v_begin=vb if world > 1 else 0, v_end=ve if world > 1 else 0)
+                 v_begin=vb if world > 1 else 0, v_end=ve if world > 1 else 0, max_task_edges=args.emax)
     torch.cuda.synchronize()
     t_part = time.perf_counter() - t0
     dtype = torch.bfloat16 if c.dtype == "bf16" else torch.float32

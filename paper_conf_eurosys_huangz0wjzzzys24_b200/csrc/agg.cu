@@ -124,6 +124,34 @@ __device__ __forceinline__ void finish_vec(const AggArgs& a, const float* acc, i
                     a.ld_out, a.F);
 }
 
+// Rows of a regular item without in-edges get the epilogue of a zero sum
+// (bias / self term), and the optional second output is zeroed.  The test is
+// one thread per row (all rows' row_ptr loads in parallel, coalesced): a
+// per-warp row loop put a dependent global load per row on the CTA's tail
+// (4096-row RGCN stage items: ~500 serial loads per warp).
+template <typename T>
+__device__ __forceinline__ void empty_rows(const AggArgs& a, const WorkItem& it, int VPR) {
+  constexpr int EPV = VT<T>::EPV;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int r0 = it.row_lo; r0 < it.row_hi; r0 += WARPS * 32) {
+    const int r = r0 + (int)threadIdx.x;
+    const bool empty = r < it.row_hi && a.row_ptr[r + 1] == a.row_ptr[r];
+    unsigned m = __ballot_sync(0xffffffffu, empty);
+    while (m) {
+      const int rr = r0 + warp * 32 + __ffs(m) - 1;
+      m &= m - 1;
+      const float zero[EPV] = {};
+      for (int vi = lane; vi < VPR; vi += 32) finish_vec<T>(a, zero, rr, vi * EPV, -1);
+    }
+  }
+  if (a.zero_out) {
+    for (int r = it.row_lo + warp; r < it.row_hi; r += WARPS) {
+      T* p = static_cast<T*>(a.zero_out) + (int64_t)r * a.ld_zero;
+      for (int c = lane * EPV; c < a.zero_cols; c += 32 * EPV) *reinterpret_cast<int4*>(p + c) = make_int4(0, 0, 0, 0);
+    }
+  }
+}
+
 // Warp-segmented gather-reduce.  Template: LPE lanes per edge row chunk, NV
 // 16-byte vectors per lane (chunk width CW = LPE*NV vectors), U edges in flight.
 template <typename T, int LPE, int NV, int U>
@@ -270,17 +298,7 @@ __global__ void __launch_bounds__(WARPS * 32, 3) k_agg(AggArgs a, int VPR) {
     __syncthreads();
   }
   if (split) return;
-  // rows without in-edges (and the optional zeroed second output)
-  for (int r = it.row_lo + warp; r < it.row_hi; r += WARPS) {
-    if (a.row_ptr[r + 1] == a.row_ptr[r]) {
-      const float zero[EPV] = {};
-      for (int vi = lane; vi < VPR; vi += 32) finish_vec<T>(a, zero, r, vi * EPV, -1);
-    }
-    if (a.zero_out) {
-      T* p = static_cast<T*>(a.zero_out) + (int64_t)r * a.ld_zero;
-      for (int c = lane * EPV; c < a.zero_cols; c += 32 * EPV) *reinterpret_cast<int4*>(p + c) = make_int4(0, 0, 0, 0);
-    }
-  }
+  empty_rows<T>(a, it, VPR);
 }
 
 // ---------------------------------------------------------------------------
@@ -493,16 +511,7 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) k_agg_cp(AggArgs a, int VPR)
     __syncthreads();
   }
   if (split) return;
-  for (int r = it.row_lo + warp; r < it.row_hi; r += WARPS) {
-    if (a.row_ptr[r + 1] == a.row_ptr[r]) {
-      const float zero[EPV] = {};
-      for (int vi = lane; vi < VPR; vi += 32) finish_vec<T>(a, zero, r, vi * EPV, -1);
-    }
-    if (a.zero_out) {
-      T* p = static_cast<T*>(a.zero_out) + (int64_t)r * a.ld_zero;
-      for (int c = lane * EPV; c < a.zero_cols; c += 32 * EPV) *reinterpret_cast<int4*>(p + c) = make_int4(0, 0, 0, 0);
-    }
-  }
+  empty_rows<T>(a, it, VPR);
 }
 
 template <typename T>

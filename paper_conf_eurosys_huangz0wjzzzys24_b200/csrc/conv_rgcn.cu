@@ -93,8 +93,9 @@ wg_status build_exec(wg_plan_s* p, const std::vector<int64_t>& rp, const std::ve
   std::vector<std::pair<int64_t, WorkItem>> L;
   int slot = 0;
   ItemList& IL = X->items;
+  // at least ~6 items per SM when the CSR is small (a few EDGE-plan gTasks)
   constexpr int64_t ITEM_ROWS = 4096, ITEM_EDGES = 4096;
-  const int64_t item_edges = std::min(E_max, ITEM_EDGES);
+  const int64_t item_edges = std::min(E_max, std::max<int64_t>(512, std::min(ITEM_EDGES, X->nnz / (148 * 6))));
   int64_t lo = 0;
   auto close = [&](int64_t hi) {
     if (hi <= lo) return;

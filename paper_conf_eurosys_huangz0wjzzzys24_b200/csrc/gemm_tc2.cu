@@ -305,13 +305,26 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
     const uint32_t tx = A_STAGE + b_bytes;
     int s = 0;
     uint32_t ph = 0;
+    // the next tile's gather row ids and relation are loaded one tile ahead,
+    // so their latency never stalls the producer between tiles
+    auto tile_meta = [&](int64_t t, int4& gi, int& grp) {
+      gi = make_int4(0, 0, 0, 0);
+      grp = 0;
+      if (t >= p.num_tiles) return;
+      const int64_t mt = t / p.n_tiles;
+      if (p.a_rows[0]) gi = __ldg(reinterpret_cast<const int4*>(p.a_rows[0] + mt * BM) + lane);
+      if (p.tile_group[0]) grp = __ldg(p.tile_group[0] + mt);
+    };
+    int4 gi_next;
+    int grp_next;
+    tile_meta(blockIdx.x, gi_next, grp_next);
     for (int64_t t = blockIdx.x; t < p.num_tiles; t += gridDim.x) {
       const int64_t mt = t / p.n_tiles;
       const int m0 = (int)(mt * BM), n0 = (int)((t % p.n_tiles) * BN);
       int part = 0, kk = 0;
-      int brow = n0 + (p.tile_group[0] ? p.tile_group[0][mt] * p.group_rows[0] : 0);
-      int4 gi = make_int4(0, 0, 0, 0);
-      if (p.a_rows[0]) gi = __ldg(reinterpret_cast<const int4*>(p.a_rows[0] + m0) + lane);
+      int4 gi = gi_next;
+      int brow = n0 + grp_next * p.group_rows[0];
+      tile_meta(t + gridDim.x, gi_next, grp_next);
       for (int kb = 0; kb < total_kb; ++kb) {
         const CUtensorMap* ta = part == 0 ? &tA0 : (part == 1 ? &tA1 : &tA2);
         const CUtensorMap* tb = part == 0 ? &tB0 : (part == 1 ? &tB1 : &tB2);
