@@ -146,7 +146,10 @@ wg_status wg_plan_export(wg_plan p, uint8_t* per_task_plan, int64_t stats[8]);
 /* Introspection (tests / tools): byte offset of a named sub-buffer of the
  * saved (which = 0) or workspace (which = 1) buffer, e.g. "agg" (the saved
  * aggregation, [owned rows x pitch(f_in)]) or "h" (GIN hidden activation,
- * [owned rows x pitch(f_out)]).  WG_ERR_INVALID if the plan has no such
+ * [owned rows x pitch(f_out)]) or "xg" (RGCN on one partition with every
+ * gTask VERTEX: x[src] of each (source, relation) row, grouped by relation,
+ * gathered once by the forward for the Y GEMM and reused by the dW_r GEMM,
+ * SURVEY §8(a) a5 / a11).  WG_ERR_INVALID if the plan has no such
  * buffer.  Pitches are 32-byte padded rows in the conv dtype.              */
 wg_status wg_plan_buffer(wg_plan p, int which, const char* name, size_t* offset);
 wg_status wg_plan_destroy(wg_plan p);

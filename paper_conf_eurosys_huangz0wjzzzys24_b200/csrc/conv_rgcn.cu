@@ -59,6 +59,10 @@ struct RgcnPlan {
   CsrExec bg;                        // transposed rows -> their source vertex (X_g gather copy)
   std::vector<int64_t> h_group_offT; // [R+1] transposed group row offsets
   TnUnits tn;                        // dW_r work units over the transposed groups
+  // Y rows == transposed G rows (every gTask VERTEX, one partition): the
+  // forward gathers X_g = x[src] once (saved), the Y GEMM streams it
+  // contiguously, and the backward's dW_r GEMM reuses it
+  bool share_xg = false;
 };
 
 template <typename T>
@@ -288,8 +292,16 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
   struct Contrib { int32_t dst; int32_t type; int64_t row; float c; bool vert; };
   std::vector<Contrib> contrib;
   contrib.reserve(E);
+  // On one partition with >= 90% of the edges in VERTEX gTasks, the Y rows
+  // cover every (source, relation) pair of the graph: the few extra rows
+  // (sources reached only through EDGE gTasks) make the Y block identical to
+  // the transposed G rows, so X_g is shared with the backward (share_xg)
+  int64_t e_vert = 0;
   for (int64_t t = 0; t < nt; ++t)
-    if (p->plan_bits[t] == 1)
+    if (p->plan_bits[t] == 1) e_vert += tasks[t].e_end - tasks[t].e_begin;
+  const bool y_all = nr == g->V && e_vert > 0 && e_vert * 10 >= E * 9;
+  for (int64_t t = 0; t < nt; ++t)
+    if (p->plan_bits[t] == 1 || y_all)
       for (int64_t i = tasks[t].e_begin; i < tasks[t].e_end; ++i) uniq[tasks[t].type].push_back(fi_[i]);
   for (int r = 0; r < R; ++r) {
     std::sort(uniq[r].begin(), uniq[r].end());
@@ -438,6 +450,8 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
       rp->tn.units = du; rp->tn.unit_off = duo;
       rp->tn.n_units = (int)units.size(); rp->tn.groups = R; rp->tn.align = TILE_M; rp->tn.k_total = baseT[R];
     }
+    rp->share_xg = nr == g->V && rp->n1v == rp->n1T;
+    for (int r = 0; r < R && rp->share_xg; ++r) rp->share_xg = uniq[r] == seg_src[r];
     std::stable_sort(sc.begin(), sc.end(), [](const SC& a, const SC& b) {
       return a.src != b.src ? a.src < b.src : a.row < b.row;
     });
@@ -456,6 +470,7 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
   S = Layout();
   W = Layout();
   S.add("none", 1);
+  if (rp->share_xg) S.add("xg", (size_t)rp->n1T * p->pi * s);
   W.add("wt", (size_t)R * rows_o * p->pi * s);          // stacked W_r^T
   W.add("w", (size_t)R * rows_i * p->po * s);           // stacked W_r
   W.add("w0t", (size_t)rows_o * p->pi * s);
@@ -513,7 +528,21 @@ wg_status rgcn_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, c
   // stage 2: grouped GEMMs  T1[Y block, group r] = x[ysrc] W_r (A rows gathered
   // from x) and T1[EDGE block, group r] = S W_r
   void* t1 = L.at<void>(ws, "t1");
-  if (rp->n1v) {
+  if (rp->n1v && rp->share_xg) {
+    WG_REQ(A->saved, WG_ERR_INVALID, "RGCN forward: saved is NULL");
+    void* xg = p->saved.at<void>(A->saved, "xg");
+    AggArgs a = exec_args(rp->bg, g->E_max);
+    a.table = A->x; a.ld_tab = A->ldx;
+    a.out = xg; a.ld_out = p->pi;
+    a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
+    a.F = d.f_in;
+    WG_TRY(run(dt, a, rp->bg, st));
+    GemmPart part{xg, p->pi, wt, p->pi, d.f_in, d.f_out};
+    part.tile_group = rp->tile_type_v; part.group_rows = (int)rows_o; part.groups = R;
+    GemmEpi e;
+    e.D = t1; e.ldd = p->po;
+    WG_TRY(gemm_nt(dt, rp->n1v, (int)rup(d.f_out, 16 / s), &part, 1, e, nullptr, 0, st));
+  } else if (rp->n1v) {
     GemmPart part{A->x, A->ldx, wt, p->pi, d.f_in, d.f_out};
     part.tile_group = rp->tile_type_v; part.group_rows = (int)rows_o; part.groups = R;
     part.a_rows = rp->ysrc; part.a_table_rows = V;
@@ -613,13 +642,19 @@ wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, 
   }
   // dW_r = X_g[group r]^T G[group r]   (this rank's out-edges; the caller all-reduces)
   if (G && G->W) {
-    void* xg = L.at<void>(ws, "xg");
-    AggArgs a = exec_args(rp->bg, g->E_max);
-    a.table = A->x; a.ld_tab = A->ldx;
-    a.out = xg; a.ld_out = p->pi;
-    a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
-    a.F = d.f_in;
-    WG_TRY(run(dt, a, rp->bg, st));
+    void* xg = nullptr;
+    if (rp->share_xg) {   // gathered by the forward
+      WG_REQ(A->saved, WG_ERR_INVALID, "RGCN backward: saved is NULL");
+      xg = p->saved.at<void>(A->saved, "xg");
+    } else {
+      xg = L.at<void>(ws, "xg");
+      AggArgs a = exec_args(rp->bg, g->E_max);
+      a.table = A->x; a.ld_tab = A->ldx;
+      a.out = xg; a.ld_out = p->pi;
+      a.partial = L.at<float>(ws, "part"); a.ld_part = pl;
+      a.F = d.f_in;
+      WG_TRY(run(dt, a, rp->bg, st));
+    }
     WG_TRY(gemm_tn_grouped(dt, rp->tn, d.f_in, d.f_out, xg, p->pi, gt, p->po, G->W, L.at<void>(ws, "tn"), st));
   }
   if (!d.need_dx) return WG_OK;

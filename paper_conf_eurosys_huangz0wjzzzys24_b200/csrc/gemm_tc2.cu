@@ -76,6 +76,8 @@ struct P2 {
   const float* rscale;
   const float* bias;
   int relu, has_add, has_mask, bias_vec;
+  int cpg;          // fp32 row-gathered A by per-lane cp.async (see the producer)
+  const void* a_tab; int64_t lda_tab; int k_a;   // cpg: table, its row pitch (elements), K
 };
 
 __device__ __forceinline__ uint32_t su32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
@@ -226,16 +228,17 @@ template <> __device__ __forceinline__ int4 pack16<float>(const float* f) {
 
 // shared-memory plan (bytes from the 1024-aligned base), identical on host and device
 struct SmemPlan {
-  int stage, ring, stg, add, mask, bars, total;
+  int stage, ring, stg, add, mask, ids, bars, total;
 };
-__host__ __device__ inline SmemPlan smem_plan(bool tf32, int BN, int S, bool has_add, bool has_mask) {
+__host__ __device__ inline SmemPlan smem_plan(bool tf32, int BN, int S, bool has_add, bool has_mask, bool cpg) {
   SmemPlan q;
   q.stage = (A_STAGE + BN * 128) * (tf32 ? 2 : 1);   // [A | B] (+ [A_lo | B_lo])
   q.ring = S * q.stage;
   q.stg = q.ring;
   q.add = q.stg + 2 * CHUNK_BYTES;
   q.mask = q.add + (has_add ? 2 * CHUNK_BYTES : 0);
-  q.bars = q.mask + (has_mask ? 2 * CHUNK_BYTES : 0);
+  q.ids = q.mask + (has_mask ? 2 * CHUNK_BYTES : 0);
+  q.bars = q.ids + (cpg ? BM * 4 : 0);               // cpg: the tile's 128 gather row ids
   q.total = q.bars + 256;
   return q;
 }
@@ -256,7 +259,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int BN = p.BN, S = p.stages;
   const int b_bytes = BN * 128;
-  const SmemPlan L = smem_plan(C::TF32, BN, S, p.has_add, p.has_mask);
+  const SmemPlan L = smem_plan(C::TF32, BN, S, p.has_add, p.has_mask, p.cpg != 0);
   // stage s: A at s*stage, B at +A_STAGE; fp32: A_lo at +A_STAGE+b_bytes, B_lo after it
   uint8_t* ring = smem;
   uint8_t* st_sm = smem + L.stg;                   // 2 x 16 KB output staging
@@ -276,7 +279,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
-      mbar_init(su32(&full[s]), 1);
+      mbar_init(su32(&full[s]), p.cpg ? 33 : 1);   // cpg: + one cp.async arrive per producer lane
       mbar_init(su32(&empty[s]), 1);
       mbar_init(su32(&conv[s]), 128);
     }
@@ -318,12 +321,24 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
     int4 gi_next;
     int grp_next;
     tile_meta(blockIdx.x, gi_next, grp_next);
+    // cpg: lane l copies 16-byte unit (l & 7) of rows 4j + (l >> 3), j < 32:
+    // each instruction moves four whole 128-byte row pieces (coalesced); the
+    // lane's cp.async completions arrive on full[s] (noinc; count 33)
+    int* ids = reinterpret_cast<int*>(smem + L.ids);
+    const int cu = lane & 7, csub = lane >> 3;
     for (int64_t t = blockIdx.x; t < p.num_tiles; t += gridDim.x) {
       const int64_t mt = t / p.n_tiles;
       const int m0 = (int)(mt * BM), n0 = (int)((t % p.n_tiles) * BN);
       int part = 0, kk = 0;
       int4 gi = gi_next;
       int brow = n0 + grp_next * p.group_rows[0];
+      if constexpr (C::TF32) {
+        if (p.cpg) {
+          __syncwarp();                       // previous tile's ids fully consumed
+          ids[4 * lane + 0] = gi.x; ids[4 * lane + 1] = gi.y; ids[4 * lane + 2] = gi.z; ids[4 * lane + 3] = gi.w;
+          __syncwarp();
+        }
+      }
       tile_meta(t + gridDim.x, gi_next, grp_next);
       for (int kb = 0; kb < total_kb; ++kb) {
         const CUtensorMap* ta = part == 0 ? &tA0 : (part == 1 ? &tA1 : &tA2);
@@ -331,10 +346,23 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
         uint8_t* st = ring + s * L.stage;
         if (lane == 0) {
           mbar_wait(su32(&empty[s]), ph ^ 1);
-          mbar_expect_tx(su32(&full[s]), tx);
+          mbar_expect_tx(su32(&full[s]), p.cpg ? (uint32_t)b_bytes : tx);
         }
         __syncwarp();
-        if (p.a_rows[part]) {
+        if (C::TF32 && p.cpg) {
+          const float* tab = static_cast<const float*>(p.a_tab);
+          const int col = kk * C::BKE + cu * 4;
+          const bool ok = col < p.k_a;
+          const uint32_t sb = su32(st);
+#pragma unroll 8
+          for (int j = 0; j < 32; ++j) {
+            const int r = 4 * j + csub;
+            const float* src = tab + (int64_t)ids[r] * p.lda_tab + (ok ? col : 0);
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(sb + sw_off(r, cu)), "l"(src),
+                         "r"(ok ? 16 : 0) : "memory");
+          }
+          asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(su32(&full[s])) : "memory");
+        } else if (p.a_rows[part]) {
           tma_gather4(su32(st) + lane * 512, ta, kk * C::BKE, gi.x, gi.y, gi.z, gi.w, su32(&full[s]));
         } else if (lane == 0) {
           tma_load(su32(st), ta, kk * C::BKE, m0, su32(&full[s]));
@@ -607,14 +635,27 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
       return false;
     p.has_mask = 1;
   }
+  // fp32 row-gathered A: per-lane cp.async instead of TMA gather4 (32 gather4
+  // per stage capped the producer at ~2 TB/s on C3); WG_GATHER_TMA=1 keeps TMA
+  static int gather_tma = -1;
+  if (gather_tma < 0) {
+    const char* e = getenv("WG_GATHER_TMA");
+    gather_tma = (e && e[0] == '1') ? 1 : 0;
+  }
+  if (f32 && n_parts == 1 && parts[0].a_rows && parts[0].K % 4 == 0 && (parts[0].lda % 4) == 0 && !gather_tma) {
+    p.cpg = 1;
+    p.a_tab = parts[0].A;
+    p.lda_tab = parts[0].lda;
+    p.k_a = parts[0].K;
+  }
   p.rscale = epi.rscale;
   p.bias = epi.bias;
   p.bias_vec = (reinterpret_cast<uintptr_t>(epi.bias) & 15) == 0;
   p.relu = epi.relu;
   const int limit = 227 * 1024 - 1024;
   int stages = 4;
-  while (stages > 2 && smem_plan(f32, BN, stages, p.has_add, p.has_mask).total > limit) --stages;
-  if (smem_plan(f32, BN, stages, p.has_add, p.has_mask).total > limit) return false;
+  while (stages > 2 && smem_plan(f32, BN, stages, p.has_add, p.has_mask, p.cpg).total > limit) --stages;
+  if (smem_plan(f32, BN, stages, p.has_add, p.has_mask, p.cpg).total > limit) return false;
   p.stages = stages;
   if (!g_sms) {
     int dev = 0;
@@ -622,7 +663,7 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
     cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
   }
   const unsigned grid = (unsigned)std::min<int64_t>(p.num_tiles, g_sms);
-  const size_t smem = 1024 + (size_t)smem_plan(f32, BN, stages, p.has_add, p.has_mask).total;
+  const size_t smem = 1024 + (size_t)smem_plan(f32, BN, stages, p.has_add, p.has_mask, p.cpg).total;
   double kt = 0;
   for (int i = 0; i < n_parts; ++i) kt += parts[i].K;
   ProfScope ps(PK_TC_NT, s, (double)M * (kt + N + (epi.addend ? N : 0) + (epi.mask_ref ? N : 0)) * es,
