@@ -438,7 +438,8 @@ def main():
                            epoch_time_ms=ms, l2="inputs larger than L2 (no flush needed)",
                            max_in_degree=int(g.max_in_degree), E_max=int(g.E_max),
                            plans=[{"edge_tasks": cv.n_edge_tasks, "vertex_tasks": cv.n_vertex_tasks,
-                                   "bwd_path": cv.bwd_path} for cv in stack.convs]),
+                                   "bwd_path": cv.bwd_path, "items": cv.n_items, "items_T": cv.n_items_T,
+                                   "split_rows": cv.n_split_rows} for cv in stack.convs]),
             "gpu_launches": int(launches), "roofline": roofline, "kernels": kernels,
             "one_off": {"partition_s": t_part, "plan_s": t_plan, "synth_s": t_gen},
             "clocks": clk, "loss": float(loss.item()), "e2e": e2e}

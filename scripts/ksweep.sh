@@ -1,0 +1,14 @@
+#!/bin/bash
+# measured sweep of the gTask edge limit E_max (the paper's
+# K sweeps, Fig 18) -- bench lines per (config, model, E_max)
+mkdir -p gpurun_out/ksweep
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { tail -30 gpurun_out/build.log; exit 1; }
+for cm in ${CMS:-"C4 sage" "C3 rgcn"}; do
+  set -- $cm
+  for k in ${KS:-1024 4096 16384 65536}; do
+    timeout 600 python bench.py --config $1 --model $2 --steps 5 --warmup 3 --no-cpu --no-e2e --emax $k \
+      > gpurun_out/ksweep/$1_$2_$k.json 2> gpurun_out/ksweep/$1_$2_$k.err
+    echo "$1 $2 E_max=$k exit $?"
+  done
+done
+python scripts/ksweep_table.py gpurun_out/ksweep/*.json

@@ -137,3 +137,22 @@ def test_rgcn_1d_partition_phases_match_oracle(policy, P):
     errs = {"y": rel_err(f64(yt[:V]), yo), "dx": rel_err(f64(dxt[:V]), dxo), "dW": rel_err(f64(tot["W"]), dWo),
             "dW0": rel_err(f64(tot["W_self"]), dW0o), "db": rel_err(f64(tot["bias"]), dbo)}
     assert all(v <= 1e-4 for v in errs.values()), str(errs)
+
+
+def test_rgcn_gather_cpasync_subprocess():
+    """The opt-in cp.async row gather of the fp32 grouped GEMM (WG_GATHER_CPASYNC=1,
+    read once per process) on a mixed plan, where the Y GEMM gathers its A rows."""
+    import os
+    import subprocess
+    import sys
+    code = ("from tests.test_gpu_conv_rgcn import run, TOL\n"
+            "import torch\n"
+            "e, _ = run(policy='random', norm='right', self_loop=True)\n"
+            "assert max(e.values()) <= TOL[torch.float32], e\n"
+            "e, _ = run(policy='random', ints=True, fi=32)\n"
+            "assert max(e.values()) == 0.0, e\n"
+            "print('ok')\n")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], cwd=root, capture_output=True, text=True, timeout=600,
+                       env=dict(os.environ, WG_GATHER_CPASYNC="1"))
+    assert r.returncode == 0 and "ok" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
