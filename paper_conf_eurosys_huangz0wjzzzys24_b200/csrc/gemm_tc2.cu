@@ -635,14 +635,16 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
       return false;
     p.has_mask = 1;
   }
-  // fp32 row-gathered A: per-lane cp.async instead of TMA gather4 (32 gather4
-  // per stage capped the producer at ~2 TB/s on C3); WG_GATHER_TMA=1 keeps TMA
-  static int gather_tma = -1;
-  if (gather_tma < 0) {
-    const char* e = getenv("WG_GATHER_TMA");
-    gather_tma = (e && e[0] == '1') ? 1 : 0;
+  // fp32 row-gathered A by per-lane cp.async instead of TMA gather4: opt-in
+  // (WG_GATHER_CPASYNC=1) -- on C3 (128-byte row pieces, 4-stage ring) it
+  // measured 6.45 ms vs 6.0 ms for gather4: both are bound by the ring's
+  // bytes in flight, not by TMA issue
+  static int gather_cp = -1;
+  if (gather_cp < 0) {
+    const char* e = getenv("WG_GATHER_CPASYNC");
+    gather_cp = (e && e[0] == '1') ? 1 : 0;
   }
-  if (f32 && n_parts == 1 && parts[0].a_rows && parts[0].K % 4 == 0 && (parts[0].lda % 4) == 0 && !gather_tma) {
+  if (f32 && n_parts == 1 && parts[0].a_rows && parts[0].K % 4 == 0 && (parts[0].lda % 4) == 0 && gather_cp) {
     p.cpg = 1;
     p.a_tab = parts[0].A;
     p.lda_tab = parts[0].lda;
