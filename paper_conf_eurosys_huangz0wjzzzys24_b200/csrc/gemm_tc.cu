@@ -151,8 +151,25 @@ __device__ __forceinline__ void mbar_arrive1(uint32_t bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
 
-// 3xTF32 stage split in shared memory: n16 16-byte units at `base` become hi
-// (in place) and lo (at base + n16 * 16); threads ct = 0..nct-1, explicit
+// 3xTF32 split of one operand region: the lo parts of n16 16-byte units at
+// `base` go to `lo` (x itself is the hi operand, see tf32_split_stage)
+__device__ __forceinline__ void tf32_split_range(uint32_t base, uint32_t lo, int n16, int ct, int nct) {
+  for (int i = ct; i < n16; i += nct) {
+    uint32_t v[4], l[4];
+    asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3])
+                 : "r"(base + (uint32_t)i * 16u));
+#pragma unroll
+    for (int k = 0; k < 4; ++k) l[k] = __float_as_uint(__uint_as_float(v[k]) - __uint_as_float(v[k] & 0xffffe000u));
+    asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(lo + (uint32_t)i * 16u), "r"(l[0]), "r"(l[1]), "r"(l[2]),
+                 "r"(l[3]) : "memory");
+  }
+}
+
+// 3xTF32 stage split in shared memory: the lo parts of n16 16-byte units at
+// `base` go to base + n16 * 16.  hi needs no rewrite: kind::tf32 reads only
+// the top 19 bits of each fp32 operand (truncation -- scripts/tf32_probe.py:
+// identical 1e-6 layer errors with and without the masked hi stored), so x
+// itself is the hi operand; threads ct = 0..nct-1, explicit
 // shared-space vector loads / stores, 4 units in flight per thread
 __device__ __forceinline__ void tf32_split_stage(uint32_t base, int n16, int ct, int nct) {
   const uint32_t lo = base + (uint32_t)n16 * 16u;
@@ -173,8 +190,6 @@ __device__ __forceinline__ void tf32_split_stage(uint32_t base, int n16, int ct,
         l[k] = __float_as_uint(__uint_as_float(v[u][k]) - __uint_as_float(h[k]));
       }
       const uint32_t off = (uint32_t)(i + u * nct) * 16u;
-      asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(base + off), "r"(h[0]), "r"(h[1]), "r"(h[2]), "r"(h[3])
-                   : "memory");
       asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(lo + off), "r"(l[0]), "r"(l[1]), "r"(l[2]), "r"(l[3])
                    : "memory");
     }
@@ -188,8 +203,6 @@ __device__ __forceinline__ void tf32_split_stage(uint32_t base, int n16, int ct,
       h[k] = v[k] & 0xffffe000u;
       l[k] = __float_as_uint(__uint_as_float(v[k]) - __uint_as_float(h[k]));
     }
-    asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(base + (uint32_t)i * 16u), "r"(h[0]), "r"(h[1]), "r"(h[2]),
-                 "r"(h[3]) : "memory");
     asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(lo + (uint32_t)i * 16u), "r"(l[0]), "r"(l[1]), "r"(l[2]),
                  "r"(l[3]) : "memory");
   }
@@ -256,7 +269,11 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
 
   if (threadIdx.x == 0) {
     // ---------------- TMA producer
-    const uint32_t tx = A_STAGE + b_stage;
+    // TN: only the A chunks holding real M columns are loaded (M = f_in may
+    // be 64: rows >= M of the M=128 MMA read stale shared memory and only
+    // feed accumulator rows the epilogue never stores)
+    const int a_chunks = MN ? (int)min((int64_t)(BM / CHE), (p.M - m0 + CHE - 1) / CHE) : 0;
+    const uint32_t tx = MN ? (uint32_t)(a_chunks * BKE * 128 + b_stage) : (uint32_t)(A_STAGE + b_stage);
     int part = 0, kk = 0;
     for (int kb = 0; kb < total_kb; ++kb) {
       const int s = kb % S;
@@ -268,7 +285,7 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
       if (MN) {
         const int krow = (int)(kz + (int64_t)kb * BKE);
 #pragma unroll
-        for (int j = 0; j < BM / CHE; ++j) tma_load_2d(ad + j * BKE * 128, &tA0, (int)m0 + CHE * j, krow, fb);
+        for (int j = 0; j < a_chunks; ++j) tma_load_2d(ad + j * BKE * 128, &tA0, (int)m0 + CHE * j, krow, fb);
         for (int j = 0; j * CHE < BN; ++j) tma_load_2d(bd + j * BKE * 128, &tB0, n0 + CHE * j, krow, fb);
       } else {
         const CUtensorMap* ta = part == 0 ? &tA0 : (part == 1 ? &tA1 : &tA2);
@@ -317,10 +334,17 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
     // ---------------- hi / lo converters
     const int ct = threadIdx.x - 128;
     const int n16 = (A_STAGE + b_stage) / 16;
+    const int a16 = MN ? (int)min((int64_t)(BM / CHE), (p.M - m0 + CHE - 1) / CHE) * BKE * 8 : 0;
     for (int kb = 0; kb < total_kb; ++kb) {
       const int s = kb % S;
       mbar_wait(smem_u32(&full[s]), (kb / S) & 1);
-      tf32_split_stage(smem_u32(ring + s * stage), n16, ct, 128);
+      if (MN) {   // [A | B | A_lo | B_lo]: split the loaded A chunks and B
+        const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE, al = bd + b_stage, bl = al + A_STAGE;
+        tf32_split_range(ad, al, a16, ct, 128);
+        tf32_split_range(bd, bl, b_stage / 16, ct, 128);
+      } else {
+        tf32_split_stage(smem_u32(ring + s * stage), n16, ct, 128);
+      }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       mbar_arrive1(smem_u32(&conv[s]));
     }
@@ -589,6 +613,7 @@ bool tc_gemm_tn_grouped(wg_dtype dt, const TnUnits& U, int M, int N, const void*
   if (!tn_setup(dt, U.k_total, M, N, A, lda, B, ldb, &t)) return false;
   TcParams p{};
   p.M = M; p.N = N; p.BN = t.BN; p.nparts = 1; p.K = U.k_total; p.part = part; p.stages = t.stages;
+ 
   p.units = U.units;
   dim3 grid((unsigned)t.m_tiles, (unsigned)t.n_tiles, (unsigned)U.n_units);
   ProfScope ps(PK_TC_TN, s, (double)U.k_total * (M + N) * t.es + (double)U.n_units * M * N * 4.0,

@@ -6,8 +6,9 @@
 // hi = x with its 13 low mantissa bits cleared and lo = x - hi (exact), and
 // D += A_hi B_hi + A_hi B_lo + A_lo B_hi (the dropped lo*lo term is ~2^-22
 // relative), so fp32 layers keep fp32-level accuracy on tensor cores.  The
-// split runs in shared memory: four converter warps rewrite each landed stage
-// (hi in place, lo into a twin buffer) before the MMA warp consumes it.
+// split runs in shared memory: four converter warps write the lo part of each
+// landed stage into a twin buffer before the MMA warp consumes it; the landed
+// x is the hi operand as is (kind::tf32 truncates to the top 19 bits).
 //
 // Grouped B (RGCN relation weights, GemmPart::tile_group): the B rows of
 // 128-row tile t start at tile_group[t] * group_rows.
@@ -142,8 +143,11 @@ __device__ __forceinline__ void mma_tf32(uint32_t tmem, uint64_t a, uint64_t b, 
       "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\ntcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem),
       "l"(a), "l"(b), "r"(idesc), "r"(acc));
 }
-// 3xTF32 stage split in shared memory: n16 16-byte units at `base` become hi
-// (in place) and lo (at base + n16 * 16); threads ct = 0..nct-1, explicit
+// 3xTF32 stage split in shared memory: the lo parts of n16 16-byte units at
+// `base` go to base + n16 * 16.  hi needs no rewrite: kind::tf32 reads only
+// the top 19 bits of each fp32 operand (truncation -- scripts/tf32_probe.py:
+// identical 1e-6 layer errors with and without the masked hi stored), so x
+// itself is the hi operand; threads ct = 0..nct-1, explicit
 // shared-space vector loads / stores, 4 units in flight per thread
 __device__ __forceinline__ void tf32_split_stage(uint32_t base, int n16, int ct, int nct) {
   const uint32_t lo = base + (uint32_t)n16 * 16u;
@@ -164,8 +168,6 @@ __device__ __forceinline__ void tf32_split_stage(uint32_t base, int n16, int ct,
         l[k] = __float_as_uint(__uint_as_float(v[u][k]) - __uint_as_float(h[k]));
       }
       const uint32_t off = (uint32_t)(i + u * nct) * 16u;
-      asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(base + off), "r"(h[0]), "r"(h[1]), "r"(h[2]), "r"(h[3])
-                   : "memory");
       asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(lo + off), "r"(l[0]), "r"(l[1]), "r"(l[2]), "r"(l[3])
                    : "memory");
     }
@@ -179,8 +181,6 @@ __device__ __forceinline__ void tf32_split_stage(uint32_t base, int n16, int ct,
       h[k] = v[k] & 0xffffe000u;
       l[k] = __float_as_uint(__uint_as_float(v[k]) - __uint_as_float(h[k]));
     }
-    asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(base + (uint32_t)i * 16u), "r"(h[0]), "r"(h[1]), "r"(h[2]),
-                 "r"(h[3]) : "memory");
     asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(lo + (uint32_t)i * 16u), "r"(l[0]), "r"(l[1]), "r"(l[2]),
                  "r"(l[3]) : "memory");
   }
