@@ -79,7 +79,10 @@ class GNNStack:
         for p in self.params:
             for v in p.values():
                 v.requires_grad_(True)
-        self.opt = torch.optim.Adam([v for p in self.params for v in p.values()], lr=lr)
+        # capturable: the step count lives on the device, so a whole training
+        # step (library launches + Adam) can be captured in one CUDA graph
+        self.opt = torch.optim.Adam([v for p in self.params for v in p.values()], lr=lr,
+                                    capturable=self.dev.type == "cuda")
 
     # -------------------------------------------------------------- helpers
     def _fwd_xchg(self, c):
