@@ -588,7 +588,12 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
   // several N tiles: BN = 256 (bf16) / 128 (fp32, the lo twins double the
   // stage) so every store box stays inside its tile (the ragged end is
   // clipped by the tensor map); one tile: BN = N
-  const int bn_max = f32 ? 128 : 256;
+  static int bn_env = -1;
+  if (bn_env < 0) {
+    const char* e = getenv("WG_NT_BNMAX");
+    bn_env = e ? atoi(e) : 0;
+  }
+  const int bn_max = (bn_env >= 64 && bn_env <= 256 && bn_env % 64 == 0) ? bn_env : (f32 ? 128 : 256);
   const int n_tiles = (int)cdiv(N, bn_max);
   const int BN = n_tiles > 1 ? bn_max : (int)rup(N, 16);
   if (epi.D2 && (epi.n_split % BN != 0)) return false;   // split must fall on a tile boundary
