@@ -436,8 +436,8 @@ def main():
                "h2d_bytes_per_step": int(xh.numel() * xh.element_size() + lh.numel() * 8),
                "d2h_bytes_per_step": 4, "loss": float(loss_h.item()),
                "input_pipeline": "double-buffered: step i+1's H2D copy overlaps step i on a second stream",
-               "launch_mode": "eager (graph replays of this leg measured slower: 1.16 vs 0.51 ms on C1, "
-                              "the pinned-memory loss read-back inside the graph serialises with the copies)"}
+               "launch_mode": "eager (graph replays of this leg, each with its loss read-back captured, "
+                              "measured slower: 1.16 vs 0.51 ms on C1)"}
 
     clk = clocks.stop()
     pk, pk_src = peaks()
