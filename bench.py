@@ -64,6 +64,10 @@ def parse():
                     help="gTask edge limit E_max (0: the Q13 rule); SURVEY §8(f) f1 K sweeps")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--rank-slice", type=int, default=0, metavar="P",
+                    help="one GPU runs rank --slice-rank of a P-way 1-D partition (its in- / out-edges only, "
+                         "collectives skipped): per-rank compute of a configuration too large for one GPU (C5)")
+    ap.add_argument("--slice-rank", type=int, default=0)
     ap.add_argument("--no-graph", action="store_true",
                     help="time eager steps instead of replaying one CUDA-graph-captured step")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
@@ -279,31 +283,61 @@ def main():
     from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack, partition_1d
 
     c, model, cfg = workload(args.config, args.model)
-    t0 = time.perf_counter()
-    src, dst, et, x_np, labels_np = make_inputs(c, model)
-    t_gen = time.perf_counter() - t0
     dev = torch.device("cuda", local)
+    P = args.rank_slice
+    if P > 1 and (world > 1 or model in ("gat", "rgcn") or c.symmetric):
+        raise SystemExit("--rank-slice: one process, directed untyped GCN / SAGE / GIN configs")
+    t0 = time.perf_counter()
+    if P > 1:
+        import synth
+        block, bounds = partition_1d(c.V, P)
+        vb, ve = bounds[args.slice_rank]
+        src, dst = synth.make_graph_slice(c.V, c.E, vb, ve, seed=c.seed * 16, alpha=c.alpha)
+        et, x_np = None, None
+        labels_np = np.random.Generator(np.random.Philox(c.seed * 16 + 5)).integers(
+            0, c.dims[-1], c.V).astype(np.int64)[vb:ve]
+        args.no_e2e, args.no_cpu = True, True
+        cfg.update(rank_slice={"P": P, "rank": args.slice_rank, "v_begin": vb, "v_end": ve,
+                               "edges_touching_block": int(src.shape[0]),
+                               "note": "per-rank compute of the P-way 1-D partition on one GPU: the rank's "
+                                       "in-edges (forward) and out-edges (backward), PRE / POST phases and "
+                                       "exchange tables; all-gathers / gradient all-reduce not executed, so "
+                                       "exchanged rows and non-owned degrees are not the global ones (timing run)",
+                               "features": "torch.randn on the device (the 111M x 128 table is not built on the host)"})
+    else:
+        src, dst, et, x_np, labels_np = make_inputs(c, model)
+    t_gen = time.perf_counter() - t0
     if world > 1 and model == "gat":
         raise SystemExit("the 1-D multi-GPU partition covers GCN / SAGE / GIN / RGCN (DESIGN.md §9)")
-    block, bounds = partition_1d(c.V, world)
-    vb, ve = bounds[rank] if world > 1 else (0, c.V)
+    if P <= 1:
+        block, bounds = partition_1d(c.V, world)
+        vb, ve = bounds[rank] if world > 1 else (0, c.V)
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     R = c.R if model == "rgcn" else 1
     g = wg.Graph(torch.from_numpy(src).to(dev), torch.from_numpy(dst).to(dev), num_vertices=c.V,
                  etype=torch.from_numpy(et).to(dev) if R > 1 else None, num_types=R,
-                 v_begin=vb if world > 1 else 0, v_end=ve if world > 1 else 0, max_task_edges=args.emax)
+                 v_begin=vb if (world > 1 or P > 1) else 0, v_end=ve if (world > 1 or P > 1) else 0,
+                 max_task_edges=args.emax)
+    if P > 1:
+        src = dst = None   # host copies of the slice are not needed any more
     torch.cuda.synchronize()
     t_part = time.perf_counter() - t0
     dtype = torch.bfloat16 if c.dtype == "bf16" else torch.float32
     t0 = time.perf_counter()
     stack = GNNStack(g, model, c.dims, dtype=dtype, policy=args.policy, group=group,
-                     block=block if world > 1 else None, heads=c.heads if model == "gat" else 1, R=R,
-                     conv_kw=conv_options(c, model))
+                     block=block if (world > 1 or P > 1) else None, heads=c.heads if model == "gat" else 1, R=R,
+                     conv_kw=conv_options(c, model), sim_world=max(P, 1))
     t_plan = time.perf_counter() - t0
     Vtab = stack.Vtab
     x = wg.padded(Vtab, c.dims[0], dtype, dev)
-    x[:c.V].copy_(torch.from_numpy(x_np).to(dev))
+    if x_np is not None:
+        x[:c.V].copy_(torch.from_numpy(x_np).to(dev))
+    else:
+        gen = torch.Generator(device=dev).manual_seed(c.seed * 16 + 2)
+        for r0 in range(0, c.V, 1 << 22):
+            r1 = min(c.V, r0 + (1 << 22))
+            x[r0:r1].copy_(torch.randn((r1 - r0, c.dims[0]), generator=gen, device=dev))
     labels = torch.from_numpy(labels_np[vb:ve] if world > 1 else labels_np).to(dev)
     stream = torch.cuda.current_stream()
 
@@ -378,7 +412,9 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
     L = len(c.dims) - 1
-    value = L * c.E / (ms / 1e3)
+    # rank slice: the edges this GPU aggregates per layer pass (its in-edges)
+    E_units = g.E_fwd if P > 1 else c.E
+    value = L * E_units / (ms / 1e3)
 
     # ---- end to end through the public API with host buffers
     e2e = None

@@ -585,11 +585,19 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
   const int VPR = (int)cdiv(a.F, EPV);
   if (VPR <= 1) return launch_cfg<T, 1, 1, 1>(a, VPR, s);
   if (VPR <= 2) return launch_cfg<T, 2, 1, 2>(a, VPR, s);
-  if (VPR <= 4) return launch_cfg<T, 4, 1, 4>(a, VPR, s);
-  static int cfg = -1;
+  static int cfg = -1, narrow = -1;
   if (cfg < 0) {
     const char* e = getenv("WG_AGG_CFG");
     cfg = e ? atoi(e) : 0;
+    const char* n = getenv("WG_AGG_NARROW");
+    narrow = n ? atoi(n) : 0;
+  }
+  if (VPR <= 4) {
+    // 33-64-byte rows (C5's 32-wide bf16 layers): the staged ring at 4 CTAs /
+    // SM (A/B on the C5 rank slice, 6 gathers / epoch: register kernel
+    // 63.0 ms, ring 4x3 @ 3/SM 53.6, 4x2 @ 4/SM 51.6, 4x4 @ 2/SM 54.5 ms)
+    if (narrow == 1) return launch_cfg<T, 4, 1, 4>(a, VPR, s);
+    return launch_cp<T, 4, 1, 4, 2, 4>(a, VPR, s);
   }
   if (!use_v2() && cfg == 1) {   // 3 CTAs / SM, ring 5 x 2
     if (VPR <= 8) return launch_cp<T, 8, 1, 5, 2, 3>(a, VPR, s);

@@ -26,19 +26,25 @@ class GNNStack:
 
     def __init__(self, graph: Graph, model: str, dims, *, dtype=torch.bfloat16, heads: int = 1, policy="auto",
                  seed: int = 0, lr: float = 1e-3, group=None, block: int | None = None, R: int = 1,
-                 conv_kw: dict | None = None, conv_factory=None, device=None):
+                 conv_kw: dict | None = None, conv_factory=None, device=None, sim_world: int = 1):
         # conv_kw: extra Conv options for every layer (e.g. RGCN norm / self_loop).
         # conv_factory / device: injection points for the multi-process CPU test
         # of this orchestration (tests/test_dist_gloo.py); the product path uses
         # Conv (libwg.so) on the graph's CUDA device.
+        # sim_world > 1 (no group): one rank of a sim_world-way 1-D partition
+        # on one GPU -- the rank's own kernels (PRE / POST phases, exchange
+        # tables) run, the collectives are skipped (timing of the per-rank
+        # compute only; exchanged rows are not filled in).
         Conv_ = conv_factory or Conv
         self.g, self.model, self.dims, self.dtype = graph, model, list(dims), dtype
         self.L = len(dims) - 1
         self.dev = device if device is not None else torch.device("cuda", graph.device)
         self.group = group
-        self.dist = group is not None and torch.distributed.get_world_size(group) > 1
-        self.world = torch.distributed.get_world_size(group) if group is not None else 1
-        self.rank = torch.distributed.get_rank(group) if group is not None else 0
+        self.sim = group is None and sim_world > 1
+        self.dist = (group is not None and torch.distributed.get_world_size(group) > 1) or self.sim
+        self.world = torch.distributed.get_world_size(group) if group is not None else sim_world
+        self.rank = torch.distributed.get_rank(group) if group is not None else (
+            graph.v_begin // block if self.sim else 0)
         self.rows = graph.n_rows
         self.vb = graph.v_begin
         self.block = block if block is not None else self.rows
@@ -60,15 +66,21 @@ class GNNStack:
                 conv.close()
                 conv = Conv_(graph, model, fi, dims[i + 1], policy=pol, **kw)
             self.convs.append(conv)
+            self._share_workspace(conv)
             self.params.append(init_params(model, fi, dims[i + 1], heads=heads, concat=not last, R=R,
                                            self_loop=bool((conv_kw or {}).get("self_loop", False)),
                                            bias=bool((conv_kw or {}).get("bias", True)),
                                            device=self.dev, seed=seed + 100 + i))
-        # activation tables: h[0] = input, h[i+1] = output of layer i (global rows when distributed)
-        self.h = [None] + [padded(self.Vtab, c.out_dim, dtype, self.dev) for c in self.convs]
+        # activation tables: h[0] = input, h[i+1] = output of layer i (global
+        # rows when distributed: the next layer gathers them; the logits of the
+        # last layer are never exchanged, so that table holds the owned rows)
+        self.h = [None] + [padded(self.Vtab if i + 1 < self.L else self.rows, c.out_dim, dtype, self.dev)
+                           for i, c in enumerate(self.convs)]
         self.saved = [c.new_saved() for c in self.convs]
-        self.dx = [None] + [padded(self.Vtab if self.dist else self.rows, self.f_in[i], dtype, self.dev)
-                            for i in range(1, self.L)]
+        # dx of layer i (= dy of layer i-1): owned rows only (the exchange
+        # tables carry what other ranks read)
+        self.dx = [None] + [padded(self.rows, self.f_in[i], dtype, self.dev) for i in range(1, self.L)]
+
         self.grads = [{k: torch.zeros_like(v) for k, v in p.items()} for p in self.params]
         self.xchg_f, self.xchg_b = [], []
         for c in self.convs:
@@ -85,6 +97,30 @@ class GNNStack:
                                     capturable=self.dev.type == "cuda")
 
     # -------------------------------------------------------------- helpers
+    def _share_workspace(self, conv):
+        """One workspace for all layers: a layer's scratch lives only inside its
+        forward / backward call (the PRE and POST phases of one layer are not
+        interleaved with another layer's calls), so every layer uses the
+        largest one; shared as each layer is created, so the per-layer buffers
+        never coexist."""
+        ws = getattr(conv, "workspace", None)
+        if not isinstance(ws, torch.Tensor):
+            return
+        shared = getattr(self, "_ws", None)
+        if shared is None or ws.numel() > shared.numel():
+            self._ws = ws
+            for c in self.convs:
+                if isinstance(getattr(c, "workspace", None), torch.Tensor):
+                    c.workspace = ws
+        else:
+            conv.workspace = shared
+        if self.dev.type == "cuda":
+            torch.cuda.empty_cache()
+
+    def _out(self, i):
+        """Rows of layer i's output table this rank writes."""
+        return self._own(self.h[i + 1]) if i + 1 < self.L else self.h[self.L]
+
     def _fwd_xchg(self, c):
         """VERTEX layers exchange Y = h W (transform before communicate); RGCN
         (per-relation transforms) and EDGE layers gather the activation itself."""
@@ -94,7 +130,7 @@ class GNNStack:
         return t[self.vb:self.vb + self.rows] if self.dist else t
 
     def _allgather(self, t):
-        if not self.dist:
+        if not self.dist or self.sim:
             return
         full = t.as_strided((self.Vtab, t.stride(0)), (t.stride(0), 1))
         mine = full[self.rank * self.block:(self.rank + 1) * self.block]
@@ -104,7 +140,7 @@ class GNNStack:
         """x: [V_tab x f0] (replicated input features); returns this rank's logits rows."""
         h = x
         for i, c in enumerate(self.convs):
-            y = self._own(self.h[i + 1])
+            y = self._out(i)
             if self._fwd_xchg(c):
                 xg = self.xchg_f[i]
                 c.forward_raw(h, self.params[i], y=y, saved=self.saved[i], phase=C.PHASE_PRE, xchg=xg)
@@ -116,7 +152,7 @@ class GNNStack:
                 self._allgather(self.h[i + 1])       # next EDGE / RGCN layer gathers raw rows
             h = self.h[i + 1]
         self.x = x
-        return self._own(self.h[self.L])
+        return self.h[self.L]
 
     fuse_masks = True
 
@@ -126,8 +162,8 @@ class GNNStack:
         for i in reversed(range(self.L)):
             c = self.convs[i]
             xin = self.x if i == 0 else self.h[i]
-            dx = self._own(self.dx[i]) if i > 0 else None
-            y = self._own(self.h[i + 1])
+            dx = self.dx[i] if i > 0 else None
+            y = self._out(i)
             # fuse layer i-1's ReLU backward into layer i's dx epilogue
             fuse = self.fuse_masks and i > 0 and getattr(self.convs[i - 1], "fuse_relu", False)
             kw = dict(grads=self.grads[i], dy_masked=masked,
@@ -141,7 +177,7 @@ class GNNStack:
                 c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, **kw)
             g = dx
             masked = fuse
-        if self.dist:
+        if self.dist and not self.sim:
             flat = torch.cat([v.reshape(-1) for gr in self.grads for v in gr.values()])
             torch.distributed.all_reduce(flat, group=self.group)
             o = 0

@@ -28,7 +28,7 @@ import dataclasses
 import numpy as np
 
 __all__ = [
-    "Config", "CONFIGS", "make_graph", "make_features", "glorot", "normal",
+    "Config", "CONFIGS", "make_graph", "make_graph_slice", "make_features", "glorot", "normal",
     "small_graph", "degree_stats",
 ]
 
@@ -120,6 +120,29 @@ def make_graph(V: int, E: int, *, seed: int, alpha: float = 0.5, symmetric: bool
             etype[lo:hi] = np.searchsorted(cdf, tr.random(hi - lo), side="right").astype(np.int32)
         np.minimum(etype, R - 1, out=etype)
     return src, dst, etype
+
+
+def make_graph_slice(V: int, E: int, lo: int, hi: int, *, seed: int, alpha: float = 0.5,
+                     chunk: int = 1 << 24):
+    """The edges of ``make_graph(V, E, seed=seed, alpha=alpha)`` (directed,
+    untyped) with ``dst`` or ``src`` in ``[lo, hi)``, in generation order,
+    without materialising all E edges: the same Philox streams are drawn
+    chunk by chunk (``Generator.random`` output does not depend on the chunk
+    split) and filtered.  Used for one rank's share of the C5 1-D partition
+    (its in-edges for the forward, its out-edges for the backward)."""
+    g = _rng(seed, 0)
+    perm_in = g.permutation(V).astype(np.int32)
+    perm_out = g.permutation(V).astype(np.int32)
+    rd, rs = _rng(seed, 1), _rng(seed, 2)
+    srcs, dsts = [], []
+    for b in range(0, E, chunk):
+        n = min(E, b + chunk) - b
+        d = _powerlaw_vertices(rd, V, n, alpha, perm_in, chunk=chunk)
+        s = _powerlaw_vertices(rs, V, n, alpha, perm_out, chunk=chunk)
+        keep = ((d >= lo) & (d < hi)) | ((s >= lo) & (s < hi))
+        srcs.append(s[keep])
+        dsts.append(d[keep])
+    return np.concatenate(srcs), np.concatenate(dsts)
 
 
 def small_graph(V: int, E: int, *, seed: int, R: int = 1, alpha: float = 0.3,
