@@ -148,3 +148,69 @@ def test_stack_training_decreases_loss(model):
     losses = [float(st.step(x, labels, V).item()) for _ in range(30)]
     # random labels: GCN / GAT (no self term) can only fit them through neighbours, slowly
     assert losses[-1] < losses[0] * (0.99 if model in ("gcn", "gat") else 0.9), losses
+
+
+@pytest.mark.parametrize("model", ["sage", "gat", "rgcn"])
+def test_stack_cuda_graph_replay_equals_eager(model):
+    """bench.py times K replays of one CUDA-graph-captured step: the replays
+    must do exactly what eager steps do (same kernels, deterministic), so the
+    parameters after n replays equal those after n eager steps bit for bit."""
+    m = wg()
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack
+    V, E = 3000, 40000
+    R = 5 if model == "rgcn" else 1
+    src, dst, et = synth.make_graph(V, E, seed=51, alpha=0.5, R=R)
+    g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V,
+                etype=torch.from_numpy(et).cuda() if R > 1 else None, num_types=R)
+    kw = dict(heads=2) if model == "gat" else dict(R=R, conv_kw={"norm": "right", "self_loop": True}) \
+        if model == "rgcn" else {}
+    dtype = torch.float32 if model == "rgcn" else torch.bfloat16
+    x = m.padded(V, 24, dtype)
+    x.copy_(torch.from_numpy(synth.make_features(V, 24, seed=52)))
+    labels = torch.from_numpy(np.random.default_rng(2).integers(0, 6, V)).cuda()
+    runs = []
+    for graph in (False, True):
+        st = GNNStack(g, model, [24, 32, 6], dtype=dtype, lr=1e-2, seed=9, **kw)
+        st.step(x, labels, V)                       # warm-up (buffers, attributes)
+        torch.cuda.synchronize()
+        if graph:
+            side = torch.cuda.Stream()
+            side.wait_stream(torch.cuda.current_stream())
+            with torch.cuda.stream(side):
+                st.step(x, labels, V)
+            torch.cuda.current_stream().wait_stream(side)
+            torch.cuda.synchronize()
+            cg = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(cg):
+                loss = st.step(x, labels, V)
+            for _ in range(3):
+                cg.replay()
+        else:                                       # warm-up + 4 = warm-up + side step + 3 replays
+            for _ in range(4):
+                loss = st.step(x, labels, V)
+        torch.cuda.synchronize()
+        runs.append(([v.detach().clone() for p in st.params for v in p.values()], float(loss.item())))
+    (pa, la), (pb, lb) = runs
+    assert la == lb
+    for a, b in zip(pa, pb):
+        assert torch.equal(a, b)
+
+
+def test_stack_rank_slice_runs():
+    """bench.py --rank-slice: one rank of a P-way 1-D partition on one GPU
+    (collectives skipped) trains with the rank's owned rows only."""
+    m = wg()
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack, partition_1d
+    V, E, P = 6000, 80000, 4
+    block, bounds = partition_1d(V, P)
+    vb, ve = bounds[1]
+    src, dst = synth.make_graph_slice(V, E, vb, ve, seed=61, alpha=0.5)
+    g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V, v_begin=vb, v_end=ve)
+    st = GNNStack(g, "sage", [24, 32, 32, 7], dtype=torch.bfloat16, block=block, sim_world=P, lr=1e-2)
+    assert st.dist and st.sim and st.rank == 1 and st.rows == ve - vb
+    x = m.padded(st.Vtab, 24, torch.bfloat16)
+    x[:V].copy_(torch.from_numpy(synth.make_features(V, 24, seed=62)))
+    labels = torch.from_numpy(np.random.default_rng(3).integers(0, 7, ve - vb)).cuda()
+    losses = [float(st.step(x, labels, V).item()) for _ in range(20)]
+    assert np.isfinite(losses).all() and losses[-1] < losses[0]
+    assert st.h[-1].shape[0] == ve - vb and all(d.shape[0] == ve - vb for d in st.dx[1:])
