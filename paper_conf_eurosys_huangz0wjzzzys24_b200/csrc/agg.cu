@@ -609,6 +609,8 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
     if (VPR <= 32) return launch_cp<T, 32, 1, 4, 2, 4>(a, VPR, s);
   } else if (!use_v2()) {
     // default: 3 CTAs (24 warps) per SM, 10 edges in flight per worker
+    // (65-128-byte rows, C4 epoch A/B: 5x2 @ 3/SM 24.0 ms; 8x2 @ 3 25.2, 5x3 @ 3 24.9,
+    //  4x2 @ 4 24.4, 8x3 @ 2 27.3, 6x3 @ 3 24.8 ms)
     // (A/B on C4: 7x3 @ 2 CTAs/SM 72 %, 6x2 @ 3/SM 83 %, 5x2 @ 3/SM 84.5 %,
     //  4x2 @ 4/SM 82 % of HBM)
     if (VPR <= 8) return launch_cp<T, 8, 1, 5, 2, 3>(a, VPR, s);

@@ -116,6 +116,104 @@ __global__ void __launch_bounds__(256) k_xent_row(int64_t M, int C, const T* x, 
   }
 }
 
+
+// small C, vectorised: groups of 8 lanes per row (4 rows per warp), lane l
+// loads / stores 16-byte vectors l, l + 8, ... of the row (NVL per lane), so a
+// row is one coalesced load and one store per lane instead of C scalar ones
+// (the rows are ld-aligned: ld * sizeof(T) is a multiple of 16 bytes).
+template <typename T> struct XV;
+template <> struct XV<float> {
+  static constexpr int EPV = 4;
+  __device__ static void unpack(const int4& q, float* f) {
+    f[0] = __int_as_float(q.x); f[1] = __int_as_float(q.y); f[2] = __int_as_float(q.z); f[3] = __int_as_float(q.w);
+  }
+  __device__ static int4 pack(const float* f) {
+    return make_int4(__float_as_int(f[0]), __float_as_int(f[1]), __float_as_int(f[2]), __float_as_int(f[3]));
+  }
+};
+template <> struct XV<__nv_bfloat16> {
+  static constexpr int EPV = 8;
+  __device__ static void unpack(const int4& q, float* f) {
+    const uint32_t w[4] = {(uint32_t)q.x, (uint32_t)q.y, (uint32_t)q.z, (uint32_t)q.w};
+#pragma unroll
+    for (int i = 0; i < 4; ++i) { f[2 * i] = __uint_as_float(w[i] << 16); f[2 * i + 1] = __uint_as_float(w[i] & 0xffff0000u); }
+  }
+  __device__ static int4 pack(const float* f) {
+    uint32_t w[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      __nv_bfloat162 h = __floats2bfloat162_rn(f[2 * i], f[2 * i + 1]);
+      w[i] = *reinterpret_cast<uint32_t*>(&h);
+    }
+    return make_int4((int)w[0], (int)w[1], (int)w[2], (int)w[3]);
+  }
+};
+
+template <typename T, int NVL>
+__global__ void __launch_bounds__(256) k_xent_vec(int64_t M, int C, const T* x, int64_t ld, const int64_t* labels,
+                                                  float scale, T* dx, int64_t ldd, float* part) {
+  constexpr int EPV = XV<T>::EPV;
+  __shared__ float wsum[8];
+  const int Cpad = (C + 7) / 8 * 8;
+  const int lane = threadIdx.x & 31, g = lane >> 3, l = lane & 7;
+  const unsigned gm = 0xffu << (g * 8);
+  float lsum = 0.f;
+  const int64_t rows_per_iter = (int64_t)gridDim.x * (blockDim.x / 8);
+  for (int64_t r = blockIdx.x * (int64_t)(blockDim.x / 8) + (threadIdx.x >> 3); r < M; r += rows_per_iter) {
+    float v[NVL][EPV];
+    float m = -INFINITY;
+#pragma unroll
+    for (int q = 0; q < NVL; ++q) {
+      const int c0 = (l + 8 * q) * EPV;
+      if (c0 < Cpad) XV<T>::unpack(__ldg(reinterpret_cast<const int4*>(x + r * ld + c0)), v[q]);
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) {
+        if (c0 + i >= C) v[q][i] = -INFINITY;
+        m = fmaxf(m, v[q][i]);
+      }
+    }
+#pragma unroll
+    for (int o = 4; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(gm, m, o, 8));
+    const int64_t lab = labels[r];
+    float s = 0.f, t_lab = 0.f;
+#pragma unroll
+    for (int q = 0; q < NVL; ++q) {
+      const int c0 = (l + 8 * q) * EPV;
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) {
+        const bool in = c0 + i < C;
+        const float t = in ? v[q][i] - m : 0.f;
+        if (c0 + i == lab) t_lab = t;
+        v[q][i] = in ? __expf(t) : 0.f;
+        s += v[q][i];
+      }
+    }
+#pragma unroll
+    for (int o = 4; o; o >>= 1) s += __shfl_xor_sync(gm, s, o, 8);
+    const float inv = 1.f / s;
+#pragma unroll
+    for (int q = 0; q < NVL; ++q) {
+      const int c0 = (l + 8 * q) * EPV;
+      if (c0 >= Cpad) continue;
+      float o[EPV];
+#pragma unroll
+      for (int i = 0; i < EPV; ++i)
+        o[i] = c0 + i < C ? scale * (v[q][i] * inv - (c0 + i == lab ? 1.f : 0.f)) : 0.f;
+      *reinterpret_cast<int4*>(dx + r * ldd + c0) = XV<T>::pack(o);
+      if (lab >= c0 && lab < c0 + EPV) lsum += scale * (logf(s) - t_lab);
+    }
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) lsum += __shfl_xor_sync(0xffffffffu, lsum, o);
+  if ((threadIdx.x & 31) == 0) wsum[threadIdx.x >> 5] = lsum;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float t = 0.f;
+    for (int w = 0; w < 8; ++w) t += wsum[w];
+    part[blockIdx.x] = t;
+  }
+}
+
 __global__ void k_sum(const float* part, int n, float* out) {
   if (threadIdx.x == 0 && blockIdx.x == 0) {
     float t = 0.f;
@@ -149,7 +247,15 @@ extern "C" wg_status wg_softmax_xent(wg_dtype dtype, int64_t M, int32_t C, const
   const int per = (C + 31) / 32;
   if (C <= 64) {
     const unsigned nb = (unsigned)std::min<int64_t>(XENT_BLKS, std::max<int64_t>(1, cdiv(M, 32)));
-    if (dtype == WG_BF16)
+    const bool vec = ((ld * (dtype == WG_BF16 ? 2 : 4)) % 16 == 0) && ((ldd * (dtype == WG_BF16 ? 2 : 4)) % 16 == 0) &&
+                     (reinterpret_cast<uintptr_t>(logits) % 16 == 0) && (reinterpret_cast<uintptr_t>(dlogits) % 16 == 0);
+    if (dtype == WG_BF16 && vec)
+      WG_LAUNCH((k_xent_vec<__nv_bfloat16, 1>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld, labels, scale,
+                (__nv_bfloat16*)dlogits, ldd, part);
+    else if (vec)
+      WG_LAUNCH((k_xent_vec<float, 2>), nb, 256, 0, s, M, C, (const float*)logits, ld, labels, scale,
+                (float*)dlogits, ldd, part);
+    else if (dtype == WG_BF16)
       WG_LAUNCH((k_xent_row<__nv_bfloat16, 8>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld, labels, scale,
                 (__nv_bfloat16*)dlogits, ldd, part);
     else

@@ -167,10 +167,10 @@ def test_stack_cuda_graph_replay_equals_eager(model):
     dtype = torch.float32 if model == "rgcn" else torch.bfloat16
     x = m.padded(V, 24, dtype)
     x.copy_(torch.from_numpy(synth.make_features(V, 24, seed=52)))
-    labels = torch.from_numpy(np.random.default_rng(2).integers(0, 6, V)).cuda()
+    labels = torch.from_numpy(np.random.default_rng(2).integers(0, 8, V)).cuda()
     runs = []
     for graph in (False, True):
-        st = GNNStack(g, model, [24, 32, 6], dtype=dtype, lr=1e-2, seed=9, **kw)
+        st = GNNStack(g, model, [24, 32, 8], dtype=dtype, lr=1e-2, seed=9, **kw)
         st.step(x, labels, V)                       # warm-up (buffers, attributes)
         torch.cuda.synchronize()
         if graph:
