@@ -274,10 +274,19 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # WG_DIST_BACKEND=gloo + WG_DIST_ONE_GPU=1: every rank on cuda:0 over gloo --
+    # a functional check of the multi-rank path where only one GPU exists
+    # (timings of such a run are meaningless; the product path is NCCL)
+    backend = os.environ.get("WG_DIST_BACKEND", "nccl")
+    if os.environ.get("WG_DIST_ONE_GPU") == "1":
+        local = 0
     torch.cuda.set_device(local)
     group = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
         group = dist.group.WORLD
     import paper_conf_eurosys_huangz0wjzzzys24_b200 as wg
     from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack, partition_1d
