@@ -60,6 +60,8 @@ def parse():
     ap.add_argument("--model", default=None, choices=["sage", "gin", "gcn", "gat", "rgcn"],
                     help="default: the config's model (C4: sage)")
     ap.add_argument("--policy", default="auto")
+    ap.add_argument("--tile", type=int, default=128,
+                    help="gTask destination-tile rows T (SURVEY §8(f) f1 sweeps; 128 = the tcgen05 M)")
     ap.add_argument("--emax", type=int, default=0,
                     help="gTask edge limit E_max (0: the Q13 rule); SURVEY §8(f) f1 K sweeps")
     ap.add_argument("--no-e2e", action="store_true")
@@ -327,7 +329,7 @@ def main():
     g = wg.Graph(torch.from_numpy(src).to(dev), torch.from_numpy(dst).to(dev), num_vertices=c.V,
                  etype=torch.from_numpy(et).to(dev) if R > 1 else None, num_types=R,
                  v_begin=vb if (world > 1 or P > 1) else 0, v_end=ve if (world > 1 or P > 1) else 0,
-                 max_task_edges=args.emax)
+                 max_task_edges=args.emax, tile_rows=args.tile)
     if P > 1:
         src = dst = None   # host copies of the slice are not needed any more
     torch.cuda.synchronize()
