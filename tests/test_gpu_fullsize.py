@@ -199,3 +199,50 @@ def test_c3_rgcn_layer1_sampled():
         for (i, j) in [(0, 0), (fi - 1, fo - 1), (17, 33)]:
             ref = entry_probe(src[sel], dst[sel], None, xo, dyo, i, j)
             assert abs(gW[r, i, j] - ref) <= 1e-4 * scale, (r, i, j, gW[r, i, j], ref)
+
+
+def test_c5_rank_slice_layer1_sampled():
+    """C5 (111 M V, 1.6 B E) at full size, in the launch configuration bench.py
+    --rank-slice 8 times: rank 0's block of the 8-way 1-D partition (its in- and
+    out-edges only).  Layer-1 SAGE forward of owned rows is exact on the slice
+    (every in-edge of an owned row is present, degrees of owned rows are
+    global), so sampled rows are compared with the oracle on their induced
+    in-neighbourhood.  The EDGE plan gathers the replicated input table
+    itself; the VERTEX plan would gather Y = x W rows that other ranks own
+    (filled by the all-gather a single process does not run)."""
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import partition_1d
+    c = synth.CONFIGS["C5"]
+    m = wg()
+    block, bounds = partition_1d(c.V, 8)
+    vb, ve = bounds[0]
+    src, dst = synth.make_graph_slice(c.V, c.E, vb, ve, seed=c.seed * 16, alpha=c.alpha)
+    g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=c.V, v_begin=vb, v_end=ve)
+    dt = torch.bfloat16
+    fi, fo = c.dims[0], c.dims[1]
+    x = m.padded(c.V, fi, dt)
+    gen = torch.Generator(device="cuda").manual_seed(5)
+    for r0 in range(0, c.V, 1 << 22):
+        r1 = min(c.V, r0 + (1 << 22))
+        x[r0:r1].copy_(torch.randn((r1 - r0, fi), generator=gen, device="cuda"))
+    conv = m.Conv(g, "sage", fi, fo, dtype=dt, fuse_relu=True, need_dx=False, policy="edge")
+    params = m.init_params("sage", fi, fo, seed=7)
+    y, saved = conv.forward_raw(x, params)
+    torch.cuda.synchronize()
+    own = (dst >= vb) & (dst < ve)
+    s_own, d_own = src[own], dst[own]
+    deg = np.bincount(d_own - vb, minlength=ve - vb)
+    rows = set((RNG.choice(ve - vb, size=1000, replace=False) + vb).tolist())
+    rows |= set((np.argsort(deg)[-20:] + vb).tolist())
+    rows = np.array(sorted(rows))
+    sel = np.isin(d_own, rows)
+    s_r, d_r = s_own[sel], d_own[sel]
+    U = np.unique(np.concatenate([rows, s_r]))
+    remap = lambda a: np.searchsorted(U, a).astype(np.int32)  # noqa: E731
+    xs = f64(x[torch.from_numpy(U).cuda()])
+    W = {k: q(v, dt) for k, v in params.items()}
+    yo = np.maximum(oracle.sage_forward(remap(s_r), remap(d_r), len(U), xs, W["W_self"], W["W"], W["bias"],
+                                        rows=remap(rows)), 0)
+    yg = f64(y)[rows - vb]
+    ref = yo[remap(rows)]
+    err = np.abs(yg - ref).max() / max(np.abs(ref).max(), 1e-30)
+    assert err <= 2e-2, err
