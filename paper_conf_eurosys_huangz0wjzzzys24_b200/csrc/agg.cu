@@ -674,7 +674,8 @@ __global__ void k_prep_weight(const float* W, int batch, int rows, int cols, int
 // 16-byte vectors per thread; block partials reduced in a fixed order.
 template <typename T>
 __global__ void __launch_bounds__(256) k_colsum(int64_t M, int N, const T* dy, int64_t lddy, const T* ref,
-                                                int64_t ldref, T* dt, int64_t ldt, float* part, int64_t rows_per_blk) {
+                                                int64_t ldref, T* dt, int64_t ldt, float* part, int64_t rows_per_blk,
+                                                const float* rs2, T* dt2, int64_t ldt2) {
   constexpr int EPV = VT<T>::EPV;
   extern __shared__ float red[];                       // [nsub][nv*EPV]
   const int nv = (N + EPV - 1) / EPV;                  // vectors per row (<= 256)
@@ -695,6 +696,13 @@ __global__ void __launch_bounds__(256) k_colsum(int64_t M, int N, const T* dy, i
 #pragma unroll
       for (int i = 0; i < EPV; ++i) if (vec * EPV + i >= N) v[i] = 0.f;
       if (dt) *reinterpret_cast<int4*>(dt + r * ldt + vec * EPV) = VT<T>::pack(v);
+      if (dt2) {
+        float w[EPV];
+        const float sc = rs2[r];
+#pragma unroll
+        for (int i = 0; i < EPV; ++i) w[i] = sc * v[i];
+        *reinterpret_cast<int4*>(dt2 + r * ldt2 + vec * EPV) = VT<T>::pack(w);
+      }
 #pragma unroll
       for (int i = 0; i < EPV; ++i) acc[i] += v[i];
     }
@@ -762,22 +770,24 @@ wg_status prep_weight(wg_dtype dt, const float* W, int rows, int cols, int trans
 size_t bias_grad_scratch(int64_t M, int N) { return sizeof(float) * (size_t)COLSUM_BLKS * N; }
 
 wg_status bias_grad_mask(wg_dtype dt, int64_t M, int N, const void* dy, int64_t lddy, const void* ref,
-                         int64_t ldref, void* dt_out, int64_t ldt, float* db, float* scratch, cudaStream_t s) {
+                         int64_t ldref, void* dt_out, int64_t ldt, float* db, float* scratch, cudaStream_t s,
+                         const float* rs2, void* dt2, int64_t ldt2) {
   const int EPV = dt == WG_BF16 ? 8 : 4;
   const int nv = (int)cdiv(N, EPV);
   WG_REQ(nv <= 256, WG_ERR_UNSUPPORTED, "bias gradient: more than 256 vectors per row");
   const int64_t rpb = std::max<int64_t>(1, cdiv(M, COLSUM_BLKS));
   const int nblk = (int)std::max<int64_t>(1, cdiv(M, rpb));
   const double es = dt == WG_BF16 ? 2.0 : 4.0;
-  ProfScope ps(PK_MISC, s, (double)M * N * es * (1 + (ref ? 1 : 0) + (dt_out ? 1 : 0)), (double)M * N);
+  ProfScope ps(PK_MISC, s, (double)M * N * es * (1 + (ref ? 1 : 0) + (dt_out ? 1 : 0) + (dt2 ? 1 : 0)), (double)M * N);
   const int threads = 256;
   const size_t smem = (size_t)(threads / nv) * nv * EPV * sizeof(float);
   if (dt == WG_BF16)
     WG_LAUNCH(k_colsum<__nv_bfloat16>, nblk, threads, smem, s, M, N, (const __nv_bfloat16*)dy, lddy,
-              (const __nv_bfloat16*)ref, ldref, (__nv_bfloat16*)dt_out, ldt, scratch, rpb);
+              (const __nv_bfloat16*)ref, ldref, (__nv_bfloat16*)dt_out, ldt, scratch, rpb, rs2, (__nv_bfloat16*)dt2,
+              ldt2);
   else
     WG_LAUNCH(k_colsum<float>, nblk, threads, smem, s, M, N, (const float*)dy, lddy, (const float*)ref, ldref,
-              (float*)dt_out, ldt, scratch, rpb);
+              (float*)dt_out, ldt, scratch, rpb, rs2, (float*)dt2, ldt2);
   if (db) WG_LAUNCH(k_colsum_reduce, (unsigned)cdiv(N, 32), 256, 0, s, scratch, nblk, N, db);
   return WG_OK;
 }

@@ -295,15 +295,25 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   // dAgg path) lives in the exchange buffer when distributed.
   // (single GPU: vb == 0 and every table is indexed by global == local rows)
   const bool gpath_lin = (path == 1 && !gin);
+  // 1-D partition: the destination scale rs[d] of the transposed gather is
+  // folded into the exchanged rows by their owner in PRE (dT rs on the G
+  // path, dAgg rs on the dAgg path), so the POST gather reads no per-edge
+  // scale -- a random 4-byte load per edge from a V-sized array (444 MB at C5)
+  const bool fold = xchg != nullptr && rs != nullptr && !gin;
+  const float* rs_own = rs ? rs + c.vb : nullptr;
   void* dt_buf = nullptr;
   int64_t ld_dtb = c.po;
-  if (gpath_lin && xchg) { dt_buf = off(xchg, c.vb, A->ld_xchg, c.s); ld_dtb = A->ld_xchg; }
+  void* dt_fold = nullptr;                 // G path, folded: the scaled rows in the exchange table
+  if (gpath_lin && xchg && fold) {
+    dt_fold = off(xchg, c.vb, A->ld_xchg, c.s);
+    if (mask_dy) dt_buf = off(L.at<void>(ws, "dt"), c.vb, c.po, c.s);
+  } else if (gpath_lin && xchg) { dt_buf = off(xchg, c.vb, A->ld_xchg, c.s); ld_dtb = A->ld_xchg; }
   else if (mask_dy) { dt_buf = off(L.at<void>(ws, "dt"), c.vb, c.po, c.s); ld_dtb = c.po; }
   if (pre) {
     float* db = gin ? (G ? G->b2 : nullptr) : (G ? G->bias : nullptr);
-    if (dt_buf || db)
+    if (dt_buf || db || dt_fold)
       WG_TRY(bias_grad_mask(c.dt, c.nr, c.fo, A->dy, A->lddy, mask_dy ? A->y : nullptr, A->ldy, dt_buf, ld_dtb,
-                            db, colsum, st));
+                            db, colsum, st, dt_fold ? rs_own : nullptr, dt_fold, A->ld_xchg));
   }
   const void* dT = dt_buf ? dt_buf : A->dy;
   const int64_t lddT = dt_buf ? ld_dtb : A->lddy;
@@ -350,19 +360,21 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
         GemmPart part{dT, lddT, wbs, c.po, c.fo, (int)(2 * c.pi)};
         GemmEpi e;
         e.D = off(dtab, c.vb, ldd, c.s); e.ldd = ldd;
+        e.rscale = fold ? rs_own : nullptr;    // dAgg only (D), not dX_s (D2)
         e.D2 = L.at<void>(ws, "dxs"); e.ldd2 = c.pi; e.n_split = (int)c.pi;
         WG_TRY(gemm_nt(c.dt, c.nr, (int)(2 * c.pi), &part, 1, e, nullptr, 0, st));
       } else if (d.need_dx) {
         GemmPart part{dTT, lddTT, w, c.po, c.fo, (int)c.wrows_i};
         GemmEpi e;
         e.D = off(dtab, c.vb, ldd, c.s); e.ldd = ldd;
+        e.rscale = fold ? rs_own : nullptr;
         WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), &part, 1, e, nullptr, 0, st));
       }
     }
     if (post && d.need_dx) {
       AggArgs a = agg_base(c, p->bt, c.g->bwd);
       a.table = dtab; a.ld_tab = ldd;
-      a.gscale = rs; a.rscale = gs;       // transposed: c_e = gs[u] * rs[d]
+      a.gscale = fold ? nullptr : rs; a.rscale = gs;   // transposed: c_e = gs[u] * rs[d]
       if (sage) { a.self_tab = L.at<void>(ws, "dxs"); a.ld_self = c.pi; a.self_coef = 1.f; }
       if (gin) { a.self_tab = off(dtab, c.vb, ldd, c.s); a.ld_self = ldd; a.self_coef = 1.f + d.gin_eps; }
       a.out = A->dx; a.ld_out = A->lddx;
@@ -380,7 +392,7 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   {
     AggArgs a = agg_base(c, p->bt, c.g->bwd);
     a.table = gtab; a.ld_tab = ldg;
-    a.gscale = rs; a.rscale = gs;
+    a.gscale = fold ? nullptr : rs; a.rscale = gs;
     if (gin) { a.self_tab = off(gtab, c.vb, ldg, c.s); a.ld_self = ldg; a.self_coef = 1.f + d.gin_eps; }
     a.out = gbuf; a.ld_out = c.po;
     a.partial = L.at<float>(ws, "partT"); a.ld_part = pl;

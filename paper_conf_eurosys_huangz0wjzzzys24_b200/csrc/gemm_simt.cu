@@ -76,7 +76,7 @@ __global__ void __launch_bounds__(256) k_gemm_nt(NTArgs a) {
     for (int j = 0; j < 4; ++j) {
       const int n = n0 + tx * 4 + j;
       if (n >= a.N) continue;
-      float v = rs * acc[i][j];
+      float v = (e.D2 && n >= e.n_split) ? acc[i][j] : rs * acc[i][j];
       if (e.addend) v += tof<T>(static_cast<const T*>(e.addend)[m * e.ld_add + n]);
       if (e.bias) v += e.bias[n];
       if (e.relu) v = fmaxf(v, 0.f);

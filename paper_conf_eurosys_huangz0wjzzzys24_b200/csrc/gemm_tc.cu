@@ -378,7 +378,7 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
           if (n >= p.N) continue;
           float* f = v + 8 * h;
 #pragma unroll
-          for (int i = 0; i < 8; ++i) f[i] *= rs;
+          for (int i = 0; i < 8; ++i) f[i] *= (e.D2 && n >= e.n_split) ? 1.f : rs;
           if (e.addend) {
             float t[8];
             bf16x8_unpack(*reinterpret_cast<const int4*>(static_cast<const __nv_bfloat16*>(e.addend) + m * e.ld_add + n), t);

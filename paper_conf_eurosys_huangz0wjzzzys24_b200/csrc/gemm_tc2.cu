@@ -468,7 +468,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
       const CUtensorMap* td = second ? &tD2 : &tD;
       const int ncol0 = second ? n0 - p.n_split : n0;
       const int64_t m = (int64_t)m0 + r;
-      const float rs = (p.rscale && m < p.M) ? p.rscale[m] : 1.f;
+      const float rs = (p.rscale && m < p.M && !second) ? p.rscale[m] : 1.f;   // D only
       mbar_wait(su32(&tfull[buf]), (j >> 1) & 1);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       for (int c = 0; c < nchunk; ++c, ++g) {

@@ -198,7 +198,7 @@ struct GemmPart {
   int64_t a_table_rows = 0;
 };
 struct GemmEpi {
-  const float* rscale = nullptr;      // per row
+  const float* rscale = nullptr;      // per row (split output: applies to D only, not D2)
   const float* bias = nullptr;        // per column [N]
   const void* addend = nullptr;       // add [M x N] (conv dtype), ld_add
   int64_t ld_add = 0;
@@ -243,9 +243,12 @@ wg_status prep_weight_batched(wg_dtype dt, const float* W, int batch, int rows, 
 wg_status prep_weight(wg_dtype dt, const float* W, int rows, int cols, int transpose,
                       void* out, int64_t ldo, int out_rows, cudaStream_t s);
 // column sums (deterministic) of dy (optionally relu-masked by ref, written to dt_out)
+// dt2 (optional): the same rows scaled by rs2[row] (the destination scale
+// folded into an exchanged table)
 wg_status bias_grad_mask(wg_dtype dt, int64_t M, int N, const void* dy, int64_t lddy,
                          const void* ref, int64_t ldref, void* dt_out, int64_t ldt,
-                         float* db, float* scratch, cudaStream_t s);
+                         float* db, float* scratch, cudaStream_t s,
+                         const float* rs2 = nullptr, void* dt2 = nullptr, int64_t ldt2 = 0);
 size_t bias_grad_scratch(int64_t M, int N);
 
 // cost-model constants (milli-femtoseconds per byte / per flop), from MEASURED_PEAKS
