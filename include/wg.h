@@ -173,7 +173,10 @@ typedef struct {
 /* Phases for the 1-D multi-GPU layer (§8(e)).  Single GPU: WG_PHASE_ALL.
  * PRE computes this rank's rows of the exchange table into
  * `xchg + row_offset * ld_xchg`; the caller all-gathers `xchg` (in place);
- * POST consumes the gathered table.  RGCN: the forward has no exchange
+ * POST consumes the gathered table.  GCN / SAGE backward tables carry the
+ * destination's normalisation already (dT * c_dst on the G path, dAgg * c_dst
+ * on the dAgg path, c_dst = 1/deg_in or deg_in^-1/2), so POST reads no
+ * per-edge scale; the table is opaque to the caller.  RGCN: the forward has no exchange
  * (x must hold all rows: PRE does nothing, POST = ALL); the backward
  * exchange table is dT = dy (masked by the fused ReLU), f_out wide.  GAT
  * plans accept only WG_PHASE_ALL (and only on a full graph, see
