@@ -629,7 +629,7 @@ wg_status launch_t(const AggArgs& a, cudaStream_t s) {
 
 wg_status launch_agg(wg_dtype dt, const AggArgs& a, cudaStream_t s) {
   if (a.n_items == 0) return WG_OK;
-  WG_REQ(a.key != nullptr, WG_ERR_STATE, "launch_agg: key array missing");
+  WG_REQ(a.key != nullptr || a.idx == nullptr, WG_ERR_STATE, "launch_agg: key array missing");  // E = 0: no key / idx
   // algorithmic bytes: per edge the index (4 B), the gathered row (F elements)
   // and the source scale if any; per row the output, row_ptr and optional
   // self / mask rows

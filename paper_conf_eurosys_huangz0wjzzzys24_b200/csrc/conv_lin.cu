@@ -61,7 +61,7 @@ void lin_layout(wg_plan_s* p) {
   S = Layout();
   W = Layout();
   const bool sage = d.model == WG_SAGE, gin = d.model == WG_GIN;
-  if (p->n_edge_tasks > 0) S.add("agg", (size_t)c.nr * c.pi * s);
+  if (edge_path(p)) S.add("agg", (size_t)c.nr * c.pi * s);
   if (gin) S.add("h", (size_t)c.nr * c.po * s);
   // prepped weights (forward: transposed [rows_o x pi]; backward: [rows_i x po])
   W.add("wt", (size_t)c.wrows_o * c.pi * s);          // W^T (GCN W, SAGE W_n, GIN W1)
@@ -148,7 +148,7 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
   WG_REQ(!sage || P->W_self, WG_ERR_INVALID, "SAGE needs W_self");
   WG_REQ(!gin || P->W2, WG_ERR_INVALID, "GIN needs W2");
   WG_REQ(A->x && A->y && A->workspace, WG_ERR_INVALID, "x / y / workspace is NULL");
-  WG_REQ(p->n_edge_tasks == 0 || A->saved, WG_ERR_INVALID, "saved is NULL");
+  WG_REQ(!edge_path(p) || A->saved, WG_ERR_INVALID, "saved is NULL");
   WG_REQ((A->ldx * c.s) % 16 == 0 && A->ldx >= c.fi && (A->ldy * c.s) % 16 == 0 && A->ldy >= c.fo, WG_ERR_INVALID,
          "ldx / ldy must be >= F and 16-byte multiples");
   const bool dist = c.nr != c.Vg;
@@ -158,7 +158,7 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
   const char* x_own = off(A->x, c.vb, A->ldx, c.s);
   const float *gs, *rs;
   gcn_scales(c, &gs, &rs);
-  const bool all_vertex = p->n_edge_tasks == 0;
+  const bool all_vertex = !edge_path(p);
   const bool has_bias = d.bias && P->bias;
   // prepped weights
   void* wt = L.at<void>(ws, "wt");
@@ -196,12 +196,12 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
     }
   }
   if (!post) return WG_OK;
-  void* agg = p->n_edge_tasks > 0 ? p->saved.at<void>(A->saved, "agg") : nullptr;
+  void* agg = edge_path(p) ? p->saved.at<void>(A->saved, "agg") : nullptr;
   void* z = p->mixed ? L.at<void>(ws, "z") : nullptr;
   void* h = gin ? p->saved.at<void>(A->saved, "h") : nullptr;
   const int64_t pl = part_ld(c);
   // ---- EDGE gTasks: Agg = A_hat x  (GIN: z = (1+eps) x + A x)
-  if (p->n_edge_tasks > 0) {
+  if (edge_path(p)) {
     AggArgs a = agg_base(c, p->fe, c.g->fwd);
     a.table = A->x; a.ld_tab = A->ldx;
     a.gscale = gs; a.rscale = rs;
@@ -234,7 +234,7 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
     WG_TRY(run_agg(c, a, p->fv, st));
   }
   // ---- EDGE transform: y = Agg W (+ x W_s) + Z + b
-  if (p->n_edge_tasks > 0) {
+  if (edge_path(p)) {
     GemmPart parts[2];
     int np = 0;
     if (sage) parts[np++] = GemmPart{x_own, A->ldx, wst, c.pi, c.fi, (int)c.wrows_o};
@@ -268,7 +268,7 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   WG_REQ(P && P->W && A->dy && A->x && A->workspace, WG_ERR_INVALID, "backward: null argument");
   WG_REQ(!d.fuse_relu || A->y || A->dy_masked, WG_ERR_INVALID, "fuse_relu backward needs y");
   WG_REQ(!d.need_dx || A->dx, WG_ERR_INVALID, "need_dx but dx is NULL");
-  WG_REQ(p->n_edge_tasks == 0 || A->saved, WG_ERR_INVALID, "saved is NULL");
+  WG_REQ(!edge_path(p) || A->saved, WG_ERR_INVALID, "saved is NULL");
   // dy already masked by the next layer (dx_mask fusion): no mask pass here
   const bool mask_dy = d.fuse_relu && !A->dy_masked;
   const bool dist = c.nr != c.Vg;

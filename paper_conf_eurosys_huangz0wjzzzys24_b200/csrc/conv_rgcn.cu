@@ -194,7 +194,8 @@ wg_status rgcn_plan(wg_plan_s* p, cudaStream_t) {
   // side holds their in-edges, its transposed side their out-edges; x / dT
   // tables are read with global row ids (replicated / all-gathered), outputs
   // are written for the owned rows only.
-  const int R = g->by_type ? g->R : 1;
+  // E = 0: no edge carries a type, but the R relation gradients still exist (all zero)
+  const int R = (g->by_type || g->E_total == 0) ? g->R : 1;
   const int64_t E = g->fwd.E, Eb = g->bwd.E, V = g->V, vb = g->vb, nr = g->ve - g->vb;
   auto* rp = new RgcnPlan();
   rp->R = R;

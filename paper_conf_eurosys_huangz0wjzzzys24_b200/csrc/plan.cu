@@ -18,8 +18,10 @@ namespace {
 
 // Build work items from one side's gTask table (untyped graphs).
 // plan: per task bit (nullptr => all EDGE).  out[0] EDGE items, out[1] VERTEX.
+// b_empty: the list that takes rows of no gTask (edgeless tiles, rows beside
+// a tile's SPLIT rows) -- one whose pass runs, so their epilogue is written.
 void build_items(const wg_graph_s* g, const Side& S, const std::vector<uint8_t>* plan, ItemList* out0,
-                 ItemList* out1, int* n_slots) {
+                 ItemList* out1, int* n_slots, int b_empty = 0) {
   const int64_t T = g->T, vb = g->vb, ve = g->ve;
   const int64_t t0 = vb / T, t1 = cdiv(ve, T);
   size_t ti = 0;
@@ -35,7 +37,7 @@ void build_items(const wg_graph_s* g, const Side& S, const std::vector<uint8_t>*
     // emit the rows [cur_lo, end) as work items, cut around SPLIT rows
     // (deg > E_max: those rows are produced by their SPLIT chunks + combine)
     auto flush = [&](int32_t end) {
-      const int b = (cur_task >= 0 && plan) ? (*plan)[cur_task] : 0;
+      const int b = cur_task >= 0 ? (plan ? (*plan)[cur_task] : 0) : b_empty;
       int32_t lo = cur_lo;
       for (int32_t r = cur_lo; r <= end; ++r) {
         const bool cut = (r == end) || (S.h_row_ptr[r + 1] - S.h_row_ptr[r] > g->E_max);
@@ -190,7 +192,9 @@ wg_status plan_create(wg_graph g, const wg_conv_desc* d, wg_plan* out) {
     if (s != WG_OK) { delete p; return s; }
   } else {
     choose_plans(p);
-    build_items(g, g->fwd, &p->plan_bits, &p->fe, &p->fv, &p->n_slots_f);
+    // all-VERTEX layers run no EDGE pass; a layer with no gTask at all (E = 0) runs the EDGE one
+    const int b_empty = (d->model != WG_GAT && p->n_edge_tasks == 0 && p->n_vert_tasks > 0) ? 1 : 0;
+    build_items(g, g->fwd, &p->plan_bits, &p->fe, &p->fv, &p->n_slots_f, b_empty);
     ItemList dummy;
     build_items(g, g->bwd, nullptr, &p->bt, &dummy, &p->n_slots_t);
     wg_status s;

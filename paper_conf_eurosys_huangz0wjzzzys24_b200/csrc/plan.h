@@ -52,6 +52,11 @@ struct wg_plan_s {
   void* gat = nullptr;
 };
 
+// The EDGE pass (aggregate, then the transform GEMM) runs when any gTask is
+// EDGE, or when the layer has no gTask at all (E = 0: every row is the
+// empty-neighbourhood epilogue, produced by that pass's items).
+inline bool edge_path(const wg_plan_s* p) { return p->n_edge_tasks > 0 || p->n_vert_tasks == 0; }
+
 namespace wg {
 wg_status rgcn_plan(wg_plan_s* p, cudaStream_t s);
 void rgcn_plan_free(wg_plan_s* p);

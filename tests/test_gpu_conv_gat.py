@@ -19,9 +19,10 @@ def wg():
     return m
 
 
-def run(dtype, H, concat, V=1200, E=15000, fi=24, fo=16, relu=False, seed=0, alpha=0.8):
+def run(dtype, H, concat, V=1200, E=15000, fi=24, fo=16, relu=False, seed=0, alpha=0.8, edges=None,
+        zero_attn=False):
     m = wg()
-    src, dst, _ = synth.make_graph(V, E, seed=seed, alpha=alpha)
+    src, dst = edges if edges is not None else synth.make_graph(V, E, seed=seed, alpha=alpha)[:2]
     g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V)
     conv = m.Conv(g, "gat", fi, fo, dtype=dtype, heads=H, concat=concat, fuse_relu=relu)
     params = m.init_params("gat", fi, fo, heads=H, concat=concat, seed=seed)
@@ -45,6 +46,10 @@ def run(dtype, H, concat, V=1200, E=15000, fi=24, fo=16, relu=False, seed=0, alp
     errs = {"y": rel_err(f64(y), yo), "dx": rel_err(f64(dx), dxo), "dW": rel_err(f64(grads["W"]), dWo),
             "da_l": rel_err(f64(grads["attn_l"]), dalo), "da_r": rel_err(f64(grads["attn_r"]), daro),
             "db": rel_err(f64(grads["bias"]), dbo)}
+    if zero_attn:   # da_l = da_r = 0 exactly (every softmax is over equal logits): rounding noise vs dW's scale
+        sc = max(np.abs(dWo).max(), 1e-30)
+        errs["da_l"] = float(np.abs(f64(grads["attn_l"]) - dalo).max() / sc)
+        errs["da_r"] = float(np.abs(f64(grads["attn_r"]) - daro).max() / sc)
     return errs, g
 
 

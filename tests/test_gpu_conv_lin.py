@@ -21,8 +21,8 @@ def wg():
     return m
 
 
-def make_inputs(V, E, fi, fo, dtype, seed, alpha=0.6, ints=False):
-    src, dst, _ = synth.make_graph(V, E, seed=seed, alpha=alpha)
+def make_inputs(V, E, fi, fo, dtype, seed, alpha=0.6, ints=False, edges=None):
+    src, dst = edges if edges is not None else synth.make_graph(V, E, seed=seed, alpha=alpha)[:2]
     if ints:
         x = torch.from_numpy(synth.small_ints((V, fi), seed=seed + 1))
         dy = torch.from_numpy(synth.small_ints((V, fo), seed=seed + 2))
@@ -52,9 +52,9 @@ def oracle_layer(model, src, dst, V, x, params, dy, dtype, norm, eps=0.0, amask=
 
 
 def run(model, dtype=torch.float32, policy="auto", V=900, E=12000, fi=37, fo=20, T=128, E_max=0, fuse_relu=False,
-        norm="both", seed=0, ints=False, need_dx=True, alpha=0.6):
+        norm="both", seed=0, ints=False, need_dx=True, alpha=0.6, edges=None):
     m = wg()
-    src, dst, x, dy = make_inputs(V, E, fi, fo, dtype, seed, alpha=alpha, ints=ints)
+    src, dst, x, dy = make_inputs(V, E, fi, fo, dtype, seed, alpha=alpha, ints=ints, edges=edges)
     g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V, tile_rows=T,
                 max_task_edges=E_max)
     conv = m.Conv(g, model, fi, fo, dtype=dtype, policy=policy, seed=seed, fuse_relu=fuse_relu, norm=norm,

@@ -20,9 +20,9 @@ def wg():
 
 
 def run(dtype=torch.float32, policy="auto", norm="none", self_loop=False, bias=False, R=5, V=1500, E=20000, fi=24,
-        fo=16, E_max=0, seed=0, ints=False, relu=False, alpha=0.6):
+        fo=16, E_max=0, seed=0, ints=False, relu=False, alpha=0.6, edges=None):
     m = wg()
-    src, dst, et = synth.make_graph(V, E, seed=seed, alpha=alpha, R=R)
+    src, dst, et = edges if edges is not None else synth.make_graph(V, E, seed=seed, alpha=alpha, R=R)
     g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V,
                 etype=None if et is None else torch.from_numpy(et).cuda(), num_types=R, max_task_edges=E_max)
     conv = m.Conv(g, "rgcn", fi, fo, dtype=dtype, policy=policy, seed=seed, norm=norm, self_loop=self_loop,
