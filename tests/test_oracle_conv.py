@@ -298,3 +298,50 @@ def test_dw_probe_matches_backward():
     v = synth.normal((fo,), seed=44).astype(float)
     _, dW, _ = oracle.gcn_backward(src, dst, V, x, W, dy, norm="none")
     assert abs(oracle.dw_probe(src, dst, x, dy, u, v) - u @ dW @ v) < 1e-10
+
+
+# ------------------------------------------------------- degenerate graphs
+def test_no_edges_closed_forms():
+    # E = 0: every neighbourhood is empty, so each model reduces to its
+    # per-vertex terms (Eq. (1) with an empty sum)
+    V, fi, fo, R, H = 12, 5, 4, 3, 2
+    e = np.zeros(0, np.int32)
+    x = synth.normal((V, fi), seed=40).astype(float)
+    W = synth.normal((fi, fo), seed=41).astype(float)
+    W2 = synth.normal((fo, fo), seed=42).astype(float)
+    b = synth.normal((fo,), seed=43).astype(float)
+    b2 = synth.normal((fo,), seed=44).astype(float)
+    for norm in ("none", "right", "both"):
+        np.testing.assert_array_equal(oracle.gcn_forward(e, e, V, x, W, b, norm=norm), np.tile(b, (V, 1)))
+    np.testing.assert_allclose(oracle.sage_forward(e, e, V, x, W, W, b),
+                               x @ W + b, rtol=1e-13, atol=1e-13)
+    np.testing.assert_allclose(oracle.gin_forward(e, e, V, x, W, b, W2, b2, 0.5),
+                               np.maximum(1.5 * x @ W + b, 0) @ W2 + b2, rtol=1e-13, atol=1e-13)
+    Wr = synth.normal((R, fi, fo), seed=45).astype(float)
+    np.testing.assert_allclose(oracle.rgcn_forward(e, e, e, V, x, Wr, W, b), x @ W + b, rtol=1e-13, atol=1e-13)
+    Wg = synth.normal((fi, H * fo), seed=46).astype(float)
+    al, ar = synth.normal((H, fo), seed=47).astype(float), synth.normal((H, fo), seed=48).astype(float)
+    bg = synth.normal((H * fo,), seed=49).astype(float)
+    np.testing.assert_array_equal(oracle.gat_forward(e, e, V, x, Wg, al, ar, bg, heads=H), np.tile(bg, (V, 1)))
+    # neighbour-path weight gradients vanish
+    dy = synth.normal((V, fo), seed=50).astype(float)
+    assert not np.any(oracle.gcn_backward(e, e, V, x, W, dy, norm="both")[1])
+    assert not np.any(oracle.sage_backward(e, e, V, x, W, W, dy)[2])
+    assert not np.any(oracle.rgcn_backward(e, e, e, V, x, Wr, dy, W)[1])
+
+
+def test_gat_equal_logits_attention_gradient_vanishes():
+    # every in-neighbourhood is copies of one source: each softmax is over
+    # equal logits, y does not depend on a_l / a_r, so da_l = da_r = 0
+    V, fi, fo, H = 20, 4, 3, 2
+    src = np.zeros(90, np.int32)
+    dst = synth.make_graph(V, 90, seed=3)[1]
+    x = synth.normal((V, fi), seed=51).astype(float)
+    W = synth.normal((fi, H * fo), seed=52).astype(float)
+    al, ar = synth.normal((H, fo), seed=53).astype(float), synth.normal((H, fo), seed=54).astype(float)
+    dy = synth.normal((V, H * fo), seed=55).astype(float)
+    y = oracle.gat_forward(src, dst, V, x, W, al, ar, heads=H)
+    has = np.bincount(dst, minlength=V) > 0
+    np.testing.assert_allclose(y[has], np.tile(x[0] @ W, (has.sum(), 1)), rtol=1e-13, atol=1e-13)
+    dx, dW, dal, dar, _ = oracle.gat_backward(src, dst, V, x, W, al, ar, dy, heads=H)
+    assert np.abs(dal).max() < 1e-12 * np.abs(dW).max() and np.abs(dar).max() < 1e-12 * np.abs(dW).max()
