@@ -83,3 +83,14 @@ def test_gat_needs_full_graph():
                 v_end=512)
     with pytest.raises(WGError, match="unsupported"):
         m.Conv(g, "gat", 16, 8, heads=2)
+
+
+@pytest.mark.parametrize("H,fo", [(3, 16), (8, 8), (12, 4), (16, 8), (5, 7)])
+@pytest.mark.parametrize("concat", [True, False])
+def test_gat_head_counts(H, fo, concat):
+    # head counts off the specialised kernels' {1, 2, 4, 8} (generic logits /
+    # der / source-major passes) and above the fused forward's 8-head limit
+    for dtype in (torch.float32, torch.bfloat16):
+        errs, _ = run(dtype, H, concat, V=700, E=7000, fi=20, fo=fo, seed=H)
+        bad = {k: v for k, v in errs.items() if not v <= TOL[dtype]}
+        assert not bad, f"H={H} fo={fo} {dtype}: {errs}"
