@@ -132,7 +132,10 @@ typedef struct {
 
 /* Errors: WG_ERR_INVALID (bad sizes / model / dtype), WG_ERR_UNSUPPORTED
  * (typed graph with a non-RGCN model; GAT on a graph that owns only a row
- * block -- the 1-D partition covers GCN / SAGE / GIN / RGCN).              */
+ * block -- the 1-D partition covers GCN / SAGE / GIN / RGCN).  GAT also
+ * needs f_out * sizeof(dtype) to be a multiple of 16 bytes (one head's row
+ * slice is a whole number of 16-byte vectors); otherwise wg_conv_forward
+ * returns WG_ERR_UNSUPPORTED.                                              */
 wg_status wg_plan_create(wg_graph g, const wg_conv_desc* desc, wg_plan* out);
 /* Bytes of the caller-owned `saved` (forward -> backward) and `workspace`
  * buffers; both 256-byte aligned device memory.                            */

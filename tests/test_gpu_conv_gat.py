@@ -85,7 +85,7 @@ def test_gat_needs_full_graph():
         m.Conv(g, "gat", 16, 8, heads=2)
 
 
-@pytest.mark.parametrize("H,fo", [(3, 16), (8, 8), (12, 4), (16, 8), (5, 7)])
+@pytest.mark.parametrize("H,fo", [(3, 16), (8, 8), (12, 8), (16, 8), (5, 24)])
 @pytest.mark.parametrize("concat", [True, False])
 def test_gat_head_counts(H, fo, concat):
     # head counts off the specialised kernels' {1, 2, 4, 8} (generic logits /
@@ -94,3 +94,12 @@ def test_gat_head_counts(H, fo, concat):
         errs, _ = run(dtype, H, concat, V=700, E=7000, fi=20, fo=fo, seed=H)
         bad = {k: v for k, v in errs.items() if not v <= TOL[dtype]}
         assert not bad, f"H={H} fo={fo} {dtype}: {errs}"
+
+
+@pytest.mark.parametrize("dtype,fo", [(torch.float32, 7), (torch.bfloat16, 4)])
+def test_gat_unaligned_head_width_is_rejected(dtype, fo):
+    # per-head rows narrower than / not a multiple of 16 bytes are refused
+    # loudly (WG_ERR_UNSUPPORTED, include/wg.h), never computed approximately
+    m = wg()
+    with pytest.raises(m.WGError, match="unsupported"):
+        run(dtype, 4, True, V=300, E=2000, fi=16, fo=fo)
