@@ -118,3 +118,12 @@ def test_fewer_edges_than_workers_and_ragged_tile():
             lin.check(lin.run(model, dtype, "random", V=V, E=5, edges=e), dtype)
     check_errs(rgcn.run(torch.float32, "random", V=V, E=5, R=3, edges=typed(e, 3))[0], torch.float32)
     check_errs(gat.run(torch.float32, 4, False, V=V, E=5, edges=e)[0], torch.float32)
+
+
+@pytest.mark.parametrize("policy", ["auto", "edge", "vertex"])
+@pytest.mark.parametrize("dtype", DT)
+def test_rgcn_many_sparse_relations(policy, dtype):
+    # C3 has 100+ relation types with a Zipf mix: on a small graph most
+    # relations hold a handful of edges and some none (their dW_r must be 0)
+    errs, _ = rgcn.run(dtype, policy, V=800, E=4000, R=120, self_loop=True, bias=True, norm="right", seed=11)
+    check_errs(errs, dtype)
