@@ -171,7 +171,10 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
   // ---- VERTEX table: Y = x W (own rows), exchanged in the distributed case
   void* ytab = nullptr;
   int64_t ldY = c.po;
-  if (p->n_vert_tasks > 0) {
+  // a rank with no VERTEX gTask of its own (e.g. no in-edge at all) still
+  // writes its rows of the exchanged Y table when the caller passes one:
+  // the other ranks' VERTEX gathers read them
+  if (p->n_vert_tasks > 0 || (A->xchg && pre)) {
     ytab = A->xchg ? A->xchg : L.at<void>(ws, "y");
     ldY = A->xchg ? A->ld_xchg : c.po;
     if (pre && sage && all_vertex) {

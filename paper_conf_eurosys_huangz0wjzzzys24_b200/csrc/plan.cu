@@ -206,7 +206,9 @@ wg_status plan_create(wg_graph g, const wg_conv_desc* d, wg_plan* out) {
     }
     p->mixed = (p->n_edge_tasks > 0 && p->n_vert_tasks > 0) ? 1 : 0;
     // backward path: dAgg (needs Agg of every row, i.e. no VERTEX task) else G
-    p->bwd_path = p->n_vert_tasks > 0 ? 1 : 0;
+    // (a VERTEX-policy plan without any gTask -- a rank owning no in-edge --
+    // takes the G path too, so every rank exchanges the same table)
+    p->bwd_path = (p->n_vert_tasks > 0 || (p->n_edge_tasks == 0 && d->policy == WG_PLAN_ALL_VERTEX)) ? 1 : 0;
     if (d->model == WG_GAT) gat_layout(p); else lin_layout(p);
   }
   g->live_plans++;

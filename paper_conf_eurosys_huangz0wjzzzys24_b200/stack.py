@@ -61,10 +61,19 @@ class GNNStack:
             pol = policy
             fi = self.f_in[i]
             conv = Conv_(graph, model, fi, dims[i + 1], policy=pol, **kw)
-            if self.dist and model != "rgcn" and conv.n_edge_tasks and conv.n_vertex_tasks:   # uniform plan per layer
-                pol = "vertex" if conv.n_vertex_tasks > conv.n_edge_tasks else "edge"
-                conv.close()
-                conv = Conv_(graph, model, fi, dims[i + 1], policy=pol, **kw)
+            if self.dist and model != "rgcn":   # one uniform plan per layer, the same on every rank
+                ne, nv = conv.n_edge_tasks, conv.n_vertex_tasks
+                if group is not None:   # ranks plan their own rows: vote by gTask counts
+                    dev = self.dev if torch.distributed.get_backend(group) == "nccl" else torch.device("cpu")
+                    votes = torch.tensor([ne, nv], dtype=torch.int64, device=dev)
+                    torch.distributed.all_reduce(votes, group=group)
+                    ne, nv = (int(v) for v in votes.tolist())
+                uni = "vertex" if nv > ne else "edge"
+                if (conv.n_vertex_tasks if uni == "edge" else conv.n_edge_tasks) or \
+                        (uni == "vertex" and not conv.n_vertex_tasks and pol != "vertex"):
+                    pol = uni
+                    conv.close()
+                    conv = Conv_(graph, model, fi, dims[i + 1], policy=pol, **kw)
             self.convs.append(conv)
             self._share_workspace(conv)
             self.params.append(init_params(model, fi, dims[i + 1], heads=heads, concat=not last, R=R,

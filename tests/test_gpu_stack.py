@@ -47,12 +47,15 @@ def test_softmax_xent(dtype, C):
 
 @pytest.mark.parametrize("model,policy", [("sage", "edge"), ("sage", "vertex"), ("gcn", "edge"), ("gin", "vertex")])
 @pytest.mark.parametrize("P", [2, 3])
-def test_1d_partition_phases_match_single(model, policy, P):
+@pytest.mark.parametrize("graph", ["powerlaw", "star"])
+def test_1d_partition_phases_match_single(model, policy, P, graph):
     m = wg()
     from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import partition_1d
     V, E, fi, fo = 3000, 40000, 48, 40
     dtype = torch.float32
     src, dst, _ = synth.make_graph(V, E, seed=31, alpha=0.6)
+    if graph == "star":   # every edge into vertex 5: ranks > 0 own no in-edge (no forward gTask)
+        dst = np.full(E, 5, np.int32)
     x = torch.from_numpy(synth.make_features(V, fi, seed=32)).cuda()
     dy = torch.from_numpy(synth.normal((V, fo), seed=33, std=0.2)).cuda()
     params = m.init_params(model, fi, fo, seed=3)
