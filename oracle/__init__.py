@@ -59,7 +59,7 @@ def _L():
         _lib.wgo_gcn_backward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P, P]
         _lib.wgo_sage_forward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P]
         _lib.wgo_sage_backward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P, P, P, P]
-        _lib.wgo_gin_forward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, f64, P, P, P, P, P, P]
+        _lib.wgo_gin_forward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, f64, P, P, P, P, P, P, P, P, P]
         _lib.wgo_gin_backward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, f64, P, P, P, P, P, P, P, P, P, P, P]
         _lib.wgo_rgcn_forward.argtypes = [i64, i64, P, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P]
         _lib.wgo_rgcn_backward.argtypes = [i64, i64, P, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P, P, P, P]
@@ -172,24 +172,32 @@ def sage_backward(src, dst, V, x, Ws, Wn, dy, rows=None, grads=True):
     return dx, dWs, dWn, db
 
 
-def gin_forward(src, dst, V, x, W1, b1, W2, b2, eps=0.0):
+def gin_forward(src, dst, V, x, W1, b1, W2, b2, eps=0.0, rows=None, return_za=False):
+    """rows: produce only these rows; return_za: also return z [V x fi] and the
+    pre-activation a = z W1 + b1 [V x fo] of the produced rows."""
     x, W1, b1, W2, b2 = map(_f64, (x, W1, b1, W2, b2))
     fi, fo = W1.shape
     y = np.zeros((V, fo))
+    z = np.zeros((V, fi)) if return_za else None
+    a = np.zeros((V, fo)) if return_za else None
     s, d = _i32(src), _i32(dst)
-    _L().wgo_gin_forward(V, s.shape[0], _p(s), _p(d), fi, fo, float(eps), _p(x), _p(W1), _p(b1), _p(W2), _p(b2), _p(y))
-    return y
+    m = _mask(V, rows)
+    _L().wgo_gin_forward(V, s.shape[0], _p(s), _p(d), fi, fo, float(eps), _p(x), _p(W1), _p(b1), _p(W2), _p(b2),
+                         _p(m), _p(y), _p(z), _p(a))
+    return (y, z, a) if return_za else y
 
 
-def gin_backward(src, dst, V, x, W1, b1, W2, dy, eps=0.0, amask=None):
-    """amask: optional [V x fo] ReLU decisions taken by the implementation under test."""
+def gin_backward(src, dst, V, x, W1, b1, W2, dy, eps=0.0, dy_rows=None):
+    """Exact gradients; the ReLU decision [a > 0] is taken here, in fp64.
+    dy_rows: rows of dy outside this set are zero (skipped); dx is still
+    produced for every vertex."""
     x, W1, b1, W2, dy = map(_f64, (x, W1, b1, W2, dy))
-    am = None if amask is None else np.ascontiguousarray(amask, dtype=np.uint8)
     fi, fo = W1.shape
     dx, dW1, db1, dW2, db2 = np.zeros((V, fi)), np.zeros((fi, fo)), np.zeros(fo), np.zeros((fo, fo)), np.zeros(fo)
     s, d = _i32(src), _i32(dst)
+    m = _mask(V, dy_rows)
     _L().wgo_gin_backward(V, s.shape[0], _p(s), _p(d), fi, fo, float(eps), _p(x), _p(W1), _p(b1), _p(W2), _p(dy),
-                          _p(am), _p(dx), _p(dW1), _p(db1), _p(dW2), _p(db2))
+                          _p(m), _p(dx), _p(dW1), _p(db1), _p(dW2), _p(db2))
     return dx, dW1, db1, dW2, db2
 
 

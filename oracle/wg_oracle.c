@@ -287,38 +287,52 @@ void wgo_sage_backward(int64_t V, int64_t E, const int32_t* src, const int32_t* 
 /* GIN (Xu et al., ICLR'19 -- not in the paper; BASELINE north_star; Q5)    */
 /*   z[v] = (1+eps) x[v] + sum_{e in in(v)} x[s_e]                           */
 /*   a = z W1 + b1 ;  h = ReLU(a) ;  y = h W2 + b2                           */
-/* saved (optional, [V x fo] each): a (pre-activation)                      */
+/* The ReLU decision is the oracle's own, [a > 0] in fp64 (ReLU'(0) = 0).   */
 /* ======================================================================== */
-static void gin_z(int64_t V, int64_t E, const int32_t* src, const int32_t* dst, int fi,
-                  double eps, const double* x, double* z) {
-    for (int64_t v = 0; v < V; ++v) for (int k = 0; k < fi; ++k) z[v * fi + k] = (1.0 + eps) * x[v * fi + k];
-    for (int64_t e = 0; e < E; ++e)
-        for (int k = 0; k < fi; ++k) z[(int64_t)dst[e] * fi + k] += x[(int64_t)src[e] * fi + k];
+static void gin_z_row(int64_t v, int fi, double eps, const double* x, double* zv) {
+    for (int k = 0; k < fi; ++k) zv[k] = (1.0 + eps) * x[v * fi + k];
 }
 
+/* z for the rows of row_mask (all rows when NULL): self term, then one pass
+ * over the edges adding x[s_e] into z[d_e] (the edge loop of Eq. (1)). */
+static void gin_z(int64_t V, int64_t E, const int32_t* src, const int32_t* dst, int fi,
+                  double eps, const double* x, const uint8_t* row_mask, double* z) {
+    for (int64_t v = 0; v < V; ++v) if (ROW_ON(row_mask, v)) gin_z_row(v, fi, eps, x, z + v * fi);
+    for (int64_t e = 0; e < E; ++e) {
+        if (!ROW_ON(row_mask, dst[e])) continue;
+        for (int k = 0; k < fi; ++k) z[(int64_t)dst[e] * fi + k] += x[(int64_t)src[e] * fi + k];
+    }
+}
+
+/* row_mask (nullable): only rows v with row_mask[v] != 0 are produced.
+ * z_out ([V x fi]) and a_out ([V x fo], the pre-activation) are optional
+ * outputs for the produced rows. */
 void wgo_gin_forward(int64_t V, int64_t E, const int32_t* src, const int32_t* dst, int fi, int fo,
                      double eps, const double* x, const double* W1, const double* b1,
-                     const double* W2, const double* b2, double* y) {
-    double* z = malloc(sizeof(double) * V * fi);
+                     const double* W2, const double* b2, const uint8_t* row_mask, double* y,
+                     double* z_out, double* a_out) {
+    double* z = z_out ? z_out : malloc(sizeof(double) * V * fi);
     double* a = malloc(sizeof(double) * fo);
-    gin_z(V, E, src, dst, fi, eps, x, z);
+    gin_z(V, E, src, dst, fi, eps, x, row_mask, z);
     for (int64_t v = 0; v < V; ++v) {
+        if (!ROW_ON(row_mask, v)) continue;
         for (int j = 0; j < fo; ++j) a[j] = b1 ? b1[j] : 0.0;
         add_msg(fi, fo, 1.0, z + v * fi, W1, a);
+        if (a_out) for (int j = 0; j < fo; ++j) a_out[v * fo + j] = a[j];
         for (int j = 0; j < fo; ++j) { a[j] = a[j] > 0.0 ? a[j] : 0.0; y[v * fo + j] = b2 ? b2[j] : 0.0; }
         add_msg(fo, fo, 1.0, a, W2, y + v * fo);
     }
-    free(z); free(a);
+    if (!z_out) free(z);
+    free(a);
 }
 
 /* dW2 = h^T dy ; da = (dy W2^T) * [a > 0] ; dW1 = z^T da ; dz = da W1^T ;
- * dx[u] = (1+eps) dz[u] + sum_{e in out(u)} dz[d_e] ; db1 = sum da ; db2 = sum dy */
-/* amask (nullable, [V x fo] bytes): the ReLU decision [a > 0] taken by the
- * implementation under test in its own precision (a float deciding an integer
- * is decided by one side only); NULL = use a > 0. */
+ * dx[u] = (1+eps) dz[u] + sum_{e in out(u)} dz[d_e] ; db1 = sum da ; db2 = sum dy
+ * dy_rows (nullable): rows of dy outside this set are ZERO (they are skipped);
+ * every output is then the exact gradient for that dy (dx for all V). */
 void wgo_gin_backward(int64_t V, int64_t E, const int32_t* src, const int32_t* dst, int fi, int fo,
                       double eps, const double* x, const double* W1, const double* b1,
-                      const double* W2, const double* dy, const uint8_t* amask, double* dx, double* dW1,
+                      const double* W2, const double* dy, const uint8_t* dy_rows, double* dx, double* dW1,
                       double* db1, double* dW2, double* db2) {
     double* z = malloc(sizeof(double) * V * fi);
     double* dz = malloc(sizeof(double) * V * fi);
@@ -326,30 +340,32 @@ void wgo_gin_backward(int64_t V, int64_t E, const int32_t* src, const int32_t* d
     double* h = malloc(sizeof(double) * fo);
     double* dh = malloc(sizeof(double) * fo);
     double* da = malloc(sizeof(double) * fo);
-    gin_z(V, E, src, dst, fi, eps, x, z);
+    gin_z(V, E, src, dst, fi, eps, x, dy_rows, z);
     memset(dz, 0, sizeof(double) * V * fi);
     if (dW1) memset(dW1, 0, sizeof(double) * fi * fo);
     if (dW2) memset(dW2, 0, sizeof(double) * fo * fo);
     if (db1) memset(db1, 0, sizeof(double) * fo);
     if (db2) memset(db2, 0, sizeof(double) * fo);
     for (int64_t v = 0; v < V; ++v) {
+        if (!ROW_ON(dy_rows, v)) continue;
         for (int j = 0; j < fo; ++j) a[j] = b1 ? b1[j] : 0.0;
         add_msg(fi, fo, 1.0, z + v * fi, W1, a);
         for (int j = 0; j < fo; ++j) {
-            int on = amask ? amask[v * fo + j] != 0 : a[j] > 0.0;
-            h[j] = on ? a[j] : 0.0;
+            h[j] = a[j] > 0.0 ? a[j] : 0.0;
             dh[j] = 0.0;
         }
         if (db2) for (int j = 0; j < fo; ++j) db2[j] += dy[v * fo + j];
         add_msg_grad(fo, fo, 1.0, h, W2, dy + v * fo, dh, dW2);
-        for (int j = 0; j < fo; ++j) da[j] = (amask ? amask[v * fo + j] != 0 : a[j] > 0.0) ? dh[j] : 0.0;
+        for (int j = 0; j < fo; ++j) da[j] = a[j] > 0.0 ? dh[j] : 0.0;
         if (db1) for (int j = 0; j < fo; ++j) db1[j] += da[j];
         add_msg_grad(fi, fo, 1.0, z + v * fi, W1, da, dz + v * fi, dW1);
     }
     if (dx) {
         for (int64_t u = 0; u < V; ++u) for (int k = 0; k < fi; ++k) dx[u * fi + k] = (1.0 + eps) * dz[u * fi + k];
-        for (int64_t e = 0; e < E; ++e)
+        for (int64_t e = 0; e < E; ++e) {
+            if (!ROW_ON(dy_rows, dst[e])) continue;
             for (int k = 0; k < fi; ++k) dx[(int64_t)src[e] * fi + k] += dz[(int64_t)dst[e] * fi + k];
+        }
     }
     free(z); free(dz); free(a); free(h); free(dh); free(da);
 }

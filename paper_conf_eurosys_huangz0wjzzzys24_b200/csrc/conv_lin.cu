@@ -77,18 +77,21 @@ void lin_layout(wg_plan_s* p) {
   if (gin) {
     W.add("w2t", (size_t)c.wrows_o * c.po * s);
     W.add("w2", (size_t)c.wrows_o * c.po * s);
-    W.add("da", (size_t)c.Vg * c.po * s);
+    W.add("da", (size_t)c.nr * c.po * s);
   }
-  if (p->n_vert_tasks > 0) W.add("y", (size_t)c.Vg * c.po * s);
+  // tables the gathers read (Y, dT, dAgg, GIN da) live here only on a full
+  // graph (nr == V); on a 1-D partition they are the caller's exchange
+  // tables (global rows), so these buffers hold owned rows only
+  if (p->n_vert_tasks > 0) W.add("y", (size_t)c.nr * c.po * s);
   if (p->mixed) W.add("z", (size_t)c.nr * c.po * s);
   const int64_t pl = part_ld(c);
   W.add("part", sizeof(float) * (size_t)std::max(1, p->n_slots_f) * pl);
   W.add("partT", sizeof(float) * (size_t)std::max(1, p->n_slots_t) * pl);
   // backward
-  W.add("dt", (size_t)c.Vg * c.po * s);
+  W.add("dt", (size_t)c.nr * c.po * s);
   W.add("colsum", bias_grad_scratch(c.nr, (int)std::max(c.po, c.pi)));
   W.add("tn", gemm_tn_scratch(c.nr, (int)c.fi, (int)c.fo) + gemm_tn_scratch(c.nr, (int)c.fo, (int)c.fo));
-  W.add("dagg", (size_t)c.Vg * c.pi * s);
+  W.add("dagg", (size_t)c.nr * c.pi * s);
   W.add("g", (size_t)c.nr * c.po * s);
 }
 
@@ -153,6 +156,12 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
          "ldx / ldy must be >= F and 16-byte multiples");
   const bool dist = c.nr != c.Vg;
   WG_REQ(!dist || !p->mixed, WG_ERR_UNSUPPORTED, "mixed EDGE/VERTEX plans are not supported with a 1-D partition");
+  // on a 1-D partition the VERTEX gathers read Y rows other ranks own: the
+  // exchange table is required (the workspace holds owned rows only)
+  WG_REQ(!dist || !post || p->n_vert_tasks == 0 || A->xchg, WG_ERR_INVALID,
+         "a VERTEX layer on a 1-D partition needs the exchange table (xchg)");
+  WG_REQ(!A->xchg || ((A->ld_xchg * c.s) % 16 == 0 && A->ld_xchg >= c.fo), WG_ERR_INVALID,
+         "ld_xchg must be >= f_out and a 16-byte multiple");
   void* ws = A->workspace;
   const Layout& L = p->ws;
   const char* x_own = off(A->x, c.vb, A->ldx, c.s);
@@ -275,6 +284,11 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   // dy already masked by the next layer (dx_mask fusion): no mask pass here
   const bool mask_dy = d.fuse_relu && !A->dy_masked;
   const bool dist = c.nr != c.Vg;
+  // on a 1-D partition the transposed gather reads rows other ranks own
+  // (dT / dAgg / GIN da): the exchange table is required
+  WG_REQ(!dist || !post || (p->bwd_path == 0 && !d.need_dx) || A->xchg, WG_ERR_INVALID,
+         "backward on a 1-D partition needs the exchange table (xchg)");
+  WG_REQ(!A->xchg || (A->ld_xchg * c.s) % 16 == 0, WG_ERR_INVALID, "ld_xchg must be a 16-byte multiple");
   void* ws = A->workspace;
   const Layout& L = p->ws;
   const char* x_own = off(A->x, c.vb, A->ldx, c.s);
@@ -309,9 +323,9 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   void* dt_fold = nullptr;                 // G path, folded: the scaled rows in the exchange table
   if (gpath_lin && xchg && fold) {
     dt_fold = off(xchg, c.vb, A->ld_xchg, c.s);
-    if (mask_dy) dt_buf = off(L.at<void>(ws, "dt"), c.vb, c.po, c.s);
+    if (mask_dy) dt_buf = L.at<void>(ws, "dt");             // owned rows, local indexing
   } else if (gpath_lin && xchg) { dt_buf = off(xchg, c.vb, A->ld_xchg, c.s); ld_dtb = A->ld_xchg; }
-  else if (mask_dy) { dt_buf = off(L.at<void>(ws, "dt"), c.vb, c.po, c.s); ld_dtb = c.po; }
+  else if (mask_dy) { dt_buf = L.at<void>(ws, "dt"); ld_dtb = c.po; }
   if (pre) {
     float* db = gin ? (G ? G->b2 : nullptr) : (G ? G->bias : nullptr);
     if (dt_buf || db || dt_fold)
@@ -333,7 +347,7 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
     void* h = p->saved.at<void>(A->saved, "h");
     gin_tab = (path == 1 && xchg) ? xchg : L.at<void>(ws, "da");
     ld_gin = (path == 1 && xchg) ? A->ld_xchg : c.po;
-    void* da = off(gin_tab, c.vb, ld_gin, c.s);
+    void* da = off(gin_tab, (path == 1 && xchg) ? c.vb : 0, ld_gin, c.s);   // ws "da": owned rows
     if (pre) {
       if (G && G->W2) WG_TRY(gemm_tn(c.dt, c.nr, c.fo, c.fo, h, c.po, dT, lddT, G->W2, tn, st));
       void* w2 = L.at<void>(ws, "w2");

@@ -9,7 +9,7 @@ import torch
 
 import oracle
 import synth
-from tests.util import TOL, f64, q, rel_err
+from tests.util import TOL, assert_mask_agrees, f64, kink_band, q, rel_err, relu_dy
 
 pytestmark = pytest.mark.gpu
 
@@ -33,15 +33,20 @@ def run(dtype, H, concat, V=1200, E=15000, fi=24, fo=16, relu=False, seed=0, alp
     dy = torch.from_numpy(synth.normal((V, FO), seed=seed + 2, std=0.3)).to(dtype)
     xd = m.pad_to(x.cuda())
     y, saved = conv.forward_raw(xd, params)
-    dx, grads = conv.backward_raw(m.pad_to(dy.cuda()), xd, y, saved, params)
     torch.cuda.synchronize()
     W = q(params["W"], dtype)
     al, ar, b = f64(params["attn_l"]), f64(params["attn_r"]), f64(params["bias"])
     yo = oracle.gat_forward(src, dst, V, f64(x), W, al, ar, b, heads=H, concat=concat)
     dyo = f64(dy)
-    if relu:
-        dyo = dyo * (f64(y) > 0)
+    if relu:   # the oracle's own ReLU decision; dy = 0 on the kink band (tests/util.py)
+        band = kink_band(yo, None, dtype)
+        assert_mask_agrees(f64(y), yo, band)
+        dy_np, dyo = relu_dy(dyo, yo, band)
+        dy = torch.from_numpy(dy_np).to(dtype)
+        dyo = f64(dy) * (yo > 0)
         yo = np.maximum(yo, 0)
+    dx, grads = conv.backward_raw(m.pad_to(dy.cuda()), xd, y, saved, params)
+    torch.cuda.synchronize()
     dxo, dWo, dalo, daro, dbo = oracle.gat_backward(src, dst, V, f64(x), W, al, ar, dyo, heads=H, concat=concat)
     errs = {"y": rel_err(f64(y), yo), "dx": rel_err(f64(dx), dxo), "dW": rel_err(f64(grads["W"]), dWo),
             "da_l": rel_err(f64(grads["attn_l"]), dalo), "da_r": rel_err(f64(grads["attn_r"]), daro),

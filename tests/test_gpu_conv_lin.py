@@ -11,7 +11,8 @@ import torch
 
 import oracle
 import synth
-from tests.util import TOL, f64, q, rel_err
+from tests.util import (TOL, assert_mask_agrees, f64, gin_inner_safe_dy, kink_band, q, rel_err,
+                        relu_dy)
 
 pytestmark = pytest.mark.gpu
 
@@ -32,23 +33,57 @@ def make_inputs(V, E, fi, fo, dtype, seed, alpha=0.6, ints=False, edges=None):
     return src, dst, x.to(dtype), dy.to(dtype)
 
 
-def oracle_layer(model, src, dst, V, x, params, dy, dtype, norm, eps=0.0, amask=None):
-    Wq = {k: q(v, dtype) for k, v in params.items()}
-    xo = f64(x)
+def oracle_fwd(model, src, dst, V, xo, Wq, norm, eps=0.0):
+    """Oracle forward (before any output ReLU); GIN also returns its inner
+    pre-activation a = z W1 + b1."""
     if model == "gcn":
-        y = oracle.gcn_forward(src, dst, V, xo, Wq["W"], Wq.get("bias"), norm=norm)
-        dx, dW, db = oracle.gcn_backward(src, dst, V, xo, Wq["W"], dy, norm=norm)
-        return y, dx, {"W": dW, "bias": db}
+        return oracle.gcn_forward(src, dst, V, xo, Wq["W"], Wq.get("bias"), norm=norm), None
     if model == "sage":
-        y = oracle.sage_forward(src, dst, V, xo, Wq["W_self"], Wq["W"], Wq.get("bias"))
-        dx, dWs, dWn, db = oracle.sage_backward(src, dst, V, xo, Wq["W_self"], Wq["W"], dy)
-        return y, dx, {"W": dWn, "W_self": dWs, "bias": db}
+        return oracle.sage_forward(src, dst, V, xo, Wq["W_self"], Wq["W"], Wq.get("bias")), None
     if model == "gin":
-        y = oracle.gin_forward(src, dst, V, xo, Wq["W"], Wq["bias"], Wq["W2"], Wq["b2"], eps)
-        dx, dW1, db1, dW2, db2 = oracle.gin_backward(src, dst, V, xo, Wq["W"], Wq["bias"], Wq["W2"], dy, eps,
-                                                     amask=amask)
-        return y, dx, {"W": dW1, "bias": db1, "W2": dW2, "b2": db2}
+        y, _, a = oracle.gin_forward(src, dst, V, xo, Wq["W"], Wq["bias"], Wq["W2"], Wq["b2"], eps, return_za=True)
+        return y, a
     raise ValueError(model)
+
+
+def oracle_bwd(model, src, dst, V, xo, Wq, dT, norm, eps=0.0):
+    if model == "gcn":
+        dx, dW, db = oracle.gcn_backward(src, dst, V, xo, Wq["W"], dT, norm=norm)
+        return dx, {"W": dW, "bias": db}
+    if model == "sage":
+        dx, dWs, dWn, db = oracle.sage_backward(src, dst, V, xo, Wq["W_self"], Wq["W"], dT)
+        return dx, {"W": dWn, "W_self": dWs, "bias": db}
+    if model == "gin":
+        dx, dW1, db1, dW2, db2 = oracle.gin_backward(src, dst, V, xo, Wq["W"], Wq["bias"], Wq["W2"], dT, eps)
+        return dx, {"W": dW1, "bias": db1, "W2": dW2, "b2": db2}
+    raise ValueError(model)
+
+
+def oracle_dy(model, src, dst, V, xo, Wq, dy, dtype, norm, fuse_relu, y_gpu=None, h_gpu=None, exact=False):
+    """Oracle forward + the kink-band-safe dy (tests/util.py): returns
+    (pre, dy_in for the kernel, dT for the oracle backward).  y_gpu / h_gpu
+    (optional) are checked to take the oracle's ReLU decisions outside the band."""
+    pre, a = oracle_fwd(model, src, dst, V, xo, Wq, norm)
+    Wabs = {k: np.abs(v) for k, v in Wq.items()}
+    mag, _, mag_a = (oracle.gin_forward(src, dst, V, np.abs(xo), Wabs["W"], Wabs["bias"], Wabs["W2"], Wabs["b2"],
+                                        return_za=True) if model == "gin"
+                     else (oracle_fwd(model, src, dst, V, np.abs(xo), Wabs, norm)[0], None, None))
+    dy = np.asarray(dy, dtype=np.float64)
+    free = None
+    if fuse_relu:
+        band = kink_band(pre, mag, dtype, exact)
+        if y_gpu is not None:
+            assert_mask_agrees(y_gpu, pre, band, "output ReLU")
+        dy, _ = relu_dy(dy, pre, band)
+        free = (pre > 0) & ~band
+    if model == "gin":
+        band_a = kink_band(a, mag_a, dtype, exact)
+        if h_gpu is not None:
+            assert_mask_agrees(h_gpu, a, band_a, "GIN inner ReLU")
+        dy = gin_inner_safe_dy(dy, a, band_a, Wq["W2"], free)
+    dy_in = torch.from_numpy(dy).to(dtype)
+    dT = f64(dy_in) * (pre > 0) if fuse_relu else f64(dy_in)
+    return pre, dy_in, dT
 
 
 def run(model, dtype=torch.float32, policy="auto", V=900, E=12000, fi=37, fo=20, T=128, E_max=0, fuse_relu=False,
@@ -68,19 +103,17 @@ def run(model, dtype=torch.float32, policy="auto", V=900, E=12000, fi=37, fo=20,
         params = {k: (v + 0.1 * torch.randn(v.shape, generator=gen, device=v.device)) for k, v in params.items()}
     xd = m.pad_to(x.cuda())
     y, saved = conv.forward_raw(xd, params)
-    dyd = m.pad_to(dy.cuda())
-    dx, grads = conv.backward_raw(dyd, xd, y, saved, params)
     torch.cuda.synchronize()
     yg = f64(y)
-    dyo = f64(dy)
-    if fuse_relu:
-        dyo = dyo * (yg > 0)       # the mask decision is the kernel's (its own output)
-    amask = None
-    if model == "gin":   # GIN's inner ReLU decision is the kernel's (taken on its fp32 accumulator)
-        amask = (f64(conv.buffer_view(saved, "h", V, fo)) > 0).astype(np.uint8)
-    yo, dxo, go = oracle_layer(model, src, dst, V, x, params, dyo, dtype, norm, amask=amask)
-    if fuse_relu:
-        yo = np.maximum(yo, 0)
+    Wq = {k: q(v, dtype) for k, v in params.items()}
+    xo = f64(x)
+    hg = f64(conv.buffer_view(saved, "h", V, fo)) if model == "gin" else None
+    pre, dy_in, dT = oracle_dy(model, src, dst, V, xo, Wq, f64(dy), dtype, norm, fuse_relu, y_gpu=yg, h_gpu=hg,
+                                exact=ints)
+    dx, grads = conv.backward_raw(m.pad_to(dy_in.cuda()), xd, y, saved, params)
+    torch.cuda.synchronize()
+    dxo, go = oracle_bwd(model, src, dst, V, xo, Wq, dT, norm)
+    yo = np.maximum(pre, 0) if fuse_relu else pre
     return dict(conv=conv, y=(yg, yo), dx=(f64(dx) if need_dx else None, dxo),
                 grads={k: (f64(grads[k]), go[k]) for k in go if k in grads})
 

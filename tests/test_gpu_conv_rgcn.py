@@ -9,7 +9,7 @@ import torch
 
 import oracle
 import synth
-from tests.util import TOL, f64, q, rel_err
+from tests.util import TOL, assert_mask_agrees, f64, kink_band, q, rel_err, relu_dy
 
 pytestmark = pytest.mark.gpu
 
@@ -40,14 +40,22 @@ def run(dtype=torch.float32, policy="auto", norm="none", self_loop=False, bias=F
         dy = torch.from_numpy(synth.normal((V, fo), seed=seed + 2, std=0.25)).to(dtype)
     xd = m.pad_to(x.cuda())
     y, saved = conv.forward_raw(xd, params)
-    dx, grads = conv.backward_raw(m.pad_to(dy.cuda()), xd, y, saved, params)
     torch.cuda.synchronize()
     Wq = {k: q(v, dtype) for k, v in params.items()}
     yo = oracle.rgcn_forward(src, dst, et, V, f64(x), Wq["W"], Wq.get("W_self"), Wq.get("bias"), norm=norm)
     dyo = f64(dy)
-    if relu:
-        dyo = dyo * (f64(y) > 0)
+    if relu:   # the oracle's own ReLU decision; dy = 0 on the kink band (tests/util.py)
+        Wa = {k: np.abs(v) for k, v in Wq.items()}
+        mag = oracle.rgcn_forward(src, dst, et, V, np.abs(f64(x)), Wa["W"], Wa.get("W_self"), Wa.get("bias"),
+                                  norm=norm)
+        band = kink_band(yo, mag, dtype, exact=ints)
+        assert_mask_agrees(f64(y), yo, band)
+        dy_np, _ = relu_dy(dyo, yo, band)
+        dy = torch.from_numpy(dy_np).to(dtype)
+        dyo = f64(dy) * (yo > 0)
         yo = np.maximum(yo, 0)
+    dx, grads = conv.backward_raw(m.pad_to(dy.cuda()), xd, y, saved, params)
+    torch.cuda.synchronize()
     dxo, dWo, dW0o, dbo = oracle.rgcn_backward(src, dst, et, V, f64(x), Wq["W"], dyo, Wq.get("W_self"), norm=norm)
     errs = {"y": rel_err(f64(y), yo), "dx": rel_err(f64(dx), dxo), "dW": rel_err(f64(grads["W"]), dWo)}
     if self_loop:
@@ -124,14 +132,22 @@ def test_rgcn_1d_partition_phases_match_oracle(policy, P):
         ranks.append((g, c, vb, ve, c.new_saved()))
     for g, c, vb, ve, sv in ranks:
         c.forward_raw(xt, params, y=yt[vb:ve], saved=sv, phase=2)
+    torch.cuda.synchronize()
+    Wq = {k: f64(v) for k, v in params.items()}
+    pre = oracle.rgcn_forward(src, dst, et, V, f64(x), Wq["W"], Wq["W_self"], Wq["bias"], norm="right")
+    Wa = {k: np.abs(v) for k, v in Wq.items()}
+    mag = oracle.rgcn_forward(src, dst, et, V, np.abs(f64(x)), Wa["W"], Wa["W_self"], Wa["bias"], norm="right")
+    band = kink_band(pre, mag, dtype)
+    assert_mask_agrees(f64(yt[:V]), pre, band)
+    dy_np, _ = relu_dy(f64(dy), pre, band)
+    dyt[:V] = torch.from_numpy(dy_np).to(dtype).cuda()
     grads = [{k: torch.zeros_like(v) for k, v in params.items()} for _ in ranks]
     for ph in (1, 2):
         for (g, c, vb, ve, sv), gr in zip(ranks, grads):
             c.backward_raw(dyt[vb:ve], xt, yt[vb:ve], sv, params, dx=dxt[vb:ve], phase=ph, xchg=xb, grads=gr)
     torch.cuda.synchronize()
-    Wq = {k: f64(v) for k, v in params.items()}
-    yo = np.maximum(oracle.rgcn_forward(src, dst, et, V, f64(x), Wq["W"], Wq["W_self"], Wq["bias"], norm="right"), 0)
-    dyo = f64(dy) * (f64(yt[:V]) > 0)
+    yo = np.maximum(pre, 0)
+    dyo = f64(dyt[:V]) * (pre > 0)
     dxo, dWo, dW0o, dbo = oracle.rgcn_backward(src, dst, et, V, f64(x), Wq["W"], dyo, Wq["W_self"], norm="right")
     tot = {k: sum(gr[k] for gr in grads) for k in params}
     errs = {"y": rel_err(f64(yt[:V]), yo), "dx": rel_err(f64(dxt[:V]), dxo), "dW": rel_err(f64(tot["W"]), dWo),

@@ -148,6 +148,57 @@ def test_gin_dense(eps):
         np.testing.assert_allclose(g, tt.grad.numpy(), rtol=1e-11, atol=1e-11)
 
 
+def test_gin_rows_za_and_dy_rows():
+    """Row-restricted forward == full forward on those rows; z and the
+    pre-activation a are the dense z = (1+eps)x + A x, a = z W1 + b1; the
+    dy_rows backward equals autograd with dy zeroed outside the rows (dx for
+    every vertex)."""
+    src, dst, _ = tgraph(8)
+    V, fi, fo, eps = 40, 5, 6, 0.5
+    x = synth.normal((V, fi), seed=20).astype(float)
+    W1 = synth.normal((fi, fo), seed=21).astype(float)
+    b1 = synth.normal((fo,), seed=22).astype(float)
+    W2 = synth.normal((fo, fo), seed=23).astype(float)
+    b2 = synth.normal((fo,), seed=24).astype(float)
+    A = dense_adj(src, dst, V)
+    rows = np.array([0, 3, 7, 11, 39])
+    y, z, a = oracle.gin_forward(src, dst, V, x, W1, b1, W2, b2, eps, rows=rows, return_za=True)
+    zr = (1 + eps) * x + A @ x
+    np.testing.assert_allclose(z[rows], zr[rows], rtol=1e-12, atol=1e-12)
+    np.testing.assert_allclose(a[rows], (zr @ W1 + b1)[rows], rtol=1e-12, atol=1e-12)
+    np.testing.assert_allclose(y[rows], (np.maximum(zr @ W1 + b1, 0) @ W2 + b2)[rows], rtol=1e-12, atol=1e-12)
+    dy = synth.normal((V, fo), seed=25).astype(float)
+    dyz = np.zeros_like(dy)
+    dyz[rows] = dy[rows]
+    t = [torch.tensor(v, requires_grad=True) for v in (x, W1, b1, W2, b2)]
+    zz = (1 + eps) * t[0] + torch.tensor(A) @ t[0]
+    (torch.relu(zz @ t[1] + t[2]) @ t[3] + t[4]).backward(torch.tensor(dyz))
+    got = oracle.gin_backward(src, dst, V, x, W1, b1, W2, dy, eps, dy_rows=rows)
+    for g, tt in zip(got, t):
+        np.testing.assert_allclose(g, tt.grad.numpy(), rtol=1e-11, atol=1e-11)
+
+
+def test_gin_relu_derivative_at_zero():
+    """Integer inputs with pre-activations exactly 0: ReLU'(0) = 0 (Q8 / SURVEY
+    c3), as torch.relu's backward."""
+    src, dst, _ = tgraph(9)
+    V, fi, fo = 40, 3, 4
+    x = synth.small_ints((V, fi), seed=30).astype(float)
+    W1 = synth.small_ints((fi, fo), seed=31).astype(float)
+    b1 = np.zeros(fo)
+    W2 = synth.small_ints((fo, fo), seed=32).astype(float)
+    _, _, a = oracle.gin_forward(src, dst, V, x, W1, b1, W2, np.zeros(fo), return_za=True)
+    assert (a == 0).any()          # the kink is hit exactly
+    dy = synth.small_ints((V, fo), seed=33).astype(float)
+    A = dense_adj(src, dst, V)
+    t = [torch.tensor(v, requires_grad=True) for v in (x, W1, b1, W2)]
+    zz = t[0] + torch.tensor(A) @ t[0]
+    (torch.relu(zz @ t[1] + t[2]) @ t[3]).backward(torch.tensor(dy))
+    got = oracle.gin_backward(src, dst, V, x, W1, b1, W2, dy)
+    for g, tt in zip((got[0], got[1], got[2], got[3]), t):
+        np.testing.assert_array_equal(g, tt.grad.numpy())
+
+
 def test_gin_special_case_neighbour_sum():
     # eps = -1, W1 = W2 = I, b = 0, x >= 0: pure neighbour sum
     src, dst, _ = tgraph(6)

@@ -22,3 +22,65 @@ def q(t, dtype):
 
 def f64(t):
     return t.to(torch.float64).cpu().numpy()
+
+
+# ---------------------------------------------------------------------------
+# ReLU decisions (DESIGN.md §2 "Kink band").  Every mask the oracle applies is
+# its own, [pre > 0] on its fp64 pre-activation.  The kernel decides on its own
+# rounded pre-activation, which may differ from the oracle's only where
+# |pre| is below the rounding-error bound of the kernel's arithmetic path:
+#   |pre_gpu - pre| <= K * u * mag,   mag = the same computation on |inputs|
+# (every value the kernel stores on the way is rounded once to the conv dtype,
+# unit roundoff u; fp32 accumulation error is << u at these depths; the fp32
+# path is 3xTF32, ~2^-21 per product).  Elements inside that band are the kink
+# band: the test input dy is chosen so that no compared value depends on the
+# decision there (dy = 0 on band elements of an output ReLU; dy rows projected
+# orthogonal to the W2 rows of band elements of GIN's inner ReLU), and outside
+# the band the kernel's decisions must EQUAL the oracle's.
+U_BAND = {torch.float32: 2.0 ** -19, torch.bfloat16: 2.0 ** -8}
+K_BAND = 2.0
+
+
+def kink_band(pre, mag, dtype, exact=False):
+    """Elements where the kernel's ReLU decision may legitimately differ
+    (empty when the inputs make every kernel operation exact: small integers)."""
+    pre = np.asarray(pre, dtype=np.float64)
+    if exact:
+        return np.zeros(pre.shape, bool)
+    if mag is None:                        # no |input| propagation available: global scale
+        mag = np.full_like(pre, np.abs(pre).max() if pre.size else 0.0)
+    return np.abs(pre) < K_BAND * U_BAND[dtype] * np.asarray(mag, dtype=np.float64)
+
+
+def relu_dy(dy, pre, band):
+    """dy zeroed on the kink band, and the oracle's dT = dy * [pre > 0]."""
+    dy = np.where(band, 0.0, np.asarray(dy, dtype=np.float64))
+    return dy, dy * (np.asarray(pre) > 0)
+
+
+def assert_mask_agrees(y_gpu, pre, band, what="ReLU"):
+    """Outside the kink band the kernel's decision [y_gpu > 0] equals [pre > 0]."""
+    got = np.asarray(y_gpu) > 0
+    ref = np.asarray(pre) > 0
+    bad = (got != ref) & ~band
+    assert not bad.any(), f"{what}: {int(bad.sum())} decisions differ outside the kink band " \
+                          f"(first at {np.argwhere(bad)[:3].tolist()})"
+
+
+def gin_inner_safe_dy(dy, a, band_a, W2, free=None):
+    """Project each row of dy (on its free coordinates) orthogonal to the rows
+    W2[j, :] of that row's inner kink-band elements j, so that
+    dh[v, j] = dy[v] . W2[j] = 0 there: the inner ReLU decision at (v, j)
+    then does not change any gradient.  free: [V x fo] bool, coordinates dy
+    may use (default all)."""
+    dy = np.array(dy, dtype=np.float64)
+    for v in np.nonzero(band_a.any(1))[0]:
+        J = np.nonzero(band_a[v])[0]
+        S = np.nonzero(free[v])[0] if free is not None else np.arange(dy.shape[1])
+        if len(S) == 0:
+            continue
+        A = W2[np.ix_(J, S)]
+        g = dy[v, S]
+        coef, *_ = np.linalg.lstsq(A @ A.T, A @ g, rcond=None)
+        dy[v, S] = g - A.T @ coef
+    return dy
