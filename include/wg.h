@@ -222,9 +222,98 @@ typedef struct {
   int32_t dy_masked;
 } wg_bwd_args;
 
+/* Forward: h^{l+1} of Eq. (1) (§2 "GNN model": "h^{l+1}[e.dst]
+ * += MLP(h^l[e.src], W^l[e.type])") for the model's message function and
+ * per-vertex terms (DESIGN.md §2 Q1-Q7); the gTask plan decides the operation
+ * order (T2 indexing swapping) but not the result.  Backward:
+ * the exact gradients of that definition (the paper is silent, Q8), the
+ * transposed gather running over the transposed gTask partition.
+ * Errors: WG_ERR_INVALID for null / misaligned arguments (ld * sizeof(dtype)
+ * not a multiple of 16, ld < F), a missing saved / workspace / exchange
+ * buffer, or a phase the plan does not accept; WG_ERR_UNSUPPORTED for
+ * combinations listed at wg_plan_create; WG_ERR_CUDA for a launch failure
+ * (kernel faults surface on a later call).  Asynchronous on `stream`.      */
 wg_status wg_conv_forward(wg_plan p, const wg_params* params, const wg_fwd_args* a, wg_stream stream);
 wg_status wg_conv_backward(wg_plan p, const wg_params* params, const wg_bwd_args* a,
                            const wg_grads* grads, wg_stream stream);
+
+/* ------------------------------------------------------------------------ */
+/* Multi-GPU layer (the paper's data-parallel scheme          */
+/* P:L2199-2229, Fig 11; transform-before-communicate P:L2279-2289).         */
+/* One process per GPU.  Rank p owns the T-aligned vertex block              */
+/* [b_p, b_{p+1}) of every activation / gradient table, the forward gTasks   */
+/* of those rows and the transposed gTasks of their out-edges.  Per layer    */
+/* the table the gathers read is exchanged over NCCL (all-gather-v of the    */
+/* row blocks) on the communicator's own high-priority stream; GCN / SAGE    */
+/* exchange tables are column-chunked so the gather of chunk k overlaps the  */
+/* exchange of chunk k+1.  Weight gradients are all-reduced (sum).           */
+/* NCCL is the process's own libnccl.so.2 (loaded by torch), resolved at    */
+/* run time; without it these calls return WG_ERR_UNSUPPORTED.               */
+/* ------------------------------------------------------------------------ */
+typedef struct wg_comm_s* wg_comm;
+#define WG_COMM_ID_BYTES 128
+
+/* 128-byte ncclUniqueId (call on one rank, broadcast it out of band, e.g.
+ * through torch.distributed).                                              */
+wg_status wg_comm_unique_id(void* id);
+/* Collective over the `world` ranks (blocking until all have joined).      */
+wg_status wg_comm_init(const void* id, int rank, int world, int device, wg_comm* out);
+/* One-GPU emulation of rank `rank` of a `world`-way partition: every
+ * exchange is a copy kernel on the communication stream that re-reads and
+ * re-writes the non-owned rows (the bytes an all-gather writes, with the SM
+ * share of an NCCL kernel: WG_EMU_CTAS CTAs, default 16); no data moves
+ * between ranks and gradients are not reduced.  For timing the overlap of
+ * exchange and gathers on one GPU (bench.py --rank-slice), not for results. */
+wg_status wg_comm_init_emulated(int rank, int world, int device, wg_comm* out);
+/* info: rank, world, device, emulated                                      */
+wg_status wg_comm_info(wg_comm c, int32_t info[4]);
+/* `stream` waits for the communicator's outstanding work (the gradient
+ * all-reduce that wg_conv_backward_dist leaves running).                   */
+wg_status wg_comm_wait(wg_comm c, wg_stream stream);
+wg_status wg_comm_destroy(wg_comm c);
+
+/* Edge-balanced 1-D partition (host computation, deterministic, so every
+ * rank computes the same bounds from the same global graph): bounds[0..world]
+ * with bounds[0] = 0, bounds[world] = V, interior bounds multiples of T
+ * (desc->tile_rows), each rank >= 1 tile, chosen greedily so each rank's
+ * in-edges + out-edges + rows are ~1/world of the total.  desc is the GLOBAL
+ * graph (pointers host or device).  WG_ERR_INVALID if V has fewer tiles than
+ * ranks.                                                                    */
+wg_status wg_partition_1d(const wg_graph_desc* desc, int world, int64_t* bounds);
+/* This rank's graph of the partition: `global` describes the whole graph (or
+ * any superset of the edges touching this rank's block); bounds (nullable:
+ * wg_partition_1d) fixes every rank's block.  Returns the owned range.      */
+wg_status wg_graph_create_dist(wg_comm c, const wg_graph_desc* global, const int64_t* bounds, int device,
+                               wg_stream stream, wg_graph* out, int64_t* v_begin, int64_t* v_end);
+/* bounds[0..n_ranks] of a graph made by wg_graph_create_dist (n_ranks = 0 otherwise). */
+wg_status wg_graph_bounds(wg_graph g, int64_t* bounds, int32_t* n_ranks);
+/* Plan with ONE layer-level plan on every rank (the ranks exchange one
+ * table): WG_PLAN_AUTO sums the ranks' a4 layer costs (an all-reduce) and
+ * takes all-EDGE or all-VERTEX; WG_PLAN_RANDOM (mixed) is UNSUPPORTED.      */
+wg_status wg_plan_create_dist(wg_comm c, wg_graph g, const wg_conv_desc* desc, wg_plan* out);
+/* Exchange table of a plan, dir 0 = forward, 1 = backward.  info[0] rows
+ * (= V, global vertex ids), info[1] row pitch of a chunk (elements),
+ * info[2] chunks C, info[3] bytes (0: the layer exchanges no table).  The
+ * table is C chunks, chunk k = [rows x info[1]] row-major at byte offset
+ * k * rows * info[1] * sizeof(dtype); pass ld_xchg = info[1].  Caller-owned
+ * device memory.                                                            */
+wg_status wg_plan_xchg(wg_plan p, int dir, int64_t info[4]);
+/* Forward of one layer on every rank (a->phase must be WG_PHASE_ALL; x is
+ * [V x ldx] global rows).  EDGE / RGCN layers gather raw rows of x: unless
+ * x_gathered, this call first all-gathers x's row blocks IN PLACE (the owned
+ * rows must be current, e.g. written by the previous layer).  VERTEX layers
+ * write Y = x W of the owned rows into a->xchg, exchange it chunk by chunk
+ * and gather each chunk as it arrives.  y holds the owned rows.  Stream-
+ * ordered on `stream`; the communicator's stream is joined before return.  */
+wg_status wg_conv_forward_dist(wg_comm c, wg_plan p, const wg_params* params, const wg_fwd_args* a, int x_gathered,
+                               wg_stream stream);
+/* Backward of one layer on every rank (phase WG_PHASE_ALL): this rank's rows
+ * of the backward table into a->xchg, chunked exchange, transposed gather
+ * over the rank's out-edges; dx / dy hold owned rows.  The weight gradients
+ * in `grads` are all-reduced (sum over ranks) on the communicator's stream
+ * AFTER this call returns: call wg_comm_wait before reading them.          */
+wg_status wg_conv_backward_dist(wg_comm c, wg_plan p, const wg_params* params, const wg_bwd_args* a,
+                                const wg_grads* grads, wg_stream stream);
 
 /* ------------------------------------------------------------------------ */
 /* Training-step utility: fused softmax cross-entropy over the last layer's

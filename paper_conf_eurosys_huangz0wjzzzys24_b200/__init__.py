@@ -18,7 +18,8 @@ import torch
 from . import _capi as C
 from ._capi import WGError, TASK_DTYPE
 
-__all__ = ["Graph", "Conv", "WGError", "TASK_DTYPE", "padded", "pad_to", "ld_of", "launch_count", "init_params"]
+__all__ = ["Graph", "Conv", "Comm", "WGError", "TASK_DTYPE", "padded", "pad_to", "ld_of", "launch_count",
+           "init_params", "partition_1d"]
 
 
 def _ptr(t):
@@ -104,37 +105,111 @@ def profile(cmd: str):
             for i, k in enumerate(C.PROF_KINDS)}
 
 
-class Graph:
-    """Device graph + forward / transposed gTask partitions (wg_graph_create)."""
+class Comm:
+    """Communicator of the 1-D multi-GPU layer (wg_comm_*): NCCL over the
+    ranks of a torch.distributed group (the 128-byte id is broadcast through
+    it), or the one-GPU emulation of one rank (emulate=(rank, world))."""
 
-    def __init__(self, src, dst=None, *, num_vertices: int, indptr=None, etype=None, num_types: int = 1,
-                 tile_rows: int = 128, max_task_edges: int = 0, v_begin: int = 0, v_end: int = 0,
-                 device: int | None = None, stream=None):
+    def __init__(self, group=None, *, device: int | None = None, emulate=None):
         L = C.lib()
-        self._keep = []
-
-        def arr(a, dt):
-            if a is None:
-                return None
-            if isinstance(a, torch.Tensor):
-                a = a.to(dt).contiguous()
-            else:
-                a = np.ascontiguousarray(a, dtype={torch.int32: np.int32, torch.int64: np.int64}[dt])
-            self._keep.append(a)
-            return a
-
-        s = arr(src, torch.int32)
-        d = arr(dst, torch.int32)
-        ip = arr(indptr, torch.int64)
-        et = arr(etype, torch.int32)
-        E = (s.shape[0] if s is not None else 0)
-        desc = C.GraphDesc(num_vertices, E, _ptr(ip), _ptr(s), _ptr(d), _ptr(et), num_types, tile_rows,
-                           max_task_edges, v_begin, v_end)
         self.device = torch.cuda.current_device() if device is None else device
         h = ctypes.c_void_p()
         with torch.cuda.device(self.device):
-            C.check(L.wg_graph_create(ctypes.byref(desc), self.device, _stream(stream), ctypes.byref(h)),
-                    "wg_graph_create")
+            if emulate is not None:
+                self.rank, self.world = emulate
+                C.check(L.wg_comm_init_emulated(self.rank, self.world, self.device, ctypes.byref(h)),
+                        "wg_comm_init_emulated")
+            else:
+                import torch.distributed as dist
+                self.rank, self.world = dist.get_rank(group), dist.get_world_size(group)
+                uid = torch.zeros(C.COMM_ID_BYTES, dtype=torch.uint8)
+                if self.rank == 0:
+                    C.check(L.wg_comm_unique_id(_ptr(uid)), "wg_comm_unique_id")
+                dev = torch.device("cuda", self.device) if dist.get_backend(group) == "nccl" else torch.device("cpu")
+                u = uid.to(dev)
+                dist.broadcast(u, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+                uid = u.cpu().contiguous()
+                C.check(L.wg_comm_init(_ptr(uid), self.rank, self.world, self.device, ctypes.byref(h)),
+                        "wg_comm_init")
+        self._h = h
+        self.emulated = emulate is not None
+
+    @property
+    def handle(self):
+        return self._h
+
+    def wait(self, stream=None):
+        """The current (or given) stream waits for outstanding communication
+        (the gradient all-reduce left running by backward_dist)."""
+        C.check(C.lib().wg_comm_wait(self._h, _stream(stream)), "wg_comm_wait")
+
+    def close(self):
+        if getattr(self, "_h", None):
+            C.lib().wg_comm_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def _graph_desc(src, dst, num_vertices, indptr, etype, num_types, tile_rows, max_task_edges, v_begin, v_end, keep):
+    def arr(a, dt):
+        if a is None:
+            return None
+        if isinstance(a, torch.Tensor):
+            a = a.to(dt).contiguous()
+        else:
+            a = np.ascontiguousarray(a, dtype={torch.int32: np.int32, torch.int64: np.int64}[dt])
+        keep.append(a)
+        return a
+
+    s = arr(src, torch.int32)
+    d = arr(dst, torch.int32)
+    ip = arr(indptr, torch.int64)
+    et = arr(etype, torch.int32)
+    E = (s.shape[0] if s is not None else 0)
+    return C.GraphDesc(num_vertices, E, _ptr(ip), _ptr(s), _ptr(d), _ptr(et), num_types, tile_rows,
+                       max_task_edges, v_begin, v_end)
+
+
+def partition_1d(src, dst=None, *, num_vertices: int, world: int, indptr=None, tile_rows: int = 128):
+    """Edge-balanced T-aligned 1-D partition bounds [world + 1] (wg_partition_1d,
+    a host computation: works without a GPU for host arrays)."""
+    keep = []
+    desc = _graph_desc(src, dst, num_vertices, indptr, None, 1, tile_rows, 0, 0, 0, keep)
+    b = np.zeros(world + 1, np.int64)
+    C.check(C.lib().wg_partition_1d(ctypes.byref(desc), world, _ptr(b)), "wg_partition_1d")
+    return b
+
+
+class Graph:
+    """Device graph + forward / transposed gTask partitions (wg_graph_create;
+    with comm=, this rank's block of the 1-D partition, wg_graph_create_dist)."""
+
+    def __init__(self, src, dst=None, *, num_vertices: int, indptr=None, etype=None, num_types: int = 1,
+                 tile_rows: int = 128, max_task_edges: int = 0, v_begin: int = 0, v_end: int = 0,
+                 device: int | None = None, stream=None, comm: Comm | None = None, bounds=None):
+        L = C.lib()
+        self._keep = []
+        desc = _graph_desc(src, dst, num_vertices, indptr, etype, num_types, tile_rows, max_task_edges,
+                           v_begin, v_end, self._keep)
+        self.device = (comm.device if comm is not None else torch.cuda.current_device()) if device is None else device
+        h = ctypes.c_void_p()
+        self.comm = comm
+        with torch.cuda.device(self.device):
+            if comm is not None:
+                b = None if bounds is None else np.ascontiguousarray(bounds, dtype=np.int64)
+                vb, ve = ctypes.c_int64(), ctypes.c_int64()
+                C.check(L.wg_graph_create_dist(comm.handle, ctypes.byref(desc), _ptr(b), self.device,
+                                               _stream(stream), ctypes.byref(h), ctypes.byref(vb),
+                                               ctypes.byref(ve)), "wg_graph_create_dist")
+                v_begin = vb.value if comm.world > 1 else 0
+            else:
+                C.check(L.wg_graph_create(ctypes.byref(desc), self.device, _stream(stream), ctypes.byref(h)),
+                        "wg_graph_create")
         self._h = h
         self._keep = []
         info = (ctypes.c_int64 * 10)()
@@ -144,6 +219,12 @@ class Graph:
         self.v_begin = v_begin
         self.num_types = num_types
         self._plans = 0
+        self.bounds = None
+        if comm is not None:
+            b = np.zeros(comm.world + 1, np.int64)
+            n = ctypes.c_int32()
+            C.check(L.wg_graph_bounds(self._h, _ptr(b), ctypes.byref(n)), "wg_graph_bounds")
+            self.bounds = b
 
     @property
     def handle(self):
@@ -195,7 +276,12 @@ class Conv:
                                int(self_loop), int(bias), int(fuse_relu), gin_eps, neg_slope, C.POLICIES[policy],
                                seed, int(need_dx))
         h = ctypes.c_void_p()
-        C.check(C.lib().wg_plan_create(graph.handle, ctypes.byref(self.desc), ctypes.byref(h)), "wg_plan_create")
+        self.comm = graph.comm
+        if self.comm is not None:   # one uniform plan on every rank (wg_plan_create_dist)
+            C.check(C.lib().wg_plan_create_dist(self.comm.handle, graph.handle, ctypes.byref(self.desc),
+                                                ctypes.byref(h)), "wg_plan_create_dist")
+        else:
+            C.check(C.lib().wg_plan_create(graph.handle, ctypes.byref(self.desc), ctypes.byref(h)), "wg_plan_create")
         self._h = h
         graph._plans += 1
         sb, wb = ctypes.c_size_t(), ctypes.c_size_t()
@@ -222,6 +308,21 @@ class Conv:
         ld = pitch(F, self.dtype)
         raw = buf[off.value: off.value + rows * ld * es]
         return raw.view(self.dtype).view(rows, ld)[:, :F]
+
+    def xchg_info(self, direction: int):
+        """(rows, chunk pitch, chunks, bytes) of the forward (0) / backward (1) exchange table."""
+        info = (ctypes.c_int64 * 4)()
+        C.check(C.lib().wg_plan_xchg(self._h, direction, info), "wg_plan_xchg")
+        return tuple(int(v) for v in info)
+
+    def new_xchg(self, direction: int):
+        """The caller-owned exchange table ([chunks x rows x pitch] in the conv
+        dtype, returned as a [chunks * rows x pitch] tensor; ld_xchg = pitch),
+        or None if the layer exchanges no table in that direction."""
+        rows, ld, chunks, nbytes = self.xchg_info(direction)
+        if nbytes == 0:
+            return None
+        return torch.zeros((chunks * rows, ld), dtype=self.dtype, device=self.workspace.device)
 
     def new_saved(self):
         return torch.empty(max(self.saved_bytes, 256), dtype=torch.uint8, device=self.workspace.device)
@@ -259,6 +360,30 @@ class Conv:
         C.check(C.lib().wg_conv_backward(self._h, ctypes.byref(pr), ctypes.byref(a), ctypes.byref(gr),
                                          _stream(stream)), "wg_conv_backward")
         return dx, grads
+
+    # ------------------------------------------------------------------ distributed
+    def forward_dist(self, x, params: dict, y, saved, xchg=None, x_gathered: bool = False, stream=None):
+        """wg_conv_forward_dist: exchange + forward of this rank's rows (see include/wg.h)."""
+        pr = C.Params(*[_ptr(params.get(n)) for n in PARAM_NAMES])
+        a = C.FwdArgs(C.PHASE_ALL, _ptr(x), ld_of(x), _ptr(y), ld_of(y), _ptr(saved), _ptr(self.workspace),
+                      _ptr(xchg), xchg.stride(0) if xchg is not None else 0)
+        C.check(C.lib().wg_conv_forward_dist(self.comm.handle, self._h, ctypes.byref(pr), ctypes.byref(a),
+                                             int(x_gathered), _stream(stream)), "wg_conv_forward_dist")
+        return y
+
+    def backward_dist(self, dy, x, y, saved, params: dict, dx=None, xchg=None, grads: dict | None = None,
+                      dx_mask=None, dy_masked: bool = False, stream=None):
+        """wg_conv_backward_dist; the gradients are all-reduced on the
+        communicator's stream after return (Comm.wait before reading them)."""
+        pr = C.Params(*[_ptr(params.get(n)) for n in PARAM_NAMES])
+        gr = C.Grads(*[_ptr((grads or {}).get(n)) for n in PARAM_NAMES])
+        a = C.BwdArgs(C.PHASE_ALL, _ptr(dy), ld_of(dy), _ptr(x), ld_of(x), _ptr(y), ld_of(y) if y is not None else 0,
+                      _ptr(saved), _ptr(dx), ld_of(dx) if dx is not None else 0, _ptr(self.workspace),
+                      _ptr(xchg), xchg.stride(0) if xchg is not None else 0,
+                      _ptr(dx_mask), ld_of(dx_mask) if dx_mask is not None else 0, int(dy_masked))
+        C.check(C.lib().wg_conv_backward_dist(self.comm.handle, self._h, ctypes.byref(pr), ctypes.byref(a),
+                                              ctypes.byref(gr), _stream(stream)), "wg_conv_backward_dist")
+        return dx
 
     # ------------------------------------------------------------------ autograd
     def __call__(self, x, params: dict):

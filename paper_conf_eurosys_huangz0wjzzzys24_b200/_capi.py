@@ -26,7 +26,11 @@ EXPORTS = [
     "wg_plan_create", "wg_plan_sizes", "wg_plan_export", "wg_plan_buffer", "wg_plan_destroy",
     "wg_conv_forward", "wg_conv_backward",
     "wg_status_string", "wg_last_error", "wg_launch_count", "wg_profile", "wg_softmax_xent",
+    "wg_comm_unique_id", "wg_comm_init", "wg_comm_init_emulated", "wg_comm_info", "wg_comm_wait",
+    "wg_comm_destroy", "wg_partition_1d", "wg_graph_create_dist", "wg_graph_bounds", "wg_plan_create_dist",
+    "wg_plan_xchg", "wg_conv_forward_dist", "wg_conv_backward_dist",
 ]
+COMM_ID_BYTES = 128
 XENT_SCRATCH_BYTES = 8192
 PROF_KINDS = ["gather_reduce", "split_combine", "tc_gemm_nt", "tc_gemm_tn", "simt_gemm", "misc", "gat", "rgcn"]
 
@@ -120,6 +124,35 @@ def lib():
     L.wg_profile.argtypes = [ctypes.c_int, P]
     L.wg_softmax_xent.restype = st
     L.wg_softmax_xent.argtypes = [ctypes.c_int, i64, i32, P, i64, P, f32, P, i64, P, P, P]
+    # multi-GPU
+    L.wg_comm_unique_id.restype = st
+    L.wg_comm_unique_id.argtypes = [P]
+    L.wg_comm_init.restype = st
+    L.wg_comm_init.argtypes = [P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.POINTER(P)]
+    L.wg_comm_init_emulated.restype = st
+    L.wg_comm_init_emulated.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.POINTER(P)]
+    L.wg_comm_info.restype = st
+    L.wg_comm_info.argtypes = [P, P]
+    L.wg_comm_wait.restype = st
+    L.wg_comm_wait.argtypes = [P, P]
+    L.wg_comm_destroy.restype = st
+    L.wg_comm_destroy.argtypes = [P]
+    L.wg_partition_1d.restype = st
+    L.wg_partition_1d.argtypes = [ctypes.POINTER(GraphDesc), ctypes.c_int, P]
+    L.wg_graph_create_dist.restype = st
+    L.wg_graph_create_dist.argtypes = [P, ctypes.POINTER(GraphDesc), P, ctypes.c_int, P, ctypes.POINTER(P),
+                                       ctypes.POINTER(i64), ctypes.POINTER(i64)]
+    L.wg_graph_bounds.restype = st
+    L.wg_graph_bounds.argtypes = [P, P, ctypes.POINTER(i32)]
+    L.wg_plan_create_dist.restype = st
+    L.wg_plan_create_dist.argtypes = [P, P, ctypes.POINTER(ConvDesc), ctypes.POINTER(P)]
+    L.wg_plan_xchg.restype = st
+    L.wg_plan_xchg.argtypes = [P, ctypes.c_int, P]
+    L.wg_conv_forward_dist.restype = st
+    L.wg_conv_forward_dist.argtypes = [P, P, ctypes.POINTER(Params), ctypes.POINTER(FwdArgs), ctypes.c_int, P]
+    L.wg_conv_backward_dist.restype = st
+    L.wg_conv_backward_dist.argtypes = [P, P, ctypes.POINTER(Params), ctypes.POINTER(BwdArgs),
+                                        ctypes.POINTER(Grads), P]
     _lib = L
     return L
 

@@ -675,7 +675,7 @@ __global__ void k_prep_weight(const float* W, int batch, int rows, int cols, int
 template <typename T>
 __global__ void __launch_bounds__(256) k_colsum(int64_t M, int N, const T* dy, int64_t lddy, const T* ref,
                                                 int64_t ldref, T* dt, int64_t ldt, float* part, int64_t rows_per_blk,
-                                                const float* rs2, T* dt2, int64_t ldt2) {
+                                                const float* rs2, T* dt2, int64_t ldt2, int fc2, int64_t cs2) {
   constexpr int EPV = VT<T>::EPV;
   extern __shared__ float red[];                       // [nsub][nv*EPV]
   const int nv = (N + EPV - 1) / EPV;                  // vectors per row (<= 256)
@@ -696,12 +696,14 @@ __global__ void __launch_bounds__(256) k_colsum(int64_t M, int N, const T* dy, i
 #pragma unroll
       for (int i = 0; i < EPV; ++i) if (vec * EPV + i >= N) v[i] = 0.f;
       if (dt) *reinterpret_cast<int4*>(dt + r * ldt + vec * EPV) = VT<T>::pack(v);
-      if (dt2) {
+      if (dt2) {   // second output: scaled by rs2 (if any), optionally column-chunked
         float w[EPV];
-        const float sc = rs2[r];
+        const float sc = rs2 ? rs2[r] : 1.f;
 #pragma unroll
         for (int i = 0; i < EPV; ++i) w[i] = sc * v[i];
-        *reinterpret_cast<int4*>(dt2 + r * ldt2 + vec * EPV) = VT<T>::pack(w);
+        const int col = vec * EPV;
+        T* q = fc2 > 0 ? dt2 + (int64_t)(col / fc2) * cs2 + r * ldt2 + col % fc2 : dt2 + r * ldt2 + col;
+        *reinterpret_cast<int4*>(q) = VT<T>::pack(w);
       }
 #pragma unroll
       for (int i = 0; i < EPV; ++i) acc[i] += v[i];
@@ -771,7 +773,7 @@ size_t bias_grad_scratch(int64_t M, int N) { return sizeof(float) * (size_t)COLS
 
 wg_status bias_grad_mask(wg_dtype dt, int64_t M, int N, const void* dy, int64_t lddy, const void* ref,
                          int64_t ldref, void* dt_out, int64_t ldt, float* db, float* scratch, cudaStream_t s,
-                         const float* rs2, void* dt2, int64_t ldt2) {
+                         const float* rs2, void* dt2, int64_t ldt2, int fc2, int64_t cs2) {
   const int EPV = dt == WG_BF16 ? 8 : 4;
   const int nv = (int)cdiv(N, EPV);
   WG_REQ(nv <= 256, WG_ERR_UNSUPPORTED, "bias gradient: more than 256 vectors per row");
@@ -784,10 +786,10 @@ wg_status bias_grad_mask(wg_dtype dt, int64_t M, int N, const void* dy, int64_t 
   if (dt == WG_BF16)
     WG_LAUNCH(k_colsum<__nv_bfloat16>, nblk, threads, smem, s, M, N, (const __nv_bfloat16*)dy, lddy,
               (const __nv_bfloat16*)ref, ldref, (__nv_bfloat16*)dt_out, ldt, scratch, rpb, rs2, (__nv_bfloat16*)dt2,
-              ldt2);
+              ldt2, fc2, cs2);
   else
     WG_LAUNCH(k_colsum<float>, nblk, threads, smem, s, M, N, (const float*)dy, lddy, (const float*)ref, ldref,
-              (float*)dt_out, ldt, scratch, rpb, rs2, (float*)dt2, ldt2);
+              (float*)dt_out, ldt, scratch, rpb, rs2, (float*)dt2, ldt2, fc2, cs2);
   if (db) WG_LAUNCH(k_colsum_reduce, (unsigned)cdiv(N, 32), 256, 0, s, scratch, nblk, N, db);
   return WG_OK;
 }

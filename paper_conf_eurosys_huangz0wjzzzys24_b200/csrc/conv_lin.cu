@@ -131,6 +131,49 @@ wg_status run_agg(const Ctx& c, AggArgs a, const ItemList& L, cudaStream_t st) {
   return WG_OK;
 }
 
+// Gather over an exchange table in layout X (chunk k = [V x Fc] at k * V * Fc
+// elements): one gather + combine per column chunk, writing columns
+// [k Fc, k Fc + Fc) of the output (aggregation is column-separable); before
+// chunk k the stream waits for its arrival (hook).  The self / mask / bias
+// operands are ordinary row-major [rows x ld] tensors.
+wg_status run_agg_x(const Ctx& c, AggArgs a, const ItemList& L, cudaStream_t st, const XLayout& X,
+                    const XHook* hk) {
+  if (X.C <= 1) {
+    if (hk) hk->wait(0, st);
+    return run_agg(c, a, L, st);
+  }
+  const int F = a.F;
+  for (int k = 0; k < X.C; ++k) {
+    const int64_t c0 = k * X.Fc;
+    if (c0 >= F) break;
+    if (hk) hk->wait(k, st);
+    AggArgs b = a;
+    b.table = static_cast<const char*>(a.table) + (size_t)k * c.Vg * X.Fc * c.s;
+    b.ld_tab = X.Fc;
+    b.F = (int)std::min<int64_t>(X.Fc, F - c0);
+    b.out = static_cast<char*>(a.out) + c0 * c.s;
+    if (a.bias) b.bias = a.bias + c0;
+    if (a.self_tab) b.self_tab = static_cast<const char*>(a.self_tab) + c0 * c.s;
+    if (a.mask_ref) b.mask_ref = static_cast<const char*>(a.mask_ref) + c0 * c.s;
+    WG_TRY(run_agg(c, b, L, st));
+  }
+  return WG_OK;
+}
+
+// GEMM output into this rank's rows of an exchange table (layout X, caller
+// pitch ld when X.C == 1)
+void epi_xchg(const Ctx& c, GemmEpi* e, void* tab, int64_t ld, const XLayout& X) {
+  if (X.C > 1) {
+    e->D = off(tab, c.vb, X.Fc, c.s);
+    e->ldd = X.Fc;
+    e->d_chunk_cols = (int)X.Fc;
+    e->d_chunk_stride = c.Vg * X.Fc;
+  } else {
+    e->D = off(tab, c.vb, ld, c.s);
+    e->ldd = ld;
+  }
+}
+
 // GCN edge coefficient c_e = gs[src] * rs[dst] (Q3)
 void gcn_scales(const Ctx& c, const float** gs_src, const float** rs_dst) {
   *gs_src = nullptr; *rs_dst = nullptr;
@@ -142,7 +185,7 @@ void gcn_scales(const Ctx& c, const float** gs_src, const float** rs_dst) {
 
 }  // namespace
 
-wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cudaStream_t st) {
+wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cudaStream_t st, const XHook* hk) {
   Ctx c = mk(p);
   const wg_conv_desc& d = p->d;
   const bool sage = d.model == WG_SAGE, gin = d.model == WG_GIN;
@@ -162,6 +205,9 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
          "a VERTEX layer on a 1-D partition needs the exchange table (xchg)");
   WG_REQ(!A->xchg || ((A->ld_xchg * c.s) % 16 == 0 && A->ld_xchg >= c.fo), WG_ERR_INVALID,
          "ld_xchg must be >= f_out and a 16-byte multiple");
+  const XLayout xl = A->xchg ? p->xf : XLayout{};
+  WG_REQ(xl.C <= 1 || A->ld_xchg == xl.Fc, WG_ERR_INVALID,
+         "chunked exchange table: ld_xchg must be the chunk width (wg_plan_xchg)");
   void* ws = A->workspace;
   const Layout& L = p->ws;
   const char* x_own = off(A->x, c.vb, A->ldx, c.s);
@@ -193,8 +239,7 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
       WG_TRY(prep_weight(c.dt, P->W_self, c.fi, c.fo, 1, off(wys, c.po, c.pi, c.s), c.pi, (int)c.po, st));
       GemmPart part{x_own, A->ldx, wys, c.pi, c.fi, (int)(2 * c.po)};
       GemmEpi e;
-      e.D = off(ytab, c.vb, ldY, c.s);
-      e.ldd = ldY;
+      epi_xchg(c, &e, ytab, ldY, xl);
       e.D2 = L.at<void>(ws, "s");
       e.ldd2 = c.po;
       e.n_split = (int)c.po;
@@ -202,8 +247,7 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
     } else if (pre) {
       GemmPart part{x_own, A->ldx, wt, c.pi, c.fi, (int)c.wrows_o};
       GemmEpi e;
-      e.D = off(ytab, c.vb, ldY, c.s);
-      e.ldd = ldY;
+      epi_xchg(c, &e, ytab, ldY, xl);
       WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fo, 16 / c.s), &part, 1, e, nullptr, 0, st));
     }
   }
@@ -243,7 +287,7 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
       a.out = z; a.ld_out = c.po;
       a.zero_out = agg; a.ld_zero = c.pi; a.zero_cols = (int)c.pi;
     }
-    WG_TRY(run_agg(c, a, p->fv, st));
+    WG_TRY(run_agg_x(c, a, p->fv, st, xl, hk));
   }
   // ---- EDGE transform: y = Agg W (+ x W_s) + Z + b
   if (edge_path(p)) {
@@ -272,7 +316,8 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
   return WG_OK;
 }
 
-wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, const wg_grads* G, cudaStream_t st) {
+wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, const wg_grads* G, cudaStream_t st,
+                       const XHook* hk) {
   Ctx c = mk(p);
   const wg_conv_desc& d = p->d;
   const bool sage = d.model == WG_SAGE, gin = d.model == WG_GIN;
@@ -318,19 +363,20 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
   // scale -- a random 4-byte load per edge from a V-sized array (444 MB at C5)
   const bool fold = xchg != nullptr && rs != nullptr && !gin;
   const float* rs_own = rs ? rs + c.vb : nullptr;
-  void* dt_buf = nullptr;
+  const XLayout xl = xchg ? p->xb : XLayout{};
+  WG_REQ(xl.C <= 1 || A->ld_xchg == xl.Fc, WG_ERR_INVALID,
+         "chunked exchange table: ld_xchg must be the chunk width (wg_plan_xchg)");
+  void* dt_buf = nullptr;                  // dT of the owned rows (row-major), when dy itself is not it
   int64_t ld_dtb = c.po;
-  void* dt_fold = nullptr;                 // G path, folded: the scaled rows in the exchange table
-  if (gpath_lin && xchg && fold) {
-    dt_fold = off(xchg, c.vb, A->ld_xchg, c.s);
-    if (mask_dy) dt_buf = L.at<void>(ws, "dt");             // owned rows, local indexing
-  } else if (gpath_lin && xchg) { dt_buf = off(xchg, c.vb, A->ld_xchg, c.s); ld_dtb = A->ld_xchg; }
-  else if (mask_dy) { dt_buf = L.at<void>(ws, "dt"); ld_dtb = c.po; }
+  void* dt_x = nullptr;                    // G path: this rank's rows of the exchange table, dT (* rs)
+  if (gpath_lin && xchg) dt_x = xl.C > 1 ? off(xchg, c.vb, xl.Fc, c.s) : off(xchg, c.vb, A->ld_xchg, c.s);
+  if (mask_dy) dt_buf = L.at<void>(ws, "dt");             // owned rows, local indexing
   if (pre) {
     float* db = gin ? (G ? G->b2 : nullptr) : (G ? G->bias : nullptr);
-    if (dt_buf || db || dt_fold)
+    if (dt_buf || db || dt_x)
       WG_TRY(bias_grad_mask(c.dt, c.nr, c.fo, A->dy, A->lddy, mask_dy ? A->y : nullptr, A->ldy, dt_buf, ld_dtb,
-                            db, colsum, st, dt_fold ? rs_own : nullptr, dt_fold, A->ld_xchg));
+                            db, colsum, st, fold ? rs_own : nullptr, dt_x, xl.C > 1 ? xl.Fc : A->ld_xchg,
+                            xl.C > 1 ? (int)xl.Fc : 0, c.Vg * xl.Fc));
   }
   const void* dT = dt_buf ? dt_buf : A->dy;
   const int64_t lddT = dt_buf ? ld_dtb : A->lddy;
@@ -376,14 +422,14 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
         WG_TRY(prep_weight(c.dt, P->W_self, c.fi, c.fo, 0, off(wbs, c.pi, c.po, c.s), c.po, (int)c.pi, st));
         GemmPart part{dT, lddT, wbs, c.po, c.fo, (int)(2 * c.pi)};
         GemmEpi e;
-        e.D = off(dtab, c.vb, ldd, c.s); e.ldd = ldd;
+        epi_xchg(c, &e, dtab, ldd, xl);
         e.rscale = fold ? rs_own : nullptr;    // dAgg only (D), not dX_s (D2)
         e.D2 = L.at<void>(ws, "dxs"); e.ldd2 = c.pi; e.n_split = (int)c.pi;
         WG_TRY(gemm_nt(c.dt, c.nr, (int)(2 * c.pi), &part, 1, e, nullptr, 0, st));
       } else if (d.need_dx) {
         GemmPart part{dTT, lddTT, w, c.po, c.fo, (int)c.wrows_i};
         GemmEpi e;
-        e.D = off(dtab, c.vb, ldd, c.s); e.ldd = ldd;
+        epi_xchg(c, &e, dtab, ldd, xl);
         e.rscale = fold ? rs_own : nullptr;
         WG_TRY(gemm_nt(c.dt, c.nr, (int)rup(c.fi, 16 / c.s), &part, 1, e, nullptr, 0, st));
       }
@@ -398,7 +444,7 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
       a.mask_ref = A->dx_mask; a.ld_mask = A->ld_dx_mask;
       a.partial = L.at<float>(ws, "partT"); a.ld_part = pl;
       a.F = c.fi;
-      WG_TRY(run_agg(c, a, p->bt, st));
+      WG_TRY(run_agg_x(c, a, p->bt, st, xl, hk));
     }
     return WG_OK;
   }
@@ -414,7 +460,7 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, c
     a.out = gbuf; a.ld_out = c.po;
     a.partial = L.at<float>(ws, "partT"); a.ld_part = pl;
     a.F = c.fo;
-    WG_TRY(run_agg(c, a, p->bt, st));
+    WG_TRY(run_agg_x(c, a, p->bt, st, xl, hk));
   }
   if (G && G->W) WG_TRY(gemm_tn(c.dt, c.nr, c.fi, c.fo, x_own, A->ldx, gbuf, c.po, G->W, tn, st));
   if (d.need_dx) {

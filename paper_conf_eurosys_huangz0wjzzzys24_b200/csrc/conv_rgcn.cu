@@ -586,7 +586,8 @@ wg_status rgcn_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, c
 }
 
 // ---------------------------------------------------------------- backward
-wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, const wg_grads* G, cudaStream_t st) {
+wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, const wg_grads* G, cudaStream_t st,
+                        const XHook* hk) {
   const wg_conv_desc& d = p->d;
   wg_graph_s* g = p->g;
   auto* rp = static_cast<RgcnPlan*>(p->rg);
@@ -631,6 +632,7 @@ wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* A, 
     }
   }
   if (!post) return WG_OK;
+  if (hk) hk->wait(0, st);        // distributed: the dT table has arrived
   // stage 1T: G_(u,r) = sum_{e: src u, type r} c_e dT[dst_e]
   void* gt = L.at<void>(ws, "gt");
   {

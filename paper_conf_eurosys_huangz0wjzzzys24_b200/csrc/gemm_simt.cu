@@ -210,6 +210,9 @@ wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_pa
   WG_REQ(n_parts >= 1 && n_parts <= 3, WG_ERR_INVALID, "gemm_nt: 1..3 parts");
   wg_status st = WG_OK;
   if (tc_gemm_nt(dt, M, N, parts, n_parts, epi, s, &st)) return st;
+  // a column-chunked output (exchange layout) is written by the persistent
+  // tcgen05 kernel's 3-D store maps only
+  WG_REQ(epi.d_chunk_cols <= 0, WG_ERR_UNSUPPORTED, "gemm_nt: chunked output needs the tcgen05 path");
   NTArgs a{};
   a.M = M; a.N = N; a.n_parts = n_parts; a.epi = epi;
   double kt = 0;

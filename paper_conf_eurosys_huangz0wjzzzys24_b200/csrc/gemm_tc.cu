@@ -493,6 +493,23 @@ bool tc_make_map_t(CUtensorMap* m, CUtensorMapDataType ty, const void* ptr, uint
   return make_map_t(m, ty, ptr, inner, outer, ld_bytes, box_in, box_out);
 }
 
+// 3-D tensor map {inner, outer, chunks} (128-byte swizzle): a column-chunked
+// output table [chunks][outer][inner]; chunk_bytes = 0 when chunks == 1
+bool tc_make_map3_t(CUtensorMap* m, CUtensorMapDataType ty, const void* ptr, uint64_t inner, uint64_t outer,
+                    uint64_t chunks, uint64_t ld_bytes, uint64_t chunk_bytes, uint32_t box_in, uint32_t box_out) {
+  auto fn = encode_fn();
+  if (!fn) return false;
+  if (chunks <= 1) chunk_bytes = ld_bytes * std::max<uint64_t>(outer, 1);
+  if ((reinterpret_cast<uintptr_t>(ptr) & 15) || (ld_bytes & 15) || (chunk_bytes & 15)) return false;
+  cuuint64_t dims[3] = {inner, outer, std::max<uint64_t>(chunks, 1)};
+  cuuint64_t strides[2] = {ld_bytes, chunk_bytes};
+  cuuint32_t box[3] = {box_in, box_out, 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  return fn(m, ty, 3, const_cast<void*>(ptr), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts, const GemmEpi& epi,
                            cudaStream_t s, wg_status* st);
 
@@ -500,7 +517,7 @@ bool tc_gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_part
                 cudaStream_t s, wg_status* st) {
   if (!tc_enabled() || n_parts > 3 || M <= 0) return false;
   if (tc_gemm_nt_persistent(dt, M, N, parts, n_parts, epi, s, st)) return true;
-  if (dt != WG_BF16) return false;
+  if (dt != WG_BF16 || epi.d_chunk_cols > 0) return false;
   for (int i = 0; i < n_parts; ++i)
     if (parts[i].tile_group || parts[i].a_rows) return false;   // grouped B / gathered A: persistent kernel only
   const int n_tiles = (int)cdiv(N, 256);

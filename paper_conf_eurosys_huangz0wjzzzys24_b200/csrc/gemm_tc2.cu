@@ -46,6 +46,8 @@ namespace wg {
 
 bool tc_make_map_t(CUtensorMap* m, CUtensorMapDataType ty, const void* ptr, uint64_t inner, uint64_t outer,
                    uint64_t ld_bytes, uint32_t box_in, uint32_t box_out);
+bool tc_make_map3_t(CUtensorMap* m, CUtensorMapDataType ty, const void* ptr, uint64_t inner, uint64_t outer,
+                    uint64_t chunks, uint64_t ld_bytes, uint64_t chunk_bytes, uint32_t box_in, uint32_t box_out);
 
 namespace {
 
@@ -78,6 +80,7 @@ struct P2 {
   const float* bias;
   int relu, has_add, has_mask, bias_vec;
   int cpg;          // fp32 row-gathered A by per-lane cp.async (see the producer)
+  int fc_d, fc_d2;  // columns per chunk of the (column-chunked) D / D2 output maps
   const void* a_tab; int64_t lda_tab; int k_a;   // cpg: table, its row pitch (elements), K
 };
 
@@ -112,10 +115,14 @@ __device__ __forceinline__ void tma_gather4(uint32_t dst, const CUtensorMap* m, 
       "l"(reinterpret_cast<uint64_t>(m)), "r"(c0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(bar)
       : "memory");
 }
-__device__ __forceinline__ void tma_store(const CUtensorMap* m, int c0, int c1, uint32_t src) {
-  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(
+// output maps are 3-D {columns of a chunk, rows, chunks}: a column-chunked
+// table [C][rows][Fc] (the exchange layout of DESIGN.md §9); C = 1 is the
+// plain row-major matrix.  A 128-byte store box never straddles a chunk
+// (Fc is a multiple of 128 bytes when C > 1).
+__device__ __forceinline__ void tma_store3(const CUtensorMap* m, int c0, int c1, int c2, uint32_t src) {
+  asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%1, %2, %3}], [%4];" ::"l"(
                    reinterpret_cast<uint64_t>(m)),
-               "r"(c0), "r"(c1), "r"(src)
+               "r"(c0), "r"(c1), "r"(c2), "r"(src)
                : "memory");
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
@@ -531,7 +538,8 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         epi_bar(grp);
         if (et == 0) {
-          tma_store(td, ncol0 + c * C::CHE, m0, su32(stg));
+          const int col = ncol0 + c * C::CHE, fc = second ? p.fc_d2 : p.fc_d;
+          tma_store3(td, col % fc, m0, col / fc, su32(stg));
           bulk_commit();
         }
       }
@@ -621,15 +629,25 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
   }
   for (int i = n_parts; i < 3; ++i) { maps[2 * i] = maps[0]; maps[2 * i + 1] = maps[1]; }
   const int n1 = epi.D2 ? epi.n_split : N;
-  if (!tc_make_map_t(&maps[6], ty, epi.D, (uint64_t)n1, (uint64_t)M, (uint64_t)epi.ldd * es, che, BM)) return false;
+  // D: column-chunked when d_chunk_cols > 0 (chunks of d_chunk_cols columns,
+  // d_chunk_stride elements apart); otherwise one chunk of n1 columns
+  const int C1 = epi.d_chunk_cols > 0 ? (int)cdiv(n1, epi.d_chunk_cols) : 1;
+  p.fc_d = C1 > 1 ? epi.d_chunk_cols : n1;
+  if (C1 > 1 && (p.fc_d % che != 0 || (epi.d_chunk_stride * es) % 16 != 0)) return false;
+  if (!tc_make_map3_t(&maps[6], ty, epi.D, (uint64_t)p.fc_d, (uint64_t)M, (uint64_t)C1, (uint64_t)epi.ldd * es,
+                      (uint64_t)(C1 > 1 ? epi.d_chunk_stride : 0) * es, che, BM))
+    return false;
   maps[7] = maps[6];
+  p.fc_d2 = p.fc_d;
   if (epi.D2) {
     p.n_split = epi.n_split;
-    if (!tc_make_map_t(&maps[7], ty, epi.D2, (uint64_t)(N - epi.n_split), (uint64_t)M, (uint64_t)epi.ldd2 * es, che,
-                       BM))
+    p.fc_d2 = N - epi.n_split;
+    if (!tc_make_map3_t(&maps[7], ty, epi.D2, (uint64_t)(N - epi.n_split), (uint64_t)M, 1, (uint64_t)epi.ldd2 * es, 0,
+                        che, BM))
       return false;
   }
-  maps[8] = maps[9] = maps[6];
+  // addend / mask maps (2-D loads) need their own maps
+  maps[8] = maps[9] = maps[0];
   if (epi.addend) {
     if (!tc_make_map_t(&maps[8], ty, epi.addend, (uint64_t)N, (uint64_t)M, (uint64_t)epi.ld_add * es, che, BM))
       return false;

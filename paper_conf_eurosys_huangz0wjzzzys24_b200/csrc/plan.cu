@@ -99,6 +99,76 @@ void build_items(const wg_graph_s* g, const Side& S, const std::vector<uint8_t>*
   *n_slots = slot;
 }
 
+}  // namespace
+
+// Per gTask (HBM bytes, both plans' common terms dropped):
+//   EDGE   t_e = n_e (A + 4) + n_rows 2A      (gather f_in rows, Agg round trip)
+//   VERTEX t_v = n_e (B + 4)                  (gather f_out rows)
+// plus per-layer terms: any VERTEX gTask needs Y = x W for every row,
+// V (A + B); a mixed layer also writes / reads / zeroes Z, 3 B per row.
+// sum = {all-EDGE, all-VERTEX, per-gTask minimum (mixed)}; the layer takes
+// the cheapest (ties -> EDGE), i.e. the least-workload DFG.
+// On a 1-D partition the ranks add their sums (wg_plan_create_dist) and take
+// one uniform plan.
+void lin_cost_sums(const wg_graph_s* g, const wg_conv_desc& d, int64_t sum[3], std::vector<uint8_t>* best) {
+  const auto& tasks = g->fwd.h_tasks;
+  const int64_t n = (int64_t)tasks.size();
+  const int s = dsize(d.dtype);
+  const int64_t A = rup((int64_t)d.f_in * s, 32), B = rup((int64_t)d.f_out * s, 32);
+  const int64_t rows = g->ve - g->vb;
+  sum[0] = 0; sum[1] = rows * (A + B); sum[2] = rows * (A + B) + rows * 3 * B;
+  if (best) best->assign(n, 0);
+  for (int64_t i = 0; i < n; ++i) {
+    const wg_task& t = tasks[i];
+    const int64_t ne = t.e_end - t.e_begin;
+    const int64_t nrows = (int64_t)t.d_hi - t.d_lo + 1;
+    const int64_t te = ne * (A + 4) + nrows * 2 * A, tv = ne * (B + 4);
+    sum[0] += te;
+    sum[1] += tv;
+    sum[2] += std::min(te, tv);
+    if (best) (*best)[i] = tv < te ? 1 : 0;
+  }
+}
+
+// Exchange-table layouts.  Widths: forward Y (f_out) for
+// GCN / SAGE / GIN VERTEX layers; backward dT (f_out) on the G path, dAgg
+// (f_in) on the dAgg path, RGCN dT (f_out).  On a graph that owns a row block
+// the GCN / SAGE tables are column-chunked into C <= 4 chunks of >= 256-byte
+// rows (each chunk a whole number of 128-byte TMA store boxes), so the gather
+// of chunk k overlaps the exchange of chunk k+1; GIN / RGCN tables stay
+// row-major (C = 1).  WG_XCHG_CHUNK_BYTES overrides the 256-byte minimum
+// (0 disables chunking).
+void xchg_layouts(wg_plan_s* p) {
+  const wg_graph_s* g = p->g;
+  const wg_conv_desc& d = p->d;
+  p->xf = XLayout{};
+  p->xb = XLayout{};
+  const bool lin = d.model == WG_GCN || d.model == WG_SAGE || d.model == WG_GIN;
+  if (lin) {
+    p->xf.width = d.f_out;
+    p->xb.width = p->bwd_path == 1 ? d.f_out : d.f_in;
+  } else if (d.model == WG_RGCN) {
+    p->xb.width = d.f_out;
+  }
+  const bool part = g->ve - g->vb != g->V;
+  if (!part || !(d.model == WG_GCN || d.model == WG_SAGE)) return;
+  static int64_t min_chunk = -1;
+  if (min_chunk < 0) {
+    const char* e = getenv("WG_XCHG_CHUNK_BYTES");
+    min_chunk = e ? atoll(e) : 256;
+  }
+  if (min_chunk <= 0) return;
+  const int es = dsize(d.dtype);
+  for (XLayout* X : {&p->xf, &p->xb}) {
+    const int64_t pe = pitch(X->width, d.dtype), rho = pe * es;
+    int C = (int)std::min<int64_t>(4, rho / min_chunk);
+    while (C > 1 && (pe % C != 0 || (pe / C * es) % 128 != 0)) --C;
+    if (C > 1) { X->C = C; X->Fc = pe / C; }
+  }
+}
+
+namespace {
+
 // per-task plan bits for the untyped models (GCN / SAGE / GIN)
 void choose_plans(wg_plan_s* p) {
   const wg_graph_s* g = p->g;
@@ -114,30 +184,11 @@ void choose_plans(wg_plan_s* p) {
     std::mt19937_64 rng(d.policy_seed);
     for (int64_t i = 0; i < n; ++i) p->plan_bits[i] = (uint8_t)(rng() & 1);
   } else if (d.policy == WG_PLAN_AUTO) {
-    // Per gTask (HBM bytes, both plans' common terms dropped):
-    //   EDGE   t_e = n_e (A + 4) + n_rows 2A      (gather f_in rows, Agg round trip)
-    //   VERTEX t_v = n_e (B + 4)                  (gather f_out rows)
-    // plus per-layer terms: any VERTEX gTask needs Y = x W for every row,
-    // V (A + B); a mixed layer also writes / reads / zeroes Z, 3 B per row.
-    // The layer takes the cheapest of all-EDGE, all-VERTEX and per-gTask
-    // minimum (ties -> EDGE), i.e. the least-workload DFG.
-    const int s = dsize(d.dtype);
-    const int64_t A = rup((int64_t)d.f_in * s, 32), B = rup((int64_t)d.f_out * s, 32);
-    const int64_t rows = g->ve - g->vb;
-    int64_t sum_e = 0, sum_v = rows * (A + B), sum_m = rows * (A + B) + rows * 3 * B;
-    std::vector<uint8_t> best(n, 0);
-    for (int64_t i = 0; i < n; ++i) {
-      const wg_task& t = tasks[i];
-      const int64_t ne = t.e_end - t.e_begin;
-      const int64_t nrows = (int64_t)t.d_hi - t.d_lo + 1;
-      const int64_t te = ne * (A + 4) + nrows * 2 * A, tv = ne * (B + 4);
-      sum_e += te;
-      sum_v += tv;
-      sum_m += std::min(te, tv);
-      best[i] = tv < te ? 1 : 0;
-    }
-    if (sum_e <= sum_v && sum_e <= sum_m) std::fill(p->plan_bits.begin(), p->plan_bits.end(), 0);
-    else if (sum_v <= sum_m) std::fill(p->plan_bits.begin(), p->plan_bits.end(), 1);
+    int64_t sum[3];
+    std::vector<uint8_t> best;
+    lin_cost_sums(g, d, sum, &best);
+    if (sum[0] <= sum[1] && sum[0] <= sum[2]) std::fill(p->plan_bits.begin(), p->plan_bits.end(), 0);
+    else if (sum[1] <= sum[2]) std::fill(p->plan_bits.begin(), p->plan_bits.end(), 1);
     else p->plan_bits = best;
   }
   // all SPLIT chunks of one row take the plan of the row's first chunk
@@ -211,6 +262,7 @@ wg_status plan_create(wg_graph g, const wg_conv_desc* d, wg_plan* out) {
     p->bwd_path = (p->n_vert_tasks > 0 || (p->n_edge_tasks == 0 && d->policy == WG_PLAN_ALL_VERTEX)) ? 1 : 0;
     if (d->model == WG_GAT) gat_layout(p); else lin_layout(p);
   }
+  xchg_layouts(p);
   g->live_plans++;
   *out = p;
   return WG_OK;

@@ -33,6 +33,28 @@ struct ItemList {
   int64_t n_edges = 0, n_rows = 0;   // totals (algorithmic-byte accounting)
 };
 
+// Column-chunked layout of an exchange table:
+// C chunks of Fc columns, chunk k = [rows x Fc] row-major at k * rows * Fc
+// elements, rows = the graph's global vertex count.  C = 1: one row-major
+// [rows x ld] table (ld chosen by the caller).  Aggregation is
+// column-separable, so the gather of chunk k can start as soon as chunk k of
+// every rank has arrived, overlapping the exchange of chunk k+1.
+struct XLayout {
+  int C = 1;
+  int64_t Fc = 0;          // columns per chunk (C > 1)
+  int64_t width = 0;       // exchanged columns (f_out or f_in)
+};
+
+// Dependency hook for the POST gathers of a distributed call: before the
+// gather of chunk k the compute stream waits for ev[k] (chunk k received).
+struct XHook {
+  const cudaEvent_t* ev = nullptr;
+  int n = 0;
+  void wait(int k, cudaStream_t s) const {
+    if (ev && n > 0) cudaStreamWaitEvent(s, ev[k < n ? k : n - 1], 0);
+  }
+};
+
 }  // namespace wg
 
 struct wg_plan_s {
@@ -47,6 +69,7 @@ struct wg_plan_s {
   int64_t pi = 0, po = 0;            // row pitches (elements) of f_in / f_out wide tensors
   wg::Layout saved, ws;
   std::vector<void*> allocs;
+  wg::XLayout xf, xb;                // exchange tables: forward (Y), backward (dT / dAgg)
   // model-specific structures (conv_rgcn.cu / conv_gat.cu)
   void* rg = nullptr;
   void* gat = nullptr;
@@ -61,11 +84,20 @@ namespace wg {
 wg_status rgcn_plan(wg_plan_s* p, cudaStream_t s);
 void rgcn_plan_free(wg_plan_s* p);
 wg_status rgcn_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* a, cudaStream_t s);
-wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, const wg_grads* G, cudaStream_t s);
+wg_status rgcn_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, const wg_grads* G, cudaStream_t s,
+                        const XHook* hk = nullptr);
 wg_status gat_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* a, cudaStream_t s);
 wg_status gat_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, const wg_grads* G, cudaStream_t s);
-wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* a, cudaStream_t s);
-wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, const wg_grads* G, cudaStream_t s);
+wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* a, cudaStream_t s,
+                      const XHook* hk = nullptr);
+wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, const wg_grads* G, cudaStream_t s,
+                       const XHook* hk = nullptr);
+// exchange layouts of a plan (set by plan_create for graphs owning a row block)
+void xchg_layouts(wg_plan_s* p);
+// a4 layer cost sums {all-EDGE, all-VERTEX, mixed} of the untyped models
+void lin_cost_sums(const wg_graph_s* g, const wg_conv_desc& d, int64_t sum[3], std::vector<uint8_t>* best);
+wg_status plan_create(wg_graph g, const wg_conv_desc* d, wg_plan* out);
+wg_status graph_create(const wg_graph_desc* d, int device, cudaStream_t st, wg_graph* out);
 void gat_layout(wg_plan_s* p);
 void gat_plan_free(wg_plan_s* p);
 void lin_layout(wg_plan_s* p);

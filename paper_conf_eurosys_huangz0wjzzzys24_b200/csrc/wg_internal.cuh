@@ -118,6 +118,7 @@ struct wg_graph_s {
   int32_t* rel_cnt = nullptr;   // [E_total] |in_r(dst_e)| by global edge id (typed graphs)
   std::vector<void*> allocs;
   int live_plans = 0;
+  std::vector<int64_t> bounds;  // 1-D partition of every rank (wg_graph_create_dist), else empty
 };
 
 namespace wg {
@@ -209,6 +210,9 @@ struct GemmEpi {
   int d_f32 = 0;
   // split output: columns >= n_split go to D2 (column n - n_split); n_split % 16 == 0
   void* D2 = nullptr; int64_t ldd2 = 0; int n_split = 0;
+  // column-chunked D (exchange layout [C][rows][Fc]): chunks of d_chunk_cols
+  // columns, d_chunk_stride elements apart; ldd is then the chunk pitch Fc
+  int d_chunk_cols = 0; int64_t d_chunk_stride = 0;
 };
 wg_status gemm_nt(wg_dtype dt, int64_t M, int N, const GemmPart* parts, int n_parts,
                   const GemmEpi& epi, void* scratch, size_t scratch_bytes, cudaStream_t s);
@@ -243,12 +247,14 @@ wg_status prep_weight_batched(wg_dtype dt, const float* W, int batch, int rows, 
 wg_status prep_weight(wg_dtype dt, const float* W, int rows, int cols, int transpose,
                       void* out, int64_t ldo, int out_rows, cudaStream_t s);
 // column sums (deterministic) of dy (optionally relu-masked by ref, written to dt_out)
-// dt2 (optional): the same rows scaled by rs2[row] (the destination scale
-// folded into an exchanged table)
+// dt2 (optional): the same rows scaled by rs2[row] (nullable: 1; the
+// destination scale folded into an exchanged table), in a column-chunked
+// layout when fc2 > 0 (chunks of fc2 columns, cs2 elements apart, pitch ldt2)
 wg_status bias_grad_mask(wg_dtype dt, int64_t M, int N, const void* dy, int64_t lddy,
                          const void* ref, int64_t ldref, void* dt_out, int64_t ldt,
                          float* db, float* scratch, cudaStream_t s,
-                         const float* rs2 = nullptr, void* dt2 = nullptr, int64_t ldt2 = 0);
+                         const float* rs2 = nullptr, void* dt2 = nullptr, int64_t ldt2 = 0, int fc2 = 0,
+                         int64_t cs2 = 0);
 size_t bias_grad_scratch(int64_t M, int N);
 
 // cost-model constants (milli-femtoseconds per byte / per flop), from MEASURED_PEAKS

@@ -11,7 +11,7 @@ import torch
 
 import oracle
 import synth
-from tests.util import (TOL, assert_mask_agrees, f64, gin_inner_safe_dy, kink_band, q, rel_err,
+from tests.util import (TOL, assert_mask_agrees, f64, gin_inner_safe_dy, gin_mags, kink_band, q, rel_err,
                         relu_dy)
 
 pytestmark = pytest.mark.gpu
@@ -63,11 +63,13 @@ def oracle_dy(model, src, dst, V, xo, Wq, dy, dtype, norm, fuse_relu, y_gpu=None
     """Oracle forward + the kink-band-safe dy (tests/util.py): returns
     (pre, dy_in for the kernel, dT for the oracle backward).  y_gpu / h_gpu
     (optional) are checked to take the oracle's ReLU decisions outside the band."""
-    pre, a = oracle_fwd(model, src, dst, V, xo, Wq, norm)
     Wabs = {k: np.abs(v) for k, v in Wq.items()}
-    mag, _, mag_a = (oracle.gin_forward(src, dst, V, np.abs(xo), Wabs["W"], Wabs["bias"], Wabs["W2"], Wabs["b2"],
-                                        return_za=True) if model == "gin"
-                     else (oracle_fwd(model, src, dst, V, np.abs(xo), Wabs, norm)[0], None, None))
+    if model == "gin":
+        pre, z, a = oracle.gin_forward(src, dst, V, xo, Wq["W"], Wq["bias"], Wq["W2"], Wq["b2"], return_za=True)
+        mag_a, mag = gin_mags(z, a, Wq["W"], Wq["bias"], Wq["W2"], Wq["b2"])
+    else:
+        pre = oracle_fwd(model, src, dst, V, xo, Wq, norm)[0]
+        mag = oracle_fwd(model, src, dst, V, np.abs(xo), Wabs, norm)[0]
     dy = np.asarray(dy, dtype=np.float64)
     free = None
     if fuse_relu:

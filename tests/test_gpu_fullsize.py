@@ -20,7 +20,7 @@ import torch
 
 import oracle
 import synth
-from tests.util import (assert_mask_agrees, f64, gin_inner_safe_dy, kink_band, q, relu_dy)
+from tests.util import (assert_mask_agrees, f64, gin_inner_safe_dy, gin_mags, kink_band, q, relu_dy)
 
 pytestmark = pytest.mark.gpu
 
@@ -196,10 +196,9 @@ def test_c4_gin_layer_sampled(c4, layer):
     xo = f64(x)
     deg = np.bincount(dst, minlength=c.V)
     D = sample_rows(deg, g.E_max, n=3000, top=10)
-    pre, _, a = oracle.gin_forward(src, dst, c.V, xo, W["W"], W["bias"], W["W2"], W["b2"], rows=D, return_za=True)
-    Wa = {k: np.abs(v) for k, v in W.items()}
-    mag, _, mag_a = oracle.gin_forward(src, dst, c.V, np.abs(xo), Wa["W"], Wa["bias"], Wa["W2"], Wa["b2"], rows=D,
-                                       return_za=True)
+    pre, z, a = oracle.gin_forward(src, dst, c.V, xo, W["W"], W["bias"], W["W2"], W["b2"], rows=D, return_za=True)
+    mag_a, mag = np.zeros_like(a), np.zeros_like(pre)
+    mag_a[D], mag[D] = gin_mags(z[D], a[D], W["W"], W["bias"], W["W2"], W["b2"])
     Dd = torch.from_numpy(D).cuda()
     yg = f64(y[Dd])
     yo = np.maximum(pre[D], 0) if relu else pre[D]

@@ -81,6 +81,18 @@ def gin_inner_safe_dy(dy, a, band_a, W2, free=None):
             continue
         A = W2[np.ix_(J, S)]
         g = dy[v, S]
-        coef, *_ = np.linalg.lstsq(A @ A.T, A @ g, rcond=None)
+        coef, *_ = np.linalg.lstsq(A.T, g, rcond=None)   # SVD: stable for near-square A
         dy[v, S] = g - A.T @ coef
     return dy
+
+
+def gin_mags(z, a, W1, b1, W2, b2):
+    """First-order error magnitudes of GIN's two pre-activations on the
+    kernel's path: a = z W1 + b1 is computed from z rounded once to the conv
+    dtype (mag_a = |z| |W1| + |b1|); y = h W2 + b2 from h = ReLU(a) rounded
+    once, h inheriting a's error (mag_y = (|h| + mag_a) |W2| + |b2|).  (The
+    oracle run on |x| would bound z by sum |x|, which for a hub row is
+    orders of magnitude above |z| and the actual rounding.)"""
+    mag_a = np.abs(z) @ np.abs(W1) + np.abs(b1)
+    mag_y = (np.maximum(a, 0) + mag_a) @ np.abs(W2) + np.abs(b2)
+    return mag_a, mag_y
