@@ -291,59 +291,69 @@ def main():
             dist.init_process_group(backend)
         group = dist.group.WORLD
     import paper_conf_eurosys_huangz0wjzzzys24_b200 as wg
-    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack, partition_1d
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack, equal_blocks
 
     c, model, cfg = workload(args.config, args.model)
     dev = torch.device("cuda", local)
     P = args.rank_slice
     if P > 1 and (world > 1 or model in ("gat", "rgcn") or c.symmetric):
         raise SystemExit("--rank-slice: one process, directed untyped GCN / SAGE / GIN configs")
+    if world > 1 and model == "gat":
+        raise SystemExit("the 1-D multi-GPU partition covers GCN / SAGE / GIN / RGCN (DESIGN.md §9)")
     t0 = time.perf_counter()
+    comm, bounds = None, None
     if P > 1:
+        # one rank of the P-way partition: only the edges touching its block
+        # exist here, so the blocks are equal T-aligned vertex ranges (the
+        # seeded permutation scatters hubs: edges balance to ~1 %)
         import synth
-        block, bounds = partition_1d(c.V, P)
-        vb, ve = bounds[args.slice_rank]
+        block, blocks = equal_blocks(c.V, P)
+        vb, ve = blocks[args.slice_rank]
+        bounds = [lo for lo, _ in blocks] + [c.V]
         src, dst = synth.make_graph_slice(c.V, c.E, vb, ve, seed=c.seed * 16, alpha=c.alpha)
         et, x_np = None, None
         labels_np = np.random.Generator(np.random.Philox(c.seed * 16 + 5)).integers(
             0, c.dims[-1], c.V).astype(np.int64)[vb:ve]
         args.no_e2e, args.no_cpu = True, True
+        comm = wg.Comm(emulate=(args.slice_rank, P), device=local)
         cfg.update(rank_slice={"P": P, "rank": args.slice_rank, "v_begin": vb, "v_end": ve,
                                "edges_touching_block": int(src.shape[0]),
                                "note": "per-rank compute of the P-way 1-D partition on one GPU: the rank's "
-                                       "in-edges (forward) and out-edges (backward), PRE / POST phases and "
-                                       "exchange tables; all-gathers / gradient all-reduce not executed, so "
-                                       "exchanged rows and non-owned degrees are not the global ones (timing run)",
+                                       "in-edges (forward) and out-edges (backward) through the library's "
+                                       "distributed calls with the EMULATED communicator: every exchange is a "
+                                       "copy kernel on the communication stream rewriting the non-owned rows "
+                                       "(WG_EMU_CTAS CTAs), overlapped chunk by chunk with the gathers as the "
+                                       "NCCL exchange would be; no data moves between ranks and non-owned "
+                                       "degrees are not the global ones (a timing run)",
                                "features": "torch.randn on the device (the 111M x 128 table is not built on the host)"})
     else:
         src, dst, et, x_np, labels_np = make_inputs(c, model)
+        if world > 1:
+            comm = wg.Comm(group, device=local)      # NCCL inside libwg (wg_comm_init)
     t_gen = time.perf_counter() - t0
-    if world > 1 and model == "gat":
-        raise SystemExit("the 1-D multi-GPU partition covers GCN / SAGE / GIN / RGCN (DESIGN.md §9)")
-    if P <= 1:
-        block, bounds = partition_1d(c.V, world)
-        vb, ve = bounds[rank] if world > 1 else (0, c.V)
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     R = c.R if model == "rgcn" else 1
     g = wg.Graph(torch.from_numpy(src).to(dev), torch.from_numpy(dst).to(dev), num_vertices=c.V,
                  etype=torch.from_numpy(et).to(dev) if R > 1 else None, num_types=R,
-                 v_begin=vb if (world > 1 or P > 1) else 0, v_end=ve if (world > 1 or P > 1) else 0,
-                 max_task_edges=args.emax, tile_rows=args.tile)
+                 max_task_edges=args.emax, tile_rows=args.tile, comm=comm, bounds=bounds)
+    vb, ve = g.v_begin, g.v_begin + g.n_rows
+    if world > 1:
+        cfg.update(partition={"bounds": [int(b) for b in g.bounds], "rank_rows": ve - vb,
+                              "rank_in_edges": int(g.E_fwd), "rank_out_edges": int(g.E_T),
+                              "rule": "edge-balanced T-aligned blocks (wg_partition_1d)"})
     if P > 1:
         src = dst = None   # host copies of the slice are not needed any more
     torch.cuda.synchronize()
     t_part = time.perf_counter() - t0
     dtype = torch.bfloat16 if c.dtype == "bf16" else torch.float32
     t0 = time.perf_counter()
-    stack = GNNStack(g, model, c.dims, dtype=dtype, policy=args.policy, group=group,
-                     block=block if (world > 1 or P > 1) else None, heads=c.heads if model == "gat" else 1, R=R,
-                     conv_kw=conv_options(c, model), sim_world=max(P, 1))
+    stack = GNNStack(g, model, c.dims, dtype=dtype, policy=args.policy, heads=c.heads if model == "gat" else 1, R=R,
+                     conv_kw=conv_options(c, model))
     t_plan = time.perf_counter() - t0
-    Vtab = stack.Vtab
-    x = wg.padded(Vtab, c.dims[0], dtype, dev)
+    x = wg.padded(c.V, c.dims[0], dtype, dev)
     if x_np is not None:
-        x[:c.V].copy_(torch.from_numpy(x_np).to(dev))
+        x.copy_(torch.from_numpy(x_np).to(dev))
     else:
         gen = torch.Generator(device=dev).manual_seed(c.seed * 16 + 2)
         for r0 in range(0, c.V, 1 << 22):
@@ -362,13 +372,15 @@ def main():
         stack.step(x, labels, c.V)
     torch.cuda.synchronize()
     barrier()
-    # One training step captured in a CUDA graph (one process per GPU, no
-    # collectives inside): the timed region replays it K times, so host
-    # launch overhead (ctypes marshalling, ~20-55 launches per step) leaves
-    # the step time.  Per-kernel times come from the profiled eager pass below
+    # One training step captured in a CUDA graph (one process per GPU; the
+    # library's NCCL exchanges and gradient all-reduces run on its
+    # communication stream, forked from and joined back into the captured
+    # stream, so they are captured too): the timed region replays it K times,
+    # so host launch overhead (ctypes marshalling, ~20-55 launches per step)
+    # leaves the step time.  Per-kernel times come from the profiled eager pass below
     # (the same launches; a graph replay has no per-kernel events).
     graph, graph_err = None, None
-    if world == 1 and not args.no_graph:
+    if not args.no_graph:
         try:
             side = torch.cuda.Stream(device=dev)
             side.wait_stream(stream)
@@ -438,7 +450,7 @@ def main():
         xh = torch.from_numpy(x_np).to(dtype).pin_memory()
         lh = torch.from_numpy(labels_np[vb:ve] if world > 1 else labels_np).pin_memory()
         loss_h = torch.empty(1, dtype=torch.float32).pin_memory()
-        xs = [x, wg.padded(Vtab, c.dims[0], dtype, dev)]
+        xs = [x, wg.padded(c.V, c.dims[0], dtype, dev)]
         ls = [labels, torch.empty_like(labels)]
         cstream = torch.cuda.Stream(device=dev)
         done = [torch.cuda.Event(), torch.cuda.Event()]
@@ -447,7 +459,7 @@ def main():
         def issue_copy(b):
             cstream.wait_event(done[b])
             with torch.cuda.stream(cstream):
-                xs[b][:c.V].copy_(xh, non_blocking=True)
+                xs[b].copy_(xh, non_blocking=True)
                 ls[b].copy_(lh, non_blocking=True)
             ready[b].record(cstream)
 

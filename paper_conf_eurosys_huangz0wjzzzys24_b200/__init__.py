@@ -134,6 +134,20 @@ class Comm:
         self._h = h
         self.emulated = emulate is not None
 
+    @classmethod
+    def single(cls, device: int | None = None):
+        """A one-rank NCCL communicator (no process group needed)."""
+        c = cls.__new__(cls)
+        L = C.lib()
+        c.device = torch.cuda.current_device() if device is None else device
+        uid = torch.zeros(C.COMM_ID_BYTES, dtype=torch.uint8)
+        h = ctypes.c_void_p()
+        with torch.cuda.device(c.device):
+            C.check(L.wg_comm_unique_id(_ptr(uid)), "wg_comm_unique_id")
+            C.check(L.wg_comm_init(_ptr(uid), 0, 1, c.device, ctypes.byref(h)), "wg_comm_init")
+        c._h, c.rank, c.world, c.emulated = h, 0, 1, False
+        return c
+
     @property
     def handle(self):
         return self._h

@@ -144,14 +144,19 @@ void xchg_layouts(wg_plan_s* p) {
   p->xf = XLayout{};
   p->xb = XLayout{};
   const bool lin = d.model == WG_GCN || d.model == WG_SAGE || d.model == WG_GIN;
+  const bool part = g->ve - g->vb != g->V;
+  if (!part) return;                         // one partition: nothing is exchanged
   if (lin) {
-    p->xf.width = d.f_out;
-    p->xb.width = p->bwd_path == 1 ? d.f_out : d.f_in;
+    // forward: VERTEX layers exchange Y (a rank with no gTask follows the
+    // layer's VERTEX policy); EDGE layers gather the caller's activation
+    if (p->n_vert_tasks > 0 || (p->n_edge_tasks == 0 && d.policy == WG_PLAN_ALL_VERTEX)) p->xf.width = d.f_out;
+    // backward: dT (G path) or dAgg (dAgg path, only when dx is needed)
+    if (p->bwd_path == 1) p->xb.width = d.f_out;
+    else if (d.need_dx) p->xb.width = d.f_in;
   } else if (d.model == WG_RGCN) {
     p->xb.width = d.f_out;
   }
-  const bool part = g->ve - g->vb != g->V;
-  if (!part || !(d.model == WG_GCN || d.model == WG_SAGE)) return;
+  if (!(d.model == WG_GCN || d.model == WG_SAGE)) return;
   static int64_t min_chunk = -1;
   if (min_chunk < 0) {
     const char* e = getenv("WG_XCHG_CHUNK_BYTES");
@@ -160,6 +165,7 @@ void xchg_layouts(wg_plan_s* p) {
   if (min_chunk <= 0) return;
   const int es = dsize(d.dtype);
   for (XLayout* X : {&p->xf, &p->xb}) {
+    if (!X->width) continue;
     const int64_t pe = pitch(X->width, d.dtype), rho = pe * es;
     int C = (int)std::min<int64_t>(4, rho / min_chunk);
     while (C > 1 && (pe % C != 0 || (pe / C * es) % 128 != 0)) --C;

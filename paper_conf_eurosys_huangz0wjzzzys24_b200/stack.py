@@ -2,16 +2,25 @@
 the 1-D multi-GPU partition of SURVEY §8(e)).
 
 Forward: layer i reads the previous activation table and writes its own rows
-straight into the next layer's table.  Distributed (one process per GPU,
-torch.distributed / NCCL): rank p owns the T-aligned vertex block
-[p*B, (p+1)*B) of every activation and gradient table; before a layer the
-table its gathers read is all-gathered in place -- the activation itself for
-EDGE (gather-then-transform) layers, or Y = h W for VERTEX layers when the
-transformed rows are narrower (transform-before-communicate, P:L2279-2289,
-Fig 11c).  Backward mirrors it: the per-layer PRE phase writes this rank's
-rows of dAgg (or dT) into the exchange table, the table is all-gathered, and
-the POST phase runs the transposed gather over the rank's out-edges.  Weight
-gradients are all-reduced (sum).  Rows >= V in the last block are padding.
+straight into the next layer's table.  Distributed (one process per GPU):
+rank p owns the T-aligned vertex block [b_p, b_{p+1}) of every activation and
+gradient table (edge-balanced bounds, wg_partition_1d); tables the next layer
+gathers hold all V rows.
+
+* Library path (the product path): the graph carries a ``Comm`` (NCCL over
+  the ranks, or the one-GPU emulation of one rank).  Each layer is one
+  ``wg_conv_forward_dist`` / ``wg_conv_backward_dist`` call: the library
+  exchanges the table its gathers read over NCCL on its communication stream
+  -- the activation itself for EDGE layers, Y = h W for VERTEX layers
+  (transform before communicate, Fig 11c), dT / dAgg in the
+  backward -- column-chunked so the gather of one chunk overlaps the exchange
+  of the next, and all-reduces the weight gradients under the next layer's
+  backward.  The plan of every layer is one uniform plan on all ranks
+  (wg_plan_create_dist).
+* torch.distributed path (multi-process CPU tests of this orchestration with
+  the test-only layers of tests/test_dist_gloo.py): the same PRE / exchange /
+  POST sequence with torch.distributed collectives (all-gather-v as one
+  broadcast per rank block) and a per-layer plan vote.
 """
 from __future__ import annotations
 
@@ -25,31 +34,32 @@ class GNNStack:
     """L gTask layers (hidden ReLU fused into the layer epilogue) + CE loss + Adam."""
 
     def __init__(self, graph: Graph, model: str, dims, *, dtype=torch.bfloat16, heads: int = 1, policy="auto",
-                 seed: int = 0, lr: float = 1e-3, group=None, block: int | None = None, R: int = 1,
-                 conv_kw: dict | None = None, conv_factory=None, device=None, sim_world: int = 1):
+                 seed: int = 0, lr: float = 1e-3, group=None, bounds=None, R: int = 1,
+                 conv_kw: dict | None = None, conv_factory=None, device=None):
         # conv_kw: extra Conv options for every layer (e.g. RGCN norm / self_loop).
-        # conv_factory / device: injection points for the multi-process CPU test
-        # of this orchestration (tests/test_dist_gloo.py); the product path uses
-        # Conv (libwg.so) on the graph's CUDA device.
-        # sim_world > 1 (no group): one rank of a sim_world-way 1-D partition
-        # on one GPU -- the rank's own kernels (PRE / POST phases, exchange
-        # tables) run, the collectives are skipped (timing of the per-rank
-        # compute only; exchanged rows are not filled in).
+        # group / bounds / conv_factory / device: the torch.distributed path
+        # (tests/test_dist_gloo.py); the product path takes the communicator
+        # and the partition from the graph (Graph(..., comm=Comm(...))).
         Conv_ = conv_factory or Conv
         self.g, self.model, self.dims, self.dtype = graph, model, list(dims), dtype
         self.L = len(dims) - 1
         self.dev = device if device is not None else torch.device("cuda", graph.device)
+        self.comm = getattr(graph, "comm", None)
         self.group = group
-        self.sim = group is None and sim_world > 1
-        self.dist = (group is not None and torch.distributed.get_world_size(group) > 1) or self.sim
-        self.world = torch.distributed.get_world_size(group) if group is not None else sim_world
-        self.rank = torch.distributed.get_rank(group) if group is not None else (
-            graph.v_begin // block if self.sim else 0)
+        self.tdist = self.comm is None and group is not None and torch.distributed.get_world_size(group) > 1
+        if self.comm is not None:
+            self.world, self.rank = self.comm.world, self.comm.rank
+        elif self.tdist:
+            self.world, self.rank = torch.distributed.get_world_size(group), torch.distributed.get_rank(group)
+        else:
+            self.world, self.rank = 1, 0
+        self.dist = self.world > 1
+        self.bounds = [int(b) for b in (graph.bounds if self.comm is not None else bounds)] if self.dist else None
         self.rows = graph.n_rows
         self.vb = graph.v_begin
-        self.block = block if block is not None else self.rows
-        self.Vtab = self.block * self.world if self.dist else graph.V
+        self.V = graph.V
         self.convs, self.params = [], []
+        self.vertex_layer = []
         # layer i reads a table of width f_in(i): dims[0], then the previous
         # layer's output width (heads * dims[i] for concatenated GAT heads)
         self.f_in = [dims[0]] + [heads * dims[i] if model == "gat" else dims[i] for i in range(1, self.L)]
@@ -58,45 +68,44 @@ class GNNStack:
             kw = dict(dtype=dtype, fuse_relu=not last, need_dx=i > 0, seed=seed + i, **(conv_kw or {}))
             if model == "gat":
                 kw.update(heads=heads, concat=not last)
-            pol = policy
             fi = self.f_in[i]
-            conv = Conv_(graph, model, fi, dims[i + 1], policy=pol, **kw)
-            if self.dist and model != "rgcn":   # one uniform plan per layer, the same on every rank
-                ne, nv = conv.n_edge_tasks, conv.n_vertex_tasks
-                if group is not None:   # ranks plan their own rows: vote by gTask counts
-                    dev = self.dev if torch.distributed.get_backend(group) == "nccl" else torch.device("cpu")
-                    votes = torch.tensor([ne, nv], dtype=torch.int64, device=dev)
-                    torch.distributed.all_reduce(votes, group=group)
-                    ne, nv = (int(v) for v in votes.tolist())
-                uni = "vertex" if nv > ne else "edge"
-                if (conv.n_vertex_tasks if uni == "edge" else conv.n_edge_tasks) or \
-                        (uni == "vertex" and not conv.n_vertex_tasks and pol != "vertex"):
-                    pol = uni
-                    conv.close()
-                    conv = Conv_(graph, model, fi, dims[i + 1], policy=pol, **kw)
+            conv = Conv_(graph, model, fi, dims[i + 1], policy=policy, **kw)
+            if self.tdist and model != "rgcn":
+                conv = self._vote(conv, Conv_, graph, model, fi, dims[i + 1], policy, kw)
+            # a VERTEX layer exchanges Y; a rank with no gTask follows the agreed policy (G path)
+            self.vertex_layer.append(model != "rgcn" and (conv.n_vertex_tasks > 0 or (
+                conv.n_edge_tasks == 0 and getattr(conv, "bwd_path", 0) == 1)))
             self.convs.append(conv)
             self._share_workspace(conv)
             self.params.append(init_params(model, fi, dims[i + 1], heads=heads, concat=not last, R=R,
                                            self_loop=bool((conv_kw or {}).get("self_loop", False)),
                                            bias=bool((conv_kw or {}).get("bias", True)),
                                            device=self.dev, seed=seed + 100 + i))
-        # activation tables: h[0] = input, h[i+1] = output of layer i (global
-        # rows when distributed: the next layer gathers them; the logits of the
-        # last layer are never exchanged, so that table holds the owned rows)
-        self.h = [None] + [padded(self.Vtab if i + 1 < self.L else self.rows, c.out_dim, dtype, self.dev)
+        # activation tables: h[0] = input, h[i+1] = output of layer i (all V
+        # rows when distributed: the next layer gathers them; the logits of
+        # the last layer are never exchanged, so that table holds owned rows)
+        self.h = [None] + [padded(self.V if i + 1 < self.L else self.rows, c.out_dim, dtype, self.dev)
                            for i, c in enumerate(self.convs)]
         self.saved = [c.new_saved() for c in self.convs]
         # dx of layer i (= dy of layer i-1): owned rows only (the exchange
         # tables carry what other ranks read)
         self.dx = [None] + [padded(self.rows, self.f_in[i], dtype, self.dev) for i in range(1, self.L)]
-
         self.grads = [{k: torch.zeros_like(v) for k, v in p.items()} for p in self.params]
         self.xchg_f, self.xchg_b = [], []
-        for c in self.convs:
-            self.xchg_f.append(padded(self.Vtab, pitch(c.f_out, dtype), dtype, self.dev)
-                               if self._fwd_xchg(c) else None)
-            wb = (c.f_out if c.bwd_path == 1 else c.f_in)
-            self.xchg_b.append(padded(self.Vtab, pitch(wb, dtype), dtype, self.dev) if self.dist else None)
+        for i, c in enumerate(self.convs):
+            if self.comm is not None and self.dist:
+                self.xchg_f.append(c.new_xchg(0))
+                self.xchg_b.append(c.new_xchg(1))
+            elif self.tdist:
+                self.xchg_f.append(padded(self.V, pitch(c.f_out, dtype), dtype, self.dev)
+                                   if self.vertex_layer[i] else None)
+                # layer 0 on the dAgg path writes no exchange rows (need_dx = False)
+                need_b = model == "rgcn" or getattr(c, "bwd_path", 0) == 1 or i > 0
+                wb = c.f_out if (model == "rgcn" or getattr(c, "bwd_path", 0) == 1) else c.f_in
+                self.xchg_b.append(padded(self.V, pitch(wb, dtype), dtype, self.dev) if need_b else None)
+            else:
+                self.xchg_f.append(None)
+                self.xchg_b.append(None)
         for p in self.params:
             for v in p.values():
                 v.requires_grad_(True)
@@ -106,6 +115,22 @@ class GNNStack:
                                     capturable=self.dev.type == "cuda")
 
     # -------------------------------------------------------------- helpers
+    def _vote(self, conv, Conv_, graph, model, fi, fo, policy, kw):
+        """torch.distributed path: every rank must run the same plan (the
+        ranks exchange one table); the ranks' EDGE / VERTEX gTask counts are
+        summed and the majority plan is rebuilt where it differs -- including
+        on a rank with no gTask, which then follows the agreed policy."""
+        ne, nv = conv.n_edge_tasks, conv.n_vertex_tasks
+        dev = self.dev if torch.distributed.get_backend(self.group) == "nccl" else torch.device("cpu")
+        votes = torch.tensor([ne, nv], dtype=torch.int64, device=dev)
+        torch.distributed.all_reduce(votes, group=self.group)
+        uni = "vertex" if int(votes[1]) > int(votes[0]) else "edge"
+        if (uni == "vertex" and conv.n_edge_tasks) or (uni == "edge" and conv.n_vertex_tasks) or \
+                (uni == "vertex" and not conv.n_vertex_tasks and policy != "vertex"):
+            conv.close()
+            conv = Conv_(graph, model, fi, fo, policy=uni, **kw)
+        return conv
+
     def _share_workspace(self, conv):
         """One workspace for all layers: a layer's scratch lives only inside its
         forward / backward call (the PRE and POST phases of one layer are not
@@ -130,35 +155,36 @@ class GNNStack:
         """Rows of layer i's output table this rank writes."""
         return self._own(self.h[i + 1]) if i + 1 < self.L else self.h[self.L]
 
-    def _fwd_xchg(self, c):
-        """VERTEX layers exchange Y = h W (transform before communicate); RGCN
-        (per-relation transforms) and EDGE layers gather the activation itself."""
-        return self.dist and c.n_vertex_tasks > 0 and c.model != "rgcn"
-
     def _own(self, t):
         return t[self.vb:self.vb + self.rows] if self.dist else t
 
-    def _allgather(self, t):
-        if not self.dist or self.sim:
-            return
-        full = t.as_strided((self.Vtab, t.stride(0)), (t.stride(0), 1))
-        mine = full[self.rank * self.block:(self.rank + 1) * self.block]
-        torch.distributed.all_gather_into_tensor(full, mine, group=self.group)
+    def _allgatherv(self, t):
+        """torch.distributed path: every rank's row block of a [V x ld] table,
+        in place (one broadcast per rank block: blocks differ in size)."""
+        full = t.as_strided((self.V, t.stride(0)), (t.stride(0), 1))
+        for q in range(self.world):
+            b0, b1 = self.bounds[q], self.bounds[q + 1]
+            blk = full[b0:b1]
+            src = torch.distributed.get_global_rank(self.group, q) if self.group is not None else q
+            torch.distributed.broadcast(blk, src=src, group=self.group)
 
+    # -------------------------------------------------------------- forward / backward
     def forward(self, x):
-        """x: [V_tab x f0] (replicated input features); returns this rank's logits rows."""
+        """x: [V x f0] (replicated input features); returns this rank's logits rows."""
         h = x
         for i, c in enumerate(self.convs):
             y = self._out(i)
-            if self._fwd_xchg(c):
+            if self.comm is not None and self.dist:
+                c.forward_dist(h, self.params[i], y, self.saved[i], xchg=self.xchg_f[i], x_gathered=i == 0)
+            elif self.tdist and self.vertex_layer[i]:
                 xg = self.xchg_f[i]
                 c.forward_raw(h, self.params[i], y=y, saved=self.saved[i], phase=C.PHASE_PRE, xchg=xg)
-                self._allgather(xg)
+                self._allgatherv(xg)
                 c.forward_raw(h, self.params[i], y=y, saved=self.saved[i], phase=C.PHASE_POST, xchg=xg)
             else:
+                if self.tdist and i > 0:
+                    self._allgatherv(h)             # EDGE / RGCN layers gather raw rows
                 c.forward_raw(h, self.params[i], y=y, saved=self.saved[i])
-            if self.dist and i + 1 < self.L and not self._fwd_xchg(self.convs[i + 1]):
-                self._allgather(self.h[i + 1])       # next EDGE / RGCN layer gathers raw rows
             h = self.h[i + 1]
         self.x = x
         return self.h[self.L]
@@ -177,16 +203,20 @@ class GNNStack:
             fuse = self.fuse_masks and i > 0 and getattr(self.convs[i - 1], "fuse_relu", False)
             kw = dict(grads=self.grads[i], dy_masked=masked,
                       dx_mask=self._own(self.h[i]) if fuse else None)
-            if self.dist:
+            if self.comm is not None and self.dist:
+                c.backward_dist(g, xin, y, self.saved[i], self.params[i], dx=dx, xchg=self.xchg_b[i], **kw)
+            elif self.tdist and self.xchg_b[i] is not None:
                 xb = self.xchg_b[i]
                 c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, phase=C.PHASE_PRE, xchg=xb, **kw)
-                self._allgather(xb)
+                self._allgatherv(xb)
                 c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, phase=C.PHASE_POST, xchg=xb, **kw)
             else:
                 c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, **kw)
             g = dx
             masked = fuse
-        if self.dist and not self.sim:
+        if self.comm is not None:
+            self.comm.wait()                        # the gradient all-reduces left running by backward_dist
+        elif self.tdist:
             flat = torch.cat([v.reshape(-1) for gr in self.grads for v in gr.values()])
             torch.distributed.all_reduce(flat, group=self.group)
             o = 0
@@ -210,7 +240,11 @@ class GNNStack:
         return self._loss
 
 
-def partition_1d(V: int, world: int, T: int = 128):
-    """Equal T-aligned vertex blocks: returns (block_rows, [(v_begin, v_end)] per rank)."""
+def equal_blocks(V: int, world: int, T: int = 128):
+    """Equal T-aligned vertex blocks: (block_rows, [(v_begin, v_end)] per rank).
+    Used where only one rank's edges exist (the C5 rank slice, one-GPU phase
+    simulations); the product partition is the edge-balanced wg_partition_1d."""
     block = -(-(-(-V // world)) // T) * T
-    return block, [(min(V, p * block), min(V, (p + 1) * block)) for p in range(world)]
+    if (world - 1) * block >= V:
+        raise ValueError(f"{world} ranks of {block} rows leave a rank without vertices (V = {V}, T = {T})")
+    return block, [(p * block, min(V, (p + 1) * block)) for p in range(world)]

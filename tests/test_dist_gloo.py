@@ -1,9 +1,11 @@
 """World-size-2 gloo test (CPU) of the 1-D multi-GPU orchestration (§8(e)).
 
-GNNStack's distributed path (T-aligned equal vertex blocks, PRE / all-gather /
-POST exchange phases for forward and backward, exchanged table = activation
-for EDGE layers or Y = x W for VERTEX layers, dAgg or dT in backward, weight-
-gradient all-reduce) runs on two CPU processes over gloo.  The layer compute is
+GNNStack's torch.distributed path (the library's edge-balanced T-aligned
+partition bounds from wg_partition_1d -- a host computation, no GPU -- PRE /
+all-gather-v / POST exchange phases for forward and backward, exchanged table
+= activation for EDGE layers or Y = x W for VERTEX layers, dAgg or dT in
+backward, one agreed plan per layer, weight-gradient all-reduce) runs on two
+CPU processes over gloo.  The layer compute is
 a test-only float64 torch implementation of GraphSAGE (and of RGCN with
 1/|N_v^r| normalisation and a self-loop: its forward reads the all-gathered
 activation, its backward exchanges dT) that honours the library's phase contract (include/wg.h, wg_fwd_args / wg_bwd_args); the CUDA
@@ -193,13 +195,13 @@ def factory(graph, model, fi, fo, **kw):
 V, E, DIMS, R = 700, 6000, [8, 6, 6, 5], 3
 
 
-def run_stack(graph, group, block, model="sage"):
+def run_stack(graph, group, bounds, model="sage"):
     from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack
     torch.manual_seed(0)
     kw = dict(R=R, conv_kw={"self_loop": True}) if model == "rgcn" else {}
-    st = GNNStack(graph, model, DIMS, dtype=torch.float64, group=group, block=block, conv_factory=factory,
+    st = GNNStack(graph, model, DIMS, dtype=torch.float64, group=group, bounds=bounds, conv_factory=factory,
                   device=torch.device("cpu"), seed=3, **kw)
-    x = torch.zeros(st.Vtab, DIMS[0], dtype=torch.float64)
+    x = torch.zeros(V, DIMS[0], dtype=torch.float64)
     x[:V] = torch.from_numpy(synth.make_features(V, DIMS[0], seed=4)).double()
     logits = st.forward(x).clone()
     dl = torch.from_numpy(synth.normal((V, DIMS[-1]), seed=5)).double()
@@ -211,13 +213,13 @@ def run_stack(graph, group, block, model="sage"):
 def worker(rank, world, port, q, model):
     os.environ["MASTER_ADDR"], os.environ["MASTER_PORT"] = "127.0.0.1", str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import partition_1d
+    from paper_conf_eurosys_huangz0wjzzzys24_b200 import partition_1d
     src, dst, et = synth.make_graph(V, E, seed=9, alpha=0.5, symmetric=model != "rgcn", R=R if model == "rgcn" else 1)
     et = et if model == "rgcn" else None
     ref_logits, ref_grads = run_stack(FakeGraph(src, dst, V, etype=et), None, None, model)
-    block, bounds = partition_1d(V, world, T=128)
-    vb, ve = bounds[rank]
-    logits, grads = run_stack(FakeGraph(src, dst, V, vb, ve, etype=et), dist.group.WORLD, block, model)
+    bounds = partition_1d(src, dst, num_vertices=V, world=world, tile_rows=128)
+    vb, ve = int(bounds[rank]), int(bounds[rank + 1])
+    logits, grads = run_stack(FakeGraph(src, dst, V, vb, ve, etype=et), dist.group.WORLD, bounds, model)
     ok = torch.allclose(logits, ref_logits[vb:ve], rtol=1e-10, atol=1e-12)
     for g1, g2 in zip(grads, ref_grads):      # fp32 gradients: all-reduce sums partials in another order
         for k in g1:
@@ -258,10 +260,36 @@ def test_gloo_1d_partition_matches_single(world, model):
     assert sorted(r[2] for r in res)[0][0] == 0
 
 
-def test_partition_1d_blocks():
-    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import partition_1d
-    for Vv, P in [(2449029, 8), (1000, 3), (128, 2), (129, 4)]:
-        block, b = partition_1d(Vv, P)
+def test_partition_1d_edge_balanced():
+    """wg_partition_1d (host computation, no GPU): T-aligned, covering, every
+    rank >= 1 tile, and each rank's in- + out-edges + rows within one tile's
+    load of 1/world of the total (greedy nearest-boundary)."""
+    from paper_conf_eurosys_huangz0wjzzzys24_b200 import partition_1d
+    for Vv, Ee, P, T in [(5000, 60000, 4, 128), (3000, 40000, 3, 128), (1000, 9000, 8, 64), (300, 2000, 2, 128)]:
+        src, dst, _ = synth.make_graph(Vv, Ee, seed=Vv, alpha=0.8)
+        b = partition_1d(src, dst, num_vertices=Vv, world=P, tile_rows=T)
+        assert b[0] == 0 and b[-1] == Vv and all(b[i] < b[i + 1] for i in range(P))
+        assert all(x % T == 0 for x in b[:-1])
+        w = np.bincount(src, minlength=Vv) + np.bincount(dst, minlength=Vv) + 1
+        loads = np.array([w[b[i]:b[i + 1]].sum() for i in range(P)])
+        tile_max = max(w[t:t + T].sum() for t in range(0, Vv, T))
+        assert np.abs(loads - w.sum() / P).max() <= tile_max + 1, (loads, w.sum() / P, tile_max)
+    # CSR input gives the same bounds as COO; too few tiles is an error
+    src, dst, _ = synth.make_graph(2000, 20000, seed=1, alpha=0.6)
+    order = np.argsort(dst, kind="stable")
+    indptr = np.concatenate([[0], np.cumsum(np.bincount(dst, minlength=2000))]).astype(np.int64)
+    np.testing.assert_array_equal(partition_1d(src[order], None, num_vertices=2000, world=4, indptr=indptr),
+                                  partition_1d(src, dst, num_vertices=2000, world=4))
+    from paper_conf_eurosys_huangz0wjzzzys24_b200 import WGError
+    with pytest.raises(WGError):
+        partition_1d(src, dst, num_vertices=2000, world=40)
+
+
+def test_equal_blocks():
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import equal_blocks
+    for Vv, P in [(2449029, 8), (1000, 3), (256, 2), (111059956, 8)]:
+        block, b = equal_blocks(Vv, P)
         assert block % 128 == 0 and b[0][0] == 0 and b[-1][1] == Vv
-        # block starts are T-aligned (a trailing empty block starts at V)
-        assert all(lo % 128 == 0 or lo == Vv for lo, _ in b) and all(b[i][1] == b[i + 1][0] for i in range(P - 1))
+        assert all(lo % 128 == 0 and lo < hi for lo, hi in b) and all(b[i][1] == b[i + 1][0] for i in range(P - 1))
+    with pytest.raises(ValueError):
+        equal_blocks(129, 4)

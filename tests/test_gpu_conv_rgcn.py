@@ -107,7 +107,7 @@ def test_rgcn_1d_partition_phases_match_oracle(policy, P):
     out-edges; the blocks' y / dx rows and the summed weight gradients equal
     the oracle (global 1/|N_v^r| coefficients, SPLIT rows via a small E_max)."""
     m = wg()
-    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import partition_1d
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import equal_blocks
     V, E, fi, fo, R = 3000, 40000, 24, 16, 6
     dtype = torch.float32
     src, dst, et = synth.make_graph(V, E, seed=41, alpha=0.7, R=R)
@@ -115,7 +115,7 @@ def test_rgcn_1d_partition_phases_match_oracle(policy, P):
     dy = torch.from_numpy(synth.normal((V, fo), seed=43, std=0.25))
     params = m.init_params("rgcn", fi, fo, R=R, self_loop=True, bias=True, seed=4)
     ts, td, tt = (torch.from_numpy(a).cuda() for a in (src, dst, et))
-    block, bounds = partition_1d(V, P)
+    block, bounds = equal_blocks(V, P)
     Vt = block * P
     xt = m.padded(Vt, fi, dtype)
     xt[:V] = x.cuda()

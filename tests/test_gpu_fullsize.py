@@ -374,10 +374,10 @@ def test_c3_rgcn_layer1_sampled():
 def c5slice():
     """Rank 0's slice of C5's 8-way 1-D partition (its in- and out-edges), the
     graph bench.py --rank-slice 8 builds."""
-    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import partition_1d
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import equal_blocks
     c = synth.CONFIGS["C5"]
     m = wg()
-    block, bounds = partition_1d(c.V, 8)
+    block, bounds = equal_blocks(c.V, 8)
     vb, ve = bounds[0]
     src, dst = synth.make_graph_slice(c.V, c.E, vb, ve, seed=c.seed * 16, alpha=c.alpha)
     g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=c.V, v_begin=vb, v_end=ve)

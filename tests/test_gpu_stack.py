@@ -50,7 +50,7 @@ def test_softmax_xent(dtype, C):
 @pytest.mark.parametrize("graph", ["powerlaw", "star"])
 def test_1d_partition_phases_match_single(model, policy, P, graph):
     m = wg()
-    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import partition_1d
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import equal_blocks
     V, E, fi, fo = 3000, 40000, 48, 40
     dtype = torch.float32
     src, dst, _ = synth.make_graph(V, E, seed=31, alpha=0.6)
@@ -67,7 +67,7 @@ def test_1d_partition_phases_match_single(model, policy, P, graph):
     y1, s1 = c1.forward_raw(xd, params)
     dx1, gr1 = c1.backward_raw(m.pad_to(dy), xd, y1, s1, params)
     # P rank-partitions sharing one exchange table
-    block, bounds = partition_1d(V, P)
+    block, bounds = equal_blocks(V, P)
     Vt = block * P
     xt = m.padded(Vt, fi, dtype)
     xt[:V] = x
@@ -201,19 +201,118 @@ def test_stack_cuda_graph_replay_equals_eager(model):
 
 def test_stack_rank_slice_runs():
     """bench.py --rank-slice: one rank of a P-way 1-D partition on one GPU
-    (collectives skipped) trains with the rank's owned rows only."""
+    with the emulated communicator (exchanges are copy kernels on the
+    communication stream, no data moves between ranks) trains with the rank's
+    owned rows only, through the library's distributed entry points."""
     m = wg()
-    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack, partition_1d
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack, equal_blocks
     V, E, P = 6000, 80000, 4
-    block, bounds = partition_1d(V, P)
+    block, bounds = equal_blocks(V, P)
     vb, ve = bounds[1]
     src, dst = synth.make_graph_slice(V, E, vb, ve, seed=61, alpha=0.5)
-    g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V, v_begin=vb, v_end=ve)
-    st = GNNStack(g, "sage", [24, 32, 32, 7], dtype=torch.bfloat16, block=block, sim_world=P, lr=1e-2)
-    assert st.dist and st.sim and st.rank == 1 and st.rows == ve - vb
-    x = m.padded(st.Vtab, 24, torch.bfloat16)
-    x[:V].copy_(torch.from_numpy(synth.make_features(V, 24, seed=62)))
+    comm = m.Comm(emulate=(1, P))
+    b = [lo for lo, _ in bounds] + [V]
+    g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V, comm=comm, bounds=b)
+    assert g.v_begin == vb and g.n_rows == ve - vb
+    st = GNNStack(g, "sage", [24, 256, 32, 7], dtype=torch.bfloat16, lr=1e-2)
+    assert st.dist and st.rank == 1 and st.rows == ve - vb
+    assert any(t is not None for t in st.xchg_f + st.xchg_b)
+    assert st.convs[1].xchg_info(1)[2] == 2 or st.convs[1].xchg_info(0)[2] == 2   # 512-byte rows: 2 chunks
+    x = m.padded(V, 24, torch.bfloat16)
+    x.copy_(torch.from_numpy(synth.make_features(V, 24, seed=62)))
     labels = torch.from_numpy(np.random.default_rng(3).integers(0, 7, ve - vb)).cuda()
     losses = [float(st.step(x, labels, V).item()) for _ in range(20)]
     assert np.isfinite(losses).all() and losses[-1] < losses[0]
     assert st.h[-1].shape[0] == ve - vb and all(d.shape[0] == ve - vb for d in st.dx[1:])
+
+
+@pytest.mark.parametrize("model,policy,F", [("sage", "vertex", 256), ("sage", "edge", 256), ("gcn", "vertex", 512),
+                                            ("gcn", "edge", 128)])
+def test_chunked_exchange_phases_match_single(model, policy, F):
+    """Column-chunked exchange tables (wg_plan_xchg): P rank
+    partitions on one GPU each write their rows of the chunked table (GEMM
+    3-D store maps, chunked second output of the bias-gradient pass) in PRE,
+    then every POST gathers chunk by chunk; the rank outputs and summed
+    weight gradients equal the single-partition layer."""
+    m = wg()
+    from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import equal_blocks
+    V, E, P = 3000, 40000, 3
+    dtype = torch.bfloat16
+    fi, fo = F, F
+    src, dst, _ = synth.make_graph(V, E, seed=71, alpha=0.6)
+    x = torch.from_numpy(synth.make_features(V, fi, seed=72)).to(dtype).cuda()
+    dy = torch.from_numpy(synth.normal((V, fo), seed=73, std=0.2)).to(dtype).cuda()
+    params = m.init_params(model, fi, fo, seed=7)
+    ts, td = torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda()
+    g1 = m.Graph(ts, td, num_vertices=V)
+    c1 = m.Conv(g1, model, fi, fo, dtype=dtype, policy=policy, fuse_relu=True)
+    xd = m.pad_to(x)
+    y1, s1 = c1.forward_raw(xd, params)
+    dx1, gr1 = c1.backward_raw(m.pad_to(dy), xd, y1, s1, params)
+    block, bounds = equal_blocks(V, P)
+    ranks = []
+    for p in range(P):
+        vb, ve = bounds[p]
+        g = m.Graph(ts, td, num_vertices=V, v_begin=vb, v_end=ve)
+        c = m.Conv(g, model, fi, fo, dtype=dtype, policy=policy, fuse_relu=True)
+        ranks.append((g, c, vb, ve, c.new_saved()))
+    c0 = ranks[0][1]
+    xf, xb = c0.new_xchg(0), c0.new_xchg(1)
+    assert xb is not None and c0.xchg_info(1)[2] == min(4, F * 2 // 256)   # >= 256-byte chunks
+    assert (xf is not None) == (policy == "vertex")
+    if xf is not None:
+        assert c0.xchg_info(0)[2] == min(4, F * 2 // 256)
+    y = m.padded(V, fo, dtype)
+    for ph in ((1, 2) if xf is not None else (0,)):
+        for g, c, vb, ve, sv in ranks:
+            c.forward_raw(xd, params, y=y[vb:ve], saved=sv, phase=ph, xchg=xf)
+    torch.cuda.synchronize()
+    assert rel_err(f64(y), f64(y1)) < 1e-2     # chunked gathers sum in another worker split
+    dx = m.padded(V, fi, dtype)
+    grads = [{k: torch.zeros_like(v) for k, v in params.items()} for _ in ranks]
+    for ph in (1, 2):
+        for (g, c, vb, ve, sv), gr in zip(ranks, grads):
+            c.backward_raw(m.pad_to(dy)[vb:ve], xd, y[vb:ve], sv, params, dx=dx[vb:ve], phase=ph, xchg=xb, grads=gr)
+    torch.cuda.synchronize()
+    assert rel_err(f64(dx), f64(dx1)) < 1e-2
+    for k in gr1:
+        tot = sum(gr[k] for gr in grads)
+        assert rel_err(f64(tot), f64(gr1[k])) < 1e-3, k
+
+
+@pytest.mark.parametrize("model", ["sage", "gin", "rgcn"])
+def test_nccl_world1_dist_calls_match_single(model):
+    """The distributed entry points over a real one-rank NCCL communicator
+    (ncclGetUniqueId / ncclCommInitRank through the library's dlopen'd NCCL)
+    give the single-partition results bit for bit."""
+    m = wg()
+    V, E, fi, fo, R = 2000, 25000, 64, 48, 4
+    src, dst, et = synth.make_graph(V, E, seed=81, alpha=0.6, R=R if model == "rgcn" else 1)
+    dtype = torch.bfloat16
+    ts, td = torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda()
+    tt = torch.from_numpy(et).cuda() if model == "rgcn" else None
+    kw = dict(etype=tt, num_types=R) if model == "rgcn" else {}
+    ckw = dict(norm="right", self_loop=True) if model == "rgcn" else {}
+    params = m.init_params(model, fi, fo, R=R, self_loop=model == "rgcn", seed=8)
+    x = m.pad_to(torch.from_numpy(synth.make_features(V, fi, seed=82)).to(dtype).cuda())
+    dy = m.pad_to(torch.from_numpy(synth.normal((V, fo), seed=83, std=0.2)).to(dtype).cuda())
+    g1 = m.Graph(ts, td, num_vertices=V, **kw)
+    c1 = m.Conv(g1, model, fi, fo, dtype=dtype, fuse_relu=True, **ckw)
+    y1, s1 = c1.forward_raw(x, params)
+    dx1, gr1 = c1.backward_raw(dy, x, y1, s1, params)
+    comm = m.Comm.single()
+    g = m.Graph(ts, td, num_vertices=V, comm=comm, **kw)
+    assert list(g.bounds) == [0, V]
+    c = m.Conv(g, model, fi, fo, dtype=dtype, fuse_relu=True, **ckw)
+    y = m.padded(V, fo, dtype)
+    sv = c.new_saved()
+    c.forward_dist(x, params, y, sv, x_gathered=True)
+    dx = m.padded(V, fi, dtype)
+    gr = {k: torch.zeros_like(v) for k, v in params.items()}
+    c.backward_dist(dy, x, y, sv, params, dx=dx, grads=gr)
+    comm.wait()
+    torch.cuda.synchronize()
+    assert torch.equal(y, y1) and torch.equal(dx, dx1)
+    for k in gr1:
+        assert torch.equal(gr[k], gr1[k]), k
+    comm.close()
