@@ -186,14 +186,41 @@ def layer_shapes(c, model):
             for i in range(L)]
 
 
-def cpu_baseline(c, model, src, dst, et, budget_s):
-    """The oracle (plain C, fp64, 1 thread) on a bounded sample: every in-edge
-    of a seeded random sample of destination rows (its induced star graph),
-    one forward + backward per layer shape of the workload."""
-    import oracle
-    rng = np.random.Generator(np.random.Philox(c.seed * 16 + 9))
+def host_info():
+    """nproc (usable cores), CPU model and sockets of this host (lscpu)."""
+    info = {"nproc": len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            if k.strip() == "Model name":
+                info["model"] = v.strip()
+            elif k.strip() == "Socket(s)":
+                info["sockets"] = int(v.strip())
+            elif k.strip() == "Core(s) per socket":
+                info["cores_per_socket"] = int(v.strip())
+            elif k.strip() == "Thread(s) per core":
+                info["threads_per_core"] = int(v.strip())
+    except Exception:
+        pass
+    return info
+
+
+def _csr_order(c, dst):
     order = np.argsort(dst, kind="stable")
     indptr = np.concatenate([[0], np.cumsum(np.bincount(dst, minlength=c.V))])
+    return order, indptr
+
+
+def _oracle_sample(c, model, src, dst, et, budget_s, seed, csr):
+    """A bounded sample of the workload for the oracle: every in-edge of a
+    seeded random sample of destination rows (its induced star graph), with
+    one forward + backward per layer shape.  Returns (n_edges, description,
+    run) where run() executes the oracle calls and returns per-layer
+    (t_fwd, t_bwd) seconds."""
+    import oracle
+    rng = np.random.Generator(np.random.Philox(seed))
+    order, indptr = csr
     shapes = layer_shapes(c, model)
     H = c.heads if model == "gat" else 1
     per_edge = sum(fi * fo * H for fi, fo, _ in shapes) * 2 * 3      # ~ fwd+bwd flops per edge (per-edge messages)
@@ -213,36 +240,82 @@ def cpu_baseline(c, model, src, dst, et, budget_s):
     s2, d2 = inv[:len(s)].astype(np.int32), inv[len(s):].astype(np.int32)
     t2 = et[eids].astype(np.int32) if (model == "rgcn" and et is not None) else None
     Vs = len(verts)
-    t_total = 0.0
+    calls = []
     for i, (fi, fo, concat) in enumerate(shapes):
-        r = lambda k, *sh: np.random.default_rng(10 * k + i).standard_normal(sh)
-        xs = r(0, Vs, fi)
-        t0 = time.perf_counter()
+        r = lambda k, *sh: np.random.default_rng(seed + 10 * k + i).standard_normal(sh)   # noqa: E731
+        xs, dy = r(0, Vs, fi), r(3, Vs, (H * fo if (model == "gat" and concat) else fo))
         if model == "sage":
-            oracle.sage_forward(s2, d2, Vs, xs, 0.05 * r(1, fi, fo), 0.05 * r(2, fi, fo), np.zeros(fo))
-            oracle.sage_backward(s2, d2, Vs, xs, 0.05 * r(1, fi, fo), 0.05 * r(2, fi, fo), r(3, Vs, fo))
+            Ws, Wn = 0.05 * r(1, fi, fo), 0.05 * r(2, fi, fo)
+            f = lambda: oracle.sage_forward(s2, d2, Vs, xs, Ws, Wn, np.zeros(fo))   # noqa: E731
+            b = lambda: oracle.sage_backward(s2, d2, Vs, xs, Ws, Wn, dy)   # noqa: E731
         elif model == "gcn":
-            oracle.gcn_forward(s2, d2, Vs, xs, 0.05 * r(1, fi, fo), np.zeros(fo))
-            oracle.gcn_backward(s2, d2, Vs, xs, 0.05 * r(1, fi, fo), r(3, Vs, fo))
+            W = 0.05 * r(1, fi, fo)
+            f = lambda: oracle.gcn_forward(s2, d2, Vs, xs, W, np.zeros(fo))   # noqa: E731
+            b = lambda: oracle.gcn_backward(s2, d2, Vs, xs, W, dy)   # noqa: E731
         elif model == "gin":
             W1, W2 = 0.05 * r(1, fi, fo), 0.05 * r(2, fo, fo)
-            oracle.gin_forward(s2, d2, Vs, xs, W1, np.zeros(fo), W2, np.zeros(fo))
-            oracle.gin_backward(s2, d2, Vs, xs, W1, np.zeros(fo), W2, r(3, Vs, fo))
+            f = lambda: oracle.gin_forward(s2, d2, Vs, xs, W1, np.zeros(fo), W2, np.zeros(fo))   # noqa: E731
+            b = lambda: oracle.gin_backward(s2, d2, Vs, xs, W1, np.zeros(fo), W2, dy)   # noqa: E731
         elif model == "gat":
             W, al, ar = 0.05 * r(1, fi, H * fo), 0.1 * r(2, H, fo), 0.1 * r(4, H, fo)
-            oracle.gat_forward(s2, d2, Vs, xs, W, al, ar, None, heads=H, concat=concat)
-            oracle.gat_backward(s2, d2, Vs, xs, W, al, ar, r(3, Vs, H * fo if concat else fo), heads=H,
-                                concat=concat)
+            f = lambda: oracle.gat_forward(s2, d2, Vs, xs, W, al, ar, None, heads=H, concat=concat)   # noqa: E731
+            b = lambda: oracle.gat_backward(s2, d2, Vs, xs, W, al, ar, dy, heads=H, concat=concat)   # noqa: E731
         else:
             W, W0 = 0.05 * r(1, c.R, fi, fo), 0.05 * r(2, fi, fo)
-            oracle.rgcn_forward(s2, d2, t2, Vs, xs, W, W0, np.zeros(fo), norm="right")
-            oracle.rgcn_backward(s2, d2, t2, Vs, xs, W, r(3, Vs, fo), W0, norm="right")
-        t_total += time.perf_counter() - t0
-    L = len(shapes)
-    return {"value": L * len(eids) / t_total, "unit": "edges/s", "cores": 1, "kind": "oracle",
-            "sample": f"all {len(eids)} in-edges of {len(rows)} random dst rows (induced star graph, {Vs} V), "
-                      f"fwd+bwd of each of the {L} layer shapes, {t_total:.1f} s",
-            "seconds": t_total}
+            f = lambda: oracle.rgcn_forward(s2, d2, t2, Vs, xs, W, W0, np.zeros(fo), norm="right")   # noqa: E731
+            b = lambda: oracle.rgcn_backward(s2, d2, t2, Vs, xs, W, dy, W0, norm="right")   # noqa: E731
+        calls.append((f, b))
+
+    def run():
+        out = []
+        for f, b in calls:
+            t0 = time.perf_counter()
+            f()
+            t1 = time.perf_counter()
+            b()
+            out.append((t1 - t0, time.perf_counter() - t1))
+        return out
+    desc = f"all {len(eids)} in-edges of {len(rows)} random dst rows (induced star graph, {Vs} V)"
+    return len(eids), desc, run
+
+
+def cpu_baseline(c, model, src, dst, et, budget_s, csr=None):
+    """The oracle as it stands (plain C, fp64, serial per call) timed on this
+    host's cores: (1) one thread on one bounded sample, per layer forward /
+    backward (the per-core rate); (2) nproc threads at once,
+    each running the unchanged oracle on its own sample (ctypes releases the
+    GIL), throughput = all edges / wall time.  The headline value is (2)."""
+    import threading
+    hi = host_info()
+    L = len(layer_shapes(c, model))
+    csr = csr or _csr_order(c, dst)
+    n1, desc1, run1 = _oracle_sample(c, model, src, dst, et, budget_s / 3, c.seed * 16 + 9, csr)
+    per_layer = run1()
+    t1 = sum(a + b for a, b in per_layer)
+    nth = max(1, int(hi["nproc"]))
+    samples = [_oracle_sample(c, model, src, dst, et, budget_s / 3, c.seed * 16 + 100 + k, csr) for k in range(nth)]
+    start = threading.Barrier(nth + 1)
+    done = [None] * nth
+
+    def work(k):
+        start.wait()
+        done[k] = samples[k][2]()
+    ths = [threading.Thread(target=work, args=(k,)) for k in range(nth)]
+    for t in ths:
+        t.start()
+    start.wait()
+    t0 = time.perf_counter()
+    for t in ths:
+        t.join()
+    wall = time.perf_counter() - t0
+    edges = sum(sm[0] for sm in samples)
+    return {"value": L * edges / wall, "unit": "edges/s", "cores": nth, "kind": "oracle",
+            "sample": f"{nth} threads, each the unchanged serial oracle on its own sample ({samples[0][1]}, ...; "
+                      f"{edges} in-edges in all), fwd+bwd of each of the {L} layer shapes, {wall:.1f} s wall",
+            "seconds": wall, "host": hi,
+            "per_core": {"value": L * n1 / t1, "unit": "edges/s", "threads": 1, "sample": desc1,
+                         "per_layer_ms": [{"fwd": 1e3 * a, "bwd": 1e3 * b, "edges_per_s": n1 / (a + b)}
+                                          for a, b in per_layer]}}
 
 
 def run_reference(args):
@@ -253,15 +326,18 @@ def run_reference(args):
     src, dst, et, _, _ = make_inputs(c, model)
     vals = []
     per = max(2.0, 60.0 / max(1, args.steps + args.warmup))
+    csr = _csr_order(c, dst)
     for i in range(args.warmup + args.steps):
-        r = cpu_baseline(c, model, src, dst, et, per)
+        r = cpu_baseline(c, model, src, dst, et, per, csr)
         if i >= args.warmup:
             vals.append(r)
     v = statistics.median([r["value"] for r in vals])
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "edges/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "dtype": "f64",
             "data": "synthetic", "config": cfg, "vs_baseline": None,
-            "cpu_baseline": {"value": v, "unit": "edges/s", "cores": 1, "kind": "oracle", "sample": vals[-1]["sample"]},
+            "cpu_baseline": {"value": v, "unit": "edges/s", "cores": vals[-1]["cores"], "kind": "oracle",
+                             "sample": vals[-1]["sample"], "host": vals[-1]["host"],
+                             "per_core": vals[-1]["per_core"]},
             "e2e": {"value": v, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line))
 
@@ -399,28 +475,45 @@ def main():
             graph, graph_err = None, f"{type(ex).__name__}: {ex}"[:200]
             torch.cuda.synchronize()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    step_ms = None
     if graph is not None:
         barrier()
         clocks.mark_start()
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps - 1)]
         ev0.record(stream)
-        for _ in range(args.steps):
+        for k in range(args.steps):
             graph.replay()
+            if k < args.steps - 1:
+                evs[k].record(stream)
         ev1.record(stream)
         torch.cuda.synchronize()
         clocks.mark_stop()
         loss = loss_g
         ms_graph = ev0.elapsed_time(ev1) / args.steps
+        marks = [ev0] + evs + [ev1]
+        step_ms = [marks[k].elapsed_time(marks[k + 1]) for k in range(args.steps)]
     wg.profile("start")
     n0 = wg.launch_count()
     torch.cuda.synchronize()
     barrier()
     if graph is None:
         clocks.mark_start()
+    stack.layer_events = []
     ev0.record(stream)
+    evs_e = []
     for _ in range(args.steps):
         loss_e = stack.step(x, labels, c.V)
+        evs_e.append(torch.cuda.Event(enable_timing=True))
+        evs_e[-1].record(stream)
     ev1.record(stream)
     torch.cuda.synchronize()
+    lay = {}
+    for key, a, b in stack.layer_events:
+        lay[key] = lay.get(key, 0.0) + a.elapsed_time(b) / args.steps
+    stack.layer_events = None
+    if step_ms is None:
+        marks = [ev0] + evs_e
+        step_ms = [marks[k].elapsed_time(marks[k + 1]) for k in range(args.steps)]
     if graph is None:
         clocks.mark_stop()
         loss = loss_e
@@ -438,6 +531,17 @@ def main():
     # rank slice: the edges this GPU aggregates per layer pass (its in-edges)
     E_units = g.E_fwd if P > 1 else c.E
     value = L * E_units / (ms / 1e3)
+    # per layer: edges/s = E / (t_fwd + t_bwd), CUDA events
+    # around each layer call in the profiled eager pass (this rank's edges)
+    per_layer = [{"layer": i, "f_in": c.dims[i], "f_out": c.dims[i + 1], "fwd_ms": lay.get(("fwd", i), 0.0),
+                  "bwd_ms": lay.get(("bwd", i), 0.0),
+                  "edges_per_s": g.E_fwd / ((lay.get(("fwd", i), 0.0) + lay.get(("bwd", i), 0.0)) / 1e3)
+                  if lay.get(("fwd", i), 0.0) + lay.get(("bwd", i), 0.0) > 0 else None}
+                 for i in range(L)]
+    qs = np.percentile(np.array(step_ms), [10, 50, 90]).tolist()
+    step_stats = {"median_ms": qs[1], "p10_ms": qs[0], "p90_ms": qs[2], "n": len(step_ms),
+                  "source": "CUDA events between graph replays" if graph is not None
+                  else "CUDA events between eager steps"}
 
     # ---- end to end through the public API with host buffers
     e2e = None
@@ -565,6 +669,7 @@ def main():
                                    "bwd_path": cv.bwd_path, "items": cv.n_items, "items_T": cv.n_items_T,
                                    "split_rows": cv.n_split_rows} for cv in stack.convs]),
             "gpu_launches": int(launches), "roofline": roofline, "kernels": kernels,
+            "step_time": step_stats, "per_layer": per_layer,
             "one_off": {"partition_s": t_part, "plan_s": t_plan, "synth_s": t_gen},
             "clocks": clk, "loss": float(loss.item()), "e2e": e2e}
     if rank == 0 and world == 1 and not args.no_cpu:

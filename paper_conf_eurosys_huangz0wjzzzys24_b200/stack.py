@@ -155,6 +155,23 @@ class GNNStack:
         """Rows of layer i's output table this rank writes."""
         return self._own(self.h[i + 1]) if i + 1 < self.L else self.h[self.L]
 
+    # per-layer timing (bench.py): CUDA events on the current stream around each
+    # layer's forward / backward when self.layer_events is a list
+    layer_events = None
+
+    def _mark(self, key):
+        if self.layer_events is None:
+            return None
+        ev = torch.cuda.Event(enable_timing=True)
+        ev.record()
+        return (key, ev)
+
+    def _close(self, m):
+        if m is not None:
+            ev = torch.cuda.Event(enable_timing=True)
+            ev.record()
+            self.layer_events.append((m[0], m[1], ev))
+
     def _own(self, t):
         return t[self.vb:self.vb + self.rows] if self.dist else t
 
@@ -173,6 +190,7 @@ class GNNStack:
         """x: [V x f0] (replicated input features); returns this rank's logits rows."""
         h = x
         for i, c in enumerate(self.convs):
+            mk = self._mark(("fwd", i))
             y = self._out(i)
             if self.comm is not None and self.dist:
                 c.forward_dist(h, self.params[i], y, self.saved[i], xchg=self.xchg_f[i], x_gathered=i == 0)
@@ -185,6 +203,7 @@ class GNNStack:
                 if self.tdist and i > 0:
                     self._allgatherv(h)             # EDGE / RGCN layers gather raw rows
                 c.forward_raw(h, self.params[i], y=y, saved=self.saved[i])
+            self._close(mk)
             h = self.h[i + 1]
         self.x = x
         return self.h[self.L]
@@ -195,6 +214,7 @@ class GNNStack:
         g = dlogits
         masked = False
         for i in reversed(range(self.L)):
+            mk = self._mark(("bwd", i))
             c = self.convs[i]
             xin = self.x if i == 0 else self.h[i]
             dx = self.dx[i] if i > 0 else None
@@ -212,6 +232,7 @@ class GNNStack:
                 c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, phase=C.PHASE_POST, xchg=xb, **kw)
             else:
                 c.backward_raw(g, xin, y, self.saved[i], self.params[i], dx=dx, **kw)
+            self._close(mk)
             g = dx
             masked = fuse
         if self.comm is not None:
