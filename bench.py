@@ -68,8 +68,11 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--rank-slice", type=int, default=0, metavar="P",
                     help="one GPU runs rank --slice-rank of a P-way 1-D partition (its in- / out-edges only, "
-                         "collectives skipped): per-rank compute of a configuration too large for one GPU (C5)")
+                         "collectives emulated): per-rank compute of a configuration too large for one GPU (C5)")
     ap.add_argument("--slice-rank", type=int, default=0)
+    ap.add_argument("--emulate-xchg", action="store_true",
+                    help="--rank-slice: time every exchange as a copy kernel on the library's communication "
+                         "stream (overlapped with the gathers as the NCCL exchange would be)")
     ap.add_argument("--no-graph", action="store_true",
                     help="time eager steps instead of replaying one CUDA-graph-captured step")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
@@ -391,15 +394,17 @@ def main():
         labels_np = np.random.Generator(np.random.Philox(c.seed * 16 + 5)).integers(
             0, c.dims[-1], c.V).astype(np.int64)[vb:ve]
         args.no_e2e, args.no_cpu = True, True
-        comm = wg.Comm(emulate=(args.slice_rank, P), device=local)
+        comm = wg.Comm(emulate=(args.slice_rank, P), device=local, emulate_copy=args.emulate_xchg)
         cfg.update(rank_slice={"P": P, "rank": args.slice_rank, "v_begin": vb, "v_end": ve,
                                "edges_touching_block": int(src.shape[0]),
+                               "exchange": "emulated copy kernels (--emulate-xchg)" if args.emulate_xchg
+                                           else "none (compute of the rank only)",
                                "note": "per-rank compute of the P-way 1-D partition on one GPU: the rank's "
                                        "in-edges (forward) and out-edges (backward) through the library's "
-                                       "distributed calls with the EMULATED communicator: every exchange is a "
-                                       "copy kernel on the communication stream rewriting the non-owned rows "
-                                       "(WG_EMU_CTAS CTAs), overlapped chunk by chunk with the gathers as the "
-                                       "NCCL exchange would be; no data moves between ranks and non-owned "
+                                       "distributed calls with the EMULATED communicator (with --emulate-xchg "
+                                       "every exchange is a copy kernel on the communication stream rewriting "
+                                       "the non-owned rows, overlapped chunk by chunk with the gathers as the "
+                                       "NCCL exchange would be); no data moves between ranks and non-owned "
                                        "degrees are not the global ones (a timing run)",
                                "features": "torch.randn on the device (the 111M x 128 table is not built on the host)"})
     else:

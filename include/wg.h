@@ -258,13 +258,14 @@ typedef struct wg_comm_s* wg_comm;
 wg_status wg_comm_unique_id(void* id);
 /* Collective over the `world` ranks (blocking until all have joined).      */
 wg_status wg_comm_init(const void* id, int rank, int world, int device, wg_comm* out);
-/* One-GPU emulation of rank `rank` of a `world`-way partition: every
- * exchange is a copy kernel on the communication stream that re-reads and
- * re-writes the non-owned rows (the bytes an all-gather writes, with the SM
- * share of an NCCL kernel: WG_EMU_CTAS CTAs, default 16); no data moves
- * between ranks and gradients are not reduced.  For timing the overlap of
- * exchange and gathers on one GPU (bench.py --rank-slice), not for results. */
-wg_status wg_comm_init_emulated(int rank, int world, int device, wg_comm* out);
+/* One-GPU emulation of rank `rank` of a `world`-way partition: with copy = 1
+ * every exchange is a copy kernel on the communication stream that re-reads
+ * and re-writes the non-owned rows (the HBM bytes an all-gather moves, with
+ * the SM share of an NCCL kernel: WG_EMU_CTAS CTAs, default 16); copy = 0
+ * skips exchanges (the rank's compute alone).  No data moves between ranks
+ * and gradients are not reduced.  For timing one rank on one GPU
+ * (bench.py --rank-slice), not for results.                                */
+wg_status wg_comm_init_emulated(int rank, int world, int device, int copy, wg_comm* out);
 /* info: rank, world, device, emulated                                      */
 wg_status wg_comm_info(wg_comm c, int32_t info[4]);
 /* `stream` waits for the communicator's outstanding work (the gradient

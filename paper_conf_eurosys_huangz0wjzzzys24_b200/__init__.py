@@ -108,16 +108,18 @@ def profile(cmd: str):
 class Comm:
     """Communicator of the 1-D multi-GPU layer (wg_comm_*): NCCL over the
     ranks of a torch.distributed group (the 128-byte id is broadcast through
-    it), or the one-GPU emulation of one rank (emulate=(rank, world))."""
+    it), or the one-GPU emulation of one rank (emulate=(rank, world); with
+    emulate_copy the exchanges are timed as copy kernels, else skipped)."""
 
-    def __init__(self, group=None, *, device: int | None = None, emulate=None):
+    def __init__(self, group=None, *, device: int | None = None, emulate=None, emulate_copy: bool = True):
         L = C.lib()
         self.device = torch.cuda.current_device() if device is None else device
         h = ctypes.c_void_p()
         with torch.cuda.device(self.device):
             if emulate is not None:
                 self.rank, self.world = emulate
-                C.check(L.wg_comm_init_emulated(self.rank, self.world, self.device, ctypes.byref(h)),
+                C.check(L.wg_comm_init_emulated(self.rank, self.world, self.device, int(emulate_copy),
+                                                ctypes.byref(h)),
                         "wg_comm_init_emulated")
             else:
                 import torch.distributed as dist

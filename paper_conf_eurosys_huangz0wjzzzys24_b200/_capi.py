@@ -130,7 +130,7 @@ def lib():
     L.wg_comm_init.restype = st
     L.wg_comm_init.argtypes = [P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.POINTER(P)]
     L.wg_comm_init_emulated.restype = st
-    L.wg_comm_init_emulated.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.POINTER(P)]
+    L.wg_comm_init_emulated.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.POINTER(P)]
     L.wg_comm_info.restype = st
     L.wg_comm_info.argtypes = [P, P]
     L.wg_comm_wait.restype = st

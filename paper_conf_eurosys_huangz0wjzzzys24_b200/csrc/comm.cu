@@ -136,6 +136,7 @@ wg_status fork_to_comm(wg_comm_s* c, cudaStream_t s) {
 wg_status exchange_rows(wg_comm_s* c, void* base, int64_t ld_bytes, const std::vector<int64_t>& b) {
   if (c->world <= 1) return WG_OK;
   char* p = static_cast<char*>(base);
+  if (c->emulated == 2) return WG_OK;          // compute-only emulation: no exchange at all
   if (c->emulated) {
     const int64_t n = b.back() * ld_bytes / 16;
     WG_LAUNCH(k_emu_xchg, c->emu_ctas, 512, 0, c->cs, reinterpret_cast<int4*>(p), b[c->rank] * ld_bytes / 16,
@@ -250,12 +251,12 @@ wg_status wg_comm_init(const void* id, int rank, int world, int device, wg_comm*
   return WG_OK;
 }
 
-wg_status wg_comm_init_emulated(int rank, int world, int device, wg_comm* out) {
+wg_status wg_comm_init_emulated(int rank, int world, int device, int copy, wg_comm* out) {
   using namespace wg;
   WG_REQ(out && world >= 1 && rank >= 0 && rank < world, WG_ERR_INVALID, "wg_comm_init_emulated: bad argument");
   WG_CK(cudaSetDevice(device));
   auto* c = new wg_comm_s();
-  c->rank = rank; c->world = world; c->device = device; c->emulated = 1;
+  c->rank = rank; c->world = world; c->device = device; c->emulated = copy ? 1 : 2;
   const char* e = getenv("WG_EMU_CTAS");
   if (e && atoi(e) > 0) c->emu_ctas = atoi(e);
   wg_status st = comm_streams(c);
