@@ -55,6 +55,8 @@ def _L():
         i64, i32, f64 = ctypes.c_int64, ctypes.c_int32, ctypes.c_double
         _lib.wgo_partition.restype = i64
         _lib.wgo_partition.argtypes = [i64, P, P, P, i32, i32, i64, P, P]
+        _lib.wgo_partition_general.restype = i64
+        _lib.wgo_partition_general.argtypes = [i64, i64, P, P, P, P, P, i32, P, P]
         _lib.wgo_gcn_forward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, P, P, P, P, P]
         _lib.wgo_gcn_backward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P, P]
         _lib.wgo_sage_forward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P]
@@ -104,6 +106,25 @@ def partition(key_vertex, other_vertex, etype=None, *, by_type=False, T=128, E_m
     tasks = np.empty(max(E, 1), TASK_DTYPE)
     n = _L().wgo_partition(E, _p(kv), _p(ov), _p(et), int(bool(by_type and et is not None)),
                            int(T), int(E_max), _p(perm), _p(tasks))
+    return perm[:E].copy(), tasks[:n].copy()
+
+
+ATTRS = {"dst": 0, "src": 1, "type": 2, "dst_degree": 3, "edge": 4}
+
+
+def partition_general(src, dst, V, restrictions, etype=None):
+    """General restriction engine (f2; Fig 7): restrictions is a
+    list of (attribute name, k) with k >= 1 (uniq(a) = k) or "min"
+    (uniq(a) = min).  Returns (perm int64[E], tasks)."""
+    s, d, et = _i32(src), _i32(dst), _i32(etype)
+    E = s.shape[0]
+    a = np.array([ATTRS[n] for n, _ in restrictions], np.int32)
+    k = np.array([-1 if v == "min" else int(v) for _, v in restrictions], np.int32)
+    perm = np.empty(max(E, 1), np.int64)
+    tasks = np.empty(max(E, 1), TASK_DTYPE)
+    n = _L().wgo_partition_general(V, E, _p(s), _p(d), _p(et), _p(a), _p(k), len(a), _p(perm), _p(tasks))
+    if n < 0:
+        raise ValueError("bad restriction spec")
     return perm[:E].copy(), tasks[:n].copy()
 
 

@@ -151,6 +151,125 @@ int64_t wgo_partition(int64_t E, const int32_t* kv, const int32_t* ov, const int
 }
 
 /* ======================================================================== */
+/* General restriction engine: the graph partition table */
+/* of §4.2 with a restriction per edge attribute:           */
+/*   uniq(a) = k  (k >= 1): at most k distinct values of a in a gTask;     */
+/*   uniq(a) = min (k = -1): gTasks with fewer distinct values preferred;  */
+/*   no entry: unrestricted.                                               */
+/* Attributes: 0 dst-id, 1 src-id, 2 edge type, 3 dst-degree (the         */
+/* in-degree of the edge's destination, an inherent attribute P:L1361),    */
+/* 4 edge-id.  Greedy of P:L1431-1451: sort by the restricted attributes,  */
+/* scan in order, add the edge if every restriction still holds, else     */
+/* start a new gTask.  Readings (Q25): the sort key is the      */
+/* uniq = 1 attributes (spec order), then the min attributes (spec        */
+/* order: sorting by them groups equal values, which minimises the        */
+/* distinct count the greedy packs), then the uniq = k > 1 attributes     */
+/* other than edge-id (spec order), then dst-id if absent, then edge-id   */
+/* (a total order).  Task record: tile = -1, type of the first edge,      */
+/* d_lo / d_hi = smallest / largest dst-id, flags 0, n_uniq_src.          */
+/* ======================================================================== */
+static int32_t g_nkey;
+static int32_t g_key[8];
+static const int32_t *g_gsrc, *g_gdst, *g_gty;
+static const int64_t* g_gdeg;
+
+static int64_t attr_value(int32_t a, int64_t e) {
+    switch (a) {
+        case 0: return g_gdst[e];
+        case 1: return g_gsrc[e];
+        case 2: return g_gty ? g_gty[e] : 0;
+        case 3: return g_gdeg[g_gdst[e]];
+        default: return e;
+    }
+}
+
+static int cmp_general(const void* pa, const void* pb) {
+    int64_t a = *(const int64_t*)pa, b = *(const int64_t*)pb;
+    for (int32_t i = 0; i < g_nkey; ++i) {
+        int64_t va = attr_value(g_key[i], a), vb = attr_value(g_key[i], b);
+        if (va != vb) return va < vb ? -1 : 1;
+    }
+    return 0;
+}
+
+/* attr[i], k[i]: n restrictions (each attribute at most once).  Returns the
+ * number of tasks; perm / tasks as wgo_partition; -1 on a bad spec. */
+int64_t wgo_partition_general(int64_t V, int64_t E, const int32_t* src, const int32_t* dst, const int32_t* etype,
+                              const int32_t* attr, const int32_t* k, int32_t n, int64_t* perm, wgo_task* tasks) {
+    int64_t* deg = (int64_t*)calloc((size_t)(V > 0 ? V : 1), sizeof(int64_t));
+    for (int64_t e = 0; e < E; ++e) deg[dst[e]]++;
+    g_gsrc = src; g_gdst = dst; g_gty = etype; g_gdeg = deg;
+    /* sort key */
+    int used[5] = {0, 0, 0, 0, 0};
+    g_nkey = 0;
+    for (int pass = 0; pass < 3; ++pass)
+        for (int32_t i = 0; i < n; ++i) {
+            if (attr[i] < 0 || attr[i] > 4) { free(deg); return -1; }
+            int take = pass == 0 ? k[i] == 1 : pass == 1 ? k[i] == -1 : (k[i] > 1 && attr[i] != 4);
+            if (take && !used[attr[i]]) { g_key[g_nkey++] = attr[i]; used[attr[i]] = 1; }
+        }
+    if (!used[0]) g_key[g_nkey++] = 0;
+    g_key[g_nkey++] = 4;
+    for (int64_t i = 0; i < E; ++i) perm[i] = i;
+    qsort(perm, (size_t)E, sizeof(int64_t), cmp_general);
+    /* greedy scan: per restricted attribute, the distinct values of the open task */
+    int64_t* vals[5] = {0, 0, 0, 0, 0};
+    int64_t cnt[5] = {0, 0, 0, 0, 0};
+    for (int32_t i = 0; i < n; ++i)
+        if (k[i] >= 1) vals[attr[i]] = (int64_t*)malloc(sizeof(int64_t) * (size_t)k[i]);
+    int64_t nt = 0, open_b = 0;
+    for (int64_t p = 0; p < E; ++p) {
+        int64_t e = perm[p];
+        int fits = 1;
+        for (int32_t i = 0; i < n && fits; ++i) {
+            if (k[i] < 1) continue;
+            int32_t a = attr[i];
+            int64_t v = attr_value(a, e), j;
+            for (j = 0; j < cnt[a]; ++j) if (vals[a][j] == v) break;
+            if (j == cnt[a] && cnt[a] == k[i]) fits = 0;      /* a new value beyond k */
+        }
+        if (!fits) {                                          /* close [open_b, p) */
+            wgo_task* t = &tasks[nt++];
+            t->e_begin = open_b; t->e_end = p;
+            open_b = p;
+            for (int a = 0; a < 5; ++a) cnt[a] = 0;
+        }
+        for (int32_t i = 0; i < n; ++i) {                     /* record the edge's values */
+            if (k[i] < 1) continue;
+            int32_t a = attr[i];
+            int64_t v = attr_value(a, e), j;
+            for (j = 0; j < cnt[a]; ++j) if (vals[a][j] == v) break;
+            if (j == cnt[a]) vals[a][cnt[a]++] = v;
+        }
+    }
+    if (E > 0) { tasks[nt].e_begin = open_b; tasks[nt].e_end = E; ++nt; }
+    for (int a = 0; a < 5; ++a) free(vals[a]);
+    /* task records */
+    int32_t* buf = (int32_t*)malloc(sizeof(int32_t) * (size_t)(E > 0 ? E : 1));
+    for (int64_t t = 0; t < nt; ++t) {
+        wgo_task* r = &tasks[t];
+        r->tile = -1;
+        r->type = etype ? etype[perm[r->e_begin]] : 0;
+        r->flags = 0;
+        r->d_lo = dst[perm[r->e_begin]]; r->d_hi = r->d_lo;
+        int64_t m = 0;
+        for (int64_t q = r->e_begin; q < r->e_end; ++q) {
+            int32_t d = dst[perm[q]];
+            if (d < r->d_lo) r->d_lo = d;
+            if (d > r->d_hi) r->d_hi = d;
+            buf[m++] = src[perm[q]];
+        }
+        qsort(buf, (size_t)m, sizeof(int32_t), cmp_i32);
+        int32_t u = 0;
+        for (int64_t q = 0; q < m; ++q) if (q == 0 || buf[q] != buf[q - 1]) ++u;
+        r->n_uniq_src = u;
+    }
+    free(buf);
+    free(deg);
+    return nt;
+}
+
+/* ======================================================================== */
 /* Helpers: degrees and the GCN / RGCN edge coefficients.                  */
 /* ======================================================================== */
 

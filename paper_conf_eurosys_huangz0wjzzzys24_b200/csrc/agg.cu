@@ -310,10 +310,17 @@ __global__ void __launch_bounds__(WARPS * 32, 3) k_agg(AggArgs a, int VPR) {
 // that is 2 CTAs x 256 lanes x D x 16 B ~ 190 KB, enough to cover HBM latency
 // at full bandwidth (Little's law: 6.5 TB/s x ~2 us / 148 SMs ~ 90 KB).
 // Edge metadata (destination row, source scale) rides in a per-worker ring.
+// Gathered rows: random accesses, whose DRAM cost is set by the L2 fill
+// granularity -- measured (scripts/gran_probe.cu, profiles/r02/gran_probe.md):
+// a random 32-128 B row fetches a whole 128-byte line by default; with the
+// .L2::64B prefetch-size hint only the 64-byte halves it touches (a 64-B row
+// 64 B instead of 128, a 96-B row 128 instead of 192 on average).  Random
+// row accesses are capped near 35 G/s either way (DRAM activations), so the
+// hint cuts bytes, not accesses.
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool pred) {
   const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
   const int n = pred ? 16 : 0;
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "r"(n) : "memory");
+  asm volatile("cp.async.cg.shared.global.L2::64B [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "r"(n) : "memory");
 }
 __device__ __forceinline__ void cp_async4(void* smem, const void* gmem, bool pred) {
   const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
@@ -397,7 +404,8 @@ __global__ void __launch_bounds__(WARPS * 32, MINB) k_agg_cp(AggArgs a, int VPR)
 #pragma unroll
           for (int q = 0; q < NV; ++q) {
             const int vi = l + q * LPE;
-            cp_async16(my_ring + (pslot + u) * RSTRIDE + q * TPB, row + vi * EPV, u < n && vi < nvec);
+            // lanes past the row's last vector point at its first one (no extra 64-B block)
+            cp_async16(my_ring + (pslot + u) * RSTRIDE + q * TPB, row + (vi < nvec ? vi : 0) * EPV, u < n && vi < nvec);
           }
         }
         if (l < RS) {
