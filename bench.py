@@ -375,13 +375,26 @@ def main():
     c, model, cfg = workload(args.config, args.model)
     dev = torch.device("cuda", local)
     P = args.rank_slice
-    if P > 1 and (world > 1 or model in ("gat", "rgcn") or c.symmetric):
-        raise SystemExit("--rank-slice: one process, directed untyped GCN / SAGE / GIN configs")
+    if P > 1 and (world > 1 or model == "gat"):
+        raise SystemExit("--rank-slice: one process, GCN / SAGE / GIN / RGCN configs")
     if world > 1 and model == "gat":
         raise SystemExit("the 1-D multi-GPU partition covers GCN / SAGE / GIN / RGCN (DESIGN.md §9)")
     t0 = time.perf_counter()
     comm, bounds = None, None
-    if P > 1:
+    if P > 1 and c.E <= (1 << 31) // 8:
+        # one rank of the P-way partition of a graph that fits this host: the
+        # library partitions it (edge-balanced wg_partition_1d) and keeps the
+        # rank's rows, in- and out-edges
+        src, dst, et, x_np, labels_np = make_inputs(c, model)
+        args.no_e2e, args.no_cpu = True, True
+        comm = wg.Comm(emulate=(args.slice_rank, P), device=local, emulate_copy=args.emulate_xchg)
+        cfg.update(rank_slice={"P": P, "rank": args.slice_rank,
+                               "exchange": "emulated copy kernels (--emulate-xchg)" if args.emulate_xchg
+                                           else "none (compute of the rank only)",
+                               "note": "one rank of the P-way 1-D partition (edge-balanced) on one GPU through "
+                                       "the library's distributed calls with the EMULATED communicator; no data "
+                                       "moves between ranks (a timing run)"})
+    elif P > 1:
         # one rank of the P-way partition: only the edges touching its block
         # exist here, so the blocks are equal T-aligned vertex ranges (the
         # seeded permutation scatters hubs: edges balance to ~1 %)
@@ -419,6 +432,10 @@ def main():
                  etype=torch.from_numpy(et).to(dev) if R > 1 else None, num_types=R,
                  max_task_edges=args.emax, tile_rows=args.tile, comm=comm, bounds=bounds)
     vb, ve = g.v_begin, g.v_begin + g.n_rows
+    if P > 1 and x_np is not None:
+        labels_np = labels_np[vb:ve]
+        cfg["rank_slice"].update(v_begin=vb, v_end=ve, bounds=[int(b) for b in g.bounds],
+                                 rank_in_edges=int(g.E_fwd), rank_out_edges=int(g.E_T))
     if world > 1:
         cfg.update(partition={"bounds": [int(b) for b in g.bounds], "rank_rows": ve - vb,
                               "rank_in_edges": int(g.E_fwd), "rank_out_edges": int(g.E_T),

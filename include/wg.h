@@ -317,6 +317,48 @@ wg_status wg_conv_backward_dist(wg_comm c, wg_plan p, const wg_params* params, c
                                 const wg_grads* grads, wg_stream stream);
 
 /* ------------------------------------------------------------------------ */
+/* General restriction engine: the graph partition table  */
+/* of §4.2 with arbitrary restrictions, the greedy of        */
+/* P:L1431-1451, Fig 7 and Fig 9 instances.   */
+/* ------------------------------------------------------------------------ */
+typedef enum { WG_ATTR_DST = 0, WG_ATTR_SRC = 1, WG_ATTR_TYPE = 2, WG_ATTR_DST_DEGREE = 3,
+               WG_ATTR_EDGE = 4 } wg_attr;
+#define WG_UNIQ_MIN (-1)
+/* uniq(attr) = k: at most k distinct values of the attribute among a
+ * gTask's edges (k >= 1); k = WG_UNIQ_MIN: uniq(attr) = min, gTasks with
+ * fewer distinct values preferred (orders the scan, never cuts a gTask).
+ * dst-degree is the in-degree of the edge's destination.          */
+typedef struct { int32_t attr, k; } wg_restriction;
+typedef struct wg_gpart_s* wg_gpart;
+/* Partition the edges of `desc` (a full graph; v_begin / v_end ignored):
+ * sort key = the uniq = 1 attributes (restriction order), then the min
+ * attributes, then the uniq = k > 1 attributes except edge-id, then dst-id if
+ * absent, then edge-id (Q25); a greedy scan then cuts a gTask
+ * whenever an edge would bring a k-th + 1 distinct value.  Each attribute at
+ * most once; the sum of k over k > 1 attributes (edge-id excluded) <= 2048
+ * (WG_ERR_UNSUPPORTED beyond).  Task records: tile = -1, type of the first
+ * edge, d_lo / d_hi = smallest / largest dst-id, flags 0, n_uniq_src.
+ * Synchronous on `stream`; pointers host or device.                         */
+wg_status wg_gpart_create(const wg_graph_desc* desc, const wg_restriction* r, int32_t n_r, int device,
+                          wg_stream stream, wg_gpart* out);
+/* info: V, E, number of gTasks                                             */
+wg_status wg_gpart_info(wg_gpart g, int64_t info[3]);
+/* HOST copies: perm[E] (edge ids in scan order), tasks[n] (either may be NULL). */
+wg_status wg_gpart_export(wg_gpart g, int64_t* perm, wg_task* tasks);
+/* Bytes of the workspace wg_gpart_aggregate needs for width F.             */
+size_t wg_gpart_workspace(wg_gpart g, int32_t F);
+/* Agg[v] = sum_{e: dst_e = v} c_e x[src_e] (the Index / Index-add pair,
+ * P:L520-536) executed over the gTasks of ANY restriction set: gTasks may
+ * share destinations, so fp32 partial rows are added with vector atomics
+ * (one per run of equal destinations) and a finishing pass applies the
+ * destination scale and the cast (RNE for bf16).  c_e per `norm` as for GCN
+ * (Q3).  Row-major x [V x ldx], out [V x ldo] in dtype; F % 4 == 0.  The
+ * atomic order varies between runs (results agree to fp32 rounding).        */
+wg_status wg_gpart_aggregate(wg_gpart g, wg_dtype dtype, int32_t F, wg_norm norm, const void* x, int64_t ldx,
+                             void* out, int64_t ldo, void* workspace, wg_stream stream);
+wg_status wg_gpart_destroy(wg_gpart g);
+
+/* ------------------------------------------------------------------------ */
 /* Training-step utility: fused softmax cross-entropy over the last layer's
  * logits [M x ld] (C classes): loss_out[0] = scale * sum_r -log softmax(x_r)[label_r],
  * dlogits = scale * (softmax(x_r) - onehot(label_r)) in the conv dtype

@@ -18,7 +18,7 @@ import torch
 from . import _capi as C
 from ._capi import WGError, TASK_DTYPE
 
-__all__ = ["Graph", "Conv", "Comm", "WGError", "TASK_DTYPE", "padded", "pad_to", "ld_of", "launch_count",
+__all__ = ["Graph", "Conv", "Comm", "GPart", "WGError", "TASK_DTYPE", "padded", "pad_to", "ld_of", "launch_count",
            "init_params", "partition_1d"]
 
 
@@ -267,6 +267,61 @@ class Graph:
             if getattr(self, "_h", None) and self._plans == 0:
                 C.lib().wg_graph_destroy(self._h)
                 self._h = None
+        except Exception:
+            pass
+
+
+class GPart:
+    """General restriction engine (wg_gpart_*): gTasks of any uniq() restriction
+    set over dst / src / type / dst_degree / edge (Fig 7), and
+    the atomic Index / Index-add executor over them.
+
+        gp = GPart(src, dst, num_vertices=V, restrictions=[("src", 32), ("type", 1)], etype=et)
+        agg = gp.aggregate(x, norm="both")
+    """
+
+    def __init__(self, src, dst=None, *, num_vertices: int, restrictions=(), indptr=None, etype=None,
+                 device: int | None = None, stream=None):
+        L = C.lib()
+        keep = []
+        desc = _graph_desc(src, dst, num_vertices, indptr, etype, 1, 128, 0, 0, 0, keep)
+        r = (ctypes.c_int32 * (2 * max(1, len(restrictions))))()
+        for i, (a, k) in enumerate(restrictions):
+            r[2 * i] = C.ATTRS[a]
+            r[2 * i + 1] = C.UNIQ_MIN if k == "min" else int(k)
+        self.device = torch.cuda.current_device() if device is None else device
+        h = ctypes.c_void_p()
+        with torch.cuda.device(self.device):
+            C.check(L.wg_gpart_create(ctypes.byref(desc), r, len(restrictions), self.device, _stream(stream),
+                                      ctypes.byref(h)), "wg_gpart_create")
+        self._h = h
+        info = (ctypes.c_int64 * 3)()
+        C.check(L.wg_gpart_info(h, info), "wg_gpart_info")
+        self.V, self.E, self.n_tasks = list(info)
+
+    def export(self):
+        perm = np.empty(max(self.E, 1), np.int64)
+        tasks = np.empty(max(self.n_tasks, 1), TASK_DTYPE)
+        C.check(C.lib().wg_gpart_export(self._h, _ptr(perm), _ptr(tasks)), "wg_gpart_export")
+        return perm[:self.E], tasks[:self.n_tasks]
+
+    def aggregate(self, x, norm: str = "none", out=None, stream=None):
+        F = x.shape[1]
+        if out is None:
+            out = padded(self.V, F, x.dtype, x.device, zero=False)
+        ws = torch.empty(max(int(C.lib().wg_gpart_workspace(self._h, F)), 256), dtype=torch.uint8, device=x.device)
+        C.check(C.lib().wg_gpart_aggregate(self._h, _dt(x.dtype), F, C.NORMS[norm], _ptr(x), ld_of(x), _ptr(out),
+                                           ld_of(out), _ptr(ws), _stream(stream)), "wg_gpart_aggregate")
+        return out
+
+    def close(self):
+        if getattr(self, "_h", None):
+            C.lib().wg_gpart_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
         except Exception:
             pass
 

@@ -29,7 +29,11 @@ EXPORTS = [
     "wg_comm_unique_id", "wg_comm_init", "wg_comm_init_emulated", "wg_comm_info", "wg_comm_wait",
     "wg_comm_destroy", "wg_partition_1d", "wg_graph_create_dist", "wg_graph_bounds", "wg_plan_create_dist",
     "wg_plan_xchg", "wg_conv_forward_dist", "wg_conv_backward_dist",
+    "wg_gpart_create", "wg_gpart_info", "wg_gpart_export", "wg_gpart_workspace", "wg_gpart_aggregate",
+    "wg_gpart_destroy",
 ]
+ATTRS = {"dst": 0, "src": 1, "type": 2, "dst_degree": 3, "edge": 4}
+UNIQ_MIN = -1
 COMM_ID_BYTES = 128
 XENT_SCRATCH_BYTES = 8192
 PROF_KINDS = ["gather_reduce", "split_combine", "tc_gemm_nt", "tc_gemm_tn", "simt_gemm", "misc", "gat", "rgcn"]
@@ -153,6 +157,19 @@ def lib():
     L.wg_conv_backward_dist.restype = st
     L.wg_conv_backward_dist.argtypes = [P, P, ctypes.POINTER(Params), ctypes.POINTER(BwdArgs),
                                         ctypes.POINTER(Grads), P]
+    # general restriction engine
+    L.wg_gpart_create.restype = st
+    L.wg_gpart_create.argtypes = [ctypes.POINTER(GraphDesc), P, i32, ctypes.c_int, P, ctypes.POINTER(P)]
+    L.wg_gpart_info.restype = st
+    L.wg_gpart_info.argtypes = [P, P]
+    L.wg_gpart_export.restype = st
+    L.wg_gpart_export.argtypes = [P, P, P]
+    L.wg_gpart_workspace.restype = ctypes.c_size_t
+    L.wg_gpart_workspace.argtypes = [P, i32]
+    L.wg_gpart_aggregate.restype = st
+    L.wg_gpart_aggregate.argtypes = [P, ctypes.c_int, i32, ctypes.c_int, P, i64, P, i64, P, P]
+    L.wg_gpart_destroy.restype = st
+    L.wg_gpart_destroy.argtypes = [P]
     _lib = L
     return L
 

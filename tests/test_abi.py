@@ -12,7 +12,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 def declared_symbols():
     src = open(os.path.join(ROOT, "include", "wg.h")).read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
-    return sorted(set(re.findall(r"^\s*(?:wg_status|const char\*|int64_t)\s+(wg_\w+)\s*\(", src, flags=re.M)))
+    return sorted(set(re.findall(r"^\s*(?:wg_status|const char\*|int64_t|size_t)\s+(wg_\w+)\s*\(", src, flags=re.M)))
 
 
 def test_header_declares_the_boundary():
