@@ -128,6 +128,8 @@ typedef struct {
   wg_plan_policy policy;
   uint64_t policy_seed;     /* WG_PLAN_RANDOM                                    */
   int32_t need_dx;          /* backward produces dx (0 for the input layer)      */
+  int32_t x_replicated;     /* 1-D partition: the layer's input rows are on every */
+                            /* rank already (the input features); 0: exchanged  */
 } wg_conv_desc;
 
 /* Errors: WG_ERR_INVALID (bad sizes / model / dtype), WG_ERR_UNSUPPORTED
@@ -142,9 +144,10 @@ wg_status wg_plan_create(wg_graph g, const wg_conv_desc* desc, wg_plan* out);
 wg_status wg_plan_sizes(wg_plan p, size_t* saved_bytes, size_t* workspace_bytes);
 /* per_task_plan (host, n_tasks bytes, may be NULL): 0 = EDGE, 1 = VERTEX.
  * stats (host, may be NULL) [0..7]: n EDGE tasks, n VERTEX tasks, backward
- * path (0 = dAgg, 1 = G), exchange width fwd, exchange width bwd (elements,
- * 0 = the exchanged table is x itself), n work items fwd, n work items T,
- * n split rows fwd.                                                        */
+ * path (0 = dAgg, 1 = G), exchange width fwd, exchange width bwd (columns
+ * of the table the layer exchanges on a 1-D partition, 0 = none: an EDGE
+ * layer's forward reads the activation itself), n work items fwd, n work
+ * items T, n split rows fwd.                                               */
 wg_status wg_plan_export(wg_plan p, uint8_t* per_task_plan, int64_t stats[8]);
 /* Introspection (tests / tools): byte offset of a named sub-buffer of the
  * saved (which = 0) or workspace (which = 1) buffer, e.g. "agg" (the saved

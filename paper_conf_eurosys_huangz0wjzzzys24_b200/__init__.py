@@ -335,7 +335,7 @@ class Conv:
     def __init__(self, graph: Graph, model: str, f_in: int, f_out: int, *, dtype=torch.float32, heads: int = 1,
                  concat: bool = True, norm: str = "both", self_loop: bool = False, bias: bool = True,
                  fuse_relu: bool = False, gin_eps: float = 0.0, neg_slope: float = 0.2, policy: str = "auto",
-                 seed: int = 0, need_dx: bool = True):
+                 seed: int = 0, need_dx: bool = True, x_replicated: bool = False):
         self.graph = graph
         self.model = model
         self.f_in, self.f_out, self.heads, self.concat = f_in, f_out, heads, concat
@@ -345,7 +345,7 @@ class Conv:
         self.need_dx = need_dx
         self.desc = C.ConvDesc(C.MODELS[model], _dt(dtype), f_in, f_out, heads, int(concat), C.NORMS[norm],
                                int(self_loop), int(bias), int(fuse_relu), gin_eps, neg_slope, C.POLICIES[policy],
-                               seed, int(need_dx))
+                               seed, int(need_dx), int(x_replicated))
         h = ctypes.c_void_p()
         self.comm = graph.comm
         if self.comm is not None:   # one uniform plan on every rank (wg_plan_create_dist)

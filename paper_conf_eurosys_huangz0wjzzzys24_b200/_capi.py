@@ -58,7 +58,7 @@ class ConvDesc(ctypes.Structure):
     _fields_ = [("model", ctypes.c_int), ("dtype", ctypes.c_int), ("f_in", i32), ("f_out", i32), ("heads", i32),
                 ("concat_heads", i32), ("norm", ctypes.c_int), ("self_loop", i32), ("bias", i32),
                 ("fuse_relu", i32), ("gin_eps", f32), ("neg_slope", f32), ("policy", ctypes.c_int),
-                ("policy_seed", u64), ("need_dx", i32)]
+                ("policy_seed", u64), ("need_dx", i32), ("x_replicated", i32)]
 
 
 class Params(ctypes.Structure):

@@ -397,20 +397,38 @@ wg_status wg_plan_create_dist(wg_comm c, wg_graph g, const wg_conv_desc* desc, w
     // one uniform plan per layer on every rank: the ranks exchange one table
     WG_REQ(d.policy != WG_PLAN_RANDOM, WG_ERR_UNSUPPORTED, "mixed (random) plans are single-partition only");
     if (d.policy == WG_PLAN_AUTO) {
+      // Operation placement by data volume (Fig 11): the a4
+      // HBM cost of each uniform plan plus the exchange it implies on this
+      // rank, pipelined over the table's column chunks.  EDGE exchanges the
+      // activation (unless replicated) and, for dx, dAgg (f_in wide);
+      // VERTEX exchanges Y = x W and dT (f_out wide).  Per-rank times are
+      // summed over the ranks (an all-reduce) and the smaller plan is taken.
       int64_t sum[3];
       lin_cost_sums(g, d, sum, nullptr);
+      const int es = dsize(d.dtype);
+      const int64_t remote = g->V - (g->ve - g->vb);
+      const int64_t rin = pitch(d.f_in, d.dtype) * es, rout = pitch(d.f_out, d.dtype) * es;
+      auto pipe = [](int64_t gather, int64_t link, int C) {   // C-chunk pipeline (milli-fs)
+        return link / C + (C - 1) * std::max(gather, link) / C + gather / C;
+      };
+      // forward gather ~ half of the layer's a4 bytes, backward the other half
+      const int64_t ge = sum[0] * K_MEM / 2, gv = sum[1] * K_MEM / 2;
+      const int64_t le_f = d.x_replicated ? 0 : remote * rin * K_LINK, le_b = d.need_dx ? remote * rin * K_LINK : 0;
+      const int64_t lv = remote * rout * K_LINK;
+      const int ci = xchg_chunks(d, d.f_in), co = xchg_chunks(d, d.f_out);
+      int64_t t[2] = {pipe(ge, le_f, 1) + pipe(ge, le_b, ci), pipe(gv, lv, co) + pipe(gv, lv, co)};
       if (!c->emulated) {   // add the ranks' layer costs (all-EDGE, all-VERTEX)
         WG_CK(cudaSetDevice(g->device));
         int64_t* dsum = nullptr;
         WG_CK(cudaMalloc(&dsum, 2 * sizeof(int64_t)));
-        cudaMemcpy(dsum, sum, 2 * sizeof(int64_t), cudaMemcpyHostToDevice);
+        cudaMemcpy(dsum, t, 2 * sizeof(int64_t), cudaMemcpyHostToDevice);
         nccl_res r = nccl().AllReduce(dsum, dsum, 2, N_INT64, N_SUM, c->comm, c->cs);
         cudaStreamSynchronize(c->cs);
-        cudaMemcpy(sum, dsum, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost);
+        cudaMemcpy(t, dsum, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost);
         cudaFree(dsum);
         if (r != 0) { set_error(std::string("ncclAllReduce: ") + nccl().GetErrorString(r)); return WG_ERR_CUDA; }
       }
-      d.policy = sum[1] < sum[0] ? WG_PLAN_ALL_VERTEX : WG_PLAN_ALL_EDGE;
+      d.policy = t[1] < t[0] ? WG_PLAN_ALL_VERTEX : WG_PLAN_ALL_EDGE;
     }
   }
   return plan_create(g, &d, out);

@@ -138,6 +138,21 @@ void lin_cost_sums(const wg_graph_s* g, const wg_conv_desc& d, int64_t sum[3], s
 // of chunk k overlaps the exchange of chunk k+1; GIN / RGCN tables stay
 // row-major (C = 1).  WG_XCHG_CHUNK_BYTES overrides the 256-byte minimum
 // (0 disables chunking).
+int xchg_chunks(const wg_conv_desc& d, int64_t width) {
+  if (!width || !(d.model == WG_GCN || d.model == WG_SAGE)) return 1;
+  static int64_t min_chunk = -1;
+  if (min_chunk < 0) {
+    const char* e = getenv("WG_XCHG_CHUNK_BYTES");
+    min_chunk = e ? atoll(e) : 256;
+  }
+  if (min_chunk <= 0) return 1;
+  const int es = dsize(d.dtype);
+  const int64_t pe = pitch(width, d.dtype), rho = pe * es;
+  int C = (int)std::min<int64_t>(4, rho / min_chunk);
+  while (C > 1 && (pe % C != 0 || (pe / C * es) % 128 != 0)) --C;
+  return std::max(C, 1);
+}
+
 void xchg_layouts(wg_plan_s* p) {
   const wg_graph_s* g = p->g;
   const wg_conv_desc& d = p->d;
@@ -156,20 +171,9 @@ void xchg_layouts(wg_plan_s* p) {
   } else if (d.model == WG_RGCN) {
     p->xb.width = d.f_out;
   }
-  if (!(d.model == WG_GCN || d.model == WG_SAGE)) return;
-  static int64_t min_chunk = -1;
-  if (min_chunk < 0) {
-    const char* e = getenv("WG_XCHG_CHUNK_BYTES");
-    min_chunk = e ? atoll(e) : 256;
-  }
-  if (min_chunk <= 0) return;
-  const int es = dsize(d.dtype);
   for (XLayout* X : {&p->xf, &p->xb}) {
-    if (!X->width) continue;
-    const int64_t pe = pitch(X->width, d.dtype), rho = pe * es;
-    int C = (int)std::min<int64_t>(4, rho / min_chunk);
-    while (C > 1 && (pe % C != 0 || (pe / C * es) % 128 != 0)) --C;
-    if (C > 1) { X->C = C; X->Fc = pe / C; }
+    const int C = xchg_chunks(d, X->width);
+    if (C > 1) { X->C = C; X->Fc = pitch(X->width, d.dtype) / C; }
   }
 }
 
@@ -296,8 +300,8 @@ wg_status wg_plan_export(wg_plan p, uint8_t* per_task_plan, int64_t stats[8]) {
     stats[0] = p->n_edge_tasks;
     stats[1] = p->n_vert_tasks;
     stats[2] = p->bwd_path;
-    stats[3] = 0;
-    stats[4] = 0;
+    stats[3] = p->xf.width;
+    stats[4] = p->xb.width;
     stats[5] = p->fe.n + p->fv.n;
     stats[6] = p->bt.n;
     stats[7] = p->fe.n_split + p->fv.n_split;

@@ -94,6 +94,8 @@ wg_status lin_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, c
                        const XHook* hk = nullptr);
 // exchange layouts of a plan (set by plan_create for graphs owning a row block)
 void xchg_layouts(wg_plan_s* p);
+// column chunks of a GCN / SAGE exchange table of `width` columns (1: row-major)
+int xchg_chunks(const wg_conv_desc& d, int64_t width);
 // a4 layer cost sums {all-EDGE, all-VERTEX, mixed} of the untyped models
 void lin_cost_sums(const wg_graph_s* g, const wg_conv_desc& d, int64_t sum[3], std::vector<uint8_t>* best);
 wg_status plan_create(wg_graph g, const wg_conv_desc* d, wg_plan* out);

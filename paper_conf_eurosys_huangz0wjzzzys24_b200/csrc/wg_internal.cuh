@@ -259,6 +259,7 @@ size_t bias_grad_scratch(int64_t M, int N);
 
 // cost-model constants (milli-femtoseconds per byte / per flop), from MEASURED_PEAKS
 constexpr int64_t K_MEM = 152952;   // 1e6 / 6.538 GB/s-per-fs
+constexpr int64_t K_LINK = 1428571; // 1e6 / 0.7 TB/s: NVLink 5 all-gather bandwidth per GPU (effective)
 constexpr int64_t K_MMA_BF16 = 720; // 1e6 / 1389.2
 constexpr int64_t K_MMA_F32 = 16000;
 

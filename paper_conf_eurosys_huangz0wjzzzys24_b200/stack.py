@@ -66,6 +66,8 @@ class GNNStack:
         for i in range(self.L):
             last = i == self.L - 1
             kw = dict(dtype=dtype, fuse_relu=not last, need_dx=i > 0, seed=seed + i, **(conv_kw or {}))
+            if conv_factory is None:
+                kw["x_replicated"] = i == 0          # the input features are on every rank
             if model == "gat":
                 kw.update(heads=heads, concat=not last)
             fi = self.f_in[i]
