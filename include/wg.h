@@ -264,7 +264,7 @@ wg_status wg_comm_init(const void* id, int rank, int world, int device, wg_comm*
 /* One-GPU emulation of rank `rank` of a `world`-way partition: with copy = 1
  * every exchange is a copy kernel on the communication stream that re-reads
  * and re-writes the non-owned rows (the HBM bytes an all-gather moves, with
- * the SM share of an NCCL kernel: WG_EMU_CTAS CTAs, default 16); copy = 0
+ * WG_EMU_CTAS CTAs, default 40: ~0.7 TB/s, an NVLink 5 all-gather's rate); copy = 0
  * skips exchanges (the rank's compute alone).  No data moves between ranks
  * and gradients are not reduced.  For timing one rank on one GPU
  * (bench.py --rank-slice), not for results.                                */

@@ -203,9 +203,9 @@ wg_status lin_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* A, cu
   // exchange table is required (the workspace holds owned rows only)
   WG_REQ(!dist || !post || p->n_vert_tasks == 0 || A->xchg, WG_ERR_INVALID,
          "a VERTEX layer on a 1-D partition needs the exchange table (xchg)");
-  WG_REQ(!A->xchg || ((A->ld_xchg * c.s) % 16 == 0 && A->ld_xchg >= c.fo), WG_ERR_INVALID,
-         "ld_xchg must be >= f_out and a 16-byte multiple");
   const XLayout xl = A->xchg ? p->xf : XLayout{};
+  WG_REQ(!A->xchg || ((A->ld_xchg * c.s) % 16 == 0 && (xl.C > 1 || A->ld_xchg >= c.fo)), WG_ERR_INVALID,
+         "ld_xchg must be >= f_out (the chunk pitch for a chunked table) and a 16-byte multiple");
   WG_REQ(xl.C <= 1 || A->ld_xchg == xl.Fc, WG_ERR_INVALID,
          "chunked exchange table: ld_xchg must be the chunk width (wg_plan_xchg)");
   void* ws = A->workspace;
