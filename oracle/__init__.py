@@ -67,6 +67,9 @@ def _L():
         _lib.wgo_rgcn_backward.argtypes = [i64, i64, P, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P, P, P, P]
         _lib.wgo_gat_forward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, f64, P, P, P, P, P, P, P]
         _lib.wgo_gat_backward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, f64, P, P, P, P, P, P, P, P, P, P]
+        _lib.wgo_sage_lstm_forward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P, P, P, P, P]
+        _lib.wgo_sage_lstm_backward.argtypes = [i64, i64, P, P, ctypes.c_int, ctypes.c_int, P, P, P, P, P, P, P, P,
+                                                P, P, P, P, P, P, P]
         _lib.wgo_dw_probe.restype = f64
         _lib.wgo_dw_probe.argtypes = [i64, P, P, P, ctypes.c_int, ctypes.c_int, P, P, P, P]
     return _lib
@@ -272,6 +275,30 @@ def gat_backward(src, dst, V, x, W, al, ar, dy, *, heads, concat=True, slope=0.2
     _L().wgo_gat_backward(V, s.shape[0], _p(s), _p(d), fi, heads, fo, int(concat), float(slope), _p(x), _p(W),
                           _p(al), _p(ar), _p(dy), _p(dx), _p(dW), _p(dal), _p(dar), _p(db))
     return dx, dW, dal, dar, db
+
+
+def sage_lstm_forward(src, dst, V, x, Ws, Wn, b, Wih, Whh, bl, rows=None, return_h=False):
+    """SAGE-LSTM forward (f4; Q26): y = b + x W_s + LSTM(x[in-nbrs in edge-id order]) W_n."""
+    x, Ws, Wn, b, Wih, Whh, bl = map(_f64, (x, Ws, Wn, b, Wih, Whh, bl))
+    fi, fo = Ws.shape
+    y = np.zeros((V, fo))
+    hN = np.zeros((V, fi)) if return_h else None
+    s, d = _i32(src), _i32(dst)
+    _L().wgo_sage_lstm_forward(V, s.shape[0], _p(s), _p(d), fi, fo, _p(x), _p(Ws), _p(Wn), _p(b), _p(Wih), _p(Whh),
+                               _p(bl), _p(_mask(V, rows)), _p(y), _p(hN))
+    return (y, hN) if return_h else y
+
+
+def sage_lstm_backward(src, dst, V, x, Ws, Wn, Wih, Whh, bl, dy, dy_rows=None):
+    """Exact gradients (BPTT per vertex): dx, dWs, dWn, db, dWih, dWhh, dbl."""
+    x, Ws, Wn, Wih, Whh, bl, dy = map(_f64, (x, Ws, Wn, Wih, Whh, bl, dy))
+    fi, fo = Ws.shape
+    out = [np.zeros((V, fi)), np.zeros((fi, fo)), np.zeros((fi, fo)), np.zeros(fo), np.zeros((fi, 4 * fi)),
+           np.zeros((fi, 4 * fi)), np.zeros(4 * fi)]
+    s, d = _i32(src), _i32(dst)
+    _L().wgo_sage_lstm_backward(V, s.shape[0], _p(s), _p(d), fi, fo, _p(x), _p(Ws), _p(Wn), _p(Wih), _p(Whh), _p(bl),
+                                _p(dy), _p(_mask(V, dy_rows)), *[_p(o) for o in out])
+    return tuple(out)
 
 
 def dw_probe(src, dst, x, dy, u, v, coef=None):

@@ -708,3 +708,135 @@ double wgo_dw_probe(int64_t E, const int32_t* src, const int32_t* dst, const dou
     }
     return acc;
 }
+
+/* ======================================================================== */
+/* GraphSAGE with the LSTM aggregator (Hamilton et al. [14]; the paper's    */
+/* fifth model, SAGE-LSTM).     */
+/* Readings (Q26): the neighbour sequence of v is its in-edges in */
+/* edge-id order; LSTM hidden size H = f_in; gates in PyTorch order         */
+/* (i, f, g, o), z = x_t W_ih + h_{t-1} W_hh + b_l with W_ih, W_hh          */
+/* [f_in x 4H] (column blocks i | f | g | o); h_0 = c_0 = 0;                 */
+/*   i = s(z_i), f = s(z_f), g = tanh(z_g), o = s(z_o),                      */
+/*   c_t = f c_{t-1} + i g,  h_t = o tanh(c_t);                              */
+/* h_N(v) = h_deg(v) (0 for an isolated v);                                  */
+/*   y[v] = b + x[v] W_s + h_N(v) W_n.                                       */
+/* ======================================================================== */
+static double sigm(double z) { return 1.0 / (1.0 + exp(-z)); }
+
+/* in-edges of every vertex in edge-id order: counting sort by dst */
+static void in_lists(int64_t V, int64_t E, const int32_t* dst, int64_t* ptr, int64_t* eid) {
+    memset(ptr, 0, sizeof(int64_t) * (V + 1));
+    for (int64_t e = 0; e < E; ++e) ptr[dst[e] + 1]++;
+    for (int64_t v = 0; v < V; ++v) ptr[v + 1] += ptr[v];
+    int64_t* fill = (int64_t*)malloc(sizeof(int64_t) * (V > 0 ? V : 1));
+    for (int64_t v = 0; v < V; ++v) fill[v] = ptr[v];
+    for (int64_t e = 0; e < E; ++e) eid[fill[dst[e]]++] = e;
+    free(fill);
+}
+
+/* one LSTM step for one vertex: z (4H) <- gates; returns activated gates in
+ * gt (4H: i, f, g, o), updates c (H) and h (H) */
+static void lstm_step(int H, const double* xt, const double* hprev, const double* Wih, const double* Whh,
+                      const double* bl, double* gt, double* c, double* h) {
+    for (int j = 0; j < 4 * H; ++j) gt[j] = bl ? bl[j] : 0.0;
+    add_msg(H, 4 * H, 1.0, xt, Wih, gt);
+    add_msg(H, 4 * H, 1.0, hprev, Whh, gt);
+    for (int j = 0; j < H; ++j) {
+        gt[j] = sigm(gt[j]);
+        gt[H + j] = sigm(gt[H + j]);
+        gt[2 * H + j] = tanh(gt[2 * H + j]);
+        gt[3 * H + j] = sigm(gt[3 * H + j]);
+        c[j] = gt[H + j] * c[j] + gt[j] * gt[2 * H + j];
+        h[j] = gt[3 * H + j] * tanh(c[j]);
+    }
+}
+
+/* row_mask: only those rows of y (and hN) are produced.  hN (nullable): [V x fi] */
+void wgo_sage_lstm_forward(int64_t V, int64_t E, const int32_t* src, const int32_t* dst, int fi, int fo,
+                           const double* x, const double* Ws, const double* Wn, const double* b, const double* Wih,
+                           const double* Whh, const double* bl, const uint8_t* row_mask, double* y, double* hN) {
+    const int H = fi;
+    int64_t* ptr = (int64_t*)malloc(sizeof(int64_t) * (V + 1));
+    int64_t* eid = (int64_t*)malloc(sizeof(int64_t) * (E > 0 ? E : 1));
+    in_lists(V, E, dst, ptr, eid);
+    double *c = malloc(sizeof(double) * H), *h = malloc(sizeof(double) * H), *gt = malloc(sizeof(double) * 4 * H);
+    for (int64_t v = 0; v < V; ++v) {
+        if (!ROW_ON(row_mask, v)) continue;
+        for (int j = 0; j < H; ++j) { c[j] = 0.0; h[j] = 0.0; }
+        for (int64_t p = ptr[v]; p < ptr[v + 1]; ++p)
+            lstm_step(H, x + (int64_t)src[eid[p]] * fi, h, Wih, Whh, bl, gt, c, h);
+        if (hN) for (int j = 0; j < H; ++j) hN[v * H + j] = h[j];
+        for (int j = 0; j < fo; ++j) y[v * fo + j] = b ? b[j] : 0.0;
+        add_msg(fi, fo, 1.0, x + v * fi, Ws, y + v * fo);
+        add_msg(H, fo, 1.0, h, Wn, y + v * fo);
+    }
+    free(ptr); free(eid); free(c); free(h); free(gt);
+}
+
+/* Exact gradients (backpropagation through each vertex's sequence).
+ * dy_rows (nullable): rows of dy outside the set are zero (skipped); every
+ * output is then the exact gradient for that dy.  Outputs nullable. */
+void wgo_sage_lstm_backward(int64_t V, int64_t E, const int32_t* src, const int32_t* dst, int fi, int fo,
+                            const double* x, const double* Ws, const double* Wn, const double* Wih,
+                            const double* Whh, const double* bl, const double* dy, const uint8_t* dy_rows,
+                            double* dx, double* dWs, double* dWn, double* db, double* dWih, double* dWhh,
+                            double* dbl) {
+    const int H = fi;
+    int64_t* ptr = (int64_t*)malloc(sizeof(int64_t) * (V + 1));
+    int64_t* eid = (int64_t*)malloc(sizeof(int64_t) * (E > 0 ? E : 1));
+    in_lists(V, E, dst, ptr, eid);
+    int64_t maxd = 0;
+    for (int64_t v = 0; v < V; ++v) if (ptr[v + 1] - ptr[v] > maxd) maxd = ptr[v + 1] - ptr[v];
+    /* per step of one sequence: activated gates, c_t, h_t (index t+1; 0 = initial) */
+    double* G = malloc(sizeof(double) * 4 * H * (maxd > 0 ? maxd : 1));
+    double* Cs = malloc(sizeof(double) * H * (maxd + 1));
+    double* Hs = malloc(sizeof(double) * H * (maxd + 1));
+    double *dh = malloc(sizeof(double) * H), *dc = malloc(sizeof(double) * H), *dz = malloc(sizeof(double) * 4 * H);
+    double* dhn = malloc(sizeof(double) * H);
+    if (dx) memset(dx, 0, sizeof(double) * V * fi);
+    if (dWs) memset(dWs, 0, sizeof(double) * fi * fo);
+    if (dWn) memset(dWn, 0, sizeof(double) * H * fo);
+    if (db) memset(db, 0, sizeof(double) * fo);
+    if (dWih) memset(dWih, 0, sizeof(double) * fi * 4 * H);
+    if (dWhh) memset(dWhh, 0, sizeof(double) * H * 4 * H);
+    if (dbl) memset(dbl, 0, sizeof(double) * 4 * H);
+    for (int64_t v = 0; v < V; ++v) {
+        if (!ROW_ON(dy_rows, v)) continue;
+        const double* dyv = dy + v * fo;
+        const int64_t T = ptr[v + 1] - ptr[v];
+        /* forward of the sequence, keeping every step */
+        for (int j = 0; j < H; ++j) { Cs[j] = 0.0; Hs[j] = 0.0; }
+        for (int64_t t = 0; t < T; ++t) {
+            for (int j = 0; j < H; ++j) Cs[(t + 1) * H + j] = Cs[t * H + j];
+            lstm_step(H, x + (int64_t)src[eid[ptr[v] + t]] * fi, Hs + t * H, Wih, Whh, bl, G + t * 4 * H,
+                      Cs + (t + 1) * H, Hs + (t + 1) * H);
+        }
+        /* y = b + x[v] W_s + h_N W_n */
+        if (db) for (int j = 0; j < fo; ++j) db[j] += dyv[j];
+        add_msg_grad(fi, fo, 1.0, x + v * fi, Ws, dyv, dx ? dx + v * fi : NULL, dWs);
+        for (int j = 0; j < H; ++j) dhn[j] = 0.0;
+        add_msg_grad(H, fo, 1.0, Hs + T * H, Wn, dyv, dhn, dWn);
+        /* backpropagation through time */
+        for (int j = 0; j < H; ++j) { dh[j] = dhn[j]; dc[j] = 0.0; }
+        for (int64_t t = T - 1; t >= 0; --t) {
+            const double* gt = G + t * 4 * H;
+            for (int j = 0; j < H; ++j) {
+                const double i = gt[j], f = gt[H + j], g = gt[2 * H + j], o = gt[3 * H + j];
+                const double tc = tanh(Cs[(t + 1) * H + j]);
+                const double dO = dh[j] * tc;
+                const double dC = dc[j] + dh[j] * o * (1.0 - tc * tc);
+                dz[j] = dC * g * i * (1.0 - i);
+                dz[H + j] = dC * Cs[t * H + j] * f * (1.0 - f);
+                dz[2 * H + j] = dC * i * (1.0 - g * g);
+                dz[3 * H + j] = dO * o * (1.0 - o);
+                dc[j] = dC * f;
+            }
+            if (dbl) for (int j = 0; j < 4 * H; ++j) dbl[j] += dz[j];
+            const int64_t s = src[eid[ptr[v] + t]];
+            add_msg_grad(fi, 4 * H, 1.0, x + s * fi, Wih, dz, dx ? dx + s * fi : NULL, dWih);
+            for (int j = 0; j < H; ++j) dh[j] = 0.0;
+            add_msg_grad(H, 4 * H, 1.0, Hs + t * H, Whh, dz, dh, dWhh);
+        }
+    }
+    free(ptr); free(eid); free(G); free(Cs); free(Hs); free(dh); free(dc); free(dz); free(dhn);
+}
