@@ -50,7 +50,9 @@ typedef enum {
   WG_ERR_STATE = 7         /* misuse of handles                             */
 } wg_status;
 
-typedef enum { WG_GCN = 0, WG_GIN = 1, WG_SAGE = 2, WG_GAT = 3, WG_RGCN = 4 } wg_model;
+/* WG_SAGE_LSTM: GraphSAGE with the LSTM aggregator (the paper's fifth model,
+ * P:L3790-3814; reading Q26): fp32, full graphs.          */
+typedef enum { WG_GCN = 0, WG_GIN = 1, WG_SAGE = 2, WG_GAT = 3, WG_RGCN = 4, WG_SAGE_LSTM = 5 } wg_model;
 typedef enum { WG_F32 = 0, WG_BF16 = 1 } wg_dtype;
 /* GCN [24] / RGCN [34] edge coefficient c_e (Q2, Q3):
  * NONE: 1; RIGHT: 1/deg_in(dst) (RGCN: 1/|in(dst) of type r|);
@@ -168,12 +170,14 @@ wg_status wg_plan_destroy(wg_plan p);
 /*   GAT : W [f_in x heads*f_out], attn_l / attn_r [heads x f_out],         */
 /*         bias [heads*f_out] (concat) or [f_out] (mean)                    */
 /*   RGCN: W [R x f_in x f_out], W_self = W_0 (self_loop), bias             */
+/*   SAGE-LSTM: W = W_n [f_in x f_out], W_self = W_s, bias, Wih / Whh       */
+/*         [f_in x 4 f_in] (gate column blocks i | f | g | o), bl [4 f_in]   */
 /* ------------------------------------------------------------------------ */
 typedef struct {
-  const float *W, *W_self, *bias, *attn_l, *attn_r, *W2, *b2;
+  const float *W, *W_self, *bias, *attn_l, *attn_r, *W2, *b2, *Wih, *Whh, *bl;
 } wg_params;
 typedef struct {
-  float *W, *W_self, *bias, *attn_l, *attn_r, *W2, *b2;   /* NULL => skip */
+  float *W, *W_self, *bias, *attn_l, *attn_r, *W2, *b2, *Wih, *Whh, *bl;   /* NULL => skip */
 } wg_grads;
 
 /* Phases for the 1-D multi-GPU layer (§8(e)).  Single GPU: WG_PHASE_ALL.

@@ -326,7 +326,7 @@ class GPart:
             pass
 
 
-PARAM_NAMES = ("W", "W_self", "bias", "attn_l", "attn_r", "W2", "b2")
+PARAM_NAMES = C.PARAM_NAMES
 
 
 class Conv:
@@ -510,6 +510,15 @@ def init_params(model: str, f_in: int, f_out: int, *, heads: int = 1, concat: bo
         p["attn_r"] = glorot(heads, f_out, fan_in=f_out, fan_out=1)
         if bias:
             p["bias"] = torch.zeros(heads * f_out if concat else f_out, device=device)
+    elif model == "sage_lstm":   # PyTorch nn.LSTM init: U(-1/sqrt(H), 1/sqrt(H)), H = f_in
+        k = 1.0 / f_in ** 0.5
+        p["W"] = glorot(f_in, f_out, fan_in=f_in, fan_out=f_out)
+        p["W_self"] = glorot(f_in, f_out, fan_in=f_in, fan_out=f_out)
+        p["Wih"] = ((torch.rand(f_in, 4 * f_in, generator=g) * 2 - 1) * k).to(device)
+        p["Whh"] = ((torch.rand(f_in, 4 * f_in, generator=g) * 2 - 1) * k).to(device)
+        p["bl"] = ((torch.rand(4 * f_in, generator=g) * 2 - 1) * k).to(device)
+        if bias:
+            p["bias"] = torch.zeros(f_out, device=device)
     elif model == "rgcn":
         p["W"] = glorot(R, f_in, f_out, fan_in=f_in, fan_out=f_out)
         if self_loop:

@@ -14,7 +14,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libwg.so")
 
 WG_OK, WG_ERR_INVALID, WG_ERR_RANGE, WG_ERR_NOMEM, WG_ERR_CUDA, WG_ERR_UNSUPPORTED, WG_ERR_STATE = 0, 1, 2, 3, 4, 6, 7
-MODELS = {"gcn": 0, "gin": 1, "sage": 2, "gat": 3, "rgcn": 4}
+MODELS = {"gcn": 0, "gin": 1, "sage": 2, "gat": 3, "rgcn": 4, "sage_lstm": 5}
 NORMS = {"none": 0, "right": 1, "both": 2}
 POLICIES = {"auto": 0, "edge": 1, "vertex": 2, "random": 3}
 WG_F32, WG_BF16 = 0, 1
@@ -61,12 +61,15 @@ class ConvDesc(ctypes.Structure):
                 ("policy_seed", u64), ("need_dx", i32), ("x_replicated", i32)]
 
 
+PARAM_NAMES = ("W", "W_self", "bias", "attn_l", "attn_r", "W2", "b2", "Wih", "Whh", "bl")
+
+
 class Params(ctypes.Structure):
-    _fields_ = [(n, P) for n in ("W", "W_self", "bias", "attn_l", "attn_r", "W2", "b2")]
+    _fields_ = [(n, P) for n in PARAM_NAMES]
 
 
 class Grads(ctypes.Structure):
-    _fields_ = [(n, P) for n in ("W", "W_self", "bias", "attn_l", "attn_r", "W2", "b2")]
+    _fields_ = [(n, P) for n in PARAM_NAMES]
 
 
 class FwdArgs(ctypes.Structure):

@@ -91,7 +91,7 @@ wg_status wg_conv_forward(wg_plan p, const wg_params* params, const wg_fwd_args*
   WG_REQ(p && params && a, WG_ERR_INVALID, "wg_conv_forward: null argument");
   WG_REQ(a->phase == WG_PHASE_ALL || a->phase == WG_PHASE_PRE || a->phase == WG_PHASE_POST, WG_ERR_INVALID,
          "wg_conv_forward: bad phase");
-  WG_REQ(a->phase == WG_PHASE_ALL || p->d.model != WG_GAT, WG_ERR_UNSUPPORTED,
+  WG_REQ(a->phase == WG_PHASE_ALL || (p->d.model != WG_GAT && p->d.model != WG_SAGE_LSTM), WG_ERR_UNSUPPORTED,
          "wg_conv_forward: PRE / POST phases are for GCN / SAGE / GIN / RGCN");
   WG_CK(cudaSetDevice(p->g->device));
   WG_CK(cudaGetLastError());
@@ -100,6 +100,7 @@ wg_status wg_conv_forward(wg_plan p, const wg_params* params, const wg_fwd_args*
     case WG_GCN: case WG_SAGE: case WG_GIN: return wg::lin_forward(p, params, a, s);
     case WG_GAT: return wg::gat_forward(p, params, a, s);
     case WG_RGCN: return wg::rgcn_forward(p, params, a, s);
+    case WG_SAGE_LSTM: return wg::lstm_forward(p, params, a, s);
   }
   return WG_ERR_INVALID;
 }
@@ -109,7 +110,7 @@ wg_status wg_conv_backward(wg_plan p, const wg_params* params, const wg_bwd_args
   WG_REQ(p && params && a, WG_ERR_INVALID, "wg_conv_backward: null argument");
   WG_REQ(a->phase == WG_PHASE_ALL || a->phase == WG_PHASE_PRE || a->phase == WG_PHASE_POST, WG_ERR_INVALID,
          "wg_conv_backward: bad phase");
-  WG_REQ(a->phase == WG_PHASE_ALL || p->d.model != WG_GAT, WG_ERR_UNSUPPORTED,
+  WG_REQ(a->phase == WG_PHASE_ALL || (p->d.model != WG_GAT && p->d.model != WG_SAGE_LSTM), WG_ERR_UNSUPPORTED,
          "wg_conv_backward: PRE / POST phases are for GCN / SAGE / GIN / RGCN");
   WG_CK(cudaSetDevice(p->g->device));
   WG_CK(cudaGetLastError());
@@ -118,6 +119,7 @@ wg_status wg_conv_backward(wg_plan p, const wg_params* params, const wg_bwd_args
     case WG_GCN: case WG_SAGE: case WG_GIN: return wg::lin_backward(p, params, a, grads, s);
     case WG_GAT: return wg::gat_backward(p, params, a, grads, s);
     case WG_RGCN: return wg::rgcn_backward(p, params, a, grads, s);
+    case WG_SAGE_LSTM: return wg::lstm_backward(p, params, a, grads, s);
   }
   return WG_ERR_INVALID;
 }

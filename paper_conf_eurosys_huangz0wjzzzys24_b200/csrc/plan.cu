@@ -186,7 +186,9 @@ void choose_plans(wg_plan_s* p) {
   const int64_t n = (int64_t)tasks.size();
   p->plan_bits.assign(n, 0);
   const wg_conv_desc& d = p->d;
-  if (d.model == WG_GAT) {  // GAT: transform-before-gather only
+  if (d.model == WG_SAGE_LSTM) {  // the LSTM aggregator is not linear: no T2 swap, EDGE only
+    std::fill(p->plan_bits.begin(), p->plan_bits.end(), 0);
+  } else if (d.model == WG_GAT) {  // GAT: transform-before-gather only
     std::fill(p->plan_bits.begin(), p->plan_bits.end(), 1);
   } else if (d.policy == WG_PLAN_ALL_VERTEX) {
     std::fill(p->plan_bits.begin(), p->plan_bits.end(), 1);
@@ -236,7 +238,7 @@ wg_status plan_create(wg_graph g, const wg_conv_desc* d, wg_plan* out) {
   WG_REQ(g && d && out, WG_ERR_INVALID, "wg_plan_create: null argument");
   WG_REQ(d->f_in >= 1 && d->f_out >= 1, WG_ERR_INVALID, "f_in / f_out must be >= 1");
   WG_REQ(d->dtype == WG_F32 || d->dtype == WG_BF16, WG_ERR_INVALID, "dtype");
-  WG_REQ(d->model >= WG_GCN && d->model <= WG_RGCN, WG_ERR_INVALID, "model");
+  WG_REQ(d->model >= WG_GCN && d->model <= WG_SAGE_LSTM, WG_ERR_INVALID, "model");
   if (d->model != WG_RGCN)
     WG_REQ(!g->by_type, WG_ERR_UNSUPPORTED, "typed graph (num_types > 1) is only supported by RGCN");
   if (d->model == WG_GAT) WG_REQ(d->heads >= 1, WG_ERR_INVALID, "GAT needs heads >= 1");
@@ -270,7 +272,14 @@ wg_status plan_create(wg_graph g, const wg_conv_desc* d, wg_plan* out) {
     // (a VERTEX-policy plan without any gTask -- a rank owning no in-edge --
     // takes the G path too, so every rank exchanges the same table)
     p->bwd_path = (p->n_vert_tasks > 0 || (p->n_edge_tasks == 0 && d->policy == WG_PLAN_ALL_VERTEX)) ? 1 : 0;
-    if (d->model == WG_GAT) gat_layout(p); else lin_layout(p);
+    if (d->model == WG_SAGE_LSTM) {
+      wg_status s2 = lstm_plan(p, 0);
+      if (s2 != WG_OK) { lstm_plan_free(p); for (void* q : p->allocs) cudaFree(q); delete p; return s2; }
+    } else if (d->model == WG_GAT) {
+      gat_layout(p);
+    } else {
+      lin_layout(p);
+    }
   }
   xchg_layouts(p);
   g->live_plans++;
@@ -324,6 +333,7 @@ wg_status wg_plan_destroy(wg_plan p) {
   cudaDeviceSynchronize();
   if (p->rg) wg::rgcn_plan_free(p);
   if (p->gat) wg::gat_plan_free(p);
+  if (p->lstm) wg::lstm_plan_free(p);
   for (void* q : p->allocs) cudaFree(q);
   p->g->live_plans--;
   delete p;

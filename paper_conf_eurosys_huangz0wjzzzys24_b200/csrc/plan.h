@@ -73,6 +73,7 @@ struct wg_plan_s {
   // model-specific structures (conv_rgcn.cu / conv_gat.cu)
   void* rg = nullptr;
   void* gat = nullptr;
+  void* lstm = nullptr;
 };
 
 // The EDGE pass (aggregate, then the transform GEMM) runs when any gTask is
@@ -101,6 +102,10 @@ void lin_cost_sums(const wg_graph_s* g, const wg_conv_desc& d, int64_t sum[3], s
 wg_status plan_create(wg_graph g, const wg_conv_desc* d, wg_plan* out);
 wg_status graph_create(const wg_graph_desc* d, int device, cudaStream_t st, wg_graph* out);
 void gat_layout(wg_plan_s* p);
+wg_status lstm_plan(wg_plan_s* p, cudaStream_t s);
+void lstm_plan_free(wg_plan_s* p);
+wg_status lstm_forward(wg_plan_s* p, const wg_params* P, const wg_fwd_args* a, cudaStream_t s);
+wg_status lstm_backward(wg_plan_s* p, const wg_params* P, const wg_bwd_args* a, const wg_grads* G, cudaStream_t s);
 void gat_plan_free(wg_plan_s* p);
 void lin_layout(wg_plan_s* p);
 }  // namespace wg

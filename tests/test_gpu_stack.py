@@ -277,7 +277,7 @@ def test_chunked_exchange_phases_match_single(model, policy, F):
     assert rel_err(f64(dx), f64(dx1)) < 1e-2
     for k in gr1:
         tot = sum(gr[k] for gr in grads)
-        assert rel_err(f64(tot), f64(gr1[k])) < 1e-3, k
+        assert rel_err(f64(tot), f64(gr1[k])) < 1e-2, k   # G rows round to bf16 after another summation split
 
 
 @pytest.mark.parametrize("model", ["sage", "gin", "rgcn"])
