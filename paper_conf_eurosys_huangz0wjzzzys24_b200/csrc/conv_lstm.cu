@@ -180,8 +180,7 @@ wg_status lstm_plan(wg_plan_s* p, cudaStream_t st) {
     WG_LAUNCH(k_tpos, grid_for(g->bwd.E), 256, 0, st, g->bwd.perm, g->bwd.E, epos, L->tpos);
   }
   WG_CK(cudaStreamSynchronize(st));
-  cudaFree(epos);
-  cudaFree(doff);
+  cudaFree(epos);                               // (doff stays in L->allocs)
   // layouts (fp32; row pitches 32-byte padded)
   const int H = d.f_in;
   p->pi = pitch(d.f_in, d.dtype);
