@@ -21,6 +21,8 @@
 //   out[r] = epi( rscale[r] * sum_{j in seg(r)} gscale[idx_j] * table[idx_j]
 //                 + self_coef * self[r] )
 //   epi(v) = mask( relu( v + bias ) )
+#include <cooperative_groups.h>
+
 #include "wg_internal.cuh"
 
 namespace wg {
@@ -548,6 +550,90 @@ __global__ void k_combine(CombineArgs a, int VPR) {
   }
 }
 
+// ---------------------------------------------------------------------------
+// Overfill gTasks ("a separate GPU kernel that
+// increases thread blocks and shared memory size", run with higher
+// priority): every destination row longer than E_max (its SPLIT chunks) is
+// reduced by one thread-block CLUSTER of HC CTAs.  Each CTA sums an equal
+// share of the row's edges (8 warps, fixed order) into shared memory; after a
+// cluster barrier the leader CTA adds the HC partial rows through distributed
+// shared memory in rank order and applies the epilogue -- no global fp32
+// scratch, no combine launch, deterministic.
+constexpr int HC = 8;                      // CTAs per heavy row (portable cluster size)
+template <typename T>
+__global__ void __launch_bounds__(WARPS * 32) k_agg_heavy(AggArgs a, const SplitRow* rows, int VPR) {
+  namespace cg = cooperative_groups;
+  cg::cluster_group cl = cg::this_cluster();
+  constexpr int EPV = VT<T>::EPV;
+  extern __shared__ __align__(16) float hsm[];            // [WARPS][VPR*EPV] then [VPR*EPV] (CTA total)
+  const int rank = (int)cl.block_rank();
+  const SplitRow sr = rows[blockIdx.x / HC];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int Fp = VPR * EPV;
+  float* cta = hsm + WARPS * Fp;
+  const int64_t eb = a.row_ptr[sr.row], ee = a.row_ptr[sr.row + 1], len = ee - eb;
+  // this CTA's share, then this warp's share of it (fixed partition of the row)
+  const int64_t cb = eb + len * rank / HC, ce = eb + len * (rank + 1) / HC;
+  const int64_t wb = cb + (ce - cb) * warp / WARPS, we = cb + (ce - cb) * (warp + 1) / WARPS;
+  const T* tab = static_cast<const T*>(a.table);
+  for (int v0 = 0; v0 < VPR; v0 += 32) {
+    const int vi = v0 + lane;
+    float acc[EPV];
+#pragma unroll
+    for (int i = 0; i < EPV; ++i) acc[i] = 0.f;
+    int64_t e = wb;
+    for (; e + 4 <= we; e += 4) {                          // 4 rows in flight per lane
+      int4 v[4];
+      float sc[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int s = a.idx[e + u];
+        sc[u] = a.gscale ? a.gscale[s] : (a.escale ? a.escale[e + u] : 1.f);
+        v[u] = vi < VPR ? ldg16(tab + (int64_t)s * a.ld_tab + vi * EPV) : make_int4(0, 0, 0, 0);
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) VT<T>::add(acc, v[u], sc[u]);
+    }
+    for (; e < we; ++e) {
+      const int s = a.idx[e];
+      const float sc = a.gscale ? a.gscale[s] : (a.escale ? a.escale[e] : 1.f);
+      if (vi < VPR) VT<T>::add(acc, ldg16(tab + (int64_t)s * a.ld_tab + vi * EPV), sc);
+    }
+    if (vi < VPR) {
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) hsm[warp * Fp + vi * EPV + i] = acc[i];
+    }
+  }
+  __syncthreads();
+  for (int c = threadIdx.x; c < Fp; c += blockDim.x) {     // CTA partial: warps in order
+    float t = 0.f;
+    for (int w = 0; w < WARPS; ++w) t += hsm[w * Fp + c];
+    cta[c] = t;
+  }
+  cl.sync();                                               // every CTA's partial is visible cluster-wide
+  if (rank == 0) {
+    for (int vi = threadIdx.x; vi < VPR; vi += blockDim.x) {
+      float t[EPV];
+#pragma unroll
+      for (int i = 0; i < EPV; ++i) t[i] = 0.f;
+      for (int r = 0; r < HC; ++r) {                       // ranks in order (deterministic)
+        const float* peer = cl.map_shared_rank(cta, r);
+#pragma unroll
+        for (int i = 0; i < EPV; ++i) t[i] += peer[vi * EPV + i];
+      }
+      const float rs = a.rscale ? a.rscale[a.row_base + sr.row] : 1.f;
+      epilogue_store<T>(t, sr.row, vi * EPV, rs, a.self_tab, a.ld_self, a.self_coef, a.bias, a.relu, a.mask_ref,
+                        a.ld_mask, a.out, a.ld_out, a.F);
+    }
+    if (a.zero_out) {
+      T* p = static_cast<T*>(a.zero_out) + (int64_t)sr.row * a.ld_zero;
+      for (int c = threadIdx.x * EPV; c < a.zero_cols; c += blockDim.x * EPV)
+        *reinterpret_cast<int4*>(p + c) = make_int4(0, 0, 0, 0);
+    }
+  }
+  cl.sync();                                               // peers keep their smem until the leader has read it
+}
+
 template <typename T, int LPE, int NV, int U>
 wg_status launch_cfg(const AggArgs& a, int VPR, cudaStream_t s) {
   constexpr int EPV = VT<T>::EPV;
@@ -656,6 +742,96 @@ wg_status launch_combine(wg_dtype dt, const CombineArgs& a, cudaStream_t s) {
   ProfScope ps(PK_COMBINE, s, (double)a.n_rows * a.F * (EPV == 8 ? 2 : 4), 0.0);
   if (dt == WG_BF16) WG_LAUNCH(k_combine<__nv_bfloat16>, a.n_rows, 128, 0, s, a, VPR);
   else WG_LAUNCH(k_combine<float>, a.n_rows, 128, 0, s, a, VPR);
+  return WG_OK;
+}
+
+// Differentiated outlier scheduling: the regular work items
+// and the overfill rows (deg > E_max) run as two kernels -- the cluster
+// kernel on a high-priority side stream ("increasing the priority of
+// execution for overfill gTasks"), the regular gather on the caller's
+// stream -- joined by events (CUDA-graph capturable).  `n_split_items`
+// leading items of `a` are the SPLIT chunks the partial path would run.
+// WG_HEAVY=0 selects the partial path (SPLIT items + k_combine).
+namespace {
+struct HeavyStreams {
+  int device = -1;
+  cudaStream_t hs = nullptr;
+  cudaEvent_t fork = nullptr, join = nullptr;
+};
+HeavyStreams& heavy_streams() {
+  static thread_local HeavyStreams h;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (h.device != dev) {
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    cudaStreamCreateWithPriority(&h.hs, cudaStreamNonBlocking, hi);
+    cudaEventCreateWithFlags(&h.fork, cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&h.join, cudaEventDisableTiming);
+    h.device = dev;
+  }
+  return h;
+}
+bool heavy_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("WG_HEAVY");
+    v = (e && e[0] == '0') ? 0 : 1;
+  }
+  return v == 1;
+}
+template <typename T>
+wg_status launch_heavy_t(const AggArgs& a, const SplitRow* rows, int n_rows, cudaStream_t s) {
+  constexpr int EPV = VT<T>::EPV;
+  const int VPR = (int)cdiv(a.F, EPV);
+  const size_t smem = sizeof(float) * (size_t)(WARPS + 1) * VPR * EPV;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_agg_heavy<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    attr = true;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(n_rows * HC));
+  cfg.blockDim = dim3(WARPS * 32);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = HC; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, k_agg_heavy<T>, a, rows, VPR);
+  ++launch_counter();
+  if (e != cudaSuccess) {
+    set_error(std::string("launch k_agg_heavy: ") + cudaGetErrorString(e));
+    return WG_ERR_CUDA;
+  }
+  return WG_OK;
+}
+}  // namespace
+
+wg_status launch_agg_outliers(wg_dtype dt, const AggArgs& a, int n_split_items, const SplitRow* split_rows,
+                              int n_split_rows, const CombineArgs& comb, cudaStream_t s) {
+  if (!heavy_enabled() || n_split_rows == 0 || a.F > 64 * (dt == WG_BF16 ? 8 : 4)) {
+    WG_TRY(launch_agg(dt, a, s));
+    return launch_combine(dt, comb, s);
+  }
+  HeavyStreams& h = heavy_streams();
+  WG_CK(cudaEventRecord(h.fork, s));
+  WG_CK(cudaStreamWaitEvent(h.hs, h.fork, 0));
+  {
+    int64_t he = 0;
+    ProfScope ps(PK_COMBINE, h.hs, 0.0, 0.0);
+    WG_TRY(dt == WG_BF16 ? launch_heavy_t<__nv_bfloat16>(a, split_rows, n_split_rows, h.hs)
+                         : launch_heavy_t<float>(a, split_rows, n_split_rows, h.hs));
+    (void)he;
+  }
+  AggArgs r = a;
+  r.items = a.items + n_split_items;
+  r.n_items = a.n_items - n_split_items;
+  if (r.n_items > 0) WG_TRY(launch_agg(dt, r, s));
+  WG_CK(cudaEventRecord(h.join, h.hs));
+  WG_CK(cudaStreamWaitEvent(s, h.join, 0));
   return WG_OK;
 }
 

@@ -126,9 +126,7 @@ CombineArgs comb_from(const AggArgs& a, const ItemList& L, int plan_filter) {
 }
 
 wg_status run_agg(const Ctx& c, AggArgs a, const ItemList& L, cudaStream_t st) {
-  WG_TRY(launch_agg(c.dt, a, st));
-  WG_TRY(launch_combine(c.dt, comb_from(a, L, -1), st));
-  return WG_OK;
+  return launch_agg_outliers(c.dt, a, L.n_split_items, L.split, L.n_split, comb_from(a, L, -1), st);
 }
 
 // Gather over an exchange table in layout X (chunk k = [V x Fc] at k * V * Fc

@@ -90,11 +90,46 @@ void build_items(const wg_graph_s* g, const Side& S, const std::vector<uint8_t>*
     ti = tj;
   }
   ItemList* outs[2] = {out0, out1};
+  // Underfill gTasks: a run of adjacent small work
+  // items (each < UNDER edges) is merged into one item of <= CAP edges --
+  // one CTA walks the run edge-wise across the gTask boundaries instead of
+  // one mostly idle CTA per gTask; merged items are the smallest, so they
+  // run last ("lower priority").  WG_UNDERFILL=0 disables.
+  static int merge = -1;
+  if (merge < 0) {
+    const char* e = getenv("WG_UNDERFILL");
+    merge = (e && e[0] == '0') ? 0 : 1;
+  }
+  constexpr int64_t UNDER = 256, CAP = 2048;
   for (int b = 0; b < 2; ++b) {
     auto& L = lists[b];
+    if (merge) {
+      std::vector<std::pair<int64_t, WorkItem>> m;
+      for (auto& e : L) {
+        const WorkItem& w = e.second;
+        const int64_t ne = w.e_hi - w.e_lo;
+        if (!m.empty() && w.split_slot < 0 && m.back().second.split_slot < 0 && ne < UNDER &&
+            m.back().first < CAP && m.back().second.row_hi == w.row_lo && m.back().first + ne <= CAP &&
+            (m.back().first < UNDER || m.back().second.task == -2)) {
+          WorkItem& p = m.back().second;
+          p.row_hi = w.row_hi;
+          p.e_hi = w.e_hi;
+          p.task = -2;                       // a merged run of gTasks
+          m.back().first += ne;
+          ++outs[b]->n_merged;
+        } else {
+          m.push_back(e);
+        }
+      }
+      L.swap(m);
+    }
     std::stable_sort(L.begin(), L.end(), [](const auto& x, const auto& y) { return x.first > y.first; });
     outs[b]->h.clear();
-    for (auto& e : L) outs[b]->h.push_back(e.second);
+    outs[b]->n_split_items = 0;
+    for (auto& e : L) {
+      outs[b]->h.push_back(e.second);
+      if (e.second.split_slot >= 0) ++outs[b]->n_split_items;
+    }
   }
   *n_slots = slot;
 }

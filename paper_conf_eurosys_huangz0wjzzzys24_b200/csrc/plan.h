@@ -31,6 +31,8 @@ struct ItemList {
   std::vector<WorkItem> h;
   std::vector<SplitRow> hs;
   int64_t n_edges = 0, n_rows = 0;   // totals (algorithmic-byte accounting)
+  int n_split_items = 0;             // leading items that are SPLIT chunks (heavy-first order)
+  int n_merged = 0;                  // underfill items merged into their neighbours
 };
 
 // Column-chunked layout of an exchange table:

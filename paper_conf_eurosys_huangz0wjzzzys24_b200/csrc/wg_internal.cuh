@@ -180,6 +180,10 @@ struct CombineArgs {
 
 wg_status launch_agg(wg_dtype dt, const AggArgs& a, cudaStream_t s);
 wg_status launch_combine(wg_dtype dt, const CombineArgs& a, cudaStream_t s);
+// regular items + overfill rows: a cluster kernel per heavy row on a
+// high-priority side stream (or, WG_HEAVY=0, SPLIT items + combine)
+wg_status launch_agg_outliers(wg_dtype dt, const AggArgs& a, int n_split_items, const SplitRow* split_rows,
+                              int n_split_rows, const CombineArgs& comb, cudaStream_t s);
 
 // GEMM: D[M x N] = sum_p A_p[M x K_p] * B_p[N x K_p]^T  (+ epilogue)
 struct GemmPart {
