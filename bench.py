@@ -70,6 +70,9 @@ def parse():
                     help="one GPU runs rank --slice-rank of a P-way 1-D partition (its in- / out-edges only, "
                          "collectives emulated): per-rank compute of a configuration too large for one GPU (C5)")
     ap.add_argument("--slice-rank", type=int, default=0)
+    ap.add_argument("--tune", action="store_true",
+                    help="choose (T, E_max) by the measured strategy search (tune.py; cached per configuration)")
+    ap.add_argument("--tune-cache", default=os.path.join(os.path.expanduser("~"), ".cache", "wg_tune.json"))
     ap.add_argument("--emulate-xchg", action="store_true",
                     help="--rank-slice: time every exchange as a copy kernel on the library's communication "
                          "stream (overlapped with the gathers as the NCCL exchange would be)")
@@ -425,9 +428,16 @@ def main():
         if world > 1:
             comm = wg.Comm(group, device=local)      # NCCL inside libwg (wg_comm_init)
     t_gen = time.perf_counter() - t0
+    R = c.R if model == "rgcn" else 1
+    if args.tune and P <= 1 and world == 1 and model != "gat":
+        from paper_conf_eurosys_huangz0wjzzzys24_b200 import tune
+        T_, Em, rep = tune.search(src, dst, c.V, model, c.dims, torch.bfloat16 if c.dtype == "bf16" else torch.float32,
+                                  etype=et if R > 1 else None, R=R, cache_path=args.tune_cache,
+                                  conv_kw=conv_options(c, model) if model != "gat" else {"heads": c.heads})
+        args.tile, args.emax = T_, Em
+        cfg["strategy_search"] = rep
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    R = c.R if model == "rgcn" else 1
     g = wg.Graph(torch.from_numpy(src).to(dev), torch.from_numpy(dst).to(dev), num_vertices=c.V,
                  etype=torch.from_numpy(et).to(dev) if R > 1 else None, num_types=R,
                  max_task_edges=args.emax, tile_rows=args.tile, comm=comm, bounds=bounds)
