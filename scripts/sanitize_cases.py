@@ -2,9 +2,10 @@
 compute-sanitizer (memcheck / racecheck / synccheck / initcheck):
 
   k_agg_cp (every ring shape: 4 / 8 / 16 / 32 lanes per row), k_agg,
-  k_combine (SPLIT rows), k_gemm_nt_p (bf16 and 3xTF32, split / chunked
+  k_combine and the overfill cluster kernel k_agg_heavy (SPLIT rows), k_gemm_nt_p (bf16 and 3xTF32, split / chunked
   outputs), k_tc_gemm (TN split-K), GAT edge kernels, RGCN stage kernels,
-  the softmax cross-entropy, the column-sum pass.
+  the softmax cross-entropy, the column-sum pass, the general restriction
+  engine (k_greedy, k_gagg), the SAGE-LSTM step kernels.
 
 Sizes are tiny (the sanitizers slow kernels down 10-100x) but span several
 tiles, a ragged tail and SPLIT chunks.  Usage:
@@ -29,6 +30,8 @@ def run(model, dtype, fi, fo, policy="auto", V=700, E=9000, E_max=64, heads=1, R
     g = m.Graph(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=V, max_task_edges=E_max,
                 **kw)
     ckw = dict(heads=heads, concat=concat) if model == "gat" else {}
+    if model == "sage_lstm":
+        policy = "auto"
     if model == "rgcn":
         ckw.update(norm="right", self_loop=True)
     conv = m.Conv(g, model, fi, fo, dtype=dtype, policy=policy, fuse_relu=True, **ckw)
@@ -76,6 +79,14 @@ def main():
         for ph in (1, 2):
             for (g, c, vb, ve), s in zip(parts, sv):
                 c.backward_raw(dy[vb:ve], x, y[vb:ve], s, params, dx=dx[vb:ve], phase=ph, xchg=xb)
+    torch.cuda.synchronize()
+    # general restriction engine + atomic executor, SAGE-LSTM
+    src, dst, et = synth.make_graph(800, 9000, seed=9, alpha=0.8, R=3)
+    for spec in ([("dst", 4)], [("src", 8), ("type", 1)], [("dst", 16), ("dst_degree", "min")], [("edge", 32)]):
+        gp = m.GPart(torch.from_numpy(src).cuda(), torch.from_numpy(dst).cuda(), num_vertices=800, restrictions=spec,
+                     etype=torch.from_numpy(et).cuda())
+        gp.aggregate(m.pad_to(torch.randn(800, 32, device="cuda").to(torch.bfloat16)), norm="both")
+    run("sage_lstm", torch.float32, 16, 8, "edge")
     torch.cuda.synchronize()
     # fused softmax cross-entropy
     lg = m.pad_to(torch.randn(3000, 47, device="cuda").to(torch.bfloat16))
