@@ -70,6 +70,8 @@ def parse():
                     help="one GPU runs rank --slice-rank of a P-way 1-D partition (its in- / out-edges only, "
                          "collectives emulated): per-rank compute of a configuration too large for one GPU (C5)")
     ap.add_argument("--slice-rank", type=int, default=0)
+    ap.add_argument("--hidden", type=int, default=0,
+                    help="replace the hidden widths of the config (a hidden-dimension sweep, Fig 20-style)")
     ap.add_argument("--tune", action="store_true",
                     help="choose (T, E_max) by the measured strategy search (tune.py; cached per configuration)")
     ap.add_argument("--tune-cache", default=os.path.join(os.path.expanduser("~"), ".cache", "wg_tune.json"))
@@ -89,9 +91,12 @@ def conv_options(c, model):
     return {}
 
 
-def workload(cfg_name, model):
+def workload(cfg_name, model, hidden=0):
+    import dataclasses
     import synth
     c = synth.CONFIGS[cfg_name]
+    if hidden:
+        c = dataclasses.replace(c, dims=(c.dims[0],) + (hidden,) * (len(c.dims) - 2) + (c.dims[-1],))
     model = model or c.model
     extra = {}
     if model == "gat":
@@ -328,7 +333,7 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    c, model, cfg = workload(args.config, args.model)
+    c, model, cfg = workload(args.config, args.model, args.hidden)
     src, dst, et, _, _ = make_inputs(c, model)
     vals = []
     per = max(2.0, 60.0 / max(1, args.steps + args.warmup))
@@ -375,7 +380,7 @@ def main():
     import paper_conf_eurosys_huangz0wjzzzys24_b200 as wg
     from paper_conf_eurosys_huangz0wjzzzys24_b200.stack import GNNStack, equal_blocks
 
-    c, model, cfg = workload(args.config, args.model)
+    c, model, cfg = workload(args.config, args.model, args.hidden)
     dev = torch.device("cuda", local)
     P = args.rank_slice
     if P > 1 and (world > 1 or model == "gat"):
