@@ -704,7 +704,8 @@ def main():
                            max_in_degree=int(g.max_in_degree), E_max=int(g.E_max),
                            plans=[{"edge_tasks": cv.n_edge_tasks, "vertex_tasks": cv.n_vertex_tasks,
                                    "bwd_path": cv.bwd_path, "items": cv.n_items, "items_T": cv.n_items_T,
-                                   "split_rows": cv.n_split_rows} for cv in stack.convs]),
+                                   "split_rows": cv.n_split_rows, "xchg_cols": [cv.xchg_fwd, cv.xchg_bwd]}
+                                  for cv in stack.convs]),
             "gpu_launches": int(launches), "roofline": roofline, "kernels": kernels,
             "step_time": step_stats, "per_layer": per_layer,
             "one_off": {"partition_s": t_part, "plan_s": t_plan, "synth_s": t_gen},
