@@ -116,7 +116,12 @@ struct GatArgs {
 };
 
 // ---------------------------------------------------------------- el / er
-template <typename T, int NV>
+// One warp per vertex row of G (fp32): el[v,h] = g[v, head h] . a_l[h],
+// er[v,h] = g[v, head h] . a_r[h].  a_l / a_r are read as float4 (one 16-byte
+// load per G vector); SEG > 0: heads are aligned groups of SEG lanes (Fo / 4,
+// a power of two <= 32), reduced by log2(SEG) xor-shuffles per vector, the
+// group's first lane stores; SEG == 0: generic head loop over the warp.
+template <typename T, int NV, int SEG>
 __global__ void k_gat_logits(int64_t V, GatArgs a, const float* al, const float* ar) {
   constexpr int EPV = GV<T>::EPV;
   const int lane = threadIdx.x & 31;
@@ -134,19 +139,41 @@ __global__ void k_gat_logits(int64_t V, GatArgs a, const float* al, const float*
       GV<T>::unpack(ld16(static_cast<const T*>(a.G) + v * a.ldg + vi * EPV), g);
       const int c0 = vi * EPV;
       hd[q] = c0 / a.Fo;
+      if (c0 + EPV <= a.HF) {
+        const float4 l4 = __ldg(reinterpret_cast<const float4*>(al + c0));
+        const float4 r4 = __ldg(reinterpret_cast<const float4*>(ar + c0));
+        pl[q] = g[0] * l4.x + g[1] * l4.y + g[2] * l4.z + g[3] * l4.w;
+        pr[q] = g[0] * r4.x + g[1] * r4.y + g[2] * r4.z + g[3] * r4.w;
+      } else {
 #pragma unroll
-      for (int i = 0; i < EPV; ++i) {
-        if (c0 + i < a.HF) { pl[q] += g[i] * al[c0 + i]; pr[q] += g[i] * ar[c0 + i]; }
+        for (int i = 0; i < EPV; ++i)
+          if (c0 + i < a.HF) { pl[q] += g[i] * al[c0 + i]; pr[q] += g[i] * ar[c0 + i]; }
       }
     }
   }
-  for (int h = 0; h < a.H; ++h) {
-    float sl = 0.f, sr = 0.f;
+  if constexpr (SEG > 0) {
 #pragma unroll
-    for (int q = 0; q < NV; ++q) if (hd[q] == h) { sl += pl[q]; sr += pr[q]; }
+    for (int q = 0; q < NV; ++q) {
+      float sl = pl[q], sr = pr[q];
 #pragma unroll
-    for (int o = 16; o; o >>= 1) { sl += __shfl_xor_sync(0xffffffffu, sl, o); sr += __shfl_xor_sync(0xffffffffu, sr, o); }
-    if (lane == 0) { const_cast<float*>(a.el)[v * a.H + h] = sl; const_cast<float*>(a.er)[v * a.H + h] = sr; }
+      for (int o = SEG / 2; o; o >>= 1) {
+        sl += __shfl_xor_sync(0xffffffffu, sl, o);
+        sr += __shfl_xor_sync(0xffffffffu, sr, o);
+      }
+      if ((lane & (SEG - 1)) == 0 && hd[q] >= 0 && hd[q] < a.H) {
+        const_cast<float*>(a.el)[v * a.H + hd[q]] = sl;
+        const_cast<float*>(a.er)[v * a.H + hd[q]] = sr;
+      }
+    }
+  } else {
+    for (int h = 0; h < a.H; ++h) {
+      float sl = 0.f, sr = 0.f;
+#pragma unroll
+      for (int q = 0; q < NV; ++q) if (hd[q] == h) { sl += pl[q]; sr += pr[q]; }
+#pragma unroll
+      for (int o = 16; o; o >>= 1) { sl += __shfl_xor_sync(0xffffffffu, sl, o); sr += __shfl_xor_sync(0xffffffffu, sr, o); }
+      if (lane == 0) { const_cast<float*>(a.el)[v * a.H + h] = sl; const_cast<float*>(a.er)[v * a.H + h] = sr; }
+    }
   }
 }
 
@@ -1043,9 +1070,22 @@ static wg_status gat_fwd_t(wg_plan_s* p, const wg_params* P, const wg_fwd_args* 
   ProfScope ps(PK_GAT, st,
                (double)g->fwd.E * (HF * 4.0 + 4.0 * H + 4) + (double)V * HF * 8.0 + (double)V * a.FO * s, 0.0);
   const unsigned wb = gs_grid(V * 32);
-  if (NV == 1) WG_LAUNCH((k_gat_logits<float, 1>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
-  else if (NV == 2) WG_LAUNCH((k_gat_logits<float, 2>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
-  else WG_LAUNCH((k_gat_logits<float, 4>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);
+  {
+    const int vph = d.f_out / 4;             // fp32 G vectors per head
+    const int SEG = (vph == 4 || vph == 8 || vph == 16 || vph == 32) ? vph : 0;
+#define WG_GAT_L(NV_)                                                                                      \
+  do {                                                                                                     \
+    if (SEG == 4) WG_LAUNCH((k_gat_logits<float, NV_, 4>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);    \
+    else if (SEG == 8) WG_LAUNCH((k_gat_logits<float, NV_, 8>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r); \
+    else if (SEG == 16) WG_LAUNCH((k_gat_logits<float, NV_, 16>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r); \
+    else if (SEG == 32) WG_LAUNCH((k_gat_logits<float, NV_, 32>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r); \
+    else WG_LAUNCH((k_gat_logits<float, NV_, 0>), wb, 256, 0, st, V, a, P->attn_l, P->attn_r);            \
+  } while (0)
+    if (NV == 1) WG_GAT_L(1);
+    else if (NV == 2) WG_GAT_L(2);
+    else WG_GAT_L(4);
+#undef WG_GAT_L
+  }
   a.idx = g->fwd.idx;
   a.chunks = gp->fwd; a.n_chunks = gp->n_fwd;
   if (gp->n_fwd) {
