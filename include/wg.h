@@ -158,7 +158,8 @@ wg_status wg_plan_export(wg_plan p, uint8_t* per_task_plan, int64_t stats[8]);
  * gTask VERTEX: x[src] of each (source, relation) row, grouped by relation,
  * gathered once by the forward for the Y GEMM and reused by the dW_r GEMM,
  * SURVEY §8(a) a5 / a11).  WG_ERR_INVALID if the plan has no such
- * buffer.  Pitches are 32-byte padded rows in the conv dtype.              */
+ * buffer.  Row pitches: <= 32 / <= 64-byte rows padded to 32 / 64 bytes,
+ * longer rows to a multiple of 128 bytes (one L2 line), in the conv dtype. */
 wg_status wg_plan_buffer(wg_plan p, int which, const char* name, size_t* offset);
 wg_status wg_plan_destroy(wg_plan p);
 

@@ -46,9 +46,14 @@ def _dt(dtype):
 
 
 def pitch(F: int, dtype) -> int:
-    """Row pitch (elements): rows padded to 32 bytes (one DRAM sector)."""
+    """Row pitch (elements) of a table the gathers read: rows of <= 32 / <= 64
+    bytes padded to 32 / 64 bytes, longer rows to a multiple of 128 bytes, so
+    a row touches the fewest 128-byte L2 lines -- random row gathers are
+    bound by line accesses (profiles/r02/gran_probe.md)."""
     s = torch.empty((), dtype=dtype).element_size()
-    return -(-F * s // 32) * 32 // s
+    b = F * s
+    q = 32 if b <= 32 else 64 if b <= 64 else 128
+    return -(-b // q) * q // s
 
 
 def padded(rows: int, F: int, dtype, device="cuda", zero=True):

@@ -64,8 +64,14 @@ struct ProfScope {
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 static inline int64_t rup(int64_t a, int64_t b) { return cdiv(a, b) * b; }
 static inline int dsize(wg_dtype t) { return t == WG_BF16 ? 2 : 4; }
-// row pitch in elements: rows padded to 32 bytes (sector size)
-static inline int64_t pitch(int64_t F, wg_dtype t) { return rup(F * dsize(t), 32) / dsize(t); }
+// row pitch in elements of a table the gathers read: <= 32 / <= 64-byte rows
+// padded to 32 / 64 bytes, longer rows to a multiple of 128 bytes, so a row
+// touches the fewest 128-byte L2 lines (random row gathers are bound by line
+// accesses: DESIGN.md §5, profiles/r02/gran_probe.md)
+static inline int64_t pitch(int64_t F, wg_dtype t) {
+  const int64_t b = F * dsize(t);
+  return rup(b, b <= 32 ? 32 : b <= 64 ? 64 : 128) / dsize(t);
+}
 
 // ------------------------------------------------------------ work items
 // A work item is the unit a CTA executes: the rows of one gTask (plus the
