@@ -559,7 +559,7 @@ __global__ void k_combine(CombineArgs a, int VPR) {
 // cluster barrier the leader CTA adds the HC partial rows through distributed
 // shared memory in rank order and applies the epilogue -- no global fp32
 // scratch, no combine launch, deterministic.
-constexpr int HC = 8;                      // CTAs per heavy row (portable cluster size)
+constexpr int HC = 16;                     // CTAs per heavy row (non-portable cluster size, opted in)
 template <typename T>
 __global__ void __launch_bounds__(WARPS * 32) k_agg_heavy(AggArgs a, const SplitRow* rows, int VPR) {
   namespace cg = cooperative_groups;
@@ -582,17 +582,21 @@ __global__ void __launch_bounds__(WARPS * 32) k_agg_heavy(AggArgs a, const Split
 #pragma unroll
     for (int i = 0; i < EPV; ++i) acc[i] = 0.f;
     int64_t e = wb;
-    for (; e + 4 <= we; e += 4) {                          // 4 rows in flight per lane
-      int4 v[4];
-      float sc[4];
+    constexpr int UH = 8;                                  // rows in flight per lane
+    for (; e + UH <= we; e += UH) {
+      int4 v[UH];
+      float sc[UH];
+      int sidx[UH];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int s = a.idx[e + u];
+      for (int u = 0; u < UH; ++u) sidx[u] = a.idx[e + u];
+#pragma unroll
+      for (int u = 0; u < UH; ++u) {
+        const int s = sidx[u];
         sc[u] = a.gscale ? a.gscale[s] : (a.escale ? a.escale[e + u] : 1.f);
         v[u] = vi < VPR ? ldg16(tab + (int64_t)s * a.ld_tab + vi * EPV) : make_int4(0, 0, 0, 0);
       }
 #pragma unroll
-      for (int u = 0; u < 4; ++u) VT<T>::add(acc, v[u], sc[u]);
+      for (int u = 0; u < UH; ++u) VT<T>::add(acc, v[u], sc[u]);
     }
     for (; e < we; ++e) {
       const int s = a.idx[e];
@@ -788,6 +792,7 @@ wg_status launch_heavy_t(const AggArgs& a, const SplitRow* rows, int n_rows, cud
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(k_agg_heavy<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    cudaFuncSetAttribute(k_agg_heavy<T>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     attr = true;
   }
   cudaLaunchConfig_t cfg = {};
