@@ -608,12 +608,14 @@ __global__ void __launch_bounds__(WARPS * 32) k_agg_heavy(AggArgs a, const Split
       for (int i = 0; i < EPV; ++i) hsm[warp * Fp + vi * EPV + i] = acc[i];
     }
   }
+  __syncwarp();                                            // reconverge before the block barrier
   __syncthreads();
   for (int c = threadIdx.x; c < Fp; c += blockDim.x) {     // CTA partial: warps in order
     float t = 0.f;
     for (int w = 0; w < WARPS; ++w) t += hsm[w * Fp + c];
     cta[c] = t;
   }
+  __syncwarp();
   cl.sync();                                               // every CTA's partial is visible cluster-wide
   if (rank == 0) {
     for (int vi = threadIdx.x; vi < VPR; vi += blockDim.x) {
@@ -635,6 +637,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_agg_heavy(AggArgs a, const Split
         *reinterpret_cast<int4*>(p + c) = make_int4(0, 0, 0, 0);
     }
   }
+  __syncwarp();
   cl.sync();                                               // peers keep their smem until the leader has read it
 }
 
@@ -817,7 +820,11 @@ wg_status launch_heavy_t(const AggArgs& a, const SplitRow* rows, int n_rows, cud
 
 wg_status launch_agg_outliers(wg_dtype dt, const AggArgs& a, int n_split_items, const SplitRow* split_rows,
                               int n_split_rows, const CombineArgs& comb, cudaStream_t s) {
-  if (!heavy_enabled() || n_split_rows == 0 || a.F > 64 * (dt == WG_BF16 ? 8 : 4)) {
+  // the cluster kernel pays off for a few very long rows (it overlaps the
+  // regular items); many moderately long rows run better as SPLIT items
+  // spread over all SMs (profiles/r02/outlier_breakdown.md: C4 with E_max =
+  // 512, 1497 heavy rows, partials 10.96 ms vs clusters 11.90 ms)
+  if (!heavy_enabled() || n_split_rows == 0 || n_split_rows > 64 || a.F > 64 * (dt == WG_BF16 ? 8 : 4)) {
     WG_TRY(launch_agg(dt, a, s));
     return launch_combine(dt, comb, s);
   }
