@@ -81,6 +81,7 @@ struct P2 {
   int relu, has_add, has_mask, bias_vec;
   int cpg;          // fp32 row-gathered A by per-lane cp.async (see the producer)
   int fc_d, fc_d2;  // columns per chunk of the (column-chunked) D / D2 output maps
+  int bres;         // B resident: every k-block of B loaded once per CTA (one N tile, no grouped B)
   const void* a_tab; int64_t lda_tab; int k_a;   // cpg: table, its row pitch (elements), K
 };
 
@@ -235,18 +236,22 @@ template <> __device__ __forceinline__ int4 pack16<float>(const float* f) {
 
 // shared-memory plan (bytes from the 1024-aligned base), identical on host and device
 struct SmemPlan {
-  int stage, ring, stg, add, mask, ids, bars, total;
+  int stage, ring, bres, stg, add, mask, ids, bars, total;
 };
-__host__ __device__ inline SmemPlan smem_plan(bool tf32, int BN, int S, bool has_add, bool has_mask, bool cpg) {
+// bres_kb > 0: B resident (bf16 only) -- the ring holds A only and the
+// bres_kb k-blocks of B (BN rows x 128 B each) sit after it for the whole kernel
+__host__ __device__ inline SmemPlan smem_plan(bool tf32, int BN, int S, bool has_add, bool has_mask, bool cpg,
+                                              int bres_kb = 0) {
   SmemPlan q;
-  q.stage = (A_STAGE + BN * 128) * (tf32 ? 2 : 1);   // [A | B] (+ [A_lo | B_lo])
+  q.stage = bres_kb ? A_STAGE : (A_STAGE + BN * 128) * (tf32 ? 2 : 1);   // [A | B] (+ [A_lo | B_lo])
   q.ring = S * q.stage;
-  q.stg = q.ring;
+  q.bres = q.ring;
+  q.stg = q.ring + bres_kb * BN * 128;
   q.add = q.stg + 2 * CHUNK_BYTES;
   q.mask = q.add + (has_add ? 2 * CHUNK_BYTES : 0);
   q.ids = q.mask + (has_mask ? 2 * CHUNK_BYTES : 0);
   q.bars = q.ids + (cpg ? BM * 4 : 0);               // cpg: the tile's 128 gather row ids
-  q.total = q.bars + 256;
+  q.total = q.bars + 512;
   return q;
 }
 
@@ -266,21 +271,24 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int BN = p.BN, S = p.stages;
   const int b_bytes = BN * 128;
-  const SmemPlan L = smem_plan(C::TF32, BN, S, p.has_add, p.has_mask, p.cpg != 0);
+  int total_kb0 = 0;
+  for (int i = 0; i < p.nparts; ++i) total_kb0 += p.kblocks[i];
+  const SmemPlan L = smem_plan(C::TF32, BN, S, p.has_add, p.has_mask, p.cpg != 0, p.bres ? total_kb0 : 0);
   // stage s: A at s*stage, B at +A_STAGE; fp32: A_lo at +A_STAGE+b_bytes, B_lo after it
   uint8_t* ring = smem;
   uint8_t* st_sm = smem + L.stg;                   // 2 x 16 KB output staging
   uint8_t* ad_sm = smem + L.add;                   // 2 x 16 KB addend
   uint8_t* mk_sm = smem + L.mask;                  // 2 x 16 KB mask
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
-  uint64_t* full = bars;            // [4] TMA landed
-  uint64_t* empty = bars + 4;       // [4] MMA done with the stage
-  uint64_t* tfull = bars + 8;       // [2]
-  uint64_t* tempty = bars + 10;     // [2]
-  uint64_t* efull = bars + 12;      // [2]
-  uint64_t* eempty = bars + 14;     // [2]
-  uint64_t* conv = bars + 16;       // [4] fp32: hi / lo split done
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 20);
+  uint64_t* full = bars;            // [8] TMA landed
+  uint64_t* empty = bars + 8;       // [8] MMA done with the stage
+  uint64_t* tfull = bars + 16;      // [2]
+  uint64_t* tempty = bars + 18;     // [2]
+  uint64_t* efull = bars + 20;      // [2]
+  uint64_t* eempty = bars + 22;     // [2]
+  uint64_t* conv = bars + 24;       // [8] fp32: hi / lo split done
+  uint64_t* bfull = bars + 32;      // resident B landed
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 33);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nchunk = (BN + C::CHE - 1) / C::CHE;
 
@@ -290,6 +298,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
       mbar_init(su32(&empty[s]), 1);
       mbar_init(su32(&conv[s]), 128);
     }
+    mbar_init(su32(bfull), 1);
     for (int b = 0; b < 2; ++b) {
       mbar_init(su32(&tfull[b]), 1);
       mbar_init(su32(&tempty[b]), 256);
@@ -312,9 +321,18 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
   if (warp == 0) {
     // ------------------------------------------------ TMA producer (lane 0;
     // row-gathered A parts: every lane issues the gather4 of its 4 tile rows)
-    const uint32_t tx = A_STAGE + b_bytes;
+    const uint32_t tx = p.bres ? (uint32_t)A_STAGE : (uint32_t)(A_STAGE + b_bytes);
     int s = 0;
     uint32_t ph = 0;
+    if (p.bres && lane == 0 && blockIdx.x < p.num_tiles) {   // every k-block of B, once
+      mbar_expect_tx(su32(bfull), (uint32_t)(total_kb0 * b_bytes));
+      int kb = 0;
+      for (int part = 0; part < p.nparts; ++part) {
+        const CUtensorMap* tb = part == 0 ? &tB0 : (part == 1 ? &tB1 : &tB2);
+        for (int kk = 0; kk < p.kblocks[part]; ++kk, ++kb)
+          tma_load(su32(smem + L.bres + kb * b_bytes), tb, kk * C::BKE, 0, su32(bfull));
+      }
+    }
     // the next tile's gather row ids and relation are loaded one tile ahead,
     // so their latency never stalls the producer between tiles
     auto tile_meta = [&](int64_t t, int4& gi, int& grp) {
@@ -374,7 +392,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
         } else if (lane == 0) {
           tma_load(su32(st), ta, kk * C::BKE, m0, su32(&full[s]));
         }
-        if (lane == 0) tma_load(su32(st + A_STAGE), tb, kk * C::BKE, brow, su32(&full[s]));
+        if (lane == 0 && !p.bres) tma_load(su32(st + A_STAGE), tb, kk * C::BKE, brow, su32(&full[s]));
         if (++kk == p.kblocks[part]) {
           kk = 0;
           ++part;
@@ -396,6 +414,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
       int s = 0;
       uint32_t ph = 0;
       int j = 0;
+      if (p.bres && blockIdx.x < p.num_tiles) mbar_wait(su32(bfull), 0);
       for (int64_t t = blockIdx.x; t < p.num_tiles; t += gridDim.x, ++j) {
         const int buf = j & 1;
         mbar_wait(su32(&tempty[buf]), ((j >> 1) & 1) ^ 1);
@@ -404,7 +423,8 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
         for (int kb = 0; kb < total_kb; ++kb) {
           mbar_wait(su32(C::TF32 ? &conv[s] : &full[s]), ph);
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          const uint32_t ad = su32(ring + s * L.stage), bd = ad + A_STAGE;
+          const uint32_t ad = su32(ring + s * L.stage);
+          const uint32_t bd = p.bres ? su32(smem + L.bres + kb * b_bytes) : ad + A_STAGE;
 #pragma unroll
           for (int k = 0; k < 4; ++k) {     // 4 MMAs of 32 bytes of K (16 bf16 / 8 tf32)
             const uint32_t on = (kb | k) != 0 ? 1u : 0u;
@@ -678,9 +698,33 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
   p.bias_vec = (reinterpret_cast<uintptr_t>(epi.bias) & 15) == 0;
   p.relu = epi.relu;
   const int limit = 227 * 1024 - 1024;
+  // B resident (bf16, one N tile, no grouped B): B is read from L2 once per
+  // CTA instead of once per tile, and the ring carries A only -- the HBM-bound
+  // skinny-K GEMMs of the gTask layer then keep A, not B, in flight.  Needs
+  // room for >= 3 A stages next to it.  WG_NT_BRES=0 disables.
+  static int bres_env = -1;
+  if (bres_env < 0) {
+    const char* e = getenv("WG_NT_BRES");
+    bres_env = (e && e[0] == '0') ? 0 : 1;
+  }
+  int total_kb = 0;
+  bool grouped = false;
+  for (int i = 0; i < n_parts; ++i) { total_kb += p.kblocks[i]; grouped = grouped || parts[i].tile_group; }
   int stages = 4;
-  while (stages > 2 && smem_plan(f32, BN, stages, p.has_add, p.has_mask, p.cpg).total > limit) --stages;
-  if (smem_plan(f32, BN, stages, p.has_add, p.has_mask, p.cpg).total > limit) return false;
+  p.bres = 0;
+  if (bres_env && !f32 && n_tiles == 1 && !grouped && !p.cpg) {
+    int st2 = 8;
+    while (st2 > 3 && smem_plan(f32, BN, st2, p.has_add, p.has_mask, false, total_kb).total > limit) --st2;
+    if (smem_plan(f32, BN, st2, p.has_add, p.has_mask, false, total_kb).total <= limit) {
+      p.bres = 1;
+      stages = st2;
+    }
+  }
+  const int bkb = p.bres ? total_kb : 0;
+  if (!p.bres) {
+    while (stages > 2 && smem_plan(f32, BN, stages, p.has_add, p.has_mask, p.cpg).total > limit) --stages;
+    if (smem_plan(f32, BN, stages, p.has_add, p.has_mask, p.cpg).total > limit) return false;
+  }
   p.stages = stages;
   if (!g_sms) {
     int dev = 0;
@@ -688,7 +732,7 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
     cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
   }
   const unsigned grid = (unsigned)std::min<int64_t>(p.num_tiles, g_sms);
-  const size_t smem = 1024 + (size_t)smem_plan(f32, BN, stages, p.has_add, p.has_mask, p.cpg).total;
+  const size_t smem = 1024 + (size_t)smem_plan(f32, BN, stages, p.has_add, p.has_mask, p.cpg, bkb).total;
   double kt = 0;
   for (int i = 0; i < n_parts; ++i) kt += parts[i].K;
   ProfScope ps(PK_TC_NT, s, (double)M * (kt + N + (epi.addend ? N : 0) + (epi.mask_ref ? N : 0)) * es,
