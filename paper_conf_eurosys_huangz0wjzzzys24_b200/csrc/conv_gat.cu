@@ -1252,10 +1252,13 @@ static wg_status gat_fwd_t(wg_plan_s* p, const wg_params* P, const wg_fwd_args* 
   a.chunks = gp->fwd; a.n_chunks = gp->n_fwd;
   if (gp->n_fwd) {
     const unsigned cbk = gs_grid((int64_t)gp->n_fwd * 32);
+    // two row chunks per warp: 40 % fewer instructions on C2 but fewer rows in
+    // flight per SM (register limit) -- measured 306 vs 290 us per forward
+    // (profiles/r02/ncu_gat_C2.csv), so opt-in (WG_GAT_HALF=1)
     static int half = -1;
     if (half < 0) {
       const char* e = getenv("WG_GAT_HALF");
-      half = (e && e[0] == '0') ? 0 : 1;
+      half = (e && e[0] == '1') ? 1 : 0;
     }
     if (H <= 4 && NV <= 2 && half) {   // two row chunks per warp (half-warps)
       const unsigned hbk = gs_grid(cdiv((int64_t)gp->n_fwd, 2) * 32);
