@@ -491,11 +491,8 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
     for (int64_t t = blockIdx.x; t < p.num_tiles; t += gridDim.x, ++j) {
       const int m0 = (int)((t / p.n_tiles) * BM), n0 = (int)((t % p.n_tiles) * BN);
       const int buf = j & 1;
-      const bool second = p.n_split > 0 && n0 >= p.n_split;
-      const CUtensorMap* td = second ? &tD2 : &tD;
-      const int ncol0 = second ? n0 - p.n_split : n0;
       const int64_t m = (int64_t)m0 + r;
-      const float rs = (p.rscale && m < p.M && !second) ? p.rscale[m] : 1.f;   // D only
+      const float rs_d = (p.rscale && m < p.M) ? p.rscale[m] : 1.f;   // D only (not the split output D2)
       mbar_wait(su32(&tfull[buf]), (j >> 1) & 1);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       for (int c = 0; c < nchunk; ++c, ++g) {
@@ -510,6 +507,9 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
         if (et == 0) bulk_wait_read<0>();
         epi_bar(grp);
         const int nc0 = n0 + c * C::CHE;
+        // split output: a 128-byte chunk belongs to D or to D2 (n_split % CHE == 0)
+        const bool second = p.n_split > 0 && nc0 >= p.n_split;
+        const float rs = second ? 1.f : rs_d;
         // one 16-byte output unit (EPV columns) at a time; FULL: every column < N
         auto units = [&](auto full_t) {
           constexpr bool FULL = decltype(full_t)::value;
@@ -558,7 +558,8 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         epi_bar(grp);
         if (et == 0) {
-          const int col = ncol0 + c * C::CHE, fc = second ? p.fc_d2 : p.fc_d;
+          const CUtensorMap* td = second ? &tD2 : &tD;
+          const int col = second ? nc0 - p.n_split : nc0, fc = second ? p.fc_d2 : p.fc_d;
           tma_store3(td, col % fc, m0, col / fc, su32(stg));
           bulk_commit();
         }
@@ -624,7 +625,7 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
   const int bn_max = (bn_env >= 64 && bn_env <= 256 && bn_env % 64 == 0) ? bn_env : (f32 ? 128 : 256);
   const int n_tiles = (int)cdiv(N, bn_max);
   const int BN = n_tiles > 1 ? bn_max : (int)rup(N, 16);
-  if (epi.D2 && (epi.n_split % BN != 0)) return false;   // split must fall on a tile boundary
+  if (epi.D2 && (epi.n_split % che != 0)) return false;  // split must fall on a 128-byte chunk boundary
   CUtensorMap maps[10];
   memset(maps, 0, sizeof(maps));
   P2 p{};
