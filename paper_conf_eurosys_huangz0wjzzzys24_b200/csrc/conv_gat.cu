@@ -1258,11 +1258,13 @@ static wg_status gat_fwd_t(wg_plan_s* p, const wg_params* P, const wg_fwd_args* 
     static int half = -1;
     if (half < 0) {
       const char* e = getenv("WG_GAT_HALF");
-      half = (e && e[0] == '1') ? 1 : 0;
+      half = e ? atoi(e) : 0;
     }
     if (H <= 4 && NV <= 2 && half) {   // two row chunks per warp (half-warps)
       const unsigned hbk = gs_grid(cdiv((int64_t)gp->n_fwd, 2) * 32);
       if (NV == 1) WG_LAUNCH((k_gat_fwd3<float, T, 2, 4, 4>), hbk, 256, 0, st, a, vb);
+      else if (half == 2) WG_LAUNCH((k_gat_fwd3<float, T, 4, 1, 4, 3>), hbk, 256, 0, st, a, vb);
+      else if (half == 3) WG_LAUNCH((k_gat_fwd3<float, T, 4, 1, 4, 4>), hbk, 256, 0, st, a, vb);
       else WG_LAUNCH((k_gat_fwd3<float, T, 4, 2, 4>), hbk, 256, 0, st, a, vb);
     } else if (H <= 4) {
       if (NV == 1) WG_LAUNCH((k_gat_fwd2<float, T, 1, 8, 4>), cbk, 256, 0, st, a, vb);
