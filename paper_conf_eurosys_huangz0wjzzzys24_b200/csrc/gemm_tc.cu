@@ -27,6 +27,7 @@ namespace wg {
 namespace {
 
 constexpr int BM = 128, BK = 64;
+constexpr int TC_CONV = 256;            // 3xTF32 converter threads (warps 4..11)
 constexpr int A_STAGE = BM * BK * 2;   // 16 KB
 
 struct TcParams {
@@ -152,9 +153,29 @@ __device__ __forceinline__ void mbar_arrive1(uint32_t bar) {
 }
 
 // 3xTF32 split of one operand region: the lo parts of n16 16-byte units at
-// `base` go to `lo` (x itself is the hi operand, see tf32_split_stage)
+// `base` go to `lo` (x itself is the hi operand, see tf32_split_stage);
+// 4 units in flight per thread (the converters are the TN's critical stage:
+// ncu shows the MMA issuer waiting on them and the TMA producer on free slots)
 __device__ __forceinline__ void tf32_split_range(uint32_t base, uint32_t lo, int n16, int ct, int nct) {
-  for (int i = ct; i < n16; i += nct) {
+  int i = ct;
+  for (; i + 3 * nct < n16; i += 4 * nct) {
+    uint32_t v[4][4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(v[u][0]), "=r"(v[u][1]), "=r"(v[u][2]), "=r"(v[u][3])
+                   : "r"(base + (uint32_t)(i + u * nct) * 16u));
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      uint32_t l[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+        l[k] = __float_as_uint(__uint_as_float(v[u][k]) - __uint_as_float(v[u][k] & 0xffffe000u));
+      asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(lo + (uint32_t)(i + u * nct) * 16u), "r"(l[0]),
+                   "r"(l[1]), "r"(l[2]), "r"(l[3]) : "memory");
+    }
+  }
+  for (; i < n16; i += nct) {
     uint32_t v[4], l[4];
     asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3])
                  : "r"(base + (uint32_t)i * 16u));
@@ -209,11 +230,15 @@ __device__ __forceinline__ void tf32_split_stage(uint32_t base, int n16, int ct,
 }
 
 // MN: TN variant (both operands MN-major, fp32 partial output).  T = float:
-// 3xTF32 with four extra converter warps (threads 128..255) that split each
-// landed stage into hi (in place) and lo (twin buffer after the stage).
+// 3xTF32 with eight extra converter warps (threads 128..383) that split each
+// landed stage into hi (the landed fp32 itself: kind::tf32 reads its top 19
+// bits) and lo.  TN: lo goes to one of two separate lo buffers (released by
+// the MMA commit), so the TMA ring holds raw stages only -- up to 6 stages of
+// K rows in flight instead of 4 stages with in-stage lo twins (the fp32 dW_r
+// GEMM was bound by bytes in flight: 3.2-3.9 TB/s).
 // Stage depth: 128 / sizeof(T) K elements (one 128-byte swizzle row).
 template <bool MN, typename T>
-__global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
+__global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
     k_tc_gemm(const __grid_constant__ CUtensorMap tA0, const __grid_constant__ CUtensorMap tB0,
               const __grid_constant__ CUtensorMap tA1, const __grid_constant__ CUtensorMap tB1,
               const __grid_constant__ CUtensorMap tA2, const __grid_constant__ CUtensorMap tB2, TcParams p) {
@@ -224,14 +249,18 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int BN = p.BN, S = p.stages;
   const int b_stage = MN ? ((BN + CHE - 1) / CHE) * BKE * 128 : BN * 128;
-  const int stage = (A_STAGE + b_stage) * (TF32 ? 2 : 1);
+  constexpr bool LOBUF = TF32 && MN;            // lo in two separate buffers
+  const int raw = A_STAGE + b_stage;
+  const int stage = (TF32 && !MN) ? 2 * raw : raw;
   uint8_t* ring = smem;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(ring + S * stage);
-  uint64_t* full = bars;
-  uint64_t* empty = bars + 4;
-  uint64_t* conv = bars + 8;
-  uint64_t* accf = bars + 12;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 13);
+  uint8_t* lo_buf = ring + S * stage;           // LOBUF: [2][A_lo | B_lo]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(lo_buf + (LOBUF ? 2 * raw : 0));
+  uint64_t* full = bars;                        // [S <= 8]
+  uint64_t* empty = bars + 8;
+  uint64_t* conv = bars + 16;
+  uint64_t* lo_empty = bars + 24;               // [2]
+  uint64_t* accf = bars + 26;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 27);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   uint32_t tcols = 32;
   while ((int)tcols < BN) tcols <<= 1;
@@ -240,8 +269,10 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
     for (int s = 0; s < S; ++s) {
       mbar_init(smem_u32(&full[s]), 1);
       mbar_init(smem_u32(&empty[s]), 1);
-      mbar_init(smem_u32(&conv[s]), 128);
+      mbar_init(smem_u32(&conv[s]), TC_CONV);
     }
+    mbar_init(smem_u32(&lo_empty[0]), 1);
+    mbar_init(smem_u32(&lo_empty[1]), 1);
     mbar_init(smem_u32(accf), 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -308,7 +339,7 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
       mbar_wait(smem_u32(TF32 ? &conv[s] : &full[s]), ph);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE;
-      const uint32_t al = bd + b_stage, bl = al + A_STAGE;
+      const uint32_t al = LOBUF ? smem_u32(lo_buf + (kb & 1) * raw) : bd + b_stage, bl = al + A_STAGE;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {   // 4 MMAs of 32 bytes of K (16 bf16 / 8 tf32)
         // MN-major: LBO = next 128-byte MN chunk, SBO = next K atom (8 rows
@@ -328,6 +359,7 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
         }
       }
       umma_commit(smem_u32(&empty[s]));
+      if (LOBUF) umma_commit(smem_u32(&lo_empty[kb & 1]));
     }
     umma_commit(smem_u32(accf));
   } else if (TF32 && warp >= 4) {
@@ -338,12 +370,14 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 256 : 128, 1)
     for (int kb = 0; kb < total_kb; ++kb) {
       const int s = kb % S;
       mbar_wait(smem_u32(&full[s]), (kb / S) & 1);
-      if (MN) {   // [A | B | A_lo | B_lo]: split the loaded A chunks and B
-        const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE, al = bd + b_stage, bl = al + A_STAGE;
-        tf32_split_range(ad, al, a16, ct, 128);
-        tf32_split_range(bd, bl, b_stage / 16, ct, 128);
+      if (MN) {   // stage [A | B] -> lo buffer kb & 1 [A_lo | B_lo], once the MMAs of kb - 2 released it
+        mbar_wait(smem_u32(&lo_empty[kb & 1]), ((kb >> 1) & 1) ^ 1);
+        const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE;
+        const uint32_t al = smem_u32(lo_buf + (kb & 1) * raw), bl = al + A_STAGE;
+        tf32_split_range(ad, al, a16, ct, TC_CONV);
+        tf32_split_range(bd, bl, b_stage / 16, ct, TC_CONV);
       } else {
-        tf32_split_stage(smem_u32(ring + s * stage), n16, ct, 128);
+        tf32_split_stage(smem_u32(ring + s * stage), n16, ct, TC_CONV);
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       mbar_arrive1(smem_u32(&conv[s]));
@@ -471,7 +505,9 @@ bool tc_enabled() {
 size_t smem_bytes(bool mn, int BN, int stages, int es = 2) {
   const int che = 128 / es, bke = 128 / es;
   const int b_stage = mn ? ((BN + che - 1) / che) * bke * 128 : BN * 128;
-  return 1024 + (size_t)stages * (A_STAGE + b_stage) * (es == 4 ? 2 : 1) + 128;
+  const size_t raw = A_STAGE + b_stage;
+  if (es == 4 && mn) return 1024 + (size_t)stages * raw + 2 * raw + 256;   // raw ring + two lo buffers
+  return 1024 + (size_t)stages * raw * (es == 4 ? 2 : 1) + 256;
 }
 
 template <bool MN, typename T>
@@ -481,7 +517,7 @@ wg_status launch(dim3 grid, size_t smem, const CUtensorMap* maps, const TcParams
     cudaFuncSetAttribute(k_tc_gemm<MN, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr = true;
   }
-  WG_LAUNCH((k_tc_gemm<MN, T>), grid, sizeof(T) == 4 ? 256 : 128, smem, s, maps[0], maps[1], maps[2], maps[3], maps[4],
+  WG_LAUNCH((k_tc_gemm<MN, T>), grid, sizeof(T) == 4 ? 128 + TC_CONV : 128, smem, s, maps[0], maps[1], maps[2], maps[3], maps[4],
             maps[5], p);
   return WG_OK;
 }
@@ -571,7 +607,7 @@ bool tn_setup(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda, 
   if (!make_map_t(&t->maps[0], ty, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda * t->es, che, bke, swz)) return false;
   if (!make_map_t(&t->maps[1], ty, B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb * t->es, che, bke, swz)) return false;
   for (int i = 2; i < 6; ++i) t->maps[i] = t->maps[i & 1];
-  t->stages = 4;
+  t->stages = t->es == 4 ? 8 : 4;
   while (t->stages > 2 && smem_bytes(true, t->BN, t->stages, t->es) > 200 * 1024) --t->stages;
   t->smem = smem_bytes(true, t->BN, t->stages, t->es);
   return t->smem <= 227 * 1024;
