@@ -28,6 +28,7 @@ namespace {
 
 constexpr int BM = 128, BK = 64;
 constexpr int TC_CONV = 256;            // 3xTF32 converter threads (warps 4..11)
+constexpr int TC_LO = 3;                // TN 3xTF32: separate lo buffers
 constexpr int A_STAGE = BM * BK * 2;   // 16 KB
 
 struct TcParams {
@@ -232,10 +233,9 @@ __device__ __forceinline__ void tf32_split_stage(uint32_t base, int n16, int ct,
 // MN: TN variant (both operands MN-major, fp32 partial output).  T = float:
 // 3xTF32 with eight extra converter warps (threads 128..383) that split each
 // landed stage into hi (the landed fp32 itself: kind::tf32 reads its top 19
-// bits) and lo.  TN: lo goes to one of two separate lo buffers (released by
-// the MMA commit), so the TMA ring holds raw stages only -- up to 6 stages of
-// K rows in flight instead of 4 stages with in-stage lo twins (the fp32 dW_r
-// GEMM was bound by bytes in flight: 3.2-3.9 TB/s).
+// bits) and lo.  TN: lo goes to one of TC_LO separate lo buffers (released by
+// the MMA commit), so the TMA ring holds raw stages only (5 stages + 3 lo
+// buffers instead of 4 stages with in-stage lo twins).
 // Stage depth: 128 / sizeof(T) K elements (one 128-byte swizzle row).
 template <bool MN, typename T>
 __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
@@ -253,14 +253,14 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
   const int raw = A_STAGE + b_stage;
   const int stage = (TF32 && !MN) ? 2 * raw : raw;
   uint8_t* ring = smem;
-  uint8_t* lo_buf = ring + S * stage;           // LOBUF: [2][A_lo | B_lo]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(lo_buf + (LOBUF ? 2 * raw : 0));
+  uint8_t* lo_buf = ring + S * stage;           // LOBUF: [TC_LO][A_lo | B_lo]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(lo_buf + (LOBUF ? TC_LO * raw : 0));
   uint64_t* full = bars;                        // [S <= 8]
   uint64_t* empty = bars + 8;
   uint64_t* conv = bars + 16;
-  uint64_t* lo_empty = bars + 24;               // [2]
-  uint64_t* accf = bars + 26;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 27);
+  uint64_t* lo_empty = bars + 24;               // [TC_LO <= 4]
+  uint64_t* accf = bars + 28;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 29);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   uint32_t tcols = 32;
   while ((int)tcols < BN) tcols <<= 1;
@@ -271,8 +271,7 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
       mbar_init(smem_u32(&empty[s]), 1);
       mbar_init(smem_u32(&conv[s]), TC_CONV);
     }
-    mbar_init(smem_u32(&lo_empty[0]), 1);
-    mbar_init(smem_u32(&lo_empty[1]), 1);
+    for (int j = 0; j < TC_LO; ++j) mbar_init(smem_u32(&lo_empty[j]), 1);
     mbar_init(smem_u32(accf), 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -339,7 +338,7 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
       mbar_wait(smem_u32(TF32 ? &conv[s] : &full[s]), ph);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE;
-      const uint32_t al = LOBUF ? smem_u32(lo_buf + (kb & 1) * raw) : bd + b_stage, bl = al + A_STAGE;
+      const uint32_t al = LOBUF ? smem_u32(lo_buf + (kb % TC_LO) * raw) : bd + b_stage, bl = al + A_STAGE;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {   // 4 MMAs of 32 bytes of K (16 bf16 / 8 tf32)
         // MN-major: LBO = next 128-byte MN chunk, SBO = next K atom (8 rows
@@ -359,7 +358,7 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
         }
       }
       umma_commit(smem_u32(&empty[s]));
-      if (LOBUF) umma_commit(smem_u32(&lo_empty[kb & 1]));
+      if (LOBUF) umma_commit(smem_u32(&lo_empty[kb % TC_LO]));
     }
     umma_commit(smem_u32(accf));
   } else if (TF32 && warp >= 4) {
@@ -370,10 +369,10 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
     for (int kb = 0; kb < total_kb; ++kb) {
       const int s = kb % S;
       mbar_wait(smem_u32(&full[s]), (kb / S) & 1);
-      if (MN) {   // stage [A | B] -> lo buffer kb & 1 [A_lo | B_lo], once the MMAs of kb - 2 released it
-        mbar_wait(smem_u32(&lo_empty[kb & 1]), ((kb >> 1) & 1) ^ 1);
+      if (MN) {   // stage [A | B] -> lo buffer kb % TC_LO [A_lo | B_lo], once the MMAs of kb - TC_LO released it
+        mbar_wait(smem_u32(&lo_empty[kb % TC_LO]), ((kb / TC_LO) & 1) ^ 1);
         const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE;
-        const uint32_t al = smem_u32(lo_buf + (kb & 1) * raw), bl = al + A_STAGE;
+        const uint32_t al = smem_u32(lo_buf + (kb % TC_LO) * raw), bl = al + A_STAGE;
         tf32_split_range(ad, al, a16, ct, TC_CONV);
         tf32_split_range(bd, bl, b_stage / 16, ct, TC_CONV);
       } else {
@@ -506,7 +505,7 @@ size_t smem_bytes(bool mn, int BN, int stages, int es = 2) {
   const int che = 128 / es, bke = 128 / es;
   const int b_stage = mn ? ((BN + che - 1) / che) * bke * 128 : BN * 128;
   const size_t raw = A_STAGE + b_stage;
-  if (es == 4 && mn) return 1024 + (size_t)stages * raw + 2 * raw + 256;   // raw ring + two lo buffers
+  if (es == 4 && mn) return 1024 + (size_t)stages * raw + TC_LO * raw + 256;   // raw ring + lo buffers
   return 1024 + (size_t)stages * raw * (es == 4 ? 2 : 1) + 256;
 }
 
