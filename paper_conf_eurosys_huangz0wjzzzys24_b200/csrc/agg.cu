@@ -930,29 +930,24 @@ __global__ void __launch_bounds__(256) k_colsum(int64_t M, int N, const T* dy, i
   }
 }
 
-// out[c] = sum_b part[b][c]: 32 columns per CTA, warp w sums blocks b = w mod 8
-// (4 loads in flight), then the 8 warp partials are added in warp order --
-// a fixed order, so the result is deterministic
-__global__ void __launch_bounds__(256) k_colsum_reduce(const float* part, int nblk, int N, float* out) {
-  __shared__ float red[8][33];
+// out[c] = sum_b part[b][c]: 32 columns per CTA, warp w of 32 sums blocks
+// b = w mod 32 (4 loads in flight), then the 32 warp partials are added in
+// warp order -- a fixed order, so the result is deterministic
+__global__ void __launch_bounds__(1024) k_colsum_reduce(const float* part, int nblk, int N, float* out) {
+  __shared__ float red[32][33];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int c = blockIdx.x * 32 + lane;
   float s = 0.f;
   if (c < N) {
-    int b = warp;
-    for (; b + 24 < nblk; b += 32) {
-      const float v0 = part[(int64_t)b * N + c], v1 = part[(int64_t)(b + 8) * N + c];
-      const float v2 = part[(int64_t)(b + 16) * N + c], v3 = part[(int64_t)(b + 24) * N + c];
-      s += v0; s += v1; s += v2; s += v3;
-    }
-    for (; b < nblk; b += 8) s += part[(int64_t)b * N + c];
+#pragma unroll 4
+    for (int b = warp; b < nblk; b += 32) s += part[(int64_t)b * N + c];
   }
   red[warp][lane] = s;
   __syncthreads();
   if (warp == 0 && c < N) {
     float t = 0.f;
 #pragma unroll
-    for (int w = 0; w < 8; ++w) t += red[w][lane];
+    for (int w = 0; w < 32; ++w) t += red[w][lane];
     out[c] = t;
   }
 }
@@ -1001,7 +996,7 @@ wg_status bias_grad_mask(wg_dtype dt, int64_t M, int N, const void* dy, int64_t 
   else
     WG_LAUNCH(k_colsum<float>, nblk, threads, smem, s, M, N, (const float*)dy, lddy, (const float*)ref, ldref,
               (float*)dt_out, ldt, scratch, rpb, rs2, (float*)dt2, ldt2, fc2, cs2);
-  if (db) WG_LAUNCH(k_colsum_reduce, (unsigned)cdiv(N, 32), 256, 0, s, scratch, nblk, N, db);
+  if (db) WG_LAUNCH(k_colsum_reduce, (unsigned)cdiv(N, 32), 1024, 0, s, scratch, nblk, N, db);
   return WG_OK;
 }
 

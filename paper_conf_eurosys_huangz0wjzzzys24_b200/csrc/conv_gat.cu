@@ -619,15 +619,15 @@ __global__ void __launch_bounds__(256) k_gat_fwd_combine(GatArgs a, const SplitR
     const float* p0 = a.part + (int64_t)sr.first_slot * a.part_ld;
     float M = -INFINITY;
     int k0 = 0;
-    for (; k0 + 4 <= sr.n_slots; k0 += 4) {      // 4 independent slot loads in flight
-      float lk[4], mk[4];
+    for (; k0 + 8 <= sr.n_slots; k0 += 8) {      // 8 independent slot loads in flight
+      float lk[8], mk[8];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
+      for (int j = 0; j < 8; ++j) {
         const float* pp = p0 + (int64_t)(k0 + j) * a.part_ld;
         lk[j] = pp[a.HF + a.H + h]; mk[j] = pp[a.HF + h];
       }
 #pragma unroll
-      for (int j = 0; j < 4; ++j) if (lk[j] > 0.f) M = fmaxf(M, mk[j]);
+      for (int j = 0; j < 8; ++j) if (lk[j] > 0.f) M = fmaxf(M, mk[j]);
     }
     for (; k0 < sr.n_slots; ++k0) {
       const float* pp = p0 + (int64_t)k0 * a.part_ld;
@@ -635,15 +635,15 @@ __global__ void __launch_bounds__(256) k_gat_fwd_combine(GatArgs a, const SplitR
     }
     float l = 0.f, o = 0.f;
     int k = 0;
-    for (; k + 4 <= sr.n_slots; k += 4) {
-      float lk[4], mk[4], ok[4];
+    for (; k + 8 <= sr.n_slots; k += 8) {
+      float lk[8], mk[8], ok[8];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
+      for (int j = 0; j < 8; ++j) {
         const float* pp = p0 + (int64_t)(k + j) * a.part_ld;
         lk[j] = pp[a.HF + a.H + h]; mk[j] = pp[a.HF + h]; ok[j] = pp[c];
       }
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
+      for (int j = 0; j < 8; ++j) {
         if (lk[j] <= 0.f) continue;
         const float sc = __expf(mk[j] - M);
         l += lk[j] * sc;
@@ -1029,7 +1029,8 @@ __global__ void k_gat_der_combine(const SplitRow* rows, int n, int64_t row_base,
   const SplitRow sr = rows[t / H];
   const int h = (int)(t % H);
   float s = 0.f;
-  for (int k = 0; k < sr.n_slots; ++k) s += part[(int64_t)(sr.first_slot + k) * part_ld + h];
+#pragma unroll 8
+  for (int k = 0; k < sr.n_slots; ++k) s += part[(int64_t)(sr.first_slot + k) * part_ld + h];   // 8 loads in flight
   der[(row_base + sr.row) * H + h] = s;
 }
 
@@ -1038,6 +1039,7 @@ __global__ void k_gat_bwd_combine(GatArgs a, const SplitRow* rows, int64_t row_b
   const int64_t u = row_base + sr.row;
   for (int c = threadIdx.x; c < a.HF + a.H; c += blockDim.x) {
     float s = 0.f;
+#pragma unroll 8
     for (int k = 0; k < sr.n_slots; ++k) s += a.part[(int64_t)(sr.first_slot + k) * a.part_ld + c];
     if (c < a.HF) a.dg[u * a.ld_dg + c] = s;
     else a.del[u * a.H + (c - a.HF)] = s;
@@ -1102,19 +1104,21 @@ __global__ void k_gat_dG(int64_t rows, int64_t row_base, GatArgs a, const float*
 
 // out0 / out1 = column sums of the [nblk x 2n] block partials (first / second
 // half): 32 columns per CTA, fixed-order warp split as k_colsum_reduce
-__global__ void __launch_bounds__(256) k_pair_reduce(const float* part, int nblk, int n, float* out0, float* out1) {
-  __shared__ float red[8][33];
+__global__ void __launch_bounds__(1024) k_pair_reduce(const float* part, int nblk, int n, float* out0, float* out1) {
+  __shared__ float red[32][33];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int c = blockIdx.x * 32 + lane;
   float s = 0.f;
-  if (c < 2 * n)
-    for (int b = warp; b < nblk; b += 8) s += part[(int64_t)b * 2 * n + c];
+  if (c < 2 * n) {
+#pragma unroll 4
+    for (int b = warp; b < nblk; b += 32) s += part[(int64_t)b * 2 * n + c];
+  }
   red[warp][lane] = s;
   __syncthreads();
   if (warp == 0 && c < 2 * n) {
     float t = 0.f;
 #pragma unroll
-    for (int w = 0; w < 8; ++w) t += red[w][lane];
+    for (int w = 0; w < 32; ++w) t += red[w][lane];
     if (c < n) { if (out0) out0[c] = t; }
     else if (out1) out1[c - n] = t;
   }
@@ -1392,7 +1396,7 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
   float* dgp = L.at<float>(ws, "dgp");
   WG_LAUNCH(k_gat_dG<T>, nblk, 256, 0, st, nr, vb, a, P->attn_l, P->attn_r, der, (T*)dG, (T*)dGlo, p->po, dgp,
             rpb);
-  WG_LAUNCH(k_pair_reduce, (unsigned)cdiv(2 * HF, 32), 256, 0, st, dgp, nblk, HF, Gr ? Gr->attn_l : nullptr,
+  WG_LAUNCH(k_pair_reduce, (unsigned)cdiv(2 * HF, 32), 1024, 0, st, dgp, nblk, HF, Gr ? Gr->attn_l : nullptr,
             Gr ? Gr->attn_r : nullptr);
   }
   // dW = x^T dG ; dx = dG W^T   (dG = hi + lo for bf16)

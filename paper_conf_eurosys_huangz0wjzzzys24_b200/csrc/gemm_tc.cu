@@ -455,7 +455,8 @@ __global__ void k_split_reduce_tc(const float* part, int splits, int64_t MN, flo
   int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= MN) return;
   float s = 0.f;
-  for (int z = 0; z < splits; ++z) s += part[z * MN + i];
+#pragma unroll 8
+  for (int z = 0; z < splits; ++z) s += part[z * MN + i];   // 8 loads in flight, split order
   D[i] = acc ? D[i] + s : s;
 }
 
@@ -655,6 +656,7 @@ __global__ void k_unit_reduce(const float* part, const int32_t* unit_off, int gr
   if (i >= MN * groups) return;
   const int64_t g = i / MN, e = i % MN;
   float s = 0.f;
+#pragma unroll 8
   for (int u = unit_off[g]; u < unit_off[g + 1]; ++u) s += part[(int64_t)u * MN + e];
   D[i] = s;
 }

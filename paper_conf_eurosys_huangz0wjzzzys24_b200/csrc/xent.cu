@@ -214,12 +214,15 @@ __global__ void __launch_bounds__(256) k_xent_vec(int64_t M, int C, const T* x, 
   }
 }
 
+// one warp: lane l sums part[l], part[l + 32], ... then a fixed xor tree
 __global__ void k_sum(const float* part, int n, float* out) {
-  if (threadIdx.x == 0 && blockIdx.x == 0) {
-    float t = 0.f;
-    for (int i = 0; i < n; ++i) t += part[i];
-    *out = t;
-  }
+  const int lane = threadIdx.x & 31;
+  float t = 0.f;
+#pragma unroll 4
+  for (int i = lane; i < n; i += 32) t += part[i];
+#pragma unroll
+  for (int o = 16; o; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+  if (lane == 0) *out = t;
 }
 
 template <typename T, int PER>
