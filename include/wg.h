@@ -377,6 +377,19 @@ wg_status wg_softmax_xent(wg_dtype dtype, int64_t M, int32_t C, const void* logi
                           const int64_t* labels, float scale, void* dlogits, int64_t ldd, float* loss_out,
                           void* scratch, wg_stream stream);
 
+/* Training-step utility: one Adam step (Kingma & Ba; the update torch.optim.Adam
+ * computes, no weight decay) over n fp32 values in one launch:
+ *   m = b1 m + (1-b1) g ; v = b2 v + (1-b2) g^2 ; t = state[0] + 1 ;
+ *   param -= lr / (1 - b1^t) * m / (sqrt(v) / sqrt(1 - b2^t) + eps).
+ * param / grad / exp_avg / exp_avg_sq: device, n floats each, 16-byte
+ * aligned, caller-owned (every parameter of a model in one flat buffer).
+ * state: device int32[2] owned by the caller, zeroed before the first step;
+ * state[0] = steps taken (advanced on the device by the launch, so a
+ * captured CUDA graph replays successive steps), state[1] internal.
+ * Concurrent calls must not share `state`.                                  */
+wg_status wg_adam_step(int64_t n, float* param, const float* grad, float* exp_avg, float* exp_avg_sq,
+                       int32_t* state, float lr, float beta1, float beta2, float eps, wg_stream stream);
+
 /* ------------------------------------------------------------------------ */
 const char* wg_status_string(wg_status s);
 const char* wg_last_error(void);

@@ -19,7 +19,7 @@ from . import _capi as C
 from ._capi import WGError, TASK_DTYPE
 
 __all__ = ["Graph", "Conv", "Comm", "GPart", "WGError", "TASK_DTYPE", "padded", "pad_to", "ld_of", "launch_count",
-           "init_params", "partition_1d"]
+           "init_params", "partition_1d", "Adam"]
 
 
 def _ptr(t):
@@ -96,6 +96,52 @@ def softmax_xent(logits: torch.Tensor, labels: torch.Tensor, scale: float, dlogi
     C.check(C.lib().wg_softmax_xent(_dt(logits.dtype), logits.shape[0], logits.shape[1], _ptr(logits), ld_of(logits),
                                     _ptr(labels), scale, _ptr(dlogits), ld_of(dlogits), _ptr(loss),
                                     _ptr(_xent_scratch[dev]), _stream(stream)), "wg_softmax_xent")
+
+
+class Adam:
+    """Adam over every parameter of a model in one flat fp32 buffer: one
+    wg_adam_step launch per step (torch.optim.Adam's update, no weight decay).
+    The parameter dicts' tensors are replaced by views of the flat buffer and
+    ``grads`` holds matching gradient views (what the conv backward writes).
+    The step count lives on the device, so a captured step replays real steps."""
+
+    ALIGN = 64          # floats: every tensor starts on a 256-byte boundary
+
+    def __init__(self, params: list, lr: float = 1e-3, betas=(0.9, 0.999), eps: float = 1e-8):
+        self.lr, self.betas, self.eps = float(lr), (float(betas[0]), float(betas[1])), float(eps)
+        ts = [t for p in params for t in p.values()]
+        if not ts:
+            raise ValueError("Adam: no parameters")
+        dev = ts[0].device
+        offs, o = [], 0
+        for t in ts:
+            if t.dtype != torch.float32:
+                raise ValueError("Adam: parameters must be fp32")
+            offs.append(o)
+            o += -(-t.numel() // self.ALIGN) * self.ALIGN
+        self.n = o
+        self.param = torch.zeros(o, dtype=torch.float32, device=dev)
+        self.grad = torch.zeros_like(self.param)
+        self.exp_avg = torch.zeros_like(self.param)
+        self.exp_avg_sq = torch.zeros_like(self.param)
+        self.state = torch.zeros(2, dtype=torch.int32, device=dev)
+        self.grads = []
+        i = 0
+        for p in params:
+            gd = {}
+            for k, t in list(p.items()):
+                a, n = offs[i], t.numel()
+                view = self.param[a:a + n].view(t.shape)
+                view.copy_(t.detach())
+                p[k] = view
+                gd[k] = self.grad[a:a + n].view(t.shape)
+                i += 1
+            self.grads.append(gd)
+
+    def step(self, stream=None):
+        C.check(C.lib().wg_adam_step(self.n, _ptr(self.param), _ptr(self.grad), _ptr(self.exp_avg),
+                                     _ptr(self.exp_avg_sq), _ptr(self.state), self.lr, self.betas[0],
+                                     self.betas[1], self.eps, _stream(stream)), "wg_adam_step")
 
 
 def profile(cmd: str):

@@ -25,7 +25,7 @@ EXPORTS = [
     "wg_graph_create", "wg_graph_info", "wg_graph_export", "wg_graph_destroy",
     "wg_plan_create", "wg_plan_sizes", "wg_plan_export", "wg_plan_buffer", "wg_plan_destroy",
     "wg_conv_forward", "wg_conv_backward",
-    "wg_status_string", "wg_last_error", "wg_launch_count", "wg_profile", "wg_softmax_xent",
+    "wg_status_string", "wg_last_error", "wg_launch_count", "wg_profile", "wg_softmax_xent", "wg_adam_step",
     "wg_comm_unique_id", "wg_comm_init", "wg_comm_init_emulated", "wg_comm_info", "wg_comm_wait",
     "wg_comm_destroy", "wg_partition_1d", "wg_graph_create_dist", "wg_graph_bounds", "wg_plan_create_dist",
     "wg_plan_xchg", "wg_conv_forward_dist", "wg_conv_backward_dist",
@@ -131,6 +131,8 @@ def lib():
     L.wg_profile.argtypes = [ctypes.c_int, P]
     L.wg_softmax_xent.restype = st
     L.wg_softmax_xent.argtypes = [ctypes.c_int, i64, i32, P, i64, P, f32, P, i64, P, P, P]
+    L.wg_adam_step.restype = st
+    L.wg_adam_step.argtypes = [i64, P, P, P, P, P, f32, f32, f32, f32, P]
     # multi-GPU
     L.wg_comm_unique_id.restype = st
     L.wg_comm_unique_id.argtypes = [P]

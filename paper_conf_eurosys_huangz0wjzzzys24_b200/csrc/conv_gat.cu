@@ -606,62 +606,84 @@ __global__ void __launch_bounds__(256, MINB) k_gat_fwd3(GatArgs a, int64_t row_b
   gat_write_y<TO>(a, ch.row, orow[wi][half], hl, 16);
 }
 
-// flash-style merge of the (m, l, acc) partials of split rows, chunk order:
-// M = max_k m_k, then l = sum_k l_k e^{m_k - M}, o = sum_k acc_k e^{m_k - M}
-// (independent loads, fixed order); writes agg, m, l and the y row
+// flash-style merge of the (m, l, acc) partials of split rows:
+// M = max_k m_k, then l = sum_k l_k e^{m_k - M}, o = sum_k acc_k e^{m_k - M};
+// writes agg, m, l and the y row.  The 8 warps of the CTA take slots
+// k = w, w + 8, ... (two independent slots in flight per lane) and their
+// sums are added in warp order (fixed order: deterministic); one thread per
+// column walking every slot was a serial latency chain (~50 us per launch).
+constexpr int CMB_HMAX = 128;   // heads <= HF / 4 <= 128
 template <typename TO>
 __global__ void __launch_bounds__(256) k_gat_fwd_combine(GatArgs a, const SplitRow* rows, int64_t row_base) {
-  __shared__ float orow[1024];
+  __shared__ float Mw[8][CMB_HMAX];
+  __shared__ float Mg[CMB_HMAX];
+  __shared__ __align__(16) float red[8][512 + CMB_HMAX];
+  __shared__ __align__(16) float orow[512];
   const SplitRow sr = rows[blockIdx.x];
   const int64_t d = row_base + sr.row;
-  for (int c = threadIdx.x; c < a.HF; c += blockDim.x) {
-    const int h = c / a.Fo;
-    const float* p0 = a.part + (int64_t)sr.first_slot * a.part_ld;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int H = a.H, HF = a.HF, VPR = HF / 4;
+  const float* p0 = a.part + (int64_t)sr.first_slot * a.part_ld;
+  // pass 1: per-head maxima over the slots with l > 0
+  for (int h = lane; h < H; h += 32) {
     float M = -INFINITY;
-    int k0 = 0;
-    for (; k0 + 8 <= sr.n_slots; k0 += 8) {      // 8 independent slot loads in flight
-      float lk[8], mk[8];
-#pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        const float* pp = p0 + (int64_t)(k0 + j) * a.part_ld;
-        lk[j] = pp[a.HF + a.H + h]; mk[j] = pp[a.HF + h];
-      }
-#pragma unroll
-      for (int j = 0; j < 8; ++j) if (lk[j] > 0.f) M = fmaxf(M, mk[j]);
-    }
-    for (; k0 < sr.n_slots; ++k0) {
-      const float* pp = p0 + (int64_t)k0 * a.part_ld;
-      if (pp[a.HF + a.H + h] > 0.f) M = fmaxf(M, pp[a.HF + h]);
-    }
-    float l = 0.f, o = 0.f;
-    int k = 0;
-    for (; k + 8 <= sr.n_slots; k += 8) {
-      float lk[8], mk[8], ok[8];
-#pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        const float* pp = p0 + (int64_t)(k + j) * a.part_ld;
-        lk[j] = pp[a.HF + a.H + h]; mk[j] = pp[a.HF + h]; ok[j] = pp[c];
-      }
-#pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        if (lk[j] <= 0.f) continue;
-        const float sc = __expf(mk[j] - M);
-        l += lk[j] * sc;
-        o += ok[j] * sc;
-      }
-    }
-    for (; k < sr.n_slots; ++k) {
+#pragma unroll 4
+    for (int k = w; k < sr.n_slots; k += 8) {    // independent loads (max is order-free)
       const float* pp = p0 + (int64_t)k * a.part_ld;
-      const float lk = pp[a.HF + a.H + h];
-      if (lk <= 0.f) continue;
-      const float sc = __expf(pp[a.HF + h] - M);
-      l += lk * sc;
-      o += pp[c] * sc;
+      const float lk = pp[HF + H + h], mk = pp[HF + h];
+      if (lk > 0.f) M = fmaxf(M, mk);
     }
-    const float val = l > 0.f ? o / l : 0.f;
+    Mw[w][h] = M;
+  }
+  __syncthreads();
+  for (int h = threadIdx.x; h < H; h += blockDim.x) {
+    float M = Mw[0][h];
+#pragma unroll
+    for (int j = 1; j < 8; ++j) M = fmaxf(M, Mw[j][h]);
+    Mg[h] = M;
+  }
+  __syncthreads();
+  // pass 2: this warp's rescaled sums (lane: float4 columns lane, lane + 32, ...)
+  float4 o[4];
+  float lh[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) { o[q] = make_float4(0.f, 0.f, 0.f, 0.f); lh[q] = 0.f; }
+#pragma unroll 2
+  for (int k = w; k < sr.n_slots; k += 8) {
+    const float* pp = p0 + (int64_t)k * a.part_ld;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int vi = lane + 32 * q;
+      if (vi < VPR) {
+        const int h = (4 * vi) / a.Fo;
+        const float lk = pp[HF + H + h];
+        const float sc = lk > 0.f ? __expf(pp[HF + h] - Mg[h]) : 0.f;
+        const float4 v = *reinterpret_cast<const float4*>(pp + 4 * vi);
+        o[q].x += v.x * sc; o[q].y += v.y * sc; o[q].z += v.z * sc; o[q].w += v.w * sc;
+      }
+      const int h = lane + 32 * q;
+      if (h < H) {
+        const float lk = pp[HF + H + h];
+        if (lk > 0.f) lh[q] += lk * __expf(pp[HF + h] - Mg[h]);
+      }
+    }
+  }
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const int vi = lane + 32 * q;
+    if (vi < VPR) *reinterpret_cast<float4*>(&red[w][4 * vi]) = o[q];
+    if (lane + 32 * q < H) red[w][512 + lane + 32 * q] = lh[q];
+  }
+  __syncthreads();
+  for (int c = threadIdx.x; c < HF; c += blockDim.x) {
+    const int h = c / a.Fo;
+    float oc = 0.f, l = 0.f;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) { oc += red[j][c]; l += red[j][512 + h]; }
+    const float val = l > 0.f ? oc / l : 0.f;
     static_cast<float*>(a.agg)[(int64_t)sr.row * a.ld_agg + c] = val;
     orow[c] = val;
-    if (c % a.Fo == 0) { a.m[d * a.H + h] = M; a.l[d * a.H + h] = l; }
+    if (c % a.Fo == 0) { a.m[d * H + h] = Mg[h]; a.l[d * H + h] = l; }
   }
   __syncthreads();
   gat_write_y<TO>(a, sr.row, orow, threadIdx.x, blockDim.x);
@@ -1022,27 +1044,57 @@ __global__ void k_gat_der3(const RowChunk* chunks, int n, int64_t row_base, cons
   }
 }
 
+// split-row sums of the slot partials: one warp per (row, column group) --
+// lane j sums slots j, j + 32, ... then a fixed xor tree (deterministic)
 __global__ void k_gat_der_combine(const SplitRow* rows, int n, int64_t row_base, const float* part, int part_ld,
                                   int H, float* der) {
-  const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const int lane = threadIdx.x & 31;
+  const int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (t >= (int64_t)n * H) return;
   const SplitRow sr = rows[t / H];
   const int h = (int)(t % H);
   float s = 0.f;
-#pragma unroll 8
-  for (int k = 0; k < sr.n_slots; ++k) s += part[(int64_t)(sr.first_slot + k) * part_ld + h];   // 8 loads in flight
-  der[(row_base + sr.row) * H + h] = s;
+#pragma unroll 4
+  for (int k = lane; k < sr.n_slots; k += 32) s += part[(int64_t)(sr.first_slot + k) * part_ld + h];
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if (lane == 0) der[(row_base + sr.row) * H + h] = s;
 }
 
-__global__ void k_gat_bwd_combine(GatArgs a, const SplitRow* rows, int64_t row_base) {
+// dg / del of a split source row: the 8 warps take slots w, w + 8, ...
+// (float4 columns per lane), summed in warp order
+__global__ void __launch_bounds__(256) k_gat_bwd_combine(GatArgs a, const SplitRow* rows, int64_t row_base) {
+  __shared__ __align__(16) float red[8][512 + CMB_HMAX];
   const SplitRow sr = rows[blockIdx.x];
   const int64_t u = row_base + sr.row;
-  for (int c = threadIdx.x; c < a.HF + a.H; c += blockDim.x) {
-    float s = 0.f;
-#pragma unroll 8
-    for (int k = 0; k < sr.n_slots; ++k) s += a.part[(int64_t)(sr.first_slot + k) * a.part_ld + c];
-    if (c < a.HF) a.dg[u * a.ld_dg + c] = s;
-    else a.del[u * a.H + (c - a.HF)] = s;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int HF = a.HF, NC = (HF + a.H + 3) / 4;   // float4 columns of a slot (acc then del)
+  float4 o[5];
+#pragma unroll
+  for (int q = 0; q < 5; ++q) o[q] = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int k = w; k < sr.n_slots; k += 8) {
+    const float4* pp = reinterpret_cast<const float4*>(a.part + (int64_t)(sr.first_slot + k) * a.part_ld);
+#pragma unroll
+    for (int q = 0; q < 5; ++q) {
+      const int vi = lane + 32 * q;
+      if (vi < NC) {
+        const float4 v = pp[vi];
+        o[q].x += v.x; o[q].y += v.y; o[q].z += v.z; o[q].w += v.w;
+      }
+    }
+  }
+#pragma unroll
+  for (int q = 0; q < 5; ++q) {
+    const int vi = lane + 32 * q;
+    if (vi < NC) *reinterpret_cast<float4*>(&red[w][4 * vi]) = o[q];
+  }
+  __syncthreads();
+  for (int c = threadIdx.x; c < HF + a.H; c += blockDim.x) {
+    float sum = 0.f;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) sum += red[j][c];
+    if (c < HF) a.dg[u * a.ld_dg + c] = sum;
+    else a.del[u * a.H + (c - HF)] = sum;
   }
 }
 
@@ -1375,7 +1427,7 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
 #undef WG_GAT_SEG
   // rows without out-edges have no chunk: their dg / del are zero
   // (chunks cover every row, including empty ones -- see build_chunks)
-  if (gp->n_bsplit) WG_LAUNCH(k_gat_bwd_combine, gp->n_bsplit, 128, 0, st, a, gp->bsplit, vb);
+  if (gp->n_bsplit) WG_LAUNCH(k_gat_bwd_combine, gp->n_bsplit, 256, 0, st, a, gp->bsplit, vb);
   float* der = L.at<float>(ws, "der");
   // (the split-row partial slots of the source-major pass were consumed by
   // k_gat_bwd_combine above: `part` is reused for the der partials)
@@ -1386,7 +1438,7 @@ static wg_status gat_bwd_t(wg_plan_s* p, const wg_params* P, const wg_bwd_args* 
     else if (H == 2) WG_LAUNCH(k_gat_der3<2>, tbk, 256, 0, st, gp->fwd, gp->n_fwd, vb, a.dt, der, a.part, a.part_ld);
     else WG_LAUNCH(k_gat_der3<8>, tbk, 256, 0, st, gp->fwd, gp->n_fwd, vb, a.dt, der, a.part, a.part_ld);
     if (gp->n_fsplit)
-      WG_LAUNCH(k_gat_der_combine, gs_grid((int64_t)gp->n_fsplit * H), 256, 0, st, gp->fsplit, gp->n_fsplit, vb,
+      WG_LAUNCH(k_gat_der_combine, gs_grid((int64_t)gp->n_fsplit * H * 32), 256, 0, st, gp->fsplit, gp->n_fsplit, vb,
                 a.part, a.part_ld, H, der);
   } else {
     WG_LAUNCH(k_gat_der, tbk32, 256, 0, st, nr, vb, g->fwd.row_ptr, a.dt, H, der);

@@ -43,6 +43,7 @@ struct TcParams {
   int64_t k_span;
   int64_t K;      // TN total K
   const int4* units;  // grouped TN: per blockIdx.z {first K row, k-blocks, -, -}
+  int a_stage;        // TN: bytes of the A part of a stage (the real M chunks only)
   GemmEpi epi;
   float* part;    // TN partial output [splits x M x N]
 };
@@ -249,8 +250,11 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int BN = p.BN, S = p.stages;
   const int b_stage = MN ? ((BN + CHE - 1) / CHE) * BKE * 128 : BN * 128;
-  constexpr bool LOBUF = TF32 && MN;            // lo in two separate buffers
-  const int raw = A_STAGE + b_stage;
+  // TN stages hold only the A chunks with real M columns (M = f_in = 64: 8 KB
+  // of A per fp32 stage, so twice the stages fit -- the TN ring is latency-bound)
+  const int a_stage = MN ? p.a_stage : A_STAGE;
+  constexpr bool LOBUF = TF32 && MN;            // lo in separate buffers
+  const int raw = a_stage + b_stage;
   const int stage = (TF32 && !MN) ? 2 * raw : raw;
   uint8_t* ring = smem;
   uint8_t* lo_buf = ring + S * stage;           // LOBUF: [TC_LO][A_lo | B_lo]
@@ -311,7 +315,7 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
       mbar_wait(smem_u32(&empty[s]), ph ^ 1);
       mbar_expect_tx(smem_u32(&full[s]), tx);
       const uint32_t fb = smem_u32(&full[s]);
-      const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE;
+      const uint32_t ad = smem_u32(ring + s * stage), bd = ad + a_stage;
       if (MN) {
         const int krow = (int)(kz + (int64_t)kb * BKE);
 #pragma unroll
@@ -337,8 +341,8 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
       const uint32_t ph = (kb / S) & 1;
       mbar_wait(smem_u32(TF32 ? &conv[s] : &full[s]), ph);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-      const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE;
-      const uint32_t al = LOBUF ? smem_u32(lo_buf + (kb % TC_LO) * raw) : bd + b_stage, bl = al + A_STAGE;
+      const uint32_t ad = smem_u32(ring + s * stage), bd = ad + a_stage;
+      const uint32_t al = LOBUF ? smem_u32(lo_buf + (kb % TC_LO) * raw) : bd + b_stage, bl = al + a_stage;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {   // 4 MMAs of 32 bytes of K (16 bf16 / 8 tf32)
         // MN-major: LBO = next 128-byte MN chunk, SBO = next K atom (8 rows
@@ -364,15 +368,15 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
   } else if (TF32 && warp >= 4) {
     // ---------------- hi / lo converters
     const int ct = threadIdx.x - 128;
-    const int n16 = (A_STAGE + b_stage) / 16;
+    const int n16 = (a_stage + b_stage) / 16;
     const int a16 = MN ? (int)min((int64_t)(BM / CHE), (p.M - m0 + CHE - 1) / CHE) * BKE * 8 : 0;
     for (int kb = 0; kb < total_kb; ++kb) {
       const int s = kb % S;
       mbar_wait(smem_u32(&full[s]), (kb / S) & 1);
       if (MN) {   // stage [A | B] -> lo buffer kb % TC_LO [A_lo | B_lo], once the MMAs of kb - TC_LO released it
         mbar_wait(smem_u32(&lo_empty[kb % TC_LO]), ((kb / TC_LO) & 1) ^ 1);
-        const uint32_t ad = smem_u32(ring + s * stage), bd = ad + A_STAGE;
-        const uint32_t al = smem_u32(lo_buf + (kb % TC_LO) * raw), bl = al + A_STAGE;
+        const uint32_t ad = smem_u32(ring + s * stage), bd = ad + a_stage;
+        const uint32_t al = smem_u32(lo_buf + (kb % TC_LO) * raw), bl = al + a_stage;
         tf32_split_range(ad, al, a16, ct, TC_CONV);
         tf32_split_range(bd, bl, b_stage / 16, ct, TC_CONV);
       } else {
@@ -502,12 +506,15 @@ bool tc_enabled() {
   return !g_tc_disabled;
 }
 
-size_t smem_bytes(bool mn, int BN, int stages, int es = 2) {
+size_t smem_bytes(bool mn, int BN, int stages, int es = 2, int a_stage = A_STAGE) {
   const int che = 128 / es, bke = 128 / es;
   const int b_stage = mn ? ((BN + che - 1) / che) * bke * 128 : BN * 128;
-  const size_t raw = A_STAGE + b_stage;
-  if (es == 4 && mn) return 1024 + (size_t)stages * raw + TC_LO * raw + 256;   // raw ring + lo buffers
-  return 1024 + (size_t)stages * raw * (es == 4 ? 2 : 1) + 256;
+  const size_t raw = (mn ? a_stage : A_STAGE) + b_stage;
+  // the M = 128 MMA reads 16 KB of A from every stage / lo buffer start: slack
+  // keeps the rows past a short A part (never stored) inside the allocation
+  const size_t slack = mn ? (size_t)(A_STAGE - a_stage) : 0;
+  if (es == 4 && mn) return 1024 + (size_t)stages * raw + TC_LO * raw + 256 + slack;   // raw ring + lo buffers
+  return 1024 + (size_t)stages * raw * (es == 4 ? 2 : 1) + 256 + slack;
 }
 
 template <bool MN, typename T>
@@ -588,7 +595,7 @@ namespace {
 // TN map pair + launch geometry shared by the plain and grouped TN GEMMs
 struct TnSetup {
   CUtensorMap maps[6];
-  int BN, n_tiles, m_tiles, stages, es;
+  int BN, n_tiles, m_tiles, stages, es, a_stage;
   size_t smem;
 };
 
@@ -607,9 +614,10 @@ bool tn_setup(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda, 
   if (!make_map_t(&t->maps[0], ty, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda * t->es, che, bke, swz)) return false;
   if (!make_map_t(&t->maps[1], ty, B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb * t->es, che, bke, swz)) return false;
   for (int i = 2; i < 6; ++i) t->maps[i] = t->maps[i & 1];
+  t->a_stage = (int)std::min<int64_t>(BM / che, cdiv(M, che)) * bke * 128;
   t->stages = t->es == 4 ? 8 : 4;
-  while (t->stages > 2 && smem_bytes(true, t->BN, t->stages, t->es) > 200 * 1024) --t->stages;
-  t->smem = smem_bytes(true, t->BN, t->stages, t->es);
+  while (t->stages > 2 && smem_bytes(true, t->BN, t->stages, t->es, t->a_stage) > 200 * 1024) --t->stages;
+  t->smem = smem_bytes(true, t->BN, t->stages, t->es, t->a_stage);
   return t->smem <= 227 * 1024;
 }
 
@@ -637,7 +645,7 @@ bool tc_gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda
   splits = cdiv(K, span);
   TcParams p{};
   p.M = M; p.N = N; p.BN = t.BN; p.nparts = 1; p.kblocks[0] = (int)(span / bke);
-  p.k_base = 0; p.k_span = span; p.K = K; p.part = part; p.stages = t.stages;
+  p.k_base = 0; p.k_span = span; p.K = K; p.part = part; p.stages = t.stages; p.a_stage = t.a_stage;
   dim3 grid((unsigned)t.m_tiles, (unsigned)t.n_tiles, (unsigned)splits);
   ProfScope ps(PK_TC_TN, s, (double)K * (M + N) * t.es + (double)M * N * 4.0, 2.0 * K * M * N);
   *st = tn_launch(dt, t, grid, p, s);
@@ -669,6 +677,7 @@ bool tc_gemm_tn_grouped(wg_dtype dt, const TnUnits& U, int M, int N, const void*
   if (!tn_setup(dt, U.k_total, M, N, A, lda, B, ldb, &t)) return false;
   TcParams p{};
   p.M = M; p.N = N; p.BN = t.BN; p.nparts = 1; p.K = U.k_total; p.part = part; p.stages = t.stages;
+  p.a_stage = t.a_stage;
  
   p.units = U.units;
   dim3 grid((unsigned)t.m_tiles, (unsigned)t.n_tiles, (unsigned)U.n_units);

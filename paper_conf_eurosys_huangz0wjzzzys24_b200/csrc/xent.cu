@@ -149,58 +149,75 @@ template <> struct XV<__nv_bfloat16> {
   }
 };
 
-template <typename T, int NVL>
+template <typename T, int NVL, int RPG>
 __global__ void __launch_bounds__(256) k_xent_vec(int64_t M, int C, const T* x, int64_t ld, const int64_t* labels,
                                                   float scale, T* dx, int64_t ldd, float* part) {
+  // RPG rows per 8-lane group per iteration: all their loads are issued
+  // before any is used (one row per group left ~24 KB in flight per SM)
   constexpr int EPV = XV<T>::EPV;
   __shared__ float wsum[8];
   const int Cpad = (C + 7) / 8 * 8;
   const int lane = threadIdx.x & 31, g = lane >> 3, l = lane & 7;
   const unsigned gm = 0xffu << (g * 8);
   float lsum = 0.f;
-  const int64_t rows_per_iter = (int64_t)gridDim.x * (blockDim.x / 8);
-  for (int64_t r = blockIdx.x * (int64_t)(blockDim.x / 8) + (threadIdx.x >> 3); r < M; r += rows_per_iter) {
-    float v[NVL][EPV];
-    float m = -INFINITY;
+  const int64_t groups = (int64_t)gridDim.x * (blockDim.x / 8);
+  const int64_t gid = blockIdx.x * (int64_t)(blockDim.x / 8) + (threadIdx.x >> 3);
+  for (int64_t r0 = gid * RPG; r0 < M; r0 += groups * RPG) {
+    float v[RPG][NVL][EPV];
+    int64_t lab[RPG];
 #pragma unroll
-    for (int q = 0; q < NVL; ++q) {
-      const int c0 = (l + 8 * q) * EPV;
-      if (c0 < Cpad) XV<T>::unpack(__ldg(reinterpret_cast<const int4*>(x + r * ld + c0)), v[q]);
+    for (int j = 0; j < RPG; ++j) {
+      const int64_t r = r0 + j;
+      lab[j] = r < M ? __ldg(labels + r) : -1;
 #pragma unroll
-      for (int i = 0; i < EPV; ++i) {
-        if (c0 + i >= C) v[q][i] = -INFINITY;
-        m = fmaxf(m, v[q][i]);
+      for (int q = 0; q < NVL; ++q) {
+        const int c0 = (l + 8 * q) * EPV;
+        if (r < M && c0 < Cpad) XV<T>::unpack(__ldg(reinterpret_cast<const int4*>(x + r * ld + c0)), v[j][q]);
       }
     }
 #pragma unroll
-    for (int o = 4; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(gm, m, o, 8));
-    const int64_t lab = labels[r];
-    float s = 0.f, t_lab = 0.f;
+    for (int j = 0; j < RPG; ++j) {
+      const int64_t r = r0 + j;
+      if (r >= M) break;                       // group-uniform
+      float m = -INFINITY;
 #pragma unroll
-    for (int q = 0; q < NVL; ++q) {
-      const int c0 = (l + 8 * q) * EPV;
+      for (int q = 0; q < NVL; ++q) {
+        const int c0 = (l + 8 * q) * EPV;
 #pragma unroll
-      for (int i = 0; i < EPV; ++i) {
-        const bool in = c0 + i < C;
-        const float t = in ? v[q][i] - m : 0.f;
-        if (c0 + i == lab) t_lab = t;
-        v[q][i] = in ? __expf(t) : 0.f;
-        s += v[q][i];
+        for (int i = 0; i < EPV; ++i) {
+          if (c0 + i >= C) v[j][q][i] = -INFINITY;
+          m = fmaxf(m, v[j][q][i]);
+        }
       }
-    }
 #pragma unroll
-    for (int o = 4; o; o >>= 1) s += __shfl_xor_sync(gm, s, o, 8);
-    const float inv = 1.f / s;
+      for (int o = 4; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(gm, m, o, 8));
+      float s = 0.f, t_lab = 0.f;
 #pragma unroll
-    for (int q = 0; q < NVL; ++q) {
-      const int c0 = (l + 8 * q) * EPV;
-      if (c0 >= Cpad) continue;
-      float o[EPV];
+      for (int q = 0; q < NVL; ++q) {
+        const int c0 = (l + 8 * q) * EPV;
 #pragma unroll
-      for (int i = 0; i < EPV; ++i)
-        o[i] = c0 + i < C ? scale * (v[q][i] * inv - (c0 + i == lab ? 1.f : 0.f)) : 0.f;
-      *reinterpret_cast<int4*>(dx + r * ldd + c0) = XV<T>::pack(o);
-      if (lab >= c0 && lab < c0 + EPV) lsum += scale * (logf(s) - t_lab);
+        for (int i = 0; i < EPV; ++i) {
+          const bool in = c0 + i < C;
+          const float t = in ? v[j][q][i] - m : 0.f;
+          if (c0 + i == lab[j]) t_lab = t;
+          v[j][q][i] = in ? __expf(t) : 0.f;
+          s += v[j][q][i];
+        }
+      }
+#pragma unroll
+      for (int o = 4; o; o >>= 1) s += __shfl_xor_sync(gm, s, o, 8);
+      const float inv = 1.f / s;
+#pragma unroll
+      for (int q = 0; q < NVL; ++q) {
+        const int c0 = (l + 8 * q) * EPV;
+        if (c0 >= Cpad) continue;
+        float o[EPV];
+#pragma unroll
+        for (int i = 0; i < EPV; ++i)
+          o[i] = c0 + i < C ? scale * (v[j][q][i] * inv - (c0 + i == lab[j] ? 1.f : 0.f)) : 0.f;
+        *reinterpret_cast<int4*>(dx + r * ldd + c0) = XV<T>::pack(o);
+        if (lab[j] >= c0 && lab[j] < c0 + EPV) lsum += scale * (logf(s) - t_lab);
+      }
     }
   }
 #pragma unroll
@@ -253,10 +270,10 @@ extern "C" wg_status wg_softmax_xent(wg_dtype dtype, int64_t M, int32_t C, const
     const bool vec = ((ld * (dtype == WG_BF16 ? 2 : 4)) % 16 == 0) && ((ldd * (dtype == WG_BF16 ? 2 : 4)) % 16 == 0) &&
                      (reinterpret_cast<uintptr_t>(logits) % 16 == 0) && (reinterpret_cast<uintptr_t>(dlogits) % 16 == 0);
     if (dtype == WG_BF16 && vec)
-      WG_LAUNCH((k_xent_vec<__nv_bfloat16, 1>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld, labels, scale,
+      WG_LAUNCH((k_xent_vec<__nv_bfloat16, 1, 4>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld, labels, scale,
                 (__nv_bfloat16*)dlogits, ldd, part);
     else if (vec)
-      WG_LAUNCH((k_xent_vec<float, 2>), nb, 256, 0, s, M, C, (const float*)logits, ld, labels, scale,
+      WG_LAUNCH((k_xent_vec<float, 2, 2>), nb, 256, 0, s, M, C, (const float*)logits, ld, labels, scale,
                 (float*)dlogits, ldd, part);
     else if (dtype == WG_BF16)
       WG_LAUNCH((k_xent_row<__nv_bfloat16, 8>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld, labels, scale,

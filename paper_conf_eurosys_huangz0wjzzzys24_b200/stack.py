@@ -26,7 +26,7 @@ from __future__ import annotations
 
 import torch
 
-from . import Conv, Graph, init_params, padded, pitch, softmax_xent
+from . import Adam, Conv, Graph, init_params, padded, pitch, softmax_xent
 from . import _capi as C
 
 
@@ -92,7 +92,14 @@ class GNNStack:
         # dx of layer i (= dy of layer i-1): owned rows only (the exchange
         # tables carry what other ranks read)
         self.dx = [None] + [padded(self.rows, self.f_in[i], dtype, self.dev) for i in range(1, self.L)]
-        self.grads = [{k: torch.zeros_like(v) for k, v in p.items()} for p in self.params]
+        # optimizer: on the GPU the library's fused Adam (one launch over one
+        # flat buffer; params / grads become views of it); the CPU orchestration
+        # tests (test-only layers on gloo) use torch's
+        if self.dev.type == "cuda":
+            self.opt = Adam(self.params, lr=lr)
+            self.grads = self.opt.grads
+        else:
+            self.grads = [{k: torch.zeros_like(v) for k, v in p.items()} for p in self.params]
         self.xchg_f, self.xchg_b = [], []
         for i, c in enumerate(self.convs):
             if self.comm is not None and self.dist:
@@ -108,13 +115,11 @@ class GNNStack:
             else:
                 self.xchg_f.append(None)
                 self.xchg_b.append(None)
-        for p in self.params:
-            for v in p.values():
-                v.requires_grad_(True)
-        # capturable: the step count lives on the device, so a whole training
-        # step (library launches + Adam) can be captured in one CUDA graph
-        self.opt = torch.optim.Adam([v for p in self.params for v in p.values()], lr=lr,
-                                    capturable=self.dev.type == "cuda")
+        if self.dev.type != "cuda":
+            for p in self.params:
+                for v in p.values():
+                    v.requires_grad_(True)
+            self.opt = torch.optim.Adam([v for p in self.params for v in p.values()], lr=lr)
 
     # -------------------------------------------------------------- helpers
     def _vote(self, conv, Conv_, graph, model, fi, fo, policy, kw):
@@ -256,10 +261,13 @@ class GNNStack:
             self._loss = torch.zeros(1, dtype=torch.float32, device=self.dev)
         softmax_xent(logits, labels, 1.0 / n_global, self._dl, self._loss)
         self.backward(self._dl)
-        for p, gr in zip(self.params, self.grads):
-            for k, v in p.items():
-                v.grad = gr[k]
-        self.opt.step()
+        if isinstance(self.opt, Adam):
+            self.opt.step()           # the step count is on the device: a captured step replays real steps
+        else:
+            for p, gr in zip(self.params, self.grads):
+                for k, v in p.items():
+                    v.grad = gr[k]
+            self.opt.step()
         return self._loss
 
 
