@@ -44,6 +44,7 @@ struct TcParams {
   int64_t K;      // TN total K
   const int4* units;  // grouped TN: per blockIdx.z {first K row, k-blocks, -, -}
   int a_stage;        // TN: bytes of the A part of a stage (the real M chunks only)
+  int fold;           // TN fp32, M <= 64: A_lo in A's MMA rows 64..127 (2 MMAs per k-step, see the kernel)
   GemmEpi epi;
   float* part;    // TN partial output [splits x M x N]
 };
@@ -256,9 +257,17 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
   constexpr bool LOBUF = TF32 && MN;            // lo in separate buffers
   const int raw = a_stage + b_stage;
   const int stage = (TF32 && !MN) ? 2 * raw : raw;
+  // M fold (TN fp32, M <= 64): the converters write A_lo into the stage's
+  // MMA rows 64..127 (A chunks 2, 3), so one M = 128 MMA computes
+  // [A_hi; A_lo]^T B and a k-step needs 2 MMAs (B_hi, B_lo) instead of 3 --
+  // the 3xTF32 GEMMs are bound by shared-memory operand reads
+  // (profiles/r02/tn_bound_experiment.md); the epilogue adds rows m and m + 64.
+  // The lo buffers then hold B_lo only.
+  const bool fold = LOBUF && p.fold;
+  const int lo_stride = fold ? b_stage : raw;
   uint8_t* ring = smem;
-  uint8_t* lo_buf = ring + S * stage;           // LOBUF: [TC_LO][A_lo | B_lo]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(lo_buf + (LOBUF ? TC_LO * raw : 0));
+  uint8_t* lo_buf = ring + S * stage;           // LOBUF: [TC_LO][A_lo | B_lo] (fold: [TC_LO][B_lo])
+  uint64_t* bars = reinterpret_cast<uint64_t*>(lo_buf + (LOBUF ? TC_LO * lo_stride : 0));
   uint64_t* full = bars;                        // [S <= 8]
   uint64_t* empty = bars + 8;
   uint64_t* conv = bars + 16;
@@ -342,7 +351,8 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
       mbar_wait(smem_u32(TF32 ? &conv[s] : &full[s]), ph);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       const uint32_t ad = smem_u32(ring + s * stage), bd = ad + a_stage;
-      const uint32_t al = LOBUF ? smem_u32(lo_buf + (kb % TC_LO) * raw) : bd + b_stage, bl = al + a_stage;
+      const uint32_t al = LOBUF ? smem_u32(lo_buf + (kb % TC_LO) * lo_stride) : bd + b_stage;
+      const uint32_t bl = fold ? al : al + a_stage;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {   // 4 MMAs of 32 bytes of K (16 bf16 / 8 tf32)
         // MN-major: LBO = next 128-byte MN chunk, SBO = next K atom (8 rows
@@ -356,7 +366,8 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
         if constexpr (TF32) {
           umma_tf32(tmem, umma_desc(ad + step, lbo, sbo, lay), umma_desc(bd + step, lbo, sbo, lay), idesc, on);
           umma_tf32(tmem, umma_desc(ad + step, lbo, sbo, lay), umma_desc(bl + step, lbo, sbo, lay), idesc, 1u);
-          umma_tf32(tmem, umma_desc(al + step, lbo, sbo, lay), umma_desc(bd + step, lbo, sbo, lay), idesc, 1u);
+          if (!fold)
+            umma_tf32(tmem, umma_desc(al + step, lbo, sbo, lay), umma_desc(bd + step, lbo, sbo, lay), idesc, 1u);
         } else {
           umma_bf16(tmem, umma_desc(ad + step, lbo, sbo, lay), umma_desc(bd + step, lbo, sbo, lay), idesc, on);
         }
@@ -376,9 +387,14 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
       if (MN) {   // stage [A | B] -> lo buffer kb % TC_LO [A_lo | B_lo], once the MMAs of kb - TC_LO released it
         mbar_wait(smem_u32(&lo_empty[kb % TC_LO]), ((kb / TC_LO) & 1) ^ 1);
         const uint32_t ad = smem_u32(ring + s * stage), bd = ad + a_stage;
-        const uint32_t al = smem_u32(lo_buf + (kb % TC_LO) * raw), bl = al + a_stage;
-        tf32_split_range(ad, al, a16, ct, TC_CONV);
-        tf32_split_range(bd, bl, b_stage / 16, ct, TC_CONV);
+        const uint32_t lb = smem_u32(lo_buf + (kb % TC_LO) * lo_stride);
+        if (fold) {
+          tf32_split_range(ad, ad + 2 * BKE * 128, a16, ct, TC_CONV);   // A_lo -> MMA rows 64..127
+          tf32_split_range(bd, lb, b_stage / 16, ct, TC_CONV);
+        } else {
+          tf32_split_range(ad, lb, a16, ct, TC_CONV);
+          tf32_split_range(bd, lb + a_stage, b_stage / 16, ct, TC_CONV);
+        }
       } else {
         tf32_split_stage(smem_u32(ring + s * stage), n16, ct, TC_CONV);
       }
@@ -395,10 +411,28 @@ __global__ void __launch_bounds__(sizeof(T) == 4 ? 128 + TC_CONV : 128, 1)
     const int64_t m = m0 + r;
     const GemmEpi& e = p.epi;
     const float rs = (!MN && e.rscale && m < p.M) ? e.rscale[m] : 1.f;
+    float* fb = reinterpret_cast<float*>(ring);   // fold: rows 64..127 (the ring is idle after accf)
+    const int ldf = BN + 1;
+    if (fold) {
+      if (warp >= 2) {
+        for (int c0 = 0; c0 < BN; c0 += 16) {
+          float v[16];
+          tmem_ld16(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0, v);
+#pragma unroll
+          for (int i = 0; i < 16; ++i) fb[(r - 64) * ldf + c0 + i] = v[i];
+        }
+      }
+      asm volatile("bar.sync 1, 128;" ::: "memory");   // the four epilogue warps
+    }
     for (int c0 = 0; c0 < BN; c0 += 16) {
+      if (fold && warp >= 2) break;
       float v[16];
       tmem_ld16(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0, v);
       if (m >= p.M) continue;
+      if (fold) {
+#pragma unroll
+        for (int i = 0; i < 16; ++i) v[i] += fb[r * ldf + c0 + i];   // A_hi^T B + A_lo^T B
+      }
       if (MN) {
         float* out = p.part + (int64_t)blockIdx.z * p.M * p.N + m * p.N;
 #pragma unroll
@@ -506,14 +540,15 @@ bool tc_enabled() {
   return !g_tc_disabled;
 }
 
-size_t smem_bytes(bool mn, int BN, int stages, int es = 2, int a_stage = A_STAGE) {
+size_t smem_bytes(bool mn, int BN, int stages, int es = 2, int a_stage = A_STAGE, bool fold = false) {
   const int che = 128 / es, bke = 128 / es;
   const int b_stage = mn ? ((BN + che - 1) / che) * bke * 128 : BN * 128;
   const size_t raw = (mn ? a_stage : A_STAGE) + b_stage;
+  const size_t lo = fold ? (size_t)b_stage : raw;   // fold: the lo buffers hold B_lo only
   // the M = 128 MMA reads 16 KB of A from every stage / lo buffer start: slack
   // keeps the rows past a short A part (never stored) inside the allocation
   const size_t slack = mn ? (size_t)(A_STAGE - a_stage) : 0;
-  if (es == 4 && mn) return 1024 + (size_t)stages * raw + TC_LO * raw + 256 + slack;   // raw ring + lo buffers
+  if (es == 4 && mn) return 1024 + (size_t)stages * raw + TC_LO * lo + 256 + slack;   // raw ring + lo buffers
   return 1024 + (size_t)stages * raw * (es == 4 ? 2 : 1) + 256 + slack;
 }
 
@@ -595,7 +630,7 @@ namespace {
 // TN map pair + launch geometry shared by the plain and grouped TN GEMMs
 struct TnSetup {
   CUtensorMap maps[6];
-  int BN, n_tiles, m_tiles, stages, es, a_stage;
+  int BN, n_tiles, m_tiles, stages, es, a_stage, fold;
   size_t smem;
 };
 
@@ -614,10 +649,17 @@ bool tn_setup(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda, 
   if (!make_map_t(&t->maps[0], ty, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda * t->es, che, bke, swz)) return false;
   if (!make_map_t(&t->maps[1], ty, B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb * t->es, che, bke, swz)) return false;
   for (int i = 2; i < 6; ++i) t->maps[i] = t->maps[i & 1];
-  t->a_stage = (int)std::min<int64_t>(BM / che, cdiv(M, che)) * bke * 128;
+  // fp32 with M <= 64: fold A_lo into the M = 128 MMA's idle rows (kernel comment)
+  static int fold_env = -1;
+  if (fold_env < 0) {
+    const char* e = getenv("WG_TN_FOLD");
+    fold_env = (e && e[0] == '0') ? 0 : 1;
+  }
+  t->fold = (t->es == 4 && M <= 64 && fold_env) ? 1 : 0;
+  t->a_stage = t->fold ? A_STAGE : (int)std::min<int64_t>(BM / che, cdiv(M, che)) * bke * 128;
   t->stages = t->es == 4 ? 8 : 4;
-  while (t->stages > 2 && smem_bytes(true, t->BN, t->stages, t->es, t->a_stage) > 200 * 1024) --t->stages;
-  t->smem = smem_bytes(true, t->BN, t->stages, t->es, t->a_stage);
+  while (t->stages > 2 && smem_bytes(true, t->BN, t->stages, t->es, t->a_stage, t->fold) > 200 * 1024) --t->stages;
+  t->smem = smem_bytes(true, t->BN, t->stages, t->es, t->a_stage, t->fold);
   return t->smem <= 227 * 1024;
 }
 
@@ -646,6 +688,7 @@ bool tc_gemm_tn(wg_dtype dt, int64_t K, int M, int N, const void* A, int64_t lda
   TcParams p{};
   p.M = M; p.N = N; p.BN = t.BN; p.nparts = 1; p.kblocks[0] = (int)(span / bke);
   p.k_base = 0; p.k_span = span; p.K = K; p.part = part; p.stages = t.stages; p.a_stage = t.a_stage;
+  p.fold = t.fold;
   dim3 grid((unsigned)t.m_tiles, (unsigned)t.n_tiles, (unsigned)splits);
   ProfScope ps(PK_TC_TN, s, (double)K * (M + N) * t.es + (double)M * N * 4.0, 2.0 * K * M * N);
   *st = tn_launch(dt, t, grid, p, s);
@@ -678,7 +721,7 @@ bool tc_gemm_tn_grouped(wg_dtype dt, const TnUnits& U, int M, int N, const void*
   TcParams p{};
   p.M = M; p.N = N; p.BN = t.BN; p.nparts = 1; p.K = U.k_total; p.part = part; p.stages = t.stages;
   p.a_stage = t.a_stage;
- 
+  p.fold = t.fold;
   p.units = U.units;
   dim3 grid((unsigned)t.m_tiles, (unsigned)t.n_tiles, (unsigned)U.n_units);
   ProfScope ps(PK_TC_TN, s, (double)U.k_total * (M + N) * t.es + (double)U.n_units * M * N * 4.0,
