@@ -98,6 +98,13 @@ def test_rgcn_c3_shape_sampled():
     assert all(v <= 1e-4 for v in errs.values()), str(errs)
 
 
+def test_rgcn_c3_layer2_shape_sampled():
+    """C3 second-layer shape (64 -> 64, R = 128): the fp32 weight gradient runs the
+    TN M fold (A_lo in the MMA's rows 64..127) with two real A chunks."""
+    errs, _ = run(torch.float32, "auto", R=128, V=20000, E=220000, fi=64, fo=64, seed=11, alpha=0.5, relu=True)
+    assert all(v <= 1e-4 for v in errs.values()), str(errs)
+
+
 @pytest.mark.parametrize("policy", ["edge", "vertex", "auto"])
 @pytest.mark.parametrize("P", [2, 3])
 def test_rgcn_1d_partition_phases_match_oracle(policy, P):
