@@ -150,7 +150,7 @@ template <> struct XV<__nv_bfloat16> {
 };
 
 template <typename T, int NVL, int RPG>
-__global__ void __launch_bounds__(256) k_xent_vec(int64_t M, int C, const T* x, int64_t ld, const int64_t* labels,
+__global__ void __launch_bounds__(256, 4) k_xent_vec(int64_t M, int C, const T* x, int64_t ld, const int64_t* labels,
                                                   float scale, T* dx, int64_t ldd, float* part) {
   // RPG rows per 8-lane group per iteration: all their loads are issued
   // before any is used (one row per group left ~24 KB in flight per SM)
@@ -163,30 +163,35 @@ __global__ void __launch_bounds__(256) k_xent_vec(int64_t M, int C, const T* x, 
   const int64_t groups = (int64_t)gridDim.x * (blockDim.x / 8);
   const int64_t gid = blockIdx.x * (int64_t)(blockDim.x / 8) + (threadIdx.x >> 3);
   for (int64_t r0 = gid * RPG; r0 < M; r0 += groups * RPG) {
-    float v[RPG][NVL][EPV];
-    int64_t lab[RPG];
+    // raw 16-byte vectors of all RPG rows in flight (4 registers each), the
+    // rows unpacked one at a time
+    int4 raw[RPG][NVL];
+    int32_t lab[RPG];
 #pragma unroll
     for (int j = 0; j < RPG; ++j) {
       const int64_t r = r0 + j;
-      lab[j] = r < M ? __ldg(labels + r) : -1;
+      lab[j] = r < M ? (int32_t)__ldg(labels + r) : -1;
 #pragma unroll
       for (int q = 0; q < NVL; ++q) {
         const int c0 = (l + 8 * q) * EPV;
-        if (r < M && c0 < Cpad) XV<T>::unpack(__ldg(reinterpret_cast<const int4*>(x + r * ld + c0)), v[j][q]);
+        raw[j][q] = (r < M && c0 < Cpad) ? __ldg(reinterpret_cast<const int4*>(x + r * ld + c0)) : make_int4(0, 0, 0, 0);
       }
     }
 #pragma unroll
     for (int j = 0; j < RPG; ++j) {
       const int64_t r = r0 + j;
       if (r >= M) break;                       // group-uniform
+      float v[1][NVL][EPV];
+#pragma unroll
+      for (int q = 0; q < NVL; ++q) XV<T>::unpack(raw[j][q], v[0][q]);
       float m = -INFINITY;
 #pragma unroll
       for (int q = 0; q < NVL; ++q) {
         const int c0 = (l + 8 * q) * EPV;
 #pragma unroll
         for (int i = 0; i < EPV; ++i) {
-          if (c0 + i >= C) v[j][q][i] = -INFINITY;
-          m = fmaxf(m, v[j][q][i]);
+          if (c0 + i >= C) v[0][q][i] = -INFINITY;
+          m = fmaxf(m, v[0][q][i]);
         }
       }
 #pragma unroll
@@ -198,10 +203,10 @@ __global__ void __launch_bounds__(256) k_xent_vec(int64_t M, int C, const T* x, 
 #pragma unroll
         for (int i = 0; i < EPV; ++i) {
           const bool in = c0 + i < C;
-          const float t = in ? v[j][q][i] - m : 0.f;
+          const float t = in ? v[0][q][i] - m : 0.f;
           if (c0 + i == lab[j]) t_lab = t;
-          v[j][q][i] = in ? __expf(t) : 0.f;
-          s += v[j][q][i];
+          v[0][q][i] = in ? __expf(t) : 0.f;
+          s += v[0][q][i];
         }
       }
 #pragma unroll
@@ -214,7 +219,7 @@ __global__ void __launch_bounds__(256) k_xent_vec(int64_t M, int C, const T* x, 
         float o[EPV];
 #pragma unroll
         for (int i = 0; i < EPV; ++i)
-          o[i] = c0 + i < C ? scale * (v[j][q][i] * inv - (c0 + i == lab[j] ? 1.f : 0.f)) : 0.f;
+          o[i] = c0 + i < C ? scale * (v[0][q][i] * inv - (c0 + i == lab[j] ? 1.f : 0.f)) : 0.f;
         *reinterpret_cast<int4*>(dx + r * ldd + c0) = XV<T>::pack(o);
         if (lab[j] >= c0 && lab[j] < c0 + EPV) lsum += scale * (logf(s) - t_lab);
       }
