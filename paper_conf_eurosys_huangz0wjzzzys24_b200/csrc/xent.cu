@@ -149,8 +149,8 @@ template <> struct XV<__nv_bfloat16> {
   }
 };
 
-template <typename T, int NVL, int RPG>
-__global__ void __launch_bounds__(256, 4) k_xent_vec(int64_t M, int C, const T* x, int64_t ld, const int64_t* labels,
+template <typename T, int NVL, int RPG, int MINB = 4>
+__global__ void __launch_bounds__(256, MINB) k_xent_vec(int64_t M, int C, const T* x, int64_t ld, const int64_t* labels,
                                                   float scale, T* dx, int64_t ldd, float* part) {
   // RPG rows per 8-lane group per iteration: all their loads are issued
   // before any is used (one row per group left ~24 KB in flight per SM)
@@ -270,10 +270,30 @@ extern "C" wg_status wg_softmax_xent(wg_dtype dtype, int64_t M, int32_t C, const
   ProfScope ps(PK_MISC, s, (double)M * C * (dtype == WG_BF16 ? 4.0 : 8.0) + M * 8.0, 0.0);
   float* part = static_cast<float*>(scratch);
   const int per = (C + 31) / 32;
+  const bool vec = ((ld * (dtype == WG_BF16 ? 2 : 4)) % 16 == 0) && ((ldd * (dtype == WG_BF16 ? 2 : 4)) % 16 == 0) &&
+                   (reinterpret_cast<uintptr_t>(logits) % 16 == 0) && (reinterpret_cast<uintptr_t>(dlogits) % 16 == 0);
+  // wider rows (C5's 172 classes): the same 8-lane groups with 3-4 vectors
+  // per lane, one row per group in flight -- the one-warp-per-row kernel
+  // below walks ~12 K rows per CTA with one dependent row at a time
+  if (vec && C > 64 && C <= (dtype == WG_BF16 ? 256 : 128)) {
+    const unsigned nb = (unsigned)std::min<int64_t>(XENT_BLKS, std::max<int64_t>(1, cdiv(M, 32)));
+    const int nvl = (int)cdiv(cdiv(C, dtype == WG_BF16 ? 8 : 4), 8);   // vectors per lane
+    if (dtype == WG_BF16) {
+      if (nvl <= 2) WG_LAUNCH((k_xent_vec<__nv_bfloat16, 2, 2, 3>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld,
+                              labels, scale, (__nv_bfloat16*)dlogits, ldd, part);
+      else WG_LAUNCH((k_xent_vec<__nv_bfloat16, 4, 1, 2>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld, labels,
+                     scale, (__nv_bfloat16*)dlogits, ldd, part);
+    } else {
+      if (nvl <= 3) WG_LAUNCH((k_xent_vec<float, 3, 1>), nb, 256, 0, s, M, C, (const float*)logits, ld, labels, scale,
+                              (float*)dlogits, ldd, part);
+      else WG_LAUNCH((k_xent_vec<float, 4, 1, 3>), nb, 256, 0, s, M, C, (const float*)logits, ld, labels, scale,
+                     (float*)dlogits, ldd, part);
+    }
+    WG_LAUNCH(k_sum, 1, 32, 0, s, part, (int)nb, loss_out);
+    return WG_OK;
+  }
   if (C <= 64) {
     const unsigned nb = (unsigned)std::min<int64_t>(XENT_BLKS, std::max<int64_t>(1, cdiv(M, 32)));
-    const bool vec = ((ld * (dtype == WG_BF16 ? 2 : 4)) % 16 == 0) && ((ldd * (dtype == WG_BF16 ? 2 : 4)) % 16 == 0) &&
-                     (reinterpret_cast<uintptr_t>(logits) % 16 == 0) && (reinterpret_cast<uintptr_t>(dlogits) % 16 == 0);
     if (dtype == WG_BF16 && vec)
       WG_LAUNCH((k_xent_vec<__nv_bfloat16, 1, 4>), nb, 256, 0, s, M, C, (const __nv_bfloat16*)logits, ld, labels, scale,
                 (__nv_bfloat16*)dlogits, ldd, part);
