@@ -272,9 +272,10 @@ extern "C" wg_status wg_softmax_xent(wg_dtype dtype, int64_t M, int32_t C, const
   const int per = (C + 31) / 32;
   const bool vec = ((ld * (dtype == WG_BF16 ? 2 : 4)) % 16 == 0) && ((ldd * (dtype == WG_BF16 ? 2 : 4)) % 16 == 0) &&
                    (reinterpret_cast<uintptr_t>(logits) % 16 == 0) && (reinterpret_cast<uintptr_t>(dlogits) % 16 == 0);
-  // wider rows (C5's 172 classes): the same 8-lane groups with 3-4 vectors
-  // per lane, one row per group in flight -- the one-warp-per-row kernel
-  // below walks ~12 K rows per CTA with one dependent row at a time
+  // wider rows (C5's 172 classes): the same 8-lane groups with 2-4 vectors
+  // per lane -- the one-warp-per-row kernel below walks ~12 K rows per CTA
+  // with one dependent row at a time (C5 rank slice: misc class 8.4 -> 6.3 ms;
+  // 16-lane groups with two rows in flight measured slower)
   if (vec && C > 64 && C <= (dtype == WG_BF16 ? 256 : 128)) {
     const unsigned nb = (unsigned)std::min<int64_t>(XENT_BLKS, std::max<int64_t>(1, cdiv(M, 32)));
     const int nvl = (int)cdiv(cdiv(C, dtype == WG_BF16 ? 8 : 4), 8);   // vectors per lane
