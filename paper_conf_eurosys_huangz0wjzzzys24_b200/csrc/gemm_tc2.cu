@@ -82,6 +82,9 @@ struct P2 {
   int cpg;          // fp32 row-gathered A by per-lane cp.async (see the producer)
   int fc_d, fc_d2;  // columns per chunk of the (column-chunked) D / D2 output maps
   int bres;         // B resident: every k-block of B loaded once per CTA (one N tile, no grouped B)
+  // direct stores of a chunk that straddles the D / D2 split (n_split not a
+  // multiple of the 128-byte chunk: C5's 32-wide [Y | S])
+  void* d_ptr; int64_t ldd, d_cstride; void* d2_ptr; int64_t ldd2;
   const void* a_tab; int64_t lda_tab; int k_a;   // cpg: table, its row pitch (elements), K
 };
 
@@ -507,8 +510,10 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
         if (et == 0) bulk_wait_read<0>();
         epi_bar(grp);
         const int nc0 = n0 + c * C::CHE;
-        // split output: a 128-byte chunk belongs to D or to D2 (n_split % CHE == 0)
+        // split output: a 128-byte chunk belongs to D or to D2, or straddles
+        // the split (stored directly from registers, 16 bytes at a time)
         const bool second = p.n_split > 0 && nc0 >= p.n_split;
+        const bool strad = p.n_split > 0 && nc0 < p.n_split && nc0 + C::CHE > p.n_split;
         const float rs = second ? 1.f : rs_d;
         // one 16-byte output unit (EPV columns) at a time; FULL: every column < N
         auto units = [&](auto full_t) {
@@ -518,7 +523,9 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
             float f[C::EPV];
             const int nc = nc0 + k * C::EPV;
 #pragma unroll
-            for (int i = 0; i < C::EPV; ++i) f[i] = rs * __uint_as_float(u[k * C::EPV + i]);
+            const float rsu = (strad && nc >= p.n_split) ? 1.f : rs;   // the row scale is D's only
+#pragma unroll
+            for (int i = 0; i < C::EPV; ++i) f[i] = rsu * __uint_as_float(u[k * C::EPV + i]);
             if constexpr ((FL & EP_ADD) != 0) {
               float a[C::EPV];
               unpack16<T>(*reinterpret_cast<const int4*>(adp + sw_off(r, k)), a);
@@ -549,7 +556,16 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
 #pragma unroll
               for (int i = 0; i < C::EPV; ++i) if (nc + i >= p.N) f[i] = 0.f;
             }
-            *reinterpret_cast<int4*>(stg + sw_off(r, k)) = pack16<T>(f);
+            if (strad) {
+              if (m < p.M && nc < p.N) {
+                T* dst = nc < p.n_split
+                             ? static_cast<T*>(p.d_ptr) + (int64_t)(nc / p.fc_d) * p.d_cstride + m * p.ldd + nc % p.fc_d
+                             : static_cast<T*>(p.d2_ptr) + m * p.ldd2 + (nc - p.n_split);
+                *reinterpret_cast<int4*>(dst) = pack16<T>(f);
+              }
+            } else {
+              *reinterpret_cast<int4*>(stg + sw_off(r, k)) = pack16<T>(f);
+            }
           }
         };
         if (nc0 + C::CHE <= p.N && p.bias_vec) units(std::true_type{});
@@ -557,7 +573,7 @@ __global__ void __launch_bounds__(Cfg<T>::NTHREADS, 1)
         if (epi_loads) mbar_arrive(su32(&eempty[grp]));
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         epi_bar(grp);
-        if (et == 0) {
+        if (et == 0 && !strad) {
           const CUtensorMap* td = second ? &tD2 : &tD;
           const int col = second ? nc0 - p.n_split : nc0, fc = second ? p.fc_d2 : p.fc_d;
           tma_store3(td, col % fc, m0, col / fc, su32(stg));
@@ -625,7 +641,8 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
   const int bn_max = (bn_env >= 64 && bn_env <= 256 && bn_env % 64 == 0) ? bn_env : (f32 ? 128 : 256);
   const int n_tiles = (int)cdiv(N, bn_max);
   const int BN = n_tiles > 1 ? bn_max : (int)rup(N, 16);
-  if (epi.D2 && (epi.n_split % che != 0)) return false;  // split must fall on a 128-byte chunk boundary
+  // a split off the 128-byte chunk grid is stored directly for the straddling chunk; 16-byte units
+  if (epi.D2 && (epi.n_split % (16 / es) != 0 || (N - epi.n_split) % (16 / es) != 0)) return false;
   CUtensorMap maps[10];
   memset(maps, 0, sizeof(maps));
   P2 p{};
@@ -655,6 +672,11 @@ bool tc_gemm_nt_persistent(wg_dtype dt, int64_t M, int N, const GemmPart* parts,
   const int C1 = epi.d_chunk_cols > 0 ? (int)cdiv(n1, epi.d_chunk_cols) : 1;
   p.fc_d = C1 > 1 ? epi.d_chunk_cols : n1;
   if (C1 > 1 && (p.fc_d % che != 0 || (epi.d_chunk_stride * es) % 16 != 0)) return false;
+  p.d_ptr = epi.D; p.ldd = epi.ldd; p.d_cstride = C1 > 1 ? epi.d_chunk_stride : 0;
+  p.d2_ptr = epi.D2; p.ldd2 = epi.ldd2;
+  if ((epi.D2 && (reinterpret_cast<uintptr_t>(epi.D2) % 16 || (epi.ldd2 * es) % 16)) ||
+      reinterpret_cast<uintptr_t>(epi.D) % 16 || (epi.ldd * es) % 16)
+    return false;
   if (!tc_make_map3_t(&maps[6], ty, epi.D, (uint64_t)p.fc_d, (uint64_t)M, (uint64_t)C1, (uint64_t)epi.ldd * es,
                       (uint64_t)(C1 > 1 ? epi.d_chunk_stride : 0) * es, che, BM))
     return false;
