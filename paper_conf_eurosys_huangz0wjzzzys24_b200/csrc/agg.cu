@@ -869,7 +869,7 @@ __global__ void k_prep_weight(const float* W, int batch, int rows, int cols, int
 // Column partial sums of (optionally ReLU-masked) dy over blocks of rows,
 // 16-byte vectors per thread; block partials reduced in a fixed order.
 template <typename T>
-__global__ void __launch_bounds__(256) k_colsum(int64_t M, int N, const T* dy, int64_t lddy, const T* ref,
+__global__ void __launch_bounds__(256, 4) k_colsum(int64_t M, int N, const T* dy, int64_t lddy, const T* ref,
                                                 int64_t ldref, T* dt, int64_t ldt, float* part, int64_t rows_per_blk,
                                                 const float* rs2, T* dt2, int64_t ldt2, int fc2, int64_t cs2) {
   constexpr int EPV = VT<T>::EPV;
