@@ -162,6 +162,16 @@ def test_widths(fi, fo):
         check(run("sage", dtype, "auto", V=700, E=6000, fi=fi, fo=fo, seed=fi), dtype)
 
 
+@pytest.mark.parametrize("fi,fo", [(32, 32), (96, 40), (32, 172)])
+@pytest.mark.parametrize("policy", ["vertex", "edge"])
+def test_split_outputs_off_chunk_grid(fi, fo, policy):
+    """SAGE's split GEMM outputs ([Y | S] forward, [dAgg | dX_s] backward) whose
+    split falls inside a 128-byte output chunk (bf16 widths not multiples of
+    64: C5's 32-wide layers) -- the straddling chunk is stored from registers."""
+    check(run("sage", torch.bfloat16, policy, V=900, E=9000, fi=fi, fo=fo, seed=fi + fo, fuse_relu=True),
+          torch.bfloat16)
+
+
 def test_need_dx_false_and_norms():
     for norm in ("none", "right", "both"):
         check(run("gcn", torch.float32, "edge", norm=norm, need_dx=False), torch.float32)
